@@ -1,0 +1,325 @@
+#!/usr/bin/env python
+"""bench.py — BFS GTEPS over an Elias-Fano-compressed graph on B200.
+
+Contract (driver): ``python bench.py --gpus N --steps K --warmup W`` prints ONE
+JSON line on rank 0.  A "step" is one full BFS (all levels: frontier
+materialisation, scan, partition, decode, visit, compaction — SURVEY §8(a)
+rows a1-a7) from one seeded source over the BASELINE.json configs[1] graph
+(RMAT scale 24, edgefactor 16) resident in HBM.
+
+  value      whole-job GTEPS = sum over ranks of traversed edges / max-over-ranks
+             device time (traversed edges = sum of degrees of reached vertices,
+             DESIGN.md reading C18)
+  e2e        the same metric through the C ABI with a pinned HOST depth buffer
+             (device->host copy of the depth array inside the timed region)
+  roofline   expand+decode kernel: algorithmic bytes (compressed list bytes of the
+             frontier + 21 B per frontier vertex) / its
+             CUDA-event time, against MEASURED_PEAKS.json hbm_gbs
+  cpu_baseline  the oracle (plain single-threaded FIFO BFS over CSR) timed on
+             this host on a bounded sample (one BFS of the same graph)
+
+``--impl reference`` runs the reference arm: the oracle, as it stands, on the
+host cores, same config/metric (each step = one oracle BFS).
+With N > 1 (torchrun) ranks run disjoint seeded sources (independent BFS
+problems, no data-path collective): "scaling": "weak".
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "BFS GTEPS on EF-compressed graph"
+UNIT = "GTEPS"
+
+
+def parse():
+    p = argparse.ArgumentParser()
+    p.add_argument("--gpus", type=int, default=1)
+    p.add_argument("--steps", type=int, default=10)
+    p.add_argument("--warmup", type=int, default=3)
+    p.add_argument("--impl", default="efg", choices=["efg", "reference"])
+    p.add_argument("--config", type=int, default=2, help="BASELINE.json config index (1-based)")
+    p.add_argument("--scale", type=int, default=None, help="override RMAT scale (debug only)")
+    p.add_argument("--no-cpu-baseline", action="store_true")
+    p.add_argument("--profile-levels", action="store_true", help="print per-level stats to stderr")
+    return p.parse_args()
+
+
+def dist_env():
+    rank = int(os.environ.get("RANK", "0"))
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    return rank, world, local
+
+
+class ClockSampler:
+    """nvidia-smi clocks / throttle reasons sampled during the timed region."""
+
+    Q = ("clocks.sm,clocks.max.sm,clocks_event_reasons.active,clocks_event_reasons.hw_slowdown,"
+         "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+         "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index: int):
+        self.index = index
+        self.proc = None
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.Q}",
+                 "--format=csv,noheader,nounits", "-lms", "100"],
+                stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+        except OSError:
+            self.proc = None
+
+    def stop(self) -> dict:
+        if self.proc is None:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        self.proc.terminate()
+        try:
+            out, _ = self.proc.communicate(timeout=5)
+        except subprocess.TimeoutExpired:
+            self.proc.kill()
+            out, _ = self.proc.communicate()
+        sm, smax, reasons = [], None, set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for line in out.strip().splitlines():
+            f = [x.strip() for x in line.split(",")]
+            if len(f) < 7:
+                continue
+            try:
+                sm.append(float(f[0]))
+                smax = float(f[1])
+            except ValueError:
+                continue
+            for nm, val in zip(names, f[3:7]):
+                if val.lower().startswith("active"):
+                    reasons.add(nm)
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": smax,
+                "reasons": sorted(reasons), "samples": len(sm)}
+
+
+def load_peak():
+    path = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(path):
+        with open(path) as f:
+            pk = json.load(f)
+        return float(pk["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs)"
+    return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
+
+
+def make_graph_edges(cfg: int, scale: int | None):
+    import synth
+    t0 = time.time()
+    n, src, dst = synth.config_edges(cfg, scale_override=scale)
+    return n, src, dst, time.time() - t0
+
+
+def cpu_count_used() -> int:
+    return 1  # the oracle is single-threaded by construction
+
+
+def run_reference(args, rank, world):
+    """Reference arm: the oracle (plain CPU BFS) on the host, rank 0 only."""
+    if rank != 0:
+        return
+    import oracle
+    import synth
+    n, src, dst, gen_s = make_graph_edges(args.config, args.scale)
+    t0 = time.time()
+    vlist, elist = oracle.csr_build(n, src, dst)
+    csr_s = time.time() - t0
+    del src, dst
+    deg = np.diff(vlist)
+    srcs = synth.sources(n, args.warmup + args.steps, seed=1000 + args.config,
+                         nonisolated_mask=deg > 0)
+    for s in srcs[:args.warmup]:
+        oracle.bfs(vlist, elist, int(s))
+    edges, secs = 0, 0.0
+    for s in srcs[args.warmup:]:
+        t = time.perf_counter()
+        d = oracle.bfs(vlist, elist, int(s))
+        secs += time.perf_counter() - t
+        edges += int(deg[d >= 0].sum())
+    v = edges / secs / 1e9
+    cfgname = synth.CONFIGS[args.config]["name"] + (f"_scale{args.scale}" if args.scale else "")
+    line = {"impl": "reference", "metric": METRIC, "value": v, "unit": UNIT, "n_gpus": args.gpus,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": secs / args.steps * 1e3,
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u32",
+            "data": "synthetic",
+            "config": {"workload": cfgname, "n": int(n), "m_directed": int(vlist[-1]),
+                       "sources": args.steps, "csr_build_s": round(csr_s, 2)},
+            "cpu_baseline": {"value": v, "unit": UNIT, "cores": 1, "kind": "oracle",
+                             "sample": f"{args.steps} single-threaded FIFO BFS over the oracle CSR"},
+            "e2e": {"value": v, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+def main():
+    args = parse()
+    rank, world, local = dist_env()
+    if args.impl == "reference":
+        run_reference(args, rank, world)
+        return
+
+    import torch
+    import synth
+    import paper_conf_ipps_gerak23_b200 as efg
+
+    if world > 1:
+        import torch.distributed as dist
+        torch.cuda.set_device(local)
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    stream = torch.cuda.Stream(device=dev)
+
+    n, src, dst, gen_s = make_graph_edges(args.config, args.scale)
+    g = efg.Graph.build(n, src, dst, device=local, stream=stream.cuda_stream)
+    del src, dst
+    info = g.info
+    vlist, nlb, offsets, _ = g.export()
+    deg = np.diff(vlist)
+    sizes = np.diff(offsets).astype(np.int64)
+
+    nsrc = args.warmup + args.steps
+    all_srcs = synth.sources(n, nsrc * world, seed=1000 + args.config, nonisolated_mask=deg > 0)
+    my = all_srcs[rank::world][:nsrc]
+
+    depth = torch.empty(n, dtype=torch.int32, device=dev)
+    with torch.cuda.stream(stream):
+        for s in my[:args.warmup]:
+            g.bfs(int(s), depth=depth)
+    torch.cuda.synchronize()
+
+    # ---- timed region: device-resident input, device depth output ----
+    if world > 1:
+        torch.distributed.barrier()
+    torch.cuda.synchronize()
+    clk = ClockSampler(local)
+    clk.start()
+    time.sleep(0.3)
+    e0 = torch.cuda.Event(enable_timing=True)
+    e1 = torch.cuda.Event(enable_timing=True)
+    stats = []
+    e0.record(stream)
+    with torch.cuda.stream(stream):
+        for s in my[args.warmup:]:
+            _, _, st = g.bfs(int(s), depth=depth, stats=True)
+            stats.append((int(s), st))
+    e1.record(stream)
+    torch.cuda.synchronize()
+    clocks = clk.stop()
+    ms = e0.elapsed_time(e1)
+    edges = sum(st["edges_traversed"] for _, st in stats)
+    launches = sum(st["kernel_launches"] for _, st in stats)
+    t_tot = torch.tensor([ms], dtype=torch.float64, device=dev)
+    e_tot = torch.tensor([edges], dtype=torch.float64, device=dev)
+    if world > 1:
+        import torch.distributed as dist
+        dist.all_reduce(t_tot, op=dist.ReduceOp.MAX)
+        dist.all_reduce(e_tot, op=dist.ReduceOp.SUM)
+    value = float(e_tot.item()) / (float(t_tot.item()) * 1e-3) / 1e9
+
+    # ---- roofline of the expand+decode kernel (per-level algorithmic bytes) ----
+    alg_bytes, exp_ms, exp_launch = 0, 0.0, 0
+    lvl_rows = []
+    for s, st in stats:
+        d = g.bfs(s)  # host depth to attribute frontier bytes per level (untimed)
+        for L in range(st["levels"]):
+            fr = d == L
+            b = int(sizes[fr].sum()) + 21 * int(fr.sum())
+            alg_bytes += b
+            lvl_rows.append((s, L, int(fr.sum()), int(st["level_edges"][L]), b,
+                             float(st["level_expand_ms"][L])))
+        exp_ms += st["expand_ms"]
+        exp_launch += st["expand_launches"]
+    peak, peak_src = load_peak()
+    achieved = alg_bytes / (exp_ms * 1e-3) / 1e9 if exp_ms > 0 else 0.0
+    if args.profile_levels and rank == 0:
+        for r in lvl_rows:
+            print("level src=%d L=%d |F|=%d E=%d bytes=%d expand_ms=%.4f GB/s=%.1f" %
+                  (*r, r[4] / max(r[5], 1e-9) / 1e6), file=sys.stderr)
+
+    # ---- e2e: through the C ABI with a pinned host depth buffer ----
+    hdepth = torch.empty(n, dtype=torch.int32, pin_memory=True)
+    e2e_edges = 0
+    torch.cuda.synchronize()
+    if world > 1:
+        torch.distributed.barrier()
+    t0 = time.perf_counter()
+    for s, st in stats:
+        g.bfs(s, depth=hdepth)  # includes the device->host copy of depth
+        e2e_edges += st["edges_traversed"]
+    e2e_s = time.perf_counter() - t0
+    e2e_t = torch.tensor([e2e_s], dtype=torch.float64, device=dev)
+    e2e_e = torch.tensor([e2e_edges], dtype=torch.float64, device=dev)
+    if world > 1:
+        import torch.distributed as dist
+        dist.all_reduce(e2e_t, op=dist.ReduceOp.MAX)
+        dist.all_reduce(e2e_e, op=dist.ReduceOp.SUM)
+    e2e_val = float(e2e_e.item()) / float(e2e_t.item()) / 1e9
+
+    # ---- cpu baseline: the oracle on a bounded sample (rank 0, N=1 only) ----
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        import oracle
+        t0 = time.time()
+        ov, oe = oracle.csr_build(n, *synth.config_edges(args.config, scale_override=args.scale)[1:])
+        csr_s = time.time() - t0
+        s0 = stats[0][0]
+        t = time.perf_counter()
+        dref = oracle.bfs(ov, oe, s0)
+        cs = time.perf_counter() - t
+        ce = int(np.diff(ov)[dref >= 0].sum())
+        ok = bool(np.array_equal(dref, g.bfs(s0)))
+        cpu = {"value": ce / cs / 1e9, "unit": UNIT, "cores": 1, "kind": "oracle",
+               "sample": f"one single-threaded FIFO BFS (source {s0}) over the oracle CSR of the "
+                         f"same graph ({cs:.1f} s; CSR build {csr_s:.1f} s untimed)",
+               "parity_bit_exact": ok}
+        del ov, oe
+
+    if rank == 0:
+        cfgname = synth.CONFIGS[args.config]["name"] + (f"_scale{args.scale}" if args.scale else "")
+        line = {
+            "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": float(t_tot.item()) / args.steps,
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u32",
+            "data": "synthetic",
+            "config": {"workload": cfgname, "n": int(n), "m_directed": int(info["m"]),
+                       "sources_per_rank": args.steps, "fwd_quantum": int(info["fwd_quantum"]),
+                       "efg_bytes_per_edge": (info["data_bytes"] + 17 * n) / info["m"],
+                       "ef_data_bytes_per_edge": info["data_bytes"] / info["m"],
+                       "csr32_over_efg": (4 * info["m"] + 4 * (n + 1)) / (info["data_bytes"] + 17 * n),
+                       "l2_policy": "inputs larger than L2 (EF data %.2f GB > 126 MB)" % (info["data_bytes"] / 1e9),
+                       "parallelism": f"{world} independent BFS replicas" if world > 1 else "1 GPU",
+                       "build_s": round(info["build_seconds"], 2), "gen_s": round(gen_s, 2)},
+            "clocks": clocks,
+            "gpu_launches": launches,
+            "roofline": {"bound": "hbm", "kernel": "expand_kernel (a4+a5+a6)",
+                         "achieved": achieved, "peak": peak, "unit": "GB/s",
+                         "frac": achieved / peak, "traffic": None, "peak_source": peak_src,
+                         "expand_launches": exp_launch, "expand_ms_total": exp_ms,
+                         "expand_share_of_step": exp_ms / ms if ms else None},
+            "e2e": {"value": e2e_val, "unit": UNIT, "h2d_bytes_per_step": 4,
+                    "d2h_bytes_per_step": 4 * n},
+            "cpu_baseline": cpu,
+        }
+        print(json.dumps(line), flush=True)
+    g.free()
+    if world > 1:
+        torch.distributed.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

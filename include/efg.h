@@ -1,0 +1,218 @@
+/*
+ * efg.h — C ABI of the B200-native Elias-Fano graph (EFG) traversal library
+ * (libefg.so).  Implements the data-parallel hot path of
+ *   P. Gera, H. Kim, "Traversing Large Compressed Graphs on GPUs", IPDPS'23
+ * cited as "P:<line> §<section>" against the extracted text PAPER.md, and
+ * SURVEY.md §8(b) for the boundary.
+ *
+ * Conventions for every call
+ *   - Plain C types only.  Sizes are element counts unless stated.
+ *   - Every call returns efg_status; on failure efg_last_error() returns a
+ *     thread-local, NUL-terminated message that stays valid until the next call
+ *     on the same thread.  No call aborts, throws, or leaves a partial handle.
+ *   - Output pointers marked "host or device" are classified with
+ *     cudaPointerGetAttributes: device (or managed) pointers are written by the
+ *     GPU in stream order, host pointers are filled by a device->host copy
+ *     before the call returns.
+ *   - A handle is not safe for concurrent calls from several threads; distinct
+ *     handles are independent.  All GPU work of a handle is issued on the
+ *     stream given at build time, and every call synchronises that stream
+ *     before returning (results are complete on return).
+ */
+#ifndef EFG_H
+#define EFG_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum efg_status {
+    EFG_OK = 0,
+    EFG_EINVAL = 1,  /* null pointer, n == 0, n > 2^32-1, bad option            */
+    EFG_ERANGE = 2,  /* a vertex id >= n (input edge, source, vertex range)      */
+    EFG_ENOMEM = 3,  /* host or device allocation failed                         */
+    EFG_ECUDA = 4,   /* a CUDA runtime error (message in efg_last_error)         */
+    EFG_ENCCL = 5,   /* a NCCL error (multi-GPU)                                 */
+    EFG_ENOTSUP = 6, /* the operation is not available on this handle            */
+    EFG_ESTATE = 7   /* handle in the wrong state (e.g. host-only handle)        */
+} efg_status;
+
+/* efg_build_opts.flags (SURVEY §8(c) readings C11, C12) */
+#define EFG_SYMMETRIZE 0x1u       /* add (d,s) for every input (s,d): "_sym" graphs  */
+#define EFG_DEDUP 0x2u            /* keep one copy of each directed (s,d)                   */
+#define EFG_DROP_SELF_LOOPS 0x4u  /* remove (v,v)                                           */
+#define EFG_DEFAULT_FLAGS (EFG_SYMMETRIZE | EFG_DEDUP | EFG_DROP_SELF_LOOPS)
+
+typedef struct efg_graph efg_graph; /* opaque: host EFG arrays + device copy */
+typedef struct efg_dist efg_dist;   /* opaque: multi-GPU communicator        */
+
+typedef struct efg_build_opts {
+    /* Forward-pointer quantum k (§VI-C; k = 512 in the paper's
+     * experiments).  0 disables forward pointers (lists are then never
+     * split across warps).  Default 512. */
+    uint32_t fwd_quantum;
+    /* EFG_* flags above.  Default EFG_DEFAULT_FLAGS. */
+    uint32_t flags;
+    /* CUDA device ordinal for the device copy; -1 = host-only handle (builder
+     * output only: efg_info / efg_export work, traversals return EFG_ESTATE). */
+    int32_t device;
+    /* Host threads for the builder; 0 = OpenMP default. */
+    uint32_t n_threads;
+    /* cudaStream_t for all device work of this handle; NULL = legacy default. */
+    void *stream;
+    /* Optional per-input-edge fp32 weights (SSSP; uncompressed).
+     * NULL = unweighted.  Weights of duplicate (s,d) pairs: the minimum is kept.
+     * With EFG_SYMMETRIZE the reverse edge gets the same weight. */
+    const float *weights;
+    /* Multi-GPU: NULL = the whole graph on `device`.  Otherwise this rank keeps
+     * the row range [row_lo, row_hi) chosen by efg_partition (1-D partition,
+     * SURVEY §8(e)); every rank passes the same edge list. */
+    efg_dist *dist;
+} efg_build_opts;
+
+/* Fill *o with the defaults above (k = 512, EFG_DEFAULT_FLAGS, device 0). */
+void efg_default_opts(efg_build_opts *o);
+
+/*
+ * efg_build — edge list -> CSR -> EFG (§III-D, §V).
+ *   n           number of vertices, 1 <= n <= 2^32-1; ids are 0..n-1
+ *   m           number of input edges
+ *   src, dst    host arrays of m vertex ids (caller-owned, read-only; they may
+ *               be freed after the call returns)
+ *   opts        NULL = defaults
+ *   out         receives the new handle (NULL on failure)
+ * Each vertex's neighbour list is sorted ascending, de-duplicated and
+ * stripped of self-loops per flags, then Elias-Fano encoded per P:81-96 with
+ * l = max{0, floor(log2(u/n))}, u = the list's last element (readings C1-C3),
+ * laid out as [forward pointers (uint32 LE)][lower bits][upper bits], each
+ * section byte-aligned, LSB-first within bytes (readings C6-C8).  The four
+ * arrays of P:113 (vlist, num_lower_bits, offsets, data) stay on the host
+ * (efg_export) and, if opts->device >= 0, are uploaded in a packed device
+ * layout.
+ * Errors: EFG_EINVAL (null pointers, n == 0, n > 2^32-1), EFG_ERANGE (an id >=
+ * n), EFG_ENOMEM, EFG_ECUDA.
+ */
+efg_status efg_build(uint64_t n, uint64_t m, const uint32_t *src, const uint32_t *dst,
+                     const efg_build_opts *opts, efg_graph **out);
+
+/* Release everything the handle owns (host and device).  NULL-safe. */
+void efg_free(efg_graph *g);
+
+typedef struct efg_info_t {
+    uint64_t n;              /* vertices                                           */
+    uint64_t m;              /* directed edges after symmetrise/dedup (= vlist[n]) */
+    uint64_t m_input;        /* input edges as given                               */
+    uint32_t fwd_quantum;    /* k                                                  */
+    uint32_t device;         /* CUDA ordinal, or 0xFFFFFFFF for host-only          */
+    uint64_t data_bytes;     /* sum of per-vertex sizes = offsets[n]               */
+    uint64_t fwd_bytes;      /* forward-pointer sections                           */
+    uint64_t lower_bytes;    /* lower-bits sections                                */
+    uint64_t upper_bytes;    /* upper-bits sections                                */
+    uint64_t apriori_bits;   /* sum over lists of n*l + n + (u >> l)  */
+    uint64_t vertex_bytes;   /* host vertex arrays: vlist 8 + offsets 8 + nlb 1     */
+    uint64_t device_bytes;   /* device memory held by the handle                   */
+    uint64_t row_lo, row_hi; /* owned row range (whole graph: 0, n)                */
+    double build_seconds;    /* host builder wall time                             */
+} efg_info_t;
+
+efg_status efg_info(const efg_graph *g, efg_info_t *info);
+
+/* Copy the P:113 arrays to caller-owned host buffers (any may be NULL):
+ * vlist[n+1] (uint64), num_lower_bits[n] (uint8), offsets[n+1] (uint64),
+ * data[offsets[n]] (uint8).  For a partitioned handle these describe the
+ * owned row range (vertices outside it have empty lists). */
+efg_status efg_export(const efg_graph *g, uint64_t *vlist, uint8_t *num_lower_bits,
+                      uint64_t *offsets, uint8_t *data);
+
+/*
+ * efg_decode — GPU decode of the neighbour lists of vertices [v0, v1) into
+ * CSR order: out[vlist[v] - vlist[v0] + i] = x_i of v (§IV-A), using
+ * the same frontier/partition/decode kernels as efg_bfs (the BFS visit step is
+ * replaced by a store).  out: host or device, vlist[v1]-vlist[v0] entries.
+ * Errors: EFG_ERANGE (v0 > v1 or v1 > n), EFG_ESTATE (host-only handle).
+ */
+efg_status efg_decode(efg_graph *g, uint32_t v0, uint32_t v1, uint32_t *out);
+
+/* Per-call statistics (all fields except level_cap / arrays are outputs). */
+typedef struct efg_stats {
+    uint32_t levels;           /* BFS levels expanded (frontiers processed)          */
+    uint32_t level_cap;        /* in: capacity of the per-level arrays (0 = none)    */
+    uint64_t edges_traversed;  /* sum of deg(f) over every expanded frontier vertex  */
+    uint64_t vertices_reached; /* vertices with depth >= 0                           */
+    float device_ms;           /* device time of the traversal (CUDA events)         */
+    float expand_ms;           /* device time inside the expand+decode kernel        */
+    uint32_t expand_launches;  /* number of expand+decode launches                   */
+    uint32_t kernel_launches;  /* all kernels launched by the call                   */
+    uint64_t expand_bytes;     /* algorithmic bytes of the expand launches (DESIGN)  */
+    uint64_t *level_frontier;  /* in/out: |F_L| per level (level_cap entries)        */
+    uint64_t *level_edges;     /* in/out: E_L = sum of frontier degrees per level    */
+    float *level_expand_ms;    /* in/out: expand kernel time per level, or NULL      */
+} efg_stats;
+
+/*
+ * efg_bfs — level-synchronous top-down BFS from `source` over the compressed
+ * graph (Alg. 1; frontier partition P:125-135; in-kernel decode
+ * P:137-177).  depth[v] = hop distance from source, -1 if unreachable
+ * (reading C15).  parent (nullable): some neighbour u with depth[u] ==
+ * depth[v]-1 (any valid one, reading C28); parent[source] = source; unreached
+ * 0xFFFFFFFF.  depth / parent: host or device, n entries, caller-allocated.
+ * With a partitioned handle the call is collective over the communicator:
+ * every rank calls it with the same source and receives the full depth array.
+ * Errors: EFG_ERANGE (source >= n), EFG_ESTATE, EFG_ECUDA, EFG_ENCCL.
+ */
+efg_status efg_bfs(efg_graph *g, uint32_t source, int32_t *depth, uint32_t *parent,
+                   efg_stats *st);
+
+/*
+ * efg_sssp — single-source shortest paths with the build-time weights (P:185
+ * §VI-F): frontier Bellman-Ford, relaxed vertices marked in a bitmap, fp32
+ * distances with single-rounding adds (dist[u] + w, no contraction; reading
+ * C20).  dist: host or device, n entries; unreached = +inf.
+ * Errors: EFG_EINVAL (graph built without weights), EFG_ERANGE, EFG_ESTATE.
+ */
+efg_status efg_sssp(efg_graph *g, uint32_t source, float *dist, efg_stats *st);
+
+/*
+ * efg_pagerank — PageRank over the compressed graph (§VI-F; capped at
+ * `iters` iterations, 50 in the paper P:201).  Reading C21: r0 = 1/N,
+ * r' = (1-d)/N + d*(sum_{u in N(v)} r(u)/deg(u) + D/N), D = rank mass on
+ * degree-0 vertices, exactly `iters` iterations, fp64 accumulation.
+ * rank: host or device, n doubles.
+ */
+efg_status efg_pagerank(efg_graph *g, double damping, uint32_t iters, double *rank,
+                        efg_stats *st);
+
+/* ---- multi-GPU: 1-D row partition, per-level exchange ---- */
+
+/* 128-byte opaque id (an ncclUniqueId).  Rank 0 creates it and the caller
+ * broadcasts it (e.g. over torch.distributed) to every rank. */
+efg_status efg_get_unique_id(uint8_t id[128]);
+
+/* Create this rank's communicator (ranks 0..world-1, one GPU per rank). */
+efg_status efg_dist_init(int rank, int world, const uint8_t id[128], int device,
+                         efg_dist **out);
+void efg_dist_free(efg_dist *d);
+
+/*
+ * efg_partition — the 1-D row partition used by efg_build with opts->dist:
+ * rank r owns vertices [bounds[r], bounds[r+1]).  Boundaries balance
+ * sum(offsets bytes) + 29 bytes per vertex and are multiples
+ * of 64 (so bitmap words have one owner).  bounds: world+1 entries.
+ * Host-only computation over the CSR degrees implied by (n, m, src, dst, flags).
+ */
+efg_status efg_partition(uint64_t n, const uint64_t *vlist, const uint64_t *offsets, int world,
+                         uint64_t *bounds);
+
+/* Thread-local message for the last failing call on this thread ("" if none). */
+const char *efg_last_error(void);
+
+/* Library version string. */
+const char *efg_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* EFG_H */

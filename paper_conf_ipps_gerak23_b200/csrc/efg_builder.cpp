@@ -1,0 +1,226 @@
+// efg_builder.cpp — host-side EFG builder (north_star (a)).
+//
+// edge list --(symmetrise, "_sym")--> directed multiset
+//           --(bucket by source, sort each list, drop self-loops/duplicates:
+//              readings C11/C12)--> CSR vlist/elist (§III-D)
+//           --(per-vertex Elias-Fano, §IV, layout P:111-117 §V,
+//              forward pointers P:157 §VI-C)--> vlist, num_lower_bits, offsets, data
+//
+// Two passes as the paper notes the size is known a priori: pass 1
+// computes every list's byte size from (n, u, k) alone, an exclusive scan gives
+// `offsets`, pass 2 encodes all lists in parallel (OpenMP).
+#include <omp.h>
+
+#include <algorithm>
+#include <chrono>
+#include <cstring>
+#include <memory>
+#include <new>
+
+#include "efg_internal.h"
+
+namespace efg {
+
+ListGeom list_geom(uint64_t n, uint64_t u, uint32_t k)
+{
+    ListGeom g{0, 0, 0, 0};
+    if (n == 0) return g;                                  // reading C10
+    const uint64_t q = u / n;                              // reading C3 (integer u/n)
+    g.l = q ? (uint32_t)(63 - __builtin_clzll(q)) : 0u;    // floor(log2(u/n)), C1
+    g.fwd = k ? 4ull * (n / k) : 0ull;                     // C8: uint32 per pointer
+    g.lower = (n * g.l + 7) / 8;                           // P:89 lower-bits array
+    g.upper = ((u >> g.l) + n + 7) / 8;                    // C4: n stop bits + (u>>l) zeros
+    return g;
+}
+
+namespace {
+
+// Exclusive scan in place over a[0..len) with a[len] = total (a has len+1 slots).
+void exclusive_scan_inplace(uint64_t *a, uint64_t len)
+{
+    uint64_t run = 0;
+    for (uint64_t i = 0; i < len; ++i) {
+        uint64_t x = a[i];
+        a[i] = run;
+        run += x;
+    }
+    a[len] = run;
+}
+
+inline uint32_t float_key(float w)
+{
+    uint32_t b;
+    std::memcpy(&b, &w, 4);
+    return b;  // weights are >= 0, so the IEEE bit pattern orders like the value
+}
+
+// Encode one sorted, duplicate-free list x[0..n) at `out` (pre-zeroed).
+void encode_list(const uint32_t *x, uint64_t n, uint32_t k, const ListGeom &g, uint8_t *out)
+{
+    const uint32_t l = g.l;
+    // forward pointers: fwd[j] = x[(j+1)k-1] >> l  (= select1(i) - i)
+    if (k) {
+        const uint64_t F = n / k;
+        for (uint64_t j = 0; j < F; ++j) {
+            const uint32_t f = x[(j + 1) * k - 1] >> l;
+            std::memcpy(out + 4 * j, &f, 4);  // little endian host
+        }
+    }
+    // lower bits: element i occupies bits [i*l, (i+1)*l), LSB first (C6)
+    uint8_t *lower = out + g.fwd;
+    if (l) {
+        const uint64_t mask = (1ull << l) - 1;
+        uint64_t acc = 0;
+        uint32_t nb = 0;
+        uint64_t p = 0;
+        for (uint64_t i = 0; i < n; ++i) {
+            acc |= ((uint64_t)x[i] & mask) << nb;
+            nb += l;
+            while (nb >= 8) {
+                lower[p++] = (uint8_t)acc;
+                acc >>= 8;
+                nb -= 8;
+            }
+        }
+        if (nb) lower[p++] = (uint8_t)acc;
+    }
+    // upper bits: stop bit of element i at position (x[i] >> l) + i
+    uint8_t *upper = lower + g.lower;
+    for (uint64_t i = 0; i < n; ++i) {
+        const uint64_t pos = ((uint64_t)(x[i] >> l)) + i;
+        upper[pos >> 3] |= (uint8_t)(1u << (pos & 7));
+    }
+}
+
+}  // namespace
+
+efg_status build_host(uint64_t n, uint64_t m, const uint32_t *src, const uint32_t *dst,
+                      const efg_build_opts &o, HostEFG &out)
+{
+    const auto t0 = std::chrono::steady_clock::now();
+    if (o.n_threads) omp_set_num_threads((int)o.n_threads);
+    const bool sym = o.flags & EFG_SYMMETRIZE;
+    const bool dedup = o.flags & EFG_DEDUP;
+    const bool noself = o.flags & EFG_DROP_SELF_LOOPS;
+    const bool weighted = o.weights != nullptr;
+    const uint32_t k = o.fwd_quantum;
+
+    // ---- validate ids (EFG_ERANGE) ----
+    uint64_t bad = 0;
+#pragma omp parallel for reduction(+ : bad) schedule(static)
+    for (int64_t e = 0; e < (int64_t)m; ++e) bad += (src[e] >= n) | (dst[e] >= n);
+    if (bad) return set_error(EFG_ERANGE, "efg_build: " + std::to_string(bad) + " edge endpoints >= n");
+
+    try {
+        // ---- directed multiset degrees ----
+        std::vector<uint64_t> start(n + 1, 0);
+#pragma omp parallel for schedule(static)
+        for (int64_t e = 0; e < (int64_t)m; ++e) {
+            __atomic_fetch_add(&start[src[e]], 1ull, __ATOMIC_RELAXED);
+            if (sym) __atomic_fetch_add(&start[dst[e]], 1ull, __ATOMIC_RELAXED);
+        }
+        exclusive_scan_inplace(start.data(), n);
+        const uint64_t total = start[n];
+
+        // ---- bucket by source (order inside a bucket is fixed by the sort below) ----
+        std::unique_ptr<uint64_t[]> cur(new uint64_t[n]);
+        std::memcpy(cur.get(), start.data(), n * sizeof(uint64_t));
+        std::unique_ptr<uint64_t[]> tmp(new uint64_t[total ? total : 1]);  // (nbr<<32)|wkey
+#pragma omp parallel for schedule(static)
+        for (int64_t e = 0; e < (int64_t)m; ++e) {
+            const uint64_t wk = weighted ? float_key(o.weights[e]) : 0u;
+            uint64_t p = __atomic_fetch_add(&cur[src[e]], 1ull, __ATOMIC_RELAXED);
+            tmp[p] = ((uint64_t)dst[e] << 32) | wk;
+            if (sym) {
+                p = __atomic_fetch_add(&cur[dst[e]], 1ull, __ATOMIC_RELAXED);
+                tmp[p] = ((uint64_t)src[e] << 32) | wk;
+            }
+        }
+        cur.reset();
+
+        // ---- sort each list; drop self loops / duplicates (keep min weight) ----
+        std::vector<uint64_t> deg(n + 1, 0);
+#pragma omp parallel for schedule(dynamic, 512)
+        for (int64_t v = 0; v < (int64_t)n; ++v) {
+            uint64_t *a = tmp.get() + start[v];
+            const uint64_t len = start[v + 1] - start[v];
+            std::sort(a, a + len);
+            uint64_t w = 0;
+            for (uint64_t i = 0; i < len; ++i) {
+                const uint32_t x = (uint32_t)(a[i] >> 32);
+                if (noself && x == (uint32_t)v) continue;
+                if (dedup && w && (uint32_t)(a[w - 1] >> 32) == x) continue;
+                a[w++] = a[i];
+            }
+            deg[v] = w;
+        }
+        // partition: keep only the owned rows' lists
+        const uint64_t lo = o.dist ? out.row_lo : 0, hi = o.dist ? out.row_hi : n;
+        for (uint64_t v = 0; v < n; ++v)
+            if (v < lo || v >= hi) deg[v] = 0;
+        out.vlist.assign(deg.begin(), deg.end());
+        exclusive_scan_inplace(out.vlist.data(), n);
+        out.m = out.vlist[n];
+        out.n = n;
+        out.m_input = m;
+        out.k = k;
+        out.row_lo = lo;
+        out.row_hi = hi;
+
+        // ---- pass 1: a-priori sizes -> offsets ----
+        if (weighted) out.weights.resize(out.m);
+        out.nlb.assign(n, 0);
+        out.offsets.assign(n + 1, 0);
+        uint64_t fb = 0, lb = 0, ub = 0, ab = 0;
+#pragma omp parallel for schedule(dynamic, 1024) reduction(+ : fb, lb, ub, ab)
+        for (int64_t v = 0; v < (int64_t)n; ++v) {
+            const uint64_t d = deg[v];
+            if (!d) continue;
+            const uint64_t *a = tmp.get() + start[v];
+            const uint32_t u = (uint32_t)(a[d - 1] >> 32);
+            const ListGeom g = list_geom(d, u, k);
+            out.nlb[v] = (uint8_t)g.l;
+            out.offsets[v] = g.fwd + g.lower + g.upper;
+            fb += g.fwd;
+            lb += g.lower;
+            ub += g.upper;
+            ab += d * g.l + d + ((uint64_t)u >> g.l);
+        }
+        exclusive_scan_inplace(out.offsets.data(), n);
+        out.fwd_bytes = fb;
+        out.lower_bytes = lb;
+        out.upper_bytes = ub;
+        out.apriori_bits = ab;
+
+        // ---- pass 2: encode (parallel over vertices) ----
+        out.data.assign(out.offsets[n], 0);
+#pragma omp parallel
+        {
+            std::vector<uint32_t> x;
+#pragma omp for schedule(dynamic, 1024)
+            for (int64_t v = 0; v < (int64_t)n; ++v) {
+                const uint64_t d = deg[v];
+                if (!d) continue;
+                const uint64_t *a = tmp.get() + start[v];
+                x.resize(d);
+                for (uint64_t i = 0; i < d; ++i) x[i] = (uint32_t)(a[i] >> 32);
+                if (weighted) {
+                    float *wo = out.weights.data() + out.vlist[v];
+                    for (uint64_t i = 0; i < d; ++i) {
+                        const uint32_t b = (uint32_t)a[i];
+                        std::memcpy(&wo[i], &b, 4);
+                    }
+                }
+                const ListGeom g = list_geom(d, x[d - 1], k);
+                encode_list(x.data(), d, k, g, out.data.data() + out.offsets[v]);
+            }
+        }
+    } catch (const std::bad_alloc &) {
+        return set_error(EFG_ENOMEM, "efg_build: host allocation failed");
+    }
+    out.build_seconds =
+        std::chrono::duration<double>(std::chrono::steady_clock::now() - t0).count();
+    return EFG_OK;
+}
+
+}  // namespace efg

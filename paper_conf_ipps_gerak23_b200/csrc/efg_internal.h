@@ -1,0 +1,123 @@
+// efg_internal.h — internal structures shared by the host builder
+// (efg_builder.cpp), the C-ABI glue (efg_api.cu) and the kernels (efg_kernels.cu).
+// Not part of the ABI.  Citations: PAPER.md "P:<line> §<section>".
+#pragma once
+
+#include <cstdint>
+#include <cstddef>
+#include <string>
+#include <vector>
+
+#include "efg.h"
+
+namespace efg {
+
+// ---------------------------------------------------------------------------
+// Host-side EFG (§V): the four arrays of the format.
+// ---------------------------------------------------------------------------
+struct HostEFG {
+    uint64_t n = 0;                 // vertices
+    uint64_t m = 0;                 // directed edges (post symmetrise/dedup)
+    uint64_t m_input = 0;
+    uint32_t k = 512;               // forward-pointer quantum
+    std::vector<uint64_t> vlist;    // n+1  (degree = vlist[v+1]-vlist[v])
+    std::vector<uint8_t> nlb;       // n    num_lower_bits
+    std::vector<uint64_t> offsets;  // n+1  exclusive sum of per-vertex byte sizes
+    std::vector<uint8_t> data;      // offsets[n] bytes (+ padding on device)
+    std::vector<float> weights;     // m (CSR order) or empty
+    uint64_t fwd_bytes = 0, lower_bytes = 0, upper_bytes = 0, apriori_bits = 0;
+    uint64_t row_lo = 0, row_hi = 0;
+    double build_seconds = 0.0;
+};
+
+// Elias-Fano parameters of one list (readings C1-C4, C7, C8).
+struct ListGeom {
+    uint32_t l;        // lower bits per element
+    uint64_t fwd;      // bytes of forward pointers = 4*floor(n/k)
+    uint64_t lower;    // bytes of lower bits = ceil(n*l/8)
+    uint64_t upper;    // bytes of upper bits = ceil(((u>>l)+n)/8)
+};
+
+ListGeom list_geom(uint64_t n, uint64_t u, uint32_t k);
+
+// Builder (efg_builder.cpp).  Returns EFG_OK or an error with set_error().
+efg_status build_host(uint64_t n, uint64_t m, const uint32_t *src, const uint32_t *dst,
+                      const efg_build_opts &o, HostEFG &out);
+
+// ---------------------------------------------------------------------------
+// Device layout
+// ---------------------------------------------------------------------------
+// Packed 16-byte vertex record: one aligned 128-bit load gives everything the
+// frontier step a1 needs (degree, data offset, l, upper-section length).
+struct alignas(16) VRec {
+    uint64_t off_l;   // bits 0..57: offsets[v] (byte offset in data); bits 58..63: l
+    uint32_t deg;     // vlist[v+1]-vlist[v]
+    uint32_t ubytes;  // upper-bits section length in bytes
+};
+static_assert(sizeof(VRec) == 16, "VRec must be 16 bytes");
+
+constexpr int kOffBits = 58;
+constexpr uint64_t kOffMask = (1ull << kOffBits) - 1;
+
+// Tile table entry (step a3): first chunk owned by an edge tile.
+struct alignas(16) TileEntry {
+    uint32_t fi;      // index into the frontier queue
+    uint32_t chunk;   // chunk index within that vertex's list
+    uint64_t e;       // global (level-local) edge index of the chunk start
+};
+static_assert(sizeof(TileEntry) == 16, "TileEntry must be 16 bytes");
+
+// Level control block (device), written by the advance kernel.
+struct LevelCtrl {
+    uint64_t nf;        // frontier size for the next expand
+    uint64_t ne;        // edges out of that frontier (E_L)
+    uint64_t ntiles;    // ceil(ne / tile_edges)
+    uint64_t pad;
+};
+
+constexpr int kExpandThreads = 128;          // 4 warps (static smem < 48 KB)
+constexpr int kAdvanceThreads = 256;         // one bitmap word per thread
+constexpr uint32_t kTileEdges = 2048;        // edges per warp tile (a3)
+
+struct DeviceGraph {
+    int device = -1;
+    void *stream = nullptr;            // cudaStream_t
+    uint64_t n = 0, nwords = 0;        // nwords = ceil(n/32) rounded up
+    uint32_t k = 512;
+    uint8_t *data = nullptr;           // EF data + padding
+    uint64_t data_bytes = 0;
+    VRec *rec = nullptr;               // n records
+    uint64_t *vlist = nullptr;         // n+1 (SSSP weight indexing / decode)
+    float *weights = nullptr;          // m or null
+    // traversal workspace
+    uint32_t *vis = nullptr;           // visited bitmap (nwords)
+    uint32_t *prev = nullptr;          // visited bitmap at the end of the last level
+    uint32_t *queue = nullptr;         // frontier queue (n)
+    TileEntry *tiles = nullptr;        // tile table (max_tiles)
+    uint64_t max_tiles = 0;
+    int32_t *depth = nullptr;          // internal depth (n)
+    uint32_t *parent = nullptr;        // internal parent (n), lazily allocated
+    uint64_t *status = nullptr;        // decoupled look-back status, 2 parities x 2 values x nblk
+    uint64_t status_blocks = 0;
+    LevelCtrl *ctrl = nullptr;         // device control block
+    LevelCtrl *ctrl_host = nullptr;    // pinned mirror
+    float *fbuf = nullptr;             // SSSP distance (n) lazily
+    double *dbuf = nullptr;            // PageRank buffers lazily (3n)
+    uint64_t device_bytes = 0;
+    int num_sms = 148;
+    int expand_blocks = 0;             // persistent grid size
+};
+
+}  // namespace efg
+
+struct efg_graph {
+    efg::HostEFG host;
+    efg::DeviceGraph dev;
+    bool on_device = false;
+};
+
+// error handling (efg_error.cpp)
+namespace efg {
+efg_status set_error(efg_status s, const std::string &msg);
+void clear_error();
+}  // namespace efg

@@ -1,0 +1,123 @@
+"""CPU-side tests of the product's host logic and C ABI (no GPU needed).
+
+* libefg.so loads and exports every symbol include/efg.h declares;
+* the host EFG builder (C++, paper_conf_ipps_gerak23_b200/csrc/efg_builder.cpp)
+  is byte-identical to the independent oracle encoder on the P:113 arrays;
+* error behaviour of the ABI (EFG_EINVAL / EFG_ERANGE / EFG_ESTATE).
+"""
+import os
+import re
+
+import numpy as np
+import pytest
+
+import oracle
+import synth
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def _declared_symbols():
+    src = open(os.path.join(ROOT, "include", "efg.h")).read()
+    return sorted(set(re.findall(r"\b(efg_[a-z_]+)\s*\(", src)) - {"efg_status"})
+
+
+def test_library_exports_every_declared_symbol():
+    import paper_conf_ipps_gerak23_b200 as efg
+    from paper_conf_ipps_gerak23_b200 import _abi
+    declared = _declared_symbols()
+    assert len(declared) >= 14
+    bound = {name for name, _, _ in _abi.SIGNATURES}
+    assert set(declared) == bound, set(declared) ^ bound
+    for name in declared:
+        assert hasattr(efg.lib, name), name
+    assert "sm_100a" in efg.version()
+
+
+def _host_graph(n, src, dst, k=512, flags=None):
+    import paper_conf_ipps_gerak23_b200 as efg
+    kw = {} if flags is None else {"flags": flags}
+    return efg.Graph.build(n, src, dst, k=k, device=-1, **kw)
+
+
+@pytest.mark.parametrize("k", [512, 8, 3, 0])
+def test_builder_byte_identical_to_oracle_random(k):
+    rng = np.random.default_rng(k + 1)
+    n = 2000
+    src = rng.integers(0, n, 30000).astype(np.uint32)
+    dst = (src + rng.integers(0, 50, 30000)).astype(np.uint32) % n
+    src[:100] = dst[:100]  # self loops
+    g = _host_graph(n, src, dst, k=k)
+    vlist, nlb, offsets, data = g.export()
+    ov, oe = oracle.csr_build(n, src, dst)
+    oo, onlb, odata = oracle.efg_encode(ov, oe, k)
+    assert np.array_equal(vlist, ov)
+    assert np.array_equal(offsets, oo)
+    assert np.array_equal(nlb, onlb)
+    assert np.array_equal(data, odata)
+    info = g.info
+    assert info["m"] == oe.size and info["data_bytes"] == odata.size
+    assert info["fwd_bytes"] + info["lower_bytes"] + info["upper_bytes"] == odata.size
+    g.free()
+
+
+def test_builder_byte_identical_rmat_c1_shape():
+    n, src, dst = synth.rmat(14, 16, seed=1)
+    g = _host_graph(n, src, dst)
+    vlist, nlb, offsets, data = g.export()
+    ov, oe = oracle.csr_build(n, src, dst)
+    oo, onlb, odata = oracle.efg_encode(ov, oe, 512)
+    assert np.array_equal(vlist, ov) and np.array_equal(offsets, oo)
+    assert np.array_equal(nlb, onlb) and np.array_equal(data, odata)
+    # a-priori size: sum over lists of n*l + n + (u >> l) bits, and
+    # the byte-rounded sections never exceed it by more than 2 bytes per list
+    deg = np.diff(ov).astype(np.int64)
+    nz = deg > 0
+    u = oe[(ov[1:][nz] - 1).astype(np.int64)].astype(np.int64)
+    l = nlb[nz].astype(np.int64)
+    bits = (deg[nz] * l + deg[nz] + (u >> l)).sum()
+    assert g.info["apriori_bits"] == bits
+    assert g.info["lower_bytes"] + g.info["upper_bytes"] - bits / 8 <= 2 * nz.sum()
+    g.free()
+
+
+def test_builder_directed_and_flags():
+    import paper_conf_ipps_gerak23_b200 as efg
+    src = np.array([0, 0, 2, 2, 2], np.uint32)
+    dst = np.array([1, 1, 0, 2, 1], np.uint32)
+    g = _host_graph(3, src, dst, flags=efg.EFG_DEDUP | efg.EFG_DROP_SELF_LOOPS)
+    vlist, nlb, offsets, data = g.export()
+    ov, oe = oracle.csr_build(3, src, dst, symmetrize=False)
+    assert np.array_equal(vlist, ov)
+    assert np.array_equal(data, oracle.efg_encode(ov, oe, 512)[2])
+
+
+def test_abi_errors():
+    import paper_conf_ipps_gerak23_b200 as efg
+    from paper_conf_ipps_gerak23_b200 import _abi
+    with pytest.raises(efg.EFGError) as e:
+        efg.Graph.build(3, np.array([0, 5], np.uint32), np.array([1, 1], np.uint32), device=-1)
+    assert e.value.status == _abi.EFG_ERANGE
+    with pytest.raises(efg.EFGError) as e:
+        efg.Graph.build(0, np.zeros(0, np.uint32), np.zeros(0, np.uint32), device=-1)
+    assert e.value.status == _abi.EFG_EINVAL
+    g = efg.Graph.build(4, np.array([0, 1], np.uint32), np.array([1, 2], np.uint32), device=-1)
+    with pytest.raises(efg.EFGError) as e:
+        g.bfs(0)
+    assert e.value.status == _abi.EFG_ESTATE
+    g.free()
+    g.free()  # idempotent
+
+
+def test_partition_balanced_and_aligned():
+    import paper_conf_ipps_gerak23_b200 as efg
+    n, src, dst = synth.rmat(13, 16, seed=1)
+    g = _host_graph(n, src, dst)
+    vlist, nlb, offsets, data = g.export()
+    for world in (1, 2, 4, 8):
+        b = efg.partition(vlist, offsets, world)
+        assert b[0] == 0 and b[-1] == n and np.all(np.diff(b.astype(np.int64)) >= 0)
+        assert all(int(x) % 64 == 0 for x in b[:-1])
+        w = (np.diff(offsets).astype(np.float64) + 29.0)
+        share = np.array([w[int(b[r]):int(b[r + 1])].sum() for r in range(world)])
+        assert share.max() <= w.sum() / world + 64 * (w.max() + 29)

@@ -1,0 +1,216 @@
+"""GPU parity tests: the CUDA path (through the C ABI) vs the CPU oracle.
+
+Bit-exact comparisons (integer work):
+  * efg_decode of every neighbour list == the oracle's CSR elist
+    (steps a1-a5: frontier/record gather, scan, tile partition, chunk bit
+    ranges via forward pointers, EF element decode);
+  * efg_bfs depth == oracle FIFO-BFS depth (steps a1-a7);
+  * parents are checked by invariant (several valid answers).
+Sizes span many edge tiles (2048 edges) and chunk boundaries (k), with ragged
+tails; special graphs cover the degenerate cases.
+"""
+import itertools
+
+import numpy as np
+import pytest
+
+import oracle
+import synth
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def efg(cuda_ok):
+    import paper_conf_ipps_gerak23_b200 as m
+    return m
+
+
+def _check_decode(efg, n, src, dst, k, **kw):
+    g = efg.Graph.build(n, src, dst, k=k, **kw)
+    ov, oe = oracle.csr_build(n, src, dst, **({} if "flags" not in kw else
+                                               {"symmetrize": bool(kw["flags"] & 1)}))
+    got = g.decode(0, n)
+    assert got.size == oe.size
+    assert np.array_equal(got, oe)
+    return g, ov, oe
+
+
+def _check_bfs(g, ov, oe, sources):
+    for s in sources:
+        d = g.bfs(int(s))
+        ref = oracle.bfs(ov, oe, int(s))
+        assert np.array_equal(d, ref), f"source {s}: {np.flatnonzero(d != ref)[:10]}"
+
+
+@pytest.mark.parametrize("k", [512, 64, 8, 0])
+def test_decode_and_bfs_rmat(efg, k):
+    n, src, dst = synth.rmat(14, 16, seed=1)
+    g, ov, oe = _check_decode(efg, n, src, dst, k)
+    _check_bfs(g, ov, oe, [0, 1, 2, 12345, n - 1])
+    g.free()
+
+
+def test_c1_rmat16_100_sources(efg):
+    # BASELINE.json configs[0]: RMAT scale 16, edgefactor 16, BFS from vertex 0
+    n, src, dst = synth.config_edges(1)
+    g, ov, oe = _check_decode(efg, n, src, dst, 512)
+    deg = np.diff(ov)
+    srcs = synth.sources(n, 100, seed=1001, nonisolated_mask=deg > 0)
+    _check_bfs(g, ov, oe, np.concatenate([[0], srcs]))
+    g.free()
+
+
+def test_decode_partial_ranges(efg):
+    n, src, dst = synth.rmat(12, 16, seed=3)
+    g = efg.Graph.build(n, src, dst, k=16)
+    ov, oe = oracle.csr_build(n, src, dst)
+    rng = np.random.default_rng(0)
+    for _ in range(20):
+        a, b = sorted(rng.integers(0, n + 1, 2))
+        got = g.decode(int(a), int(b))
+        assert np.array_equal(got, oe[ov[a]:ov[b]])
+    g.free()
+
+
+def test_decode_to_device_buffer(efg):
+    import torch
+    n, src, dst = synth.rmat(12, 8, seed=4)
+    g = efg.Graph.build(n, src, dst)
+    ov, oe = oracle.csr_build(n, src, dst)
+    out = torch.empty(oe.size, dtype=torch.int32, device="cuda")
+    g.decode(0, n, out)
+    torch.cuda.synchronize()
+    assert np.array_equal(out.cpu().numpy().view(np.uint32), oe)
+    # depth into a device buffer
+    d = torch.empty(n, dtype=torch.int32, device="cuda")
+    g.bfs(0, depth=d)
+    torch.cuda.synchronize()
+    assert np.array_equal(d.cpu().numpy(), oracle.bfs(ov, oe, 0))
+    g.free()
+
+
+def test_long_lists_cross_forward_pointers(efg):
+    # hubs with degrees around 1x, 2x, 3x k and many small lists; wide ids
+    rng = np.random.default_rng(9)
+    n = 200_000
+    srcs, dsts = [], []
+    for hub, deg in [(0, 511), (1, 512), (2, 513), (3, 1024), (4, 1537), (n - 1, 5000), (7, 70000)]:
+        nb = rng.choice(n, size=deg, replace=False).astype(np.uint32)
+        srcs.append(np.full(deg, hub, np.uint32))
+        dsts.append(nb)
+    srcs.append(rng.integers(0, n, 300000).astype(np.uint32))
+    dsts.append(rng.integers(0, n, 300000).astype(np.uint32))
+    src, dst = np.concatenate(srcs), np.concatenate(dsts)
+    for k in (512, 32):
+        g, ov, oe = _check_decode(efg, n, src, dst, k)
+        _check_bfs(g, ov, oe, [0, 7, n - 1, 12345])
+        g.free()
+
+
+def test_dense_lists_l0(efg):
+    # complete graph: every list has u < n -> l = 0; also two cliques, disconnected
+    pairs = list(itertools.combinations(range(300), 2))
+    src = np.array([p[0] for p in pairs], np.uint32)
+    dst = np.array([p[1] for p in pairs], np.uint32)
+    src = np.concatenate([src, src + 400])
+    dst = np.concatenate([dst, dst + 400])
+    n = 800
+    g, ov, oe = _check_decode(efg, n, src, dst, 512)
+    _check_bfs(g, ov, oe, [0, 299, 400, 350, 799])
+    g.free()
+
+
+def test_special_graphs(efg):
+    # path (depth = index), star, isolated source, self-loop-only vertex
+    n = 10000
+    src = np.arange(n - 1, dtype=np.uint32)
+    g, ov, oe = _check_decode(efg, n, src, src + 1, 512)
+    d = g.bfs(0)
+    assert np.array_equal(d, np.arange(n))
+    g.free()
+    src = np.zeros(n - 1, np.uint32)
+    g, ov, oe = _check_decode(efg, n, src, np.arange(1, n, dtype=np.uint32), 512)
+    _check_bfs(g, ov, oe, [0, 5, n - 1])
+    g.free()
+    g = efg.Graph.build(5, np.array([1, 4], np.uint32), np.array([2, 4], np.uint32))
+    assert list(g.bfs(0)) == [0, -1, -1, -1, -1]
+    assert list(g.bfs(4)) == [-1, -1, -1, -1, 0]
+    assert list(g.bfs(2)) == [-1, 1, 0, -1, -1]
+    g.free()
+
+
+def test_directed_graph(efg):
+    n, src, dst = synth.rmat(12, 8, seed=5)
+    g = efg.Graph.build(n, src, dst, flags=efg.EFG_DEDUP | efg.EFG_DROP_SELF_LOOPS)
+    ov, oe = oracle.csr_build(n, src, dst, symmetrize=False)
+    assert np.array_equal(g.decode(0, n), oe)
+    _check_bfs(g, ov, oe, [0, 1, 100])
+    g.free()
+
+
+def test_random_graphs_many_shapes(efg):
+    rng = np.random.default_rng(21)
+    for t in range(25):
+        n = int(rng.integers(1, 5000))
+        m = int(rng.integers(0, 20 * n))
+        src = rng.integers(0, n, m).astype(np.uint32)
+        dst = rng.integers(0, n, m).astype(np.uint32)
+        k = int(rng.choice([0, 4, 8, 100, 512]))
+        g, ov, oe = _check_decode(efg, n, src, dst, k)
+        _check_bfs(g, ov, oe, rng.integers(0, n, 3))
+        g.free()
+
+
+def test_parents_valid(efg):
+    n, src, dst = synth.rmat(14, 16, seed=1)
+    g = efg.Graph.build(n, src, dst)
+    ov, oe = oracle.csr_build(n, src, dst)
+    for s in (0, 77):
+        d, par, st = g.bfs(s, parent=True, stats=True)
+        ref = oracle.bfs(ov, oe, s)
+        assert np.array_equal(d, ref)
+        reached = d >= 0
+        assert par[s] == s
+        assert np.all(par[~reached] == 0xFFFFFFFF)
+        for v in np.flatnonzero(reached):
+            if v == s:
+                continue
+            p = int(par[v])
+            assert d[p] == d[v] - 1
+            assert v in oe[ov[p]:ov[p + 1]]
+        assert st["vertices_reached"] == reached.sum()
+        assert st["edges_traversed"] == int(np.diff(ov)[reached].sum())
+    g.free()
+
+
+def test_stats_levels(efg):
+    n, src, dst = synth.rmat(13, 16, seed=2)
+    g = efg.Graph.build(n, src, dst)
+    ov, oe = oracle.csr_build(n, src, dst)
+    d, _, st = g.bfs(0, stats=True)
+    ref = oracle.bfs(ov, oe, 0)
+    assert st["levels"] == ref.max() + 1
+    for L in range(st["levels"]):
+        lvl = ref == L
+        assert st["level_frontier"][L] == lvl.sum()
+        assert st["level_edges"][L] == np.diff(ov)[lvl].sum()
+    g.free()
+
+
+@pytest.mark.slow
+def test_c2_rmat24_full_size(efg):
+    # BASELINE.json configs[1] at full size, bench launch configuration
+    n, src, dst = synth.config_edges(2)
+    g = efg.Graph.build(n, src, dst)
+    ov, oe = oracle.csr_build(n, src, dst)
+    del src, dst
+    deg = np.diff(ov)
+    srcs = synth.sources(n, 2, seed=1002, nonisolated_mask=deg > 0)
+    for s in np.concatenate([[0], srcs]):
+        d = g.bfs(int(s))
+        assert np.array_equal(d, oracle.bfs(ov, oe, int(s)))
+    # decode of sampled vertex ranges (hubs and tail)
+    for a, b in [(0, 64), (n // 2, n // 2 + 4096), (n - 5000, n)]:
+        assert np.array_equal(g.decode(a, b), oe[ov[a]:ov[b]])
+    g.free()
