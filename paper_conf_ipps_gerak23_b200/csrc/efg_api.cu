@@ -127,7 +127,7 @@ efg_status upload(efg_graph *g, const efg_build_opts &o)
     EFG_TRY(dev_alloc(d, &d.vis, d.nwords));
     EFG_TRY(dev_alloc(d, &d.prev, d.nwords));
     EFG_TRY(dev_alloc(d, &d.queue, h.n));
-    d.max_tiles = h.m / kTileEdges + 2;
+    d.max_tiles = (h.m + (uint64_t)kVertexWork * h.n) / kTileWork + 2;
     EFG_TRY(dev_alloc(d, &d.tiles, d.max_tiles));
     EFG_TRY(dev_alloc(d, &d.depth, h.n));
     EFG_TRY(dev_alloc(d, &d.status, 4 * d.status_blocks));

@@ -63,7 +63,7 @@ constexpr uint64_t kOffMask = (1ull << kOffBits) - 1;
 struct alignas(16) TileEntry {
     uint32_t fi;      // index into the frontier queue
     uint32_t chunk;   // chunk index within that vertex's list
-    uint64_t e;       // global (level-local) edge index of the chunk start
+    uint64_t w;       // work position of the chunk start (see kTileWork)
 };
 static_assert(sizeof(TileEntry) == 16, "TileEntry must be 16 bytes");
 
@@ -71,13 +71,17 @@ static_assert(sizeof(TileEntry) == 16, "TileEntry must be 16 bytes");
 struct LevelCtrl {
     uint64_t nf;        // frontier size for the next expand
     uint64_t ne;        // edges out of that frontier (E_L)
-    uint64_t ntiles;    // ceil(ne / tile_edges)
-    uint64_t pad;
+    uint64_t ntiles;    // ceil(nwork / kTileWork)
+    uint64_t nwork;     // work units = ne + kVertexWork * nf
 };
 
 constexpr int kExpandThreads = 128;          // 4 warps (static smem < 48 KB)
 constexpr int kAdvanceThreads = 256;         // one bitmap word per thread
-constexpr uint32_t kTileEdges = 2048;        // edges per warp tile (a3)
+// Step a3 partitions "work units" rather than bare edges: a frontier vertex
+// costs kVertexWork units (its record gather and list set-up) plus one per edge,
+// so a tile of kTileWork units holds at most kTileWork/kVertexWork short lists.
+constexpr uint32_t kTileWork = 2048;         // work units per warp tile (a3)
+constexpr uint32_t kVertexWork = 32;         // per-vertex overhead in work units
 
 struct DeviceGraph {
     int device = -1;

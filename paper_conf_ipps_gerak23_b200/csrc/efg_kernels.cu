@@ -132,33 +132,42 @@ __device__ uint64_t lookback(const uint64_t *st, uint64_t b)
 // --------------------------------------------------------------------------
 // advance_kernel: a7 + a1 + a2 + a3
 //   new = vis & ~prev per 32-vertex word; depth[new] = level; sorted queue of
-//   the new frontier; per-vertex degree (a1) scanned into edge offsets (a2);
-//   edge tiles of kTileEdges -> first owned chunk (a3, Fig. 4 rule with
-//   boundaries snapped to k-aligned chunk starts).
+//   the new frontier; per-vertex degree (a1) scanned (a2) into work offsets
+//   W_v = sum over earlier frontier vertices of (kVertexWork + deg); tiles of
+//   kTileWork units -> first owned chunk (a3: the Fig. 4 maxle rule applied
+//   once per tile, with boundaries snapped to k-aligned chunk starts).
+//   Vertex v occupies work [W_v, W_v + kVertexWork + deg_v); its chunk 0
+//   starts at W_v, chunk c > 0 at W_v + kVertexWork + c*k.
 // --------------------------------------------------------------------------
 struct HubItem {
-    uint64_t q, e, d;
+    uint64_t q, w, d;
 };
 
-__device__ __forceinline__ void write_tiles(TileEntry *tiles, uint64_t q, uint64_t e, uint64_t d,
+__device__ __forceinline__ void write_tiles(TileEntry *tiles, uint64_t q, uint64_t W, uint64_t d,
                                             uint64_t ch, uint64_t w_begin, uint64_t w_step)
 {
-    // tiles w with w*T in [e, e+d): first chunk start >= w*T
-    const uint64_t T = kTileEdges;
-    for (uint64_t w = (e + T - 1) / T + w_begin; w * T < e + d; w += w_step) {
-        const uint64_t off = w * T - e;
-        const uint64_t c = (off + ch - 1) / ch;
+    const uint64_t T = kTileWork, A = kVertexWork;
+    for (uint64_t t = (W + T - 1) / T + w_begin; t * T < W + A + d; t += w_step) {
+        const uint64_t o = t * T - W;
         TileEntry te;
-        if (c * ch < d) {
+        if (o == 0) {
             te.fi = (uint32_t)q;
-            te.chunk = (uint32_t)c;
-            te.e = e + c * ch;
-        } else {
-            te.fi = (uint32_t)(q + 1);
             te.chunk = 0;
-            te.e = e + d;
+            te.w = W;
+        } else {
+            uint64_t c = o > A ? (o - A + ch - 1) / ch : 1;
+            if (c == 0) c = 1;
+            if (c * ch < d) {
+                te.fi = (uint32_t)q;
+                te.chunk = (uint32_t)c;
+                te.w = W + A + c * ch;
+            } else {
+                te.fi = (uint32_t)(q + 1);
+                te.chunk = 0;
+                te.w = W + A + d;
+            }
         }
-        tiles[w] = te;
+        tiles[t] = te;
     }
 }
 
@@ -167,8 +176,8 @@ __global__ void __launch_bounds__(kAdvanceThreads) advance_kernel(AdvanceArgs a)
     constexpr int NW = kAdvanceThreads / 32;
     constexpr int kHubCap = 32;
     __shared__ uint32_t s_wcnt[NW];
-    __shared__ uint64_t s_wedge[NW];
-    __shared__ uint64_t s_block_q, s_block_e;
+    __shared__ uint64_t s_wwork[NW];
+    __shared__ uint64_t s_block_q, s_block_w;
     __shared__ HubItem s_hub[kHubCap];
     __shared__ uint32_t s_nhub;
 
@@ -188,69 +197,66 @@ __global__ void __launch_bounds__(kAdvanceThreads) advance_kernel(AdvanceArgs a)
     if (nb) a.prev[wi] = x;
 
     // a1: degree lookup of the new frontier vertices (+ depth of the level)
-    uint64_t edges = 0;
+    uint64_t work = 0;
     for (uint32_t t = nb; t; t &= t - 1) {
         const uint64_t v = wi * 32 + (__ffs(t) - 1);
-        edges += a.rec[v].deg;
+        work += kVertexWork + a.rec[v].deg;
         a.depth[v] = a.depth_value;
     }
     const uint32_t cnt = __popc(nb);
 
-    // a2: block scan of (cnt, edges)
+    // a2: block scan of (cnt, work)
     uint32_t wtot_c;
-    uint64_t wtot_e;
+    uint64_t wtot_w;
     const uint32_t ex_c = warp_excl_u32(cnt, wtot_c);
-    const uint64_t ex_e = warp_excl_u64(edges, wtot_e);
+    const uint64_t ex_w = warp_excl_u64(work, wtot_w);
     if (lane == 31) {
         s_wcnt[wid] = wtot_c;
-        s_wedge[wid] = wtot_e;
+        s_wwork[wid] = wtot_w;
     }
     __syncthreads();
     uint32_t pre_c = 0;
-    uint64_t pre_e = 0, blk_c = 0, blk_e = 0;
+    uint64_t pre_w = 0, blk_c = 0, blk_w = 0;
 #pragma unroll
     for (int w = 0; w < NW; ++w) {
         if (w < (int)wid) {
             pre_c += s_wcnt[w];
-            pre_e += s_wedge[w];
+            pre_w += s_wwork[w];
         }
         blk_c += s_wcnt[w];
-        blk_e += s_wedge[w];
+        blk_w += s_wwork[w];
     }
 
     // decoupled look-back across blocks (single pass)
     uint64_t *st_c = a.status + (uint64_t)(a.parity * 2 + 0) * a.nblocks;
-    uint64_t *st_e = a.status + (uint64_t)(a.parity * 2 + 1) * a.nblocks;
+    uint64_t *st_w = a.status + (uint64_t)(a.parity * 2 + 1) * a.nblocks;
     if (wid == 0) {
         if (lane == 0) {
             // clear this block's slots of the other parity for the next launch
             a.status[(uint64_t)((a.parity ^ 1) * 2 + 0) * a.nblocks + b] = 0;
             a.status[(uint64_t)((a.parity ^ 1) * 2 + 1) * a.nblocks + b] = 0;
-            if (b == 0) {
-                st_release_u64(st_c + b, kFlagIncl | blk_c);
-                st_release_u64(st_e + b, kFlagIncl | blk_e);
-            } else {
-                st_release_u64(st_c + b, kFlagAgg | blk_c);
-                st_release_u64(st_e + b, kFlagAgg | blk_e);
-            }
+            const uint64_t f = b == 0 ? kFlagIncl : kFlagAgg;
+            st_release_u64(st_c + b, f | blk_c);
+            st_release_u64(st_w + b, f | blk_w);
         }
-        uint64_t bq = 0, be = 0;
+        uint64_t bq = 0, bw = 0;
         if (b > 0) {
             bq = lookback(st_c, b);
-            be = lookback(st_e, b);
+            bw = lookback(st_w, b);
             if (lane == 0) {
                 st_release_u64(st_c + b, kFlagIncl | (bq + blk_c));
-                st_release_u64(st_e + b, kFlagIncl | (be + blk_e));
+                st_release_u64(st_w + b, kFlagIncl | (bw + blk_w));
             }
         }
         if (lane == 0) {
             s_block_q = bq;
-            s_block_e = be;
+            s_block_w = bw;
             if (b == a.nblocks - 1) {
-                const uint64_t nf = bq + blk_c, ne = be + blk_e;
+                const uint64_t nf = bq + blk_c, nwork = bw + blk_w;
                 a.ctrl->nf = nf;
-                a.ctrl->ne = ne;
-                a.ctrl->ntiles = (ne + kTileEdges - 1) / kTileEdges;
+                a.ctrl->nwork = nwork;
+                a.ctrl->ne = nwork - (uint64_t)kVertexWork * nf;
+                a.ctrl->ntiles = (nwork + kTileWork - 1) / kTileWork;
             }
         }
     }
@@ -258,46 +264,48 @@ __global__ void __launch_bounds__(kAdvanceThreads) advance_kernel(AdvanceArgs a)
 
     // a7 queue + a3 tile table
     uint64_t q = s_block_q + pre_c + ex_c;
-    uint64_t e = s_block_e + pre_e + ex_e;
+    uint64_t W = s_block_w + pre_w + ex_w;
     for (uint32_t t = nb; t; t &= t - 1) {
         const uint64_t v = wi * 32 + (__ffs(t) - 1);
         const uint64_t d = a.rec[v].deg;
         a.queue[q] = (uint32_t)v;
-        if (d) {
-            bool done = false;
-            if (d >= 64ull * kTileEdges) {  // hub: hand the tile writes to the whole block
-                const uint32_t slot = atomicAdd(&s_nhub, 1u);
-                if (slot < kHubCap) {
-                    s_hub[slot] = HubItem{q, e, d};
-                    done = true;
-                }
+        bool done = false;
+        if (d >= 64ull * kTileWork) {  // hub: hand the tile writes to the whole block
+            const uint32_t slot = atomicAdd(&s_nhub, 1u);
+            if (slot < kHubCap) {
+                s_hub[slot] = HubItem{q, W, d};
+                done = true;
             }
-            if (!done) write_tiles(a.tiles, q, e, d, ch, 0, 1);
         }
+        if (!done) write_tiles(a.tiles, q, W, d, ch, 0, 1);
         ++q;
-        e += d;
+        W += kVertexWork + d;
     }
     __syncthreads();
     const uint32_t nhub = min(s_nhub, (uint32_t)kHubCap);
     for (uint32_t h = 0; h < nhub; ++h)
-        write_tiles(a.tiles, s_hub[h].q, s_hub[h].e, s_hub[h].d, ch, tid, kAdvanceThreads);
+        write_tiles(a.tiles, s_hub[h].q, s_hub[h].w, s_hub[h].d, ch, tid, kAdvanceThreads);
 }
 
 // --------------------------------------------------------------------------
 // expand_kernel: a4 + a5 + a6 (P:137-177 generalised, Alg. 1 lines 3-6)
 //
-// One warp per edge tile (persistent grid-stride over tiles).  A tile's work
-// is a run of "chunks": k-aligned pieces of frontier lists, so every
-// chunk starts at a forward pointer and needs no select to find its first bit.
-// Chunks are taken 32 at a time ("batch"; several short lists per warp: the
-// multi-list case).  The batch's upper-bit words are laid end to end
-// and processed 32 words per step (one aligned 32-bit word per lane, coalesced):
+// One warp per tile (persistent grid-stride over tiles).  A tile's work is a
+// run of "chunks": k-aligned pieces of frontier lists, so every chunk
+// starts right after a forward pointer and needs no select to find its first
+// bit.  Chunks are taken 32 at a time ("batch"; many short lists per warp: the
+// multi-list case).  The batch's upper-bit words are laid end to
+// end and processed 32 words per step (one aligned 32-bit word per lane,
+// coalesced; the next step's word is loaded before the current one is used):
 //   popcount + warp exclusive scan  -> element slot of each word's first bit
-//   set-bit enumeration (ffs)        -> select1(i) - i for every element
-//                                       (staged in shared memory by rank)
-//   balanced pass, one element per lane -> lower bits by a funnel shift of two
-//                                       words, value = hi << l | lo, visit.
+//   set-bit enumeration (ffs)        -> select1(i) - i for every element,
+//                                       staged in shared memory by slot
+//   balanced pass, kUnroll elements per lane in flight
+//                                    -> lower bits by a funnel shift of two
+//                                       words, x = hi << l | lo, visit.
 // --------------------------------------------------------------------------
+constexpr int kUnroll = 4;
+
 struct SlotGeom {
     uint64_t A0, A1, U0;  // absolute bit range of the chunk's upper bits; upper start
     uint32_t wb, eb;      // exclusive word / element prefix within the batch
@@ -310,24 +318,32 @@ struct SlotMeta {
     uint64_t aux;      // parent: source vertex; decode: output index base
 };
 
-template <int MODE>
-__device__ __forceinline__ void visit(const ExpandArgs &a, uint32_t x, const SlotMeta &m,
-                                      uint64_t ei)
+struct WordLd {
+    uint32_t word;
+    int s;
+    uint64_t wi;
+};
+
+__device__ __forceinline__ WordLd load_word(const uint32_t *data32, const SlotGeom *geom,
+                                            uint32_t wb, uint32_t g, uint32_t W)
 {
-    if (MODE == kModeDecode) {
-        a.out[m.aux + ei] = x;
-    } else {
-        uint32_t *wp = a.vis + (x >> 5);
-        const uint32_t bit = 1u << (x & 31);
-        if (!(*wp & bit)) {  // Alg. 1 line 3 (stale reads are benign: the atomic decides)
-            if (MODE == kModeVisit) {
-                atomicOr(wp, bit);  // line 4; the advance pass finds the new bits
-            } else {
-                const uint32_t old = atomicOr(wp, bit);
-                if (!(old & bit)) a.out[x] = (uint32_t)m.aux;
-            }
+    WordLd r;
+    r.s = warp_maxle_u32(wb, g);
+    r.word = 0;
+    r.wi = 0;
+    if (g < W) {
+        const SlotGeom &sg = geom[r.s];
+        const uint64_t w0 = sg.A0 >> 5, wl = (sg.A1 - 1) >> 5;
+        r.wi = w0 + (g - sg.wb);
+        uint32_t word = ldg_u32(data32 + r.wi);
+        if (r.wi == w0) word &= FULL << (uint32_t)(sg.A0 & 31);
+        if (r.wi == wl) {
+            const uint32_t hb = (uint32_t)(sg.A1 - wl * 32);  // 1..32 valid bits
+            if (hb < 32) word &= (1u << hb) - 1;
         }
+        r.word = word;
     }
+    return r;
 }
 
 template <int MODE>
@@ -339,18 +355,19 @@ __global__ void __launch_bounds__(kExpandThreads, 6) expand_kernel(ExpandArgs a)
     __shared__ SlotMeta s_meta[kWarps][32];
 
     const uint32_t lane = lane_id(), wid = threadIdx.x >> 5;
-    const uint64_t ntiles = a.ctrl->ntiles, nf = a.ctrl->nf, ne = a.ctrl->ne;
+    const uint64_t ntiles = a.ctrl->ntiles, nf = a.ctrl->nf, nwork = a.ctrl->nwork;
     const uint32_t *data32 = reinterpret_cast<const uint32_t *>(a.data);
     const uint64_t CH = a.k ? a.k : (1ull << 40);
+    const uint64_t A = kVertexWork;
     const uint64_t gw = (uint64_t)blockIdx.x * kWarps + wid;
     const uint64_t nwarps = (uint64_t)gridDim.x * kWarps;
 
     for (uint64_t tile = gw; tile < ntiles; tile += nwarps) {
         const TileEntry te = a.tiles[tile];
-        uint64_t fi = te.fi, c0 = te.chunk, E = te.e;
-        const uint64_t Eend = min((tile + 1) * (uint64_t)kTileEdges, ne);
+        uint64_t fi = te.fi, c0 = te.chunk, P = te.w;
+        const uint64_t Pend = min((tile + 1) * (uint64_t)kTileWork, nwork);
 
-        while (E < Eend && fi < nf) {
+        while (P < Pend && fi < nf) {
             // ---- a1 (gather): up to 32 frontier vertices, one per lane ----
             const uint64_t fv = fi + lane;
             uint32_t v = 0, deg = 0, ubytes = 0;
@@ -365,30 +382,34 @@ __global__ void __launch_bounds__(kExpandThreads, 6) expand_kernel(ExpandArgs a)
             const uint64_t first = lane == 0 ? c0 : 0;
             const uint64_t nch = deg ? (deg + CH - 1) / CH : 0;
             const uint32_t nrem = (uint32_t)(nch > first ? nch - first : 0);
-            const uint64_t erem = nrem ? deg - first * CH : 0;
+            // work still ahead of this vertex (from its first remaining chunk on)
+            const uint64_t wrem = fv < nf ? (first == 0 ? A + deg : deg - first * CH) : 0;
             uint32_t totc;
             const uint32_t cb = warp_excl_u32(nrem, totc);
-            uint64_t tote;
-            const uint64_t eb = warp_excl_u64(erem, tote);
+            uint64_t totw;
+            const uint64_t wbv = warp_excl_u64(wrem, totw);
+            // W_v of each vertex (work position of its chunk 0)
+            const uint64_t Wv = P + wbv - (first ? A + first * CH : 0);
             if (totc == 0) {  // 32 empty lists
                 fi += 32;
                 c0 = 0;
+                P += totw;
                 continue;
             }
 
-            // ---- a3 (within tile): chunk slot t = lane -> owning vertex lane j ----
+            // ---- chunk slot t = lane -> owning vertex lane j (maxle, C13) ----
             const int j = warp_maxle_u32(cb, lane);
             const uint32_t deg_j = __shfl_sync(FULL, deg, j);
             const uint64_t offl_j = __shfl_sync(FULL, offl, j);
             const uint32_t ub_j = __shfl_sync(FULL, ubytes, j);
             const uint32_t cb_j = __shfl_sync(FULL, cb, j);
-            const uint64_t eb_j = __shfl_sync(FULL, eb, j);
+            const uint64_t Wv_j = __shfl_sync(FULL, Wv, j);
             const uint32_t v_j = __shfl_sync(FULL, v, j);
             const uint64_t nch_j = __shfl_sync(FULL, nch, j);
             const uint64_t cc = (j == 0 ? c0 : 0) + (lane - cb_j);
             const uint64_t r0 = cc * CH;
-            const uint64_t chunk_e = E + eb_j + (uint64_t)(lane - cb_j) * CH;
-            const bool valid = lane < totc && chunk_e < Eend;
+            const uint64_t cstart = Wv_j + (cc ? A + cc * CH : 0);
+            const bool valid = lane < totc && cstart < Pend;
             const uint32_t count = __popc(__ballot_sync(FULL, valid));
             if (count == 0) break;
 
@@ -420,7 +441,11 @@ __global__ void __launch_bounds__(kExpandThreads, 6) expand_kernel(ExpandArgs a)
                 s_geom[wid][lane] = SlotGeom{A0, A1, U0, wb, ebt, r0};
                 uint64_t aux = 0;
                 if (MODE == kModeVisitParent) aux = v_j;
-                if (MODE == kModeDecode) aux = chunk_e - ebt;
+                if (MODE == kModeDecode) {
+                    // CSR position of the chunk's first element: E_v + r0, E_v = W_v - A*q_v
+                    const uint64_t qv = fi + (uint64_t)j;
+                    aux = Wv_j - A * qv + r0 - ebt;
+                }
                 s_meta[wid][lane] = SlotMeta{lbase | ((uint64_t)l << kOffBits), (int64_t)r0 - (int64_t)ebt, aux};
             }
             // state after this batch: continue after the last valid chunk
@@ -429,66 +454,91 @@ __global__ void __launch_bounds__(kExpandThreads, 6) expand_kernel(ExpandArgs a)
                 const uint64_t last_cc = __shfl_sync(FULL, cc, tl);
                 const uint64_t last_nch = __shfl_sync(FULL, nch_j, tl);
                 const int last_j = __shfl_sync(FULL, j, tl);
-                const uint64_t last_end = __shfl_sync(FULL, chunk_e, tl) + __shfl_sync(FULL, nel, tl);
+                const uint64_t last_W = __shfl_sync(FULL, Wv_j, tl);
+                const uint32_t last_deg = __shfl_sync(FULL, deg_j, tl);
                 if (last_cc + 1 < last_nch) {
                     fi += last_j;
                     c0 = last_cc + 1;
+                    P = last_W + A + c0 * CH;
                 } else {
                     fi += last_j + 1;
                     c0 = 0;
+                    P = last_W + A + last_deg;
                 }
-                E = last_end;
             }
             __syncwarp();
 
             // ---- a5 + a6: 32 upper-bit words per step ----
             uint32_t run = 0;
+            WordLd nxt = load_word(data32, s_geom[wid], wb, lane, W);
             for (uint32_t g0 = 0; g0 < W; g0 += 32) {
-                const uint32_t g = g0 + lane;
-                const int s = warp_maxle_u32(wb, g);
-                uint32_t word = 0;
-                uint64_t wi = 0;
-                if (g < W) {
-                    const SlotGeom &sg = s_geom[wid][s];
-                    const uint64_t w0 = sg.A0 >> 5, wl = (sg.A1 - 1) >> 5;
-                    wi = w0 + (g - sg.wb);
-                    word = ldg_u32(data32 + wi);
-                    if (wi == w0) word &= FULL << (uint32_t)(sg.A0 & 31);
-                    if (wi == wl) {
-                        const uint32_t hb = (uint32_t)(sg.A1 - wl * 32);  // 1..32 valid bits
-                        if (hb < 32) word &= (1u << hb) - 1;
-                    }
-                }
+                const WordLd cur = nxt;
+                if (g0 + 32 < W) nxt = load_word(data32, s_geom[wid], wb, g0 + 32 + lane, W);
                 uint32_t tot;
-                const uint32_t ep = warp_excl_u32(__popc(word), tot);
-                if (word) {
-                    const SlotGeom &sg = s_geom[wid][s];
+                const uint32_t ep = warp_excl_u32(__popc(cur.word), tot);
+                if (cur.word) {
+                    const SlotGeom &sg = s_geom[wid][cur.s];
                     const uint64_t rank = sg.r0 + run + ep - sg.eb;  // rank of the first set bit
-                    const uint64_t hb = wi * 32 - sg.U0 - rank;      // hi = hb + p - jj
-                    uint32_t w = word, jj = 0;
+                    const uint64_t hb = cur.wi * 32 - sg.U0 - rank;  // hi = hb + p - jj
+                    uint32_t w = cur.word, jj = 0;
                     while (w) {
                         const uint32_t p = __ffs(w) - 1;
                         w &= w - 1;
                         s_hi[wid][ep + jj] = (uint32_t)(hb + p - jj);  // select1(i) - i
-                        s_cs[wid][ep + jj] = (uint8_t)s;
+                        s_cs[wid][ep + jj] = (uint8_t)cur.s;
                         ++jj;
                     }
                 }
                 __syncwarp();
-                for (uint32_t e = lane; e < tot; e += 32) {
-                    const uint32_t hi = s_hi[wid][e];
-                    const SlotMeta m = s_meta[wid][s_cs[wid][e]];
-                    const uint32_t ll = (uint32_t)(m.lbase_l >> kOffBits);
-                    uint32_t lo = 0;
-                    if (ll) {
-                        const uint64_t rank = (uint64_t)(m.rankoff + (int64_t)(run + e));
-                        const uint64_t ba = (m.lbase_l & kOffMask) + rank * ll;
-                        const uint64_t bw = ba >> 5;
-                        lo = __funnelshift_r(ldg_u32(data32 + bw), ldg_u32(data32 + bw + 1),
-                                             (uint32_t)(ba & 31)) &
-                             ((1u << ll) - 1);
+                for (uint32_t base = 0; base < tot; base += 32 * kUnroll) {
+                    uint32_t xv[kUnroll];
+                    uint64_t ax[kUnroll];
+                    bool ok[kUnroll];
+#pragma unroll
+                    for (int u = 0; u < kUnroll; ++u) {
+                        const uint32_t e = base + u * 32 + lane;
+                        ok[u] = e < tot;
+                        xv[u] = 0;
+                        ax[u] = 0;
+                        if (ok[u]) {
+                            const uint32_t hi = s_hi[wid][e];
+                            const SlotMeta m = s_meta[wid][s_cs[wid][e]];
+                            const uint32_t ll = (uint32_t)(m.lbase_l >> kOffBits);
+                            uint32_t lo = 0;
+                            if (ll) {
+                                const uint64_t rank = (uint64_t)(m.rankoff + (int64_t)(run + e));
+                                const uint64_t ba = (m.lbase_l & kOffMask) + rank * ll;
+                                const uint64_t bw = ba >> 5;
+                                lo = __funnelshift_r(ldg_u32(data32 + bw), ldg_u32(data32 + bw + 1),
+                                                     (uint32_t)(ba & 31)) &
+                                     ((1u << ll) - 1);
+                            }
+                            xv[u] = (hi << ll) | lo;
+                            ax[u] = MODE == kModeDecode ? m.aux + run + e : m.aux;
+                        }
                     }
-                    visit<MODE>(a, (hi << ll) | lo, m, run + e);
+                    if (MODE == kModeDecode) {
+#pragma unroll
+                        for (int u = 0; u < kUnroll; ++u)
+                            if (ok[u]) a.out[ax[u]] = xv[u];
+                    } else {
+                        uint32_t vw[kUnroll];
+#pragma unroll
+                        for (int u = 0; u < kUnroll; ++u)
+                            vw[u] = ok[u] ? a.vis[xv[u] >> 5] : FULL;  // Alg. 1 line 3 probe
+#pragma unroll
+                        for (int u = 0; u < kUnroll; ++u) {
+                            const uint32_t bit = 1u << (xv[u] & 31);
+                            if (!(vw[u] & bit)) {  // stale reads are benign: the atomic decides
+                                if (MODE == kModeVisit) {
+                                    atomicOr(a.vis + (xv[u] >> 5), bit);  // line 4
+                                } else {
+                                    const uint32_t old = atomicOr(a.vis + (xv[u] >> 5), bit);
+                                    if (!(old & bit)) a.out[xv[u]] = (uint32_t)ax[u];
+                                }
+                            }
+                        }
+                    }
                 }
                 __syncwarp();
                 run += tot;
@@ -496,6 +546,7 @@ __global__ void __launch_bounds__(kExpandThreads, 6) expand_kernel(ExpandArgs a)
         }
     }
 }
+
 
 __global__ void set_range_bits_kernel(uint32_t *vis, uint64_t v0, uint64_t v1)
 {
