@@ -26,7 +26,6 @@ namespace {
 
 constexpr uint32_t FULL = 0xffffffffu;
 constexpr int kWarps = kExpandThreads / 32;
-constexpr int kStage = 1024;  // max set bits in 32 words of 32 bits
 
 // --------------------------------------------------------------------------
 // warp / block primitives (§III-C: exclusive scan, bounded search)
@@ -297,14 +296,15 @@ __global__ void __launch_bounds__(kAdvanceThreads) advance_kernel(AdvanceArgs a)
 // multi-list case).  The batch's upper-bit words are laid end to
 // end and processed 32 words per step (one aligned 32-bit word per lane,
 // coalesced; the next step's word is loaded before the current one is used):
-//   popcount + warp exclusive scan  -> element slot of each word's first bit
-//   set-bit enumeration (ffs)        -> select1(i) - i for every element,
-//                                       staged in shared memory by slot
-//   balanced pass, kUnroll elements per lane in flight
-//                                    -> lower bits by a funnel shift of two
-//                                       words, x = hi << l | lo, visit.
+//   popcount + warp exclusive scan  -> rank of each word's first stop bit
+//                                      (the segmented scan of P:171-177: the
+//                                      segments are chunks, whose element
+//                                      prefix is subtracted)
+//   per lane, serially over its word -> select1(i) - i by ffs-and-clear, the
+//                                      lower bits from a bit buffer streamed
+//                                      over the lower section, x = hi<<l | lo,
+//                                      then the visit with one probe in flight.
 // --------------------------------------------------------------------------
-constexpr int kUnroll = 4;
 
 struct SlotGeom {
     uint64_t A0, A1, U0;  // absolute bit range of the chunk's upper bits; upper start
@@ -347,10 +347,8 @@ __device__ __forceinline__ WordLd load_word(const uint32_t *data32, const SlotGe
 }
 
 template <int MODE>
-__global__ void __launch_bounds__(kExpandThreads, 6) expand_kernel(ExpandArgs a)
+__global__ void __launch_bounds__(kExpandThreads, 8) expand_kernel(ExpandArgs a)
 {
-    __shared__ uint32_t s_hi[kWarps][kStage];
-    __shared__ uint8_t s_cs[kWarps][kStage];
     __shared__ SlotGeom s_geom[kWarps][32];
     __shared__ SlotMeta s_meta[kWarps][32];
 
@@ -468,7 +466,12 @@ __global__ void __launch_bounds__(kExpandThreads, 6) expand_kernel(ExpandArgs a)
             }
             __syncwarp();
 
-            // ---- a5 + a6: 32 upper-bit words per step ----
+            // ---- a5 + a6: 32 upper-bit words per step, one word per lane ----
+            // Each lane decodes the elements whose stop bits lie in its word,
+            // serially: select1(i) - i by ffs-and-clear, the lower bits from a
+            // per-lane bit buffer streamed over the chunk's lower section, then
+            // the visit.  Lanes start at ranks given by the warp scan of the
+            // words' popcounts.
             uint32_t run = 0;
             WordLd nxt = load_word(data32, s_geom[wid], wb, lane, W);
             for (uint32_t g0 = 0; g0 < W; g0 += 32) {
@@ -478,69 +481,71 @@ __global__ void __launch_bounds__(kExpandThreads, 6) expand_kernel(ExpandArgs a)
                 const uint32_t ep = warp_excl_u32(__popc(cur.word), tot);
                 if (cur.word) {
                     const SlotGeom &sg = s_geom[wid][cur.s];
-                    const uint64_t rank = sg.r0 + run + ep - sg.eb;  // rank of the first set bit
-                    const uint64_t hb = cur.wi * 32 - sg.U0 - rank;  // hi = hb + p - jj
+                    const SlotMeta m = s_meta[wid][cur.s];
+                    const uint64_t rank = sg.r0 + run + ep - sg.eb;         // rank of the first set bit
+                    const uint32_t hb = (uint32_t)(cur.wi * 32 - sg.U0 - rank);  // hi = hb + p - jj
+                    const uint32_t ll = (uint32_t)(m.lbase_l >> kOffBits);
+                    const uint32_t lmask = ll ? (0xffffffffu >> (32 - ll)) : 0u;
+                    // lower-bit stream at bit lbase + rank*l
+                    const uint64_t lpos = (m.lbase_l & kOffMask) + rank * ll;
+                    const uint32_t *lp = data32 + (lpos >> 5);
+                    uint64_t buf = 0;
+                    uint32_t nb = 64;
+                    uint32_t pre = 0;
+                    if (ll) {
+                        const uint32_t sh = (uint32_t)(lpos & 31);
+                        buf = (((uint64_t)ldg_u32(lp + 1) << 32) | ldg_u32(lp)) >> sh;
+                        nb = 64 - sh;
+                        pre = ldg_u32(lp + 2);
+                        lp += 3;
+                    }
+                    const uint64_t obase = m.aux + run + ep;  // decode: output index of jj = 0
                     uint32_t w = cur.word, jj = 0;
+                    // one probe in flight: issue the load of element i, then
+                    // resolve element i-1 (Alg. 1 lines 3-4)
+                    uint32_t px = 0, pw = FULL;
                     while (w) {
                         const uint32_t p = __ffs(w) - 1;
                         w &= w - 1;
-                        s_hi[wid][ep + jj] = (uint32_t)(hb + p - jj);  // select1(i) - i
-                        s_cs[wid][ep + jj] = (uint8_t)cur.s;
-                        ++jj;
-                    }
-                }
-                __syncwarp();
-                for (uint32_t base = 0; base < tot; base += 32 * kUnroll) {
-                    uint32_t xv[kUnroll];
-                    uint64_t ax[kUnroll];
-                    bool ok[kUnroll];
-#pragma unroll
-                    for (int u = 0; u < kUnroll; ++u) {
-                        const uint32_t e = base + u * 32 + lane;
-                        ok[u] = e < tot;
-                        xv[u] = 0;
-                        ax[u] = 0;
-                        if (ok[u]) {
-                            const uint32_t hi = s_hi[wid][e];
-                            const SlotMeta m = s_meta[wid][s_cs[wid][e]];
-                            const uint32_t ll = (uint32_t)(m.lbase_l >> kOffBits);
-                            uint32_t lo = 0;
-                            if (ll) {
-                                const uint64_t rank = (uint64_t)(m.rankoff + (int64_t)(run + e));
-                                const uint64_t ba = (m.lbase_l & kOffMask) + rank * ll;
-                                const uint64_t bw = ba >> 5;
-                                lo = __funnelshift_r(ldg_u32(data32 + bw), ldg_u32(data32 + bw + 1),
-                                                     (uint32_t)(ba & 31)) &
-                                     ((1u << ll) - 1);
+                        const uint32_t hi = hb + p - jj;  // select1(i) - i
+                        uint32_t lo = 0;
+                        if (ll) {
+                            if (nb < ll) {
+                                buf |= (uint64_t)pre << nb;
+                                nb += 32;
+                                pre = ldg_u32(lp++);
                             }
-                            xv[u] = (hi << ll) | lo;
-                            ax[u] = MODE == kModeDecode ? m.aux + run + e : m.aux;
+                            lo = (uint32_t)buf & lmask;
+                            buf >>= ll;
+                            nb -= ll;
                         }
-                    }
-                    if (MODE == kModeDecode) {
-#pragma unroll
-                        for (int u = 0; u < kUnroll; ++u)
-                            if (ok[u]) a.out[ax[u]] = xv[u];
-                    } else {
-                        uint32_t vw[kUnroll];
-#pragma unroll
-                        for (int u = 0; u < kUnroll; ++u)
-                            vw[u] = ok[u] ? a.vis[xv[u] >> 5] : FULL;  // Alg. 1 line 3 probe
-#pragma unroll
-                        for (int u = 0; u < kUnroll; ++u) {
-                            const uint32_t bit = 1u << (xv[u] & 31);
-                            if (!(vw[u] & bit)) {  // stale reads are benign: the atomic decides
+                        const uint32_t x = (hi << ll) | lo;
+                        if (MODE == kModeDecode) {
+                            a.out[obase + jj] = x;
+                        } else {
+                            const uint32_t xw = a.vis[x >> 5];
+                            if (!(pw & (1u << (px & 31)))) {
                                 if (MODE == kModeVisit) {
-                                    atomicOr(a.vis + (xv[u] >> 5), bit);  // line 4
+                                    atomicOr(a.vis + (px >> 5), 1u << (px & 31));
                                 } else {
-                                    const uint32_t old = atomicOr(a.vis + (xv[u] >> 5), bit);
-                                    if (!(old & bit)) a.out[xv[u]] = (uint32_t)ax[u];
+                                    const uint32_t old = atomicOr(a.vis + (px >> 5), 1u << (px & 31));
+                                    if (!(old & (1u << (px & 31)))) a.out[px] = (uint32_t)m.aux;
                                 }
                             }
+                            px = x;
+                            pw = xw;
+                        }
+                        ++jj;
+                    }
+                    if (MODE != kModeDecode && !(pw & (1u << (px & 31)))) {
+                        if (MODE == kModeVisit) {
+                            atomicOr(a.vis + (px >> 5), 1u << (px & 31));
+                        } else {
+                            const uint32_t old = atomicOr(a.vis + (px >> 5), 1u << (px & 31));
+                            if (!(old & (1u << (px & 31)))) a.out[px] = (uint32_t)m.aux;
                         }
                     }
                 }
-                __syncwarp();
                 run += tot;
             }
         }
