@@ -303,8 +303,10 @@ __global__ void __launch_bounds__(kAdvanceThreads) advance_kernel(AdvanceArgs a)
 //   per lane, serially over its word -> select1(i) - i by ffs-and-clear, the
 //                                      lower bits from a bit buffer streamed
 //                                      over the lower section, x = hi<<l | lo,
-//                                      then the visit with one probe in flight.
+//                                      then the visits, kGroup probes in flight.
 // --------------------------------------------------------------------------
+
+constexpr int kGroup = 8;  // probes in flight per lane
 
 struct SlotGeom {
     uint64_t A0, A1, U0;  // absolute bit range of the chunk's upper bits; upper start
@@ -483,15 +485,14 @@ __global__ void __launch_bounds__(kExpandThreads, 8) expand_kernel(ExpandArgs a)
                     const SlotGeom &sg = s_geom[wid][cur.s];
                     const SlotMeta m = s_meta[wid][cur.s];
                     const uint64_t rank = sg.r0 + run + ep - sg.eb;         // rank of the first set bit
-                    const uint32_t hb = (uint32_t)(cur.wi * 32 - sg.U0 - rank);  // hi = hb + p - jj
+                    uint32_t hb = (uint32_t)(cur.wi * 32 - sg.U0 - rank);  // hi = hb + p - jj
                     const uint32_t ll = (uint32_t)(m.lbase_l >> kOffBits);
                     const uint32_t lmask = ll ? (0xffffffffu >> (32 - ll)) : 0u;
-                    // lower-bit stream at bit lbase + rank*l
+                    // lower-bit stream at bit lbase + rank*l (bit buffer `buf` holds nb bits)
                     const uint64_t lpos = (m.lbase_l & kOffMask) + rank * ll;
                     const uint32_t *lp = data32 + (lpos >> 5);
                     uint64_t buf = 0;
-                    uint32_t nb = 64;
-                    uint32_t pre = 0;
+                    uint32_t nb = 64, pre = 0;
                     if (ll) {
                         const uint32_t sh = (uint32_t)(lpos & 31);
                         buf = (((uint64_t)ldg_u32(lp + 1) << 32) | ldg_u32(lp)) >> sh;
@@ -499,50 +500,57 @@ __global__ void __launch_bounds__(kExpandThreads, 8) expand_kernel(ExpandArgs a)
                         pre = ldg_u32(lp + 2);
                         lp += 3;
                     }
-                    const uint64_t obase = m.aux + run + ep;  // decode: output index of jj = 0
-                    uint32_t w = cur.word, jj = 0;
-                    // one probe in flight: issue the load of element i, then
-                    // resolve element i-1 (Alg. 1 lines 3-4)
-                    uint32_t px = 0, pw = FULL;
+                    uint64_t obase = m.aux + run + ep;  // decode: output index of the next element
+                    uint32_t w = cur.word;
                     while (w) {
-                        const uint32_t p = __ffs(w) - 1;
-                        w &= w - 1;
-                        const uint32_t hi = hb + p - jj;  // select1(i) - i
-                        uint32_t lo = 0;
-                        if (ll) {
-                            if (nb < ll) {
-                                buf |= (uint64_t)pre << nb;
-                                nb += 32;
-                                pre = ldg_u32(lp++);
+                        // decode up to kGroup elements, then resolve their probes together
+                        uint32_t xs[kGroup];
+                        uint32_t valid = 0;
+#pragma unroll
+                        for (int u = 0; u < kGroup; ++u) {
+                            xs[u] = 0;
+                            if (w) {
+                                const uint32_t p = __ffs(w) - 1;
+                                w &= w - 1;
+                                const uint32_t hi = hb + p;  // select1(i) - i
+                                hb -= 1;
+                                uint32_t lo = 0;
+                                if (ll) {
+                                    if (nb < ll) {
+                                        buf |= (uint64_t)pre << nb;
+                                        nb += 32;
+                                        pre = ldg_u32(lp++);
+                                    }
+                                    lo = (uint32_t)buf & lmask;
+                                    buf >>= ll;
+                                    nb -= ll;
+                                }
+                                xs[u] = (hi << ll) | lo;
+                                valid |= 1u << u;
                             }
-                            lo = (uint32_t)buf & lmask;
-                            buf >>= ll;
-                            nb -= ll;
                         }
-                        const uint32_t x = (hi << ll) | lo;
                         if (MODE == kModeDecode) {
-                            a.out[obase + jj] = x;
+#pragma unroll
+                            for (int u = 0; u < kGroup; ++u)
+                                if (valid >> u & 1) a.out[obase + u] = xs[u];
+                            obase += __popc(valid);
                         } else {
-                            const uint32_t xw = a.vis[x >> 5];
-                            if (!(pw & (1u << (px & 31)))) {
-                                if (MODE == kModeVisit) {
-                                    atomicOr(a.vis + (px >> 5), 1u << (px & 31));
-                                } else {
-                                    const uint32_t old = atomicOr(a.vis + (px >> 5), 1u << (px & 31));
-                                    if (!(old & (1u << (px & 31)))) a.out[px] = (uint32_t)m.aux;
+                            uint32_t ws[kGroup];
+#pragma unroll
+                            for (int u = 0; u < kGroup; ++u)  // Alg. 1 line 3: probes in flight together
+                                ws[u] = (valid >> u & 1) ? a.vis[xs[u] >> 5] : FULL;
+#pragma unroll
+                            for (int u = 0; u < kGroup; ++u) {
+                                const uint32_t bit = 1u << (xs[u] & 31);
+                                if (!(ws[u] & bit)) {  // stale reads are benign: the atomic decides
+                                    if (MODE == kModeVisit) {
+                                        atomicOr(a.vis + (xs[u] >> 5), bit);  // line 4
+                                    } else {
+                                        const uint32_t old = atomicOr(a.vis + (xs[u] >> 5), bit);
+                                        if (!(old & bit)) a.out[xs[u]] = (uint32_t)m.aux;
+                                    }
                                 }
                             }
-                            px = x;
-                            pw = xw;
-                        }
-                        ++jj;
-                    }
-                    if (MODE != kModeDecode && !(pw & (1u << (px & 31)))) {
-                        if (MODE == kModeVisit) {
-                            atomicOr(a.vis + (px >> 5), 1u << (px & 31));
-                        } else {
-                            const uint32_t old = atomicOr(a.vis + (px >> 5), 1u << (px & 31));
-                            if (!(old & (1u << (px & 31)))) a.out[px] = (uint32_t)m.aux;
                         }
                     }
                 }
