@@ -122,8 +122,8 @@ efg_status upload(efg_graph *g, const efg_build_opts &o)
 
     // traversal workspace
     const uint64_t words = (h.n + 31) / 32;
-    d.nwords = (words + kAdvanceThreads - 1) / kAdvanceThreads * kAdvanceThreads;
-    d.status_blocks = d.nwords / kAdvanceThreads;
+    d.nwords = (words + kAdvanceWords - 1) / kAdvanceWords * kAdvanceWords;
+    d.status_blocks = d.nwords / kAdvanceWords;
     EFG_TRY(dev_alloc(d, &d.vis, d.nwords));
     EFG_TRY(dev_alloc(d, &d.prev, d.nwords));
     EFG_TRY(dev_alloc(d, &d.queue, h.n));

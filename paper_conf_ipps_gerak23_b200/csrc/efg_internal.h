@@ -76,7 +76,9 @@ struct LevelCtrl {
 };
 
 constexpr int kExpandThreads = 128;          // 4 warps (static smem < 48 KB)
-constexpr int kAdvanceThreads = 256;         // one bitmap word per thread
+constexpr int kAdvanceThreads = 256;         // 8 warps
+constexpr int kAdvanceRounds = 4;            // runs of 32 words per warp
+constexpr int kAdvanceWords = kAdvanceThreads * kAdvanceRounds;  // bitmap words per block
 // Step a3 partitions "work units" rather than bare edges: a frontier vertex
 // costs kVertexWork units (its record gather and list set-up) plus one per edge,
 // so a tile of kTileWork units holds at most kTileWork/kVertexWork short lists.

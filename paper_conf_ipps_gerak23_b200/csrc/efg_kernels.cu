@@ -105,27 +105,52 @@ constexpr uint64_t kFlagAgg = 1ull << 62;
 constexpr uint64_t kFlagIncl = 2ull << 62;
 constexpr uint64_t kValMask = (1ull << 62) - 1;
 
-// Warp-cooperative decoupled look-back: exclusive prefix of block b from the
-// status words of its predecessors (each word: flag | value).
-__device__ uint64_t lookback(const uint64_t *st, uint64_t b)
+// Decoupled look-back (single-pass scan across blocks) over a pair of values
+// (frontier count, work).  Each block publishes two 64-bit words, flag | value,
+// with the same flag in both; a reader accepts a predecessor only when both
+// words carry the same non-zero flag, so no fence is needed (each value travels
+// in the same single-copy-atomic word as its flag).  Warp 0 looks back 32
+// predecessors at a time and stops at the nearest inclusive prefix.
+__device__ __forceinline__ uint64_t ld_relaxed_u64(const uint64_t *p)
+{
+    uint64_t v;
+    asm volatile("ld.relaxed.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+    return v;
+}
+
+__device__ __forceinline__ void st_relaxed_u64(uint64_t *p, uint64_t v)
+{
+    asm volatile("st.relaxed.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+
+__device__ void lookback2(const uint64_t *st, uint64_t b, uint64_t &ex_c, uint64_t &ex_w)
 {
     const uint32_t lane = lane_id();
-    uint64_t excl = 0;
+    uint64_t c_acc = 0, w_acc = 0;
     int64_t pred = (int64_t)b - 1;
     while (pred >= 0) {
         const int64_t idx = pred - (int64_t)lane;
-        uint64_t s;
+        uint64_t c, w;
         for (;;) {
-            s = idx >= 0 ? ld_acquire_u64(st + idx) : kFlagIncl;
-            if (!__any_sync(FULL, (s >> 62) == 0)) break;
+            if (idx >= 0) {
+                c = ld_relaxed_u64(st + 2 * idx);
+                w = ld_relaxed_u64(st + 2 * idx + 1);
+            } else {
+                c = kFlagIncl;
+                w = kFlagIncl;
+            }
+            const bool ok = (c >> 62) != 0 && (c >> 62) == (w >> 62);
+            if (__all_sync(FULL, ok)) break;
         }
-        const uint32_t incl = __ballot_sync(FULL, (s >> 62) == 2);
+        const uint32_t incl = __ballot_sync(FULL, (c >> 62) == 2);
         const int first = incl ? __ffs(incl) - 1 : 31;
-        excl += warp_sum_u64((int)lane <= first ? (s & kValMask) : 0);
+        c_acc += warp_sum_u64((int)lane <= first ? (c & kValMask) : 0);
+        w_acc += warp_sum_u64((int)lane <= first ? (w & kValMask) : 0);
         if (incl) break;
         pred -= 32;
     }
-    return excl;
+    ex_c = c_acc;
+    ex_w = w_acc;
 }
 
 // --------------------------------------------------------------------------
@@ -137,6 +162,9 @@ __device__ uint64_t lookback(const uint64_t *st, uint64_t b)
 //   once per tile, with boundaries snapped to k-aligned chunk starts).
 //   Vertex v occupies work [W_v, W_v + kVertexWork + deg_v); its chunk 0
 //   starts at W_v, chunk c > 0 at W_v + kVertexWork + c*k.
+//   Layout: a block covers kAdvanceWords bitmap words; warp w owns
+//   kAdvanceRounds runs of 32 consecutive words; the 32 vertices of a word are
+//   handled by the 32 lanes (coalesced record loads, depth and queue stores).
 // --------------------------------------------------------------------------
 struct HubItem {
     uint64_t q, w, d;
@@ -173,6 +201,7 @@ __device__ __forceinline__ void write_tiles(TileEntry *tiles, uint64_t q, uint64
 __global__ void __launch_bounds__(kAdvanceThreads) advance_kernel(AdvanceArgs a)
 {
     constexpr int NW = kAdvanceThreads / 32;
+    constexpr int R = kAdvanceRounds;
     constexpr int kHubCap = 32;
     __shared__ uint32_t s_wcnt[NW];
     __shared__ uint64_t s_wwork[NW];
@@ -182,40 +211,63 @@ __global__ void __launch_bounds__(kAdvanceThreads) advance_kernel(AdvanceArgs a)
 
     const uint32_t tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
     const uint64_t b = blockIdx.x;
-    const uint64_t wi = b * kAdvanceThreads + tid;
     const uint64_t ch = a.k ? a.k : (1ull << 40);
+    const uint64_t A = kVertexWork;
+    // first word of this warp's run r: wbase + r*32
+    const uint64_t wbase = b * (uint64_t)kAdvanceWords + (uint64_t)wid * 32 * R;
 
     if (tid == 0) s_nhub = 0;
 
-    uint32_t x = 0, p = 0;
-    if (wi < a.nwords) {
-        x = a.vis[wi];
-        p = a.prev[wi];
+    // ---- pass 1: new bits, depth, per-word (count, work) ----
+    uint32_t nbr[R];
+    uint32_t wc[R];   // lane j: count of word (r, j)
+    uint64_t ww[R];   // lane j: work of word (r, j)
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+        const uint64_t wi = wbase + (uint64_t)r * 32 + lane;
+        uint32_t x = 0, p = 0;
+        if (wi < a.nwords) {
+            x = a.vis[wi];
+            p = a.prev[wi];
+        }
+        const uint32_t nb = x & ~p;
+        if (nb) a.prev[wi] = x;
+        nbr[r] = nb;
+        wc[r] = __popc(nb);
+        ww[r] = 0;
+        uint32_t todo = __ballot_sync(FULL, nb != 0);
+        while (todo) {
+            const int j = __ffs(todo) - 1;
+            todo &= todo - 1;
+            const uint32_t nbw = __shfl_sync(FULL, nb, j);
+            const bool bit = (nbw >> lane) & 1;
+            uint64_t wk = 0;
+            if (bit) {
+                const uint64_t v = (wbase + (uint64_t)r * 32 + j) * 32 + lane;
+                wk = A + a.rec[v].deg;  // a1: degree lookup
+                a.depth[v] = a.depth_value;
+            }
+            const uint64_t sum = warp_sum_u64(wk);
+            if ((int)lane == j) ww[r] = sum;
+        }
     }
-    const uint32_t nb = x & ~p;
-    if (nb) a.prev[wi] = x;
-
-    // a1: degree lookup of the new frontier vertices (+ depth of the level)
-    uint64_t work = 0;
-    for (uint32_t t = nb; t; t &= t - 1) {
-        const uint64_t v = wi * 32 + (__ffs(t) - 1);
-        work += kVertexWork + a.rec[v].deg;
-        a.depth[v] = a.depth_value;
+    // warp totals
+    uint64_t tot_c = 0, tot_w = 0;
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+        uint32_t tc;
+        uint64_t tw;
+        warp_excl_u32(wc[r], tc);
+        warp_excl_u64(ww[r], tw);
+        tot_c += tc;
+        tot_w += tw;
     }
-    const uint32_t cnt = __popc(nb);
-
-    // a2: block scan of (cnt, work)
-    uint32_t wtot_c;
-    uint64_t wtot_w;
-    const uint32_t ex_c = warp_excl_u32(cnt, wtot_c);
-    const uint64_t ex_w = warp_excl_u64(work, wtot_w);
-    if (lane == 31) {
-        s_wcnt[wid] = wtot_c;
-        s_wwork[wid] = wtot_w;
+    if (lane == 0) {
+        s_wcnt[wid] = (uint32_t)tot_c;
+        s_wwork[wid] = tot_w;
     }
     __syncthreads();
-    uint32_t pre_c = 0;
-    uint64_t pre_w = 0, blk_c = 0, blk_w = 0;
+    uint64_t pre_c = 0, pre_w = 0, blk_c = 0, blk_w = 0;
 #pragma unroll
     for (int w = 0; w < NW; ++w) {
         if (w < (int)wid) {
@@ -226,25 +278,24 @@ __global__ void __launch_bounds__(kAdvanceThreads) advance_kernel(AdvanceArgs a)
         blk_w += s_wwork[w];
     }
 
-    // decoupled look-back across blocks (single pass)
-    uint64_t *st_c = a.status + (uint64_t)(a.parity * 2 + 0) * a.nblocks;
-    uint64_t *st_w = a.status + (uint64_t)(a.parity * 2 + 1) * a.nblocks;
+    // ---- a2 across blocks: decoupled look-back ----
+    uint64_t *st = a.status + (uint64_t)a.parity * 2 * a.nblocks;
     if (wid == 0) {
         if (lane == 0) {
             // clear this block's slots of the other parity for the next launch
-            a.status[(uint64_t)((a.parity ^ 1) * 2 + 0) * a.nblocks + b] = 0;
-            a.status[(uint64_t)((a.parity ^ 1) * 2 + 1) * a.nblocks + b] = 0;
+            uint64_t *other = a.status + (uint64_t)(a.parity ^ 1) * 2 * a.nblocks;
+            other[2 * b] = 0;
+            other[2 * b + 1] = 0;
             const uint64_t f = b == 0 ? kFlagIncl : kFlagAgg;
-            st_release_u64(st_c + b, f | blk_c);
-            st_release_u64(st_w + b, f | blk_w);
+            st_relaxed_u64(st + 2 * b, f | blk_c);
+            st_relaxed_u64(st + 2 * b + 1, f | blk_w);
         }
         uint64_t bq = 0, bw = 0;
         if (b > 0) {
-            bq = lookback(st_c, b);
-            bw = lookback(st_w, b);
+            lookback2(st, b, bq, bw);
             if (lane == 0) {
-                st_release_u64(st_c + b, kFlagIncl | (bq + blk_c));
-                st_release_u64(st_w + b, kFlagIncl | (bw + blk_w));
+                st_relaxed_u64(st + 2 * b, kFlagIncl | (bq + blk_c));
+                st_relaxed_u64(st + 2 * b + 1, kFlagIncl | (bw + blk_w));
             }
         }
         if (lane == 0) {
@@ -254,37 +305,57 @@ __global__ void __launch_bounds__(kAdvanceThreads) advance_kernel(AdvanceArgs a)
                 const uint64_t nf = bq + blk_c, nwork = bw + blk_w;
                 a.ctrl->nf = nf;
                 a.ctrl->nwork = nwork;
-                a.ctrl->ne = nwork - (uint64_t)kVertexWork * nf;
+                a.ctrl->ne = nwork - A * nf;
                 a.ctrl->ntiles = (nwork + kTileWork - 1) / kTileWork;
             }
         }
     }
     __syncthreads();
 
-    // a7 queue + a3 tile table
-    uint64_t q = s_block_q + pre_c + ex_c;
-    uint64_t W = s_block_w + pre_w + ex_w;
-    for (uint32_t t = nb; t; t &= t - 1) {
-        const uint64_t v = wi * 32 + (__ffs(t) - 1);
-        const uint64_t d = a.rec[v].deg;
-        a.queue[q] = (uint32_t)v;
-        bool done = false;
-        if (d >= 64ull * kTileWork) {  // hub: hand the tile writes to the whole block
-            const uint32_t slot = atomicAdd(&s_nhub, 1u);
-            if (slot < kHubCap) {
-                s_hub[slot] = HubItem{q, W, d};
-                done = true;
+    // ---- pass 2: a7 queue + a3 tile table ----
+    uint64_t run_c = s_block_q + pre_c, run_w = s_block_w + pre_w;
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+        uint32_t tc;
+        uint64_t tw;
+        const uint64_t word_q = run_c + warp_excl_u32(wc[r], tc);
+        const uint64_t word_w = run_w + warp_excl_u64(ww[r], tw);
+        run_c += tc;
+        run_w += tw;
+        uint32_t todo = __ballot_sync(FULL, nbr[r] != 0);
+        while (todo) {
+            const int j = __ffs(todo) - 1;
+            todo &= todo - 1;
+            const uint32_t nbw = __shfl_sync(FULL, nbr[r], j);
+            const uint64_t q0 = __shfl_sync(FULL, word_q, j);
+            const uint64_t w0 = __shfl_sync(FULL, word_w, j);
+            const bool bit = (nbw >> lane) & 1;
+            const uint64_t v = (wbase + (uint64_t)r * 32 + j) * 32 + lane;
+            const uint64_t d = bit ? a.rec[v].deg : 0;
+            uint64_t dummy;
+            const uint64_t wex = warp_excl_u64(bit ? A + d : 0, dummy);
+            if (bit) {
+                const uint64_t q = q0 + __popc(nbw & ((1u << lane) - 1));
+                const uint64_t W = w0 + wex;
+                a.queue[q] = (uint32_t)v;
+                bool done = false;
+                if (d >= 64ull * kTileWork) {  // hub: hand the tile writes to the whole block
+                    const uint32_t slot = atomicAdd(&s_nhub, 1u);
+                    if (slot < kHubCap) {
+                        s_hub[slot] = HubItem{q, W, d};
+                        done = true;
+                    }
+                }
+                if (!done) write_tiles(a.tiles, q, W, d, ch, 0, 1);
             }
         }
-        if (!done) write_tiles(a.tiles, q, W, d, ch, 0, 1);
-        ++q;
-        W += kVertexWork + d;
     }
     __syncthreads();
     const uint32_t nhub = min(s_nhub, (uint32_t)kHubCap);
     for (uint32_t h = 0; h < nhub; ++h)
         write_tiles(a.tiles, s_hub[h].q, s_hub[h].w, s_hub[h].d, ch, tid, kAdvanceThreads);
 }
+
 
 // --------------------------------------------------------------------------
 // expand_kernel: a4 + a5 + a6 (P:137-177 generalised, Alg. 1 lines 3-6)
