@@ -59,6 +59,7 @@ void free_device(DeviceGraph &d)
     if (d.device >= 0) cudaSetDevice(d.device);
     cudaFree(d.data);
     cudaFree(d.rec);
+    cudaFree(d.deg32);
     cudaFree(d.vlist);
     cudaFree(d.weights);
     cudaFree(d.vis);
@@ -113,6 +114,16 @@ efg_status upload(efg_graph *g, const efg_build_opts &o)
     }
     EFG_TRY(dev_alloc(d, &d.rec, h.n));
     CUDA_TRY(cudaMemcpyAsync(d.rec, rec.data(), h.n * sizeof(VRec), cudaMemcpyHostToDevice, s));
+    {
+        const uint64_t words = (h.n + 31) / 32;
+        const uint64_t nw = (words + kAdvanceWords - 1) / kAdvanceWords * kAdvanceWords;
+        std::vector<uint32_t> deg(nw * 32, 0);
+#pragma omp parallel for schedule(static)
+        for (int64_t v = 0; v < (int64_t)h.n; ++v) deg[v] = (uint32_t)(h.vlist[v + 1] - h.vlist[v]);
+        EFG_TRY(dev_alloc(d, &d.deg32, nw * 32));
+        CUDA_TRY(cudaMemcpyAsync(d.deg32, deg.data(), nw * 32 * 4, cudaMemcpyHostToDevice, s));
+        CUDA_TRY(cudaStreamSynchronize(s));
+    }
     EFG_TRY(dev_alloc(d, &d.vlist, h.n + 1));
     CUDA_TRY(cudaMemcpyAsync(d.vlist, h.vlist.data(), (h.n + 1) * 8, cudaMemcpyHostToDevice, s));
     if (!h.weights.empty()) {
@@ -154,6 +165,7 @@ efg_status run_advance(DeviceGraph &d, int32_t *depth, int32_t depth_value)
     a.vis = d.vis;
     a.prev = d.prev;
     a.rec = d.rec;
+    a.deg32 = d.deg32;
     a.depth = depth;
     a.queue = d.queue;
     a.tiles = d.tiles;

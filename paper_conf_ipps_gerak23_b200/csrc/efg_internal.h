@@ -93,6 +93,7 @@ struct DeviceGraph {
     uint8_t *data = nullptr;           // EF data + padding
     uint64_t data_bytes = 0;
     VRec *rec = nullptr;               // n records
+    uint32_t *deg32 = nullptr;         // n degrees (padded to the bitmap size)
     uint64_t *vlist = nullptr;         // n+1 (SSSP weight indexing / decode)
     float *weights = nullptr;          // m or null
     // traversal workspace

@@ -105,12 +105,14 @@ constexpr uint64_t kFlagAgg = 1ull << 62;
 constexpr uint64_t kFlagIncl = 2ull << 62;
 constexpr uint64_t kValMask = (1ull << 62) - 1;
 
-// Decoupled look-back (single-pass scan across blocks) over a pair of values
-// (frontier count, work).  Each block publishes two 64-bit words, flag | value,
-// with the same flag in both; a reader accepts a predecessor only when both
-// words carry the same non-zero flag, so no fence is needed (each value travels
-// in the same single-copy-atomic word as its flag).  Warp 0 looks back 32
-// predecessors at a time and stops at the nearest inclusive prefix.
+// Cross-block exclusive prefix for the advance scan (a2).  Every block
+// publishes its aggregate pair (frontier count, work) as two 64-bit words
+// flag | value (same flag in both, so no fence is needed: each value travels in
+// the same single-copy-atomic word as its flag).  A block then sums the
+// aggregates of ALL its predecessors directly, 32 lanes x several independent
+// loads per step: latency is a couple of L2 round trips regardless of the block
+// index, instead of a look-back chain that grows with the grid when every
+// block is resident at once.
 __device__ __forceinline__ uint64_t ld_relaxed_u64(const uint64_t *p)
 {
     uint64_t v;
@@ -123,34 +125,35 @@ __device__ __forceinline__ void st_relaxed_u64(uint64_t *p, uint64_t v)
     asm volatile("st.relaxed.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
 }
 
-__device__ void lookback2(const uint64_t *st, uint64_t b, uint64_t &ex_c, uint64_t &ex_w)
+__device__ void prefix_of_block(const uint64_t *st, uint64_t b, uint64_t &ex_c, uint64_t &ex_w)
 {
     const uint32_t lane = lane_id();
     uint64_t c_acc = 0, w_acc = 0;
-    int64_t pred = (int64_t)b - 1;
-    while (pred >= 0) {
-        const int64_t idx = pred - (int64_t)lane;
-        uint64_t c, w;
-        for (;;) {
-            if (idx >= 0) {
-                c = ld_relaxed_u64(st + 2 * idx);
-                w = ld_relaxed_u64(st + 2 * idx + 1);
-            } else {
-                c = kFlagIncl;
-                w = kFlagIncl;
+    for (uint64_t base = 0; base < b; base += 32 * 4) {
+        uint64_t c[4], w[4];
+#pragma unroll
+        for (int u = 0; u < 4; ++u) {
+            const uint64_t idx = base + u * 32 + lane;
+            c[u] = kFlagAgg;
+            w[u] = kFlagAgg;
+            if (idx < b) {
+                c[u] = ld_relaxed_u64(st + 2 * idx);
+                w[u] = ld_relaxed_u64(st + 2 * idx + 1);
             }
-            const bool ok = (c >> 62) != 0 && (c >> 62) == (w >> 62);
-            if (__all_sync(FULL, ok)) break;
         }
-        const uint32_t incl = __ballot_sync(FULL, (c >> 62) == 2);
-        const int first = incl ? __ffs(incl) - 1 : 31;
-        c_acc += warp_sum_u64((int)lane <= first ? (c & kValMask) : 0);
-        w_acc += warp_sum_u64((int)lane <= first ? (w & kValMask) : 0);
-        if (incl) break;
-        pred -= 32;
+#pragma unroll
+        for (int u = 0; u < 4; ++u) {
+            const uint64_t idx = base + u * 32 + lane;
+            while (idx < b && ((c[u] >> 62) == 0 || (w[u] >> 62) == 0)) {
+                c[u] = ld_relaxed_u64(st + 2 * idx);
+                w[u] = ld_relaxed_u64(st + 2 * idx + 1);
+            }
+            c_acc += c[u] & kValMask;
+            w_acc += w[u] & kValMask;
+        }
     }
-    ex_c = c_acc;
-    ex_w = w_acc;
+    ex_c = warp_sum_u64(c_acc);
+    ex_w = warp_sum_u64(w_acc);
 }
 
 // --------------------------------------------------------------------------
@@ -162,9 +165,10 @@ __device__ void lookback2(const uint64_t *st, uint64_t b, uint64_t &ex_c, uint64
 //   once per tile, with boundaries snapped to k-aligned chunk starts).
 //   Vertex v occupies work [W_v, W_v + kVertexWork + deg_v); its chunk 0
 //   starts at W_v, chunk c > 0 at W_v + kVertexWork + c*k.
-//   Layout: a block covers kAdvanceWords bitmap words; warp w owns
-//   kAdvanceRounds runs of 32 consecutive words; the 32 vertices of a word are
-//   handled by the 32 lanes (coalesced record loads, depth and queue stores).
+//   Layout: a block covers kAdvanceWords bitmap words; thread t owns
+//   kAdvanceRounds consecutive words (one 16-byte load per bitmap).  Degrees
+//   come from the compact deg32 array: a word with many new bits loads its 32
+//   degrees as eight 16-byte loads, a sparse word loads per bit.
 // --------------------------------------------------------------------------
 struct HubItem {
     uint64_t q, w, d;
@@ -198,10 +202,35 @@ __device__ __forceinline__ void write_tiles(TileEntry *tiles, uint64_t q, uint64
     }
 }
 
+constexpr int kDenseBits = 6;  // words with at least this many new bits load all 32 degrees
+
+// sum over the set bits b of nb of (A + deg[32*word + b])
+__device__ __forceinline__ uint64_t word_work(const uint32_t *deg32, uint64_t word, uint32_t nb)
+{
+    uint64_t work = 0;
+    if (__popc(nb) >= kDenseBits) {
+        const uint4 *p = reinterpret_cast<const uint4 *>(deg32 + word * 32);
+        uint4 d[8];
+#pragma unroll
+        for (int i = 0; i < 8; ++i) d[i] = __ldg(p + i);
+#pragma unroll
+        for (int i = 0; i < 8; ++i) {
+            work += (nb >> (4 * i + 0) & 1) ? (uint64_t)d[i].x + kVertexWork : 0;
+            work += (nb >> (4 * i + 1) & 1) ? (uint64_t)d[i].y + kVertexWork : 0;
+            work += (nb >> (4 * i + 2) & 1) ? (uint64_t)d[i].z + kVertexWork : 0;
+            work += (nb >> (4 * i + 3) & 1) ? (uint64_t)d[i].w + kVertexWork : 0;
+        }
+    } else {
+        for (uint32_t t = nb; t; t &= t - 1) work += kVertexWork + __ldg(deg32 + word * 32 + (__ffs(t) - 1));
+    }
+    return work;
+}
+
 __global__ void __launch_bounds__(kAdvanceThreads) advance_kernel(AdvanceArgs a)
 {
     constexpr int NW = kAdvanceThreads / 32;
     constexpr int R = kAdvanceRounds;
+    static_assert(R == 4, "one uint4 of bitmap words per thread");
     constexpr int kHubCap = 32;
     __shared__ uint32_t s_wcnt[NW];
     __shared__ uint64_t s_wwork[NW];
@@ -213,58 +242,33 @@ __global__ void __launch_bounds__(kAdvanceThreads) advance_kernel(AdvanceArgs a)
     const uint64_t b = blockIdx.x;
     const uint64_t ch = a.k ? a.k : (1ull << 40);
     const uint64_t A = kVertexWork;
-    // first word of this warp's run r: wbase + r*32
-    const uint64_t wbase = b * (uint64_t)kAdvanceWords + (uint64_t)wid * 32 * R;
+    const uint64_t w0 = b * (uint64_t)kAdvanceWords + (uint64_t)tid * R;  // first owned word
 
     if (tid == 0) s_nhub = 0;
 
-    // ---- pass 1: new bits, depth, per-word (count, work) ----
-    uint32_t nbr[R];
-    uint32_t wc[R];   // lane j: count of word (r, j)
-    uint64_t ww[R];   // lane j: work of word (r, j)
+    // ---- pass 1: new bits, depth, (count, work) of this thread's words ----
+    const uint4 xv = *reinterpret_cast<const uint4 *>(a.vis + w0);
+    const uint4 pv = *reinterpret_cast<const uint4 *>(a.prev + w0);
+    const uint32_t nb[R] = {xv.x & ~pv.x, xv.y & ~pv.y, xv.z & ~pv.z, xv.w & ~pv.w};
+    if (nb[0] | nb[1] | nb[2] | nb[3]) *reinterpret_cast<uint4 *>(a.prev + w0) = xv;
+    uint32_t cnt = 0;
+    uint64_t work = 0;
 #pragma unroll
     for (int r = 0; r < R; ++r) {
-        const uint64_t wi = wbase + (uint64_t)r * 32 + lane;
-        uint32_t x = 0, p = 0;
-        if (wi < a.nwords) {
-            x = a.vis[wi];
-            p = a.prev[wi];
-        }
-        const uint32_t nb = x & ~p;
-        if (nb) a.prev[wi] = x;
-        nbr[r] = nb;
-        wc[r] = __popc(nb);
-        ww[r] = 0;
-        uint32_t todo = __ballot_sync(FULL, nb != 0);
-        while (todo) {
-            const int j = __ffs(todo) - 1;
-            todo &= todo - 1;
-            const uint32_t nbw = __shfl_sync(FULL, nb, j);
-            const bool bit = (nbw >> lane) & 1;
-            uint64_t wk = 0;
-            if (bit) {
-                const uint64_t v = (wbase + (uint64_t)r * 32 + j) * 32 + lane;
-                wk = A + a.rec[v].deg;  // a1: degree lookup
-                a.depth[v] = a.depth_value;
-            }
-            const uint64_t sum = warp_sum_u64(wk);
-            if ((int)lane == j) ww[r] = sum;
-        }
+        if (!nb[r]) continue;
+        cnt += __popc(nb[r]);
+        work += word_work(a.deg32, w0 + r, nb[r]);  // a1: degree lookup
+        for (uint32_t t = nb[r]; t; t &= t - 1) a.depth[(w0 + r) * 32 + (__ffs(t) - 1)] = a.depth_value;
     }
-    // warp totals
-    uint64_t tot_c = 0, tot_w = 0;
-#pragma unroll
-    for (int r = 0; r < R; ++r) {
-        uint32_t tc;
-        uint64_t tw;
-        warp_excl_u32(wc[r], tc);
-        warp_excl_u64(ww[r], tw);
-        tot_c += tc;
-        tot_w += tw;
-    }
-    if (lane == 0) {
-        s_wcnt[wid] = (uint32_t)tot_c;
-        s_wwork[wid] = tot_w;
+
+    // ---- a2: block scan of (cnt, work) ----
+    uint32_t wtot_c;
+    uint64_t wtot_w;
+    const uint32_t ex_c = warp_excl_u32(cnt, wtot_c);
+    const uint64_t ex_w = warp_excl_u64(work, wtot_w);
+    if (lane == 31) {
+        s_wcnt[wid] = wtot_c;
+        s_wwork[wid] = wtot_w;
     }
     __syncthreads();
     uint64_t pre_c = 0, pre_w = 0, blk_c = 0, blk_w = 0;
@@ -278,7 +282,7 @@ __global__ void __launch_bounds__(kAdvanceThreads) advance_kernel(AdvanceArgs a)
         blk_w += s_wwork[w];
     }
 
-    // ---- a2 across blocks: decoupled look-back ----
+    // ---- a2 across blocks ----
     uint64_t *st = a.status + (uint64_t)a.parity * 2 * a.nblocks;
     if (wid == 0) {
         if (lane == 0) {
@@ -286,18 +290,11 @@ __global__ void __launch_bounds__(kAdvanceThreads) advance_kernel(AdvanceArgs a)
             uint64_t *other = a.status + (uint64_t)(a.parity ^ 1) * 2 * a.nblocks;
             other[2 * b] = 0;
             other[2 * b + 1] = 0;
-            const uint64_t f = b == 0 ? kFlagIncl : kFlagAgg;
-            st_relaxed_u64(st + 2 * b, f | blk_c);
-            st_relaxed_u64(st + 2 * b + 1, f | blk_w);
+            st_relaxed_u64(st + 2 * b, kFlagAgg | blk_c);
+            st_relaxed_u64(st + 2 * b + 1, kFlagAgg | blk_w);
         }
-        uint64_t bq = 0, bw = 0;
-        if (b > 0) {
-            lookback2(st, b, bq, bw);
-            if (lane == 0) {
-                st_relaxed_u64(st + 2 * b, kFlagIncl | (bq + blk_c));
-                st_relaxed_u64(st + 2 * b + 1, kFlagIncl | (bw + blk_w));
-            }
-        }
+        uint64_t bq, bw;
+        prefix_of_block(st, b, bq, bw);
         if (lane == 0) {
             s_block_q = bq;
             s_block_w = bw;
@@ -313,41 +310,25 @@ __global__ void __launch_bounds__(kAdvanceThreads) advance_kernel(AdvanceArgs a)
     __syncthreads();
 
     // ---- pass 2: a7 queue + a3 tile table ----
-    uint64_t run_c = s_block_q + pre_c, run_w = s_block_w + pre_w;
+    uint64_t q = s_block_q + pre_c + ex_c;
+    uint64_t W = s_block_w + pre_w + ex_w;
 #pragma unroll
     for (int r = 0; r < R; ++r) {
-        uint32_t tc;
-        uint64_t tw;
-        const uint64_t word_q = run_c + warp_excl_u32(wc[r], tc);
-        const uint64_t word_w = run_w + warp_excl_u64(ww[r], tw);
-        run_c += tc;
-        run_w += tw;
-        uint32_t todo = __ballot_sync(FULL, nbr[r] != 0);
-        while (todo) {
-            const int j = __ffs(todo) - 1;
-            todo &= todo - 1;
-            const uint32_t nbw = __shfl_sync(FULL, nbr[r], j);
-            const uint64_t q0 = __shfl_sync(FULL, word_q, j);
-            const uint64_t w0 = __shfl_sync(FULL, word_w, j);
-            const bool bit = (nbw >> lane) & 1;
-            const uint64_t v = (wbase + (uint64_t)r * 32 + j) * 32 + lane;
-            const uint64_t d = bit ? a.rec[v].deg : 0;
-            uint64_t dummy;
-            const uint64_t wex = warp_excl_u64(bit ? A + d : 0, dummy);
-            if (bit) {
-                const uint64_t q = q0 + __popc(nbw & ((1u << lane) - 1));
-                const uint64_t W = w0 + wex;
-                a.queue[q] = (uint32_t)v;
-                bool done = false;
-                if (d >= 64ull * kTileWork) {  // hub: hand the tile writes to the whole block
-                    const uint32_t slot = atomicAdd(&s_nhub, 1u);
-                    if (slot < kHubCap) {
-                        s_hub[slot] = HubItem{q, W, d};
-                        done = true;
-                    }
+        for (uint32_t t = nb[r]; t; t &= t - 1) {
+            const uint64_t v = (w0 + r) * 32 + (__ffs(t) - 1);
+            const uint64_t d = __ldg(a.deg32 + v);
+            a.queue[q] = (uint32_t)v;
+            bool done = false;
+            if (d >= 64ull * kTileWork) {  // hub: hand the tile writes to the whole block
+                const uint32_t slot = atomicAdd(&s_nhub, 1u);
+                if (slot < kHubCap) {
+                    s_hub[slot] = HubItem{q, W, d};
+                    done = true;
                 }
-                if (!done) write_tiles(a.tiles, q, W, d, ch, 0, 1);
             }
+            if (!done) write_tiles(a.tiles, q, W, d, ch, 0, 1);
+            ++q;
+            W += A + d;
         }
     }
     __syncthreads();
@@ -356,7 +337,7 @@ __global__ void __launch_bounds__(kAdvanceThreads) advance_kernel(AdvanceArgs a)
         write_tiles(a.tiles, s_hub[h].q, s_hub[h].w, s_hub[h].d, ch, tid, kAdvanceThreads);
 }
 
-
+// --------------------------------------------------------------------------
 // --------------------------------------------------------------------------
 // expand_kernel: a4 + a5 + a6 (P:137-177 generalised, Alg. 1 lines 3-6)
 //

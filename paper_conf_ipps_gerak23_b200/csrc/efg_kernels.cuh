@@ -28,6 +28,7 @@ struct AdvanceArgs {
     uint32_t *vis;             // visited bitmap
     uint32_t *prev;            // visited bitmap after the previous advance
     const VRec *rec;
+    const uint32_t *deg32;     // degrees (compact copy for the frontier step a1)
     int32_t *depth;            // depth output (may be the caller's device buffer)
     uint32_t *queue;           // next frontier (sorted by vertex id)
     TileEntry *tiles;          // tile table of the next level
