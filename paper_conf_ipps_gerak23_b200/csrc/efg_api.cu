@@ -157,7 +157,13 @@ struct Ctx {
     uint32_t parity;
 };
 
-uint32_t g_epoch = 0;  // parity source for the decoupled look-back status
+uint32_t g_epoch = 0;
+
+int kshift_of(uint32_t k)
+{
+    if (k == 0 || (k & (k - 1))) return -1;
+    return __builtin_ctz(k);
+}  // parity source for the decoupled look-back status
 
 efg_status run_advance(DeviceGraph &d, int32_t *depth, int32_t depth_value)
 {
@@ -176,6 +182,7 @@ efg_status run_advance(DeviceGraph &d, int32_t *depth, int32_t depth_value)
     a.depth_value = depth_value;
     a.parity = (g_epoch++) & 1u;
     a.k = d.k;
+    a.kshift = kshift_of(d.k);
     CUDA_TRY(launch_advance(a, static_cast<cudaStream_t>(d.stream)));
     return EFG_OK;
 }
@@ -191,6 +198,7 @@ efg_status run_expand(DeviceGraph &d, int mode, uint32_t *out)
     a.vis = d.vis;
     a.out = out;
     a.k = d.k;
+    a.kshift = kshift_of(d.k);
     const int blocks = d.num_sms * expand_occupancy(mode);
     CUDA_TRY(launch_expand(mode, a, blocks, static_cast<cudaStream_t>(d.stream)));
     return EFG_OK;

@@ -105,6 +105,23 @@ constexpr uint64_t kFlagAgg = 1ull << 62;
 constexpr uint64_t kFlagIncl = 2ull << 62;
 constexpr uint64_t kValMask = (1ull << 62) - 1;
 
+// Chunk length CH = k (forward-pointer quantum), or 2^40 when k = 0 (lists are
+// never split).  Divisions by CH use a shift when k is a power of two (the
+// paper's k = 512), the generic 64-bit divide otherwise.
+struct ChunkLen {
+    uint64_t ch;
+    int shift;  // log2(ch) or -1
+    __device__ __forceinline__ uint64_t div(uint64_t x) const { return shift >= 0 ? x >> shift : x / ch; }
+};
+
+__device__ __forceinline__ ChunkLen make_chunk(uint32_t k, int kshift)
+{
+    ChunkLen c;
+    c.ch = k ? k : (1ull << 40);
+    c.shift = k ? kshift : 40;
+    return c;
+}
+
 // Cross-block exclusive prefix for the advance scan (a2).  Every block
 // publishes its aggregate pair (frontier count, work) as two 64-bit words
 // flag | value (same flag in both, so no fence is needed: each value travels in
@@ -175,8 +192,9 @@ struct HubItem {
 };
 
 __device__ __forceinline__ void write_tiles(TileEntry *tiles, uint64_t q, uint64_t W, uint64_t d,
-                                            uint64_t ch, uint64_t w_begin, uint64_t w_step)
+                                            const ChunkLen &cl, uint64_t w_begin, uint64_t w_step)
 {
+    const uint64_t ch = cl.ch;
     const uint64_t T = kTileWork, A = kVertexWork;
     for (uint64_t t = (W + T - 1) / T + w_begin; t * T < W + A + d; t += w_step) {
         const uint64_t o = t * T - W;
@@ -186,7 +204,7 @@ __device__ __forceinline__ void write_tiles(TileEntry *tiles, uint64_t q, uint64
             te.chunk = 0;
             te.w = W;
         } else {
-            uint64_t c = o > A ? (o - A + ch - 1) / ch : 1;
+            uint64_t c = o > A ? cl.div(o - A + ch - 1) : 1;
             if (c == 0) c = 1;
             if (c * ch < d) {
                 te.fi = (uint32_t)q;
@@ -231,7 +249,7 @@ __global__ void __launch_bounds__(kAdvanceThreads) advance_kernel(AdvanceArgs a)
     constexpr int NW = kAdvanceThreads / 32;
     constexpr int R = kAdvanceRounds;
     static_assert(R == 4, "one uint4 of bitmap words per thread");
-    constexpr int kHubCap = 32;
+    constexpr int kHubCap = 256;
     __shared__ uint32_t s_wcnt[NW];
     __shared__ uint64_t s_wwork[NW];
     __shared__ uint64_t s_block_q, s_block_w;
@@ -240,7 +258,7 @@ __global__ void __launch_bounds__(kAdvanceThreads) advance_kernel(AdvanceArgs a)
 
     const uint32_t tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
     const uint64_t b = blockIdx.x;
-    const uint64_t ch = a.k ? a.k : (1ull << 40);
+    const ChunkLen cl = make_chunk(a.k, a.kshift);
     const uint64_t A = kVertexWork;
     const uint64_t w0 = b * (uint64_t)kAdvanceWords + (uint64_t)tid * R;  // first owned word
 
@@ -319,14 +337,14 @@ __global__ void __launch_bounds__(kAdvanceThreads) advance_kernel(AdvanceArgs a)
             const uint64_t d = __ldg(a.deg32 + v);
             a.queue[q] = (uint32_t)v;
             bool done = false;
-            if (d >= 64ull * kTileWork) {  // hub: hand the tile writes to the whole block
+            if (d >= 8ull * kTileWork) {  // long list: hand its tile writes to the whole block
                 const uint32_t slot = atomicAdd(&s_nhub, 1u);
                 if (slot < kHubCap) {
                     s_hub[slot] = HubItem{q, W, d};
                     done = true;
                 }
             }
-            if (!done) write_tiles(a.tiles, q, W, d, ch, 0, 1);
+            if (!done) write_tiles(a.tiles, q, W, d, cl, 0, 1);
             ++q;
             W += A + d;
         }
@@ -334,7 +352,7 @@ __global__ void __launch_bounds__(kAdvanceThreads) advance_kernel(AdvanceArgs a)
     __syncthreads();
     const uint32_t nhub = min(s_nhub, (uint32_t)kHubCap);
     for (uint32_t h = 0; h < nhub; ++h)
-        write_tiles(a.tiles, s_hub[h].q, s_hub[h].w, s_hub[h].d, ch, tid, kAdvanceThreads);
+        write_tiles(a.tiles, s_hub[h].q, s_hub[h].w, s_hub[h].d, cl, tid, kAdvanceThreads);
 }
 
 // --------------------------------------------------------------------------
@@ -409,7 +427,8 @@ __global__ void __launch_bounds__(kExpandThreads, 8) expand_kernel(ExpandArgs a)
     const uint32_t lane = lane_id(), wid = threadIdx.x >> 5;
     const uint64_t ntiles = a.ctrl->ntiles, nf = a.ctrl->nf, nwork = a.ctrl->nwork;
     const uint32_t *data32 = reinterpret_cast<const uint32_t *>(a.data);
-    const uint64_t CH = a.k ? a.k : (1ull << 40);
+    const ChunkLen cl = make_chunk(a.k, a.kshift);
+    const uint64_t CH = cl.ch;
     const uint64_t A = kVertexWork;
     const uint64_t gw = (uint64_t)blockIdx.x * kWarps + wid;
     const uint64_t nwarps = (uint64_t)gridDim.x * kWarps;
@@ -432,7 +451,7 @@ __global__ void __launch_bounds__(kExpandThreads, 8) expand_kernel(ExpandArgs a)
                 ubytes = r.w;
             }
             const uint64_t first = lane == 0 ? c0 : 0;
-            const uint64_t nch = deg ? (deg + CH - 1) / CH : 0;
+            const uint64_t nch = deg ? cl.div(deg + CH - 1) : 0;
             const uint32_t nrem = (uint32_t)(nch > first ? nch - first : 0);
             // work still ahead of this vertex (from its first remaining chunk on)
             const uint64_t wrem = fv < nf ? (first == 0 ? A + deg : deg - first * CH) : 0;
@@ -472,7 +491,7 @@ __global__ void __launch_bounds__(kExpandThreads, 8) expand_kernel(ExpandArgs a)
             if (valid) {
                 const uint64_t off = offl_j & kOffMask;
                 l = (uint32_t)(offl_j >> kOffBits);
-                const uint64_t F = a.k ? deg_j / a.k : 0;
+                const uint64_t F = a.k ? cl.div(deg_j) : 0;
                 const uint64_t L = ((uint64_t)deg_j * l + 7) >> 3;
                 lbase = (off + 4 * F) * 8;
                 U0 = (off + 4 * F + L) * 8;

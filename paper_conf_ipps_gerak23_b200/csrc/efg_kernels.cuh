@@ -22,6 +22,7 @@ struct ExpandArgs {
     uint32_t *vis;             // visited bitmap (modes 0, 1)
     uint32_t *out;             // parent (mode 1) or decode output (mode 2)
     uint32_t k;                // forward-pointer quantum (chunk length); 0 = none
+    int32_t kshift;            // log2(k) if k is a power of two, else -1
 };
 
 struct AdvanceArgs {
@@ -39,6 +40,7 @@ struct AdvanceArgs {
     int32_t depth_value;       // depth assigned to newly discovered vertices
     uint32_t parity;           // status parity of this launch
     uint32_t k;                // chunk length (0 = whole lists)
+    int32_t kshift;            // log2(k) if k is a power of two, else -1
 };
 
 cudaError_t launch_expand(int mode, const ExpandArgs &a, int blocks, cudaStream_t s);
