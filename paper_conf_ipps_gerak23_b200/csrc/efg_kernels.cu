@@ -220,31 +220,37 @@ __device__ __forceinline__ void write_tiles(TileEntry *tiles, uint64_t q, uint64
     }
 }
 
-constexpr int kDenseBits = 6;  // words with at least this many new bits load all 32 degrees
-
-// sum over the set bits b of nb of (A + deg[32*word + b])
-__device__ __forceinline__ uint64_t word_work(const uint32_t *deg32, uint64_t word, uint32_t nb)
+// Tile entries for one frontier vertex; long lists are queued for the whole block.
+__device__ __noinline__ void place_tiles(TileEntry *tiles, uint64_t q, uint64_t W, uint64_t d,
+                                         const ChunkLen &cl, HubItem *hub, uint32_t *nhub, uint32_t cap)
 {
-    uint64_t work = 0;
-    if (__popc(nb) >= kDenseBits) {
-        const uint4 *p = reinterpret_cast<const uint4 *>(deg32 + word * 32);
-        uint4 d[8];
-#pragma unroll
-        for (int i = 0; i < 8; ++i) d[i] = __ldg(p + i);
-#pragma unroll
-        for (int i = 0; i < 8; ++i) {
-            work += (nb >> (4 * i + 0) & 1) ? (uint64_t)d[i].x + kVertexWork : 0;
-            work += (nb >> (4 * i + 1) & 1) ? (uint64_t)d[i].y + kVertexWork : 0;
-            work += (nb >> (4 * i + 2) & 1) ? (uint64_t)d[i].z + kVertexWork : 0;
-            work += (nb >> (4 * i + 3) & 1) ? (uint64_t)d[i].w + kVertexWork : 0;
+    if (d >= 8ull * kTileWork) {
+        const uint32_t slot = atomicAdd(nhub, 1u);
+        if (slot < cap) {
+            hub[slot] = HubItem{q, W, d};
+            return;
         }
-    } else {
-        for (uint32_t t = nb; t; t &= t - 1) work += kVertexWork + __ldg(deg32 + word * 32 + (__ffs(t) - 1));
     }
-    return work;
+    write_tiles(tiles, q, W, d, cl, 0, 1);
 }
 
-__global__ void __launch_bounds__(kAdvanceThreads) advance_kernel(AdvanceArgs a)
+// The 32 degrees of one bitmap word: eight 16-byte loads issued together.
+struct DegWord {
+    uint4 d[8];
+    __device__ __forceinline__ void load(const uint32_t *deg32, uint64_t word)
+    {
+        const uint4 *p = reinterpret_cast<const uint4 *>(deg32 + word * 32);
+#pragma unroll
+        for (int i = 0; i < 8; ++i) d[i] = __ldg(p + i);
+    }
+    __device__ __forceinline__ uint32_t at(int b) const  // b is a compile-time constant after unrolling
+    {
+        const uint4 &x = d[b >> 2];
+        return (b & 3) == 0 ? x.x : (b & 3) == 1 ? x.y : (b & 3) == 2 ? x.z : x.w;
+    }
+};
+
+__global__ void __launch_bounds__(kAdvanceThreads, 3) advance_kernel(AdvanceArgs a)
 {
     constexpr int NW = kAdvanceThreads / 32;
     constexpr int R = kAdvanceRounds;
@@ -273,10 +279,25 @@ __global__ void __launch_bounds__(kAdvanceThreads) advance_kernel(AdvanceArgs a)
     uint64_t work = 0;
 #pragma unroll
     for (int r = 0; r < R; ++r) {
-        if (!nb[r]) continue;
-        cnt += __popc(nb[r]);
-        work += word_work(a.deg32, w0 + r, nb[r]);  // a1: degree lookup
-        for (uint32_t t = nb[r]; t; t &= t - 1) a.depth[(w0 + r) * 32 + (__ffs(t) - 1)] = a.depth_value;
+        const uint32_t m = nb[r];
+        if (!m) continue;
+        const uint64_t v0 = (w0 + r) * 32;
+        cnt += __popc(m);
+        if (m & (m - 1)) {  // >= 2 new vertices: all 32 degrees at once (a1)
+            DegWord dw;
+            dw.load(a.deg32, w0 + r);
+#pragma unroll
+            for (int bb = 0; bb < 32; ++bb) {
+                if (m >> bb & 1) {
+                    work += A + dw.at(bb);
+                    a.depth[v0 + bb] = a.depth_value;
+                }
+            }
+        } else {
+            const uint64_t v = v0 + (__ffs(m) - 1);
+            work += A + __ldg(a.deg32 + v);
+            a.depth[v] = a.depth_value;
+        }
     }
 
     // ---- a2: block scan of (cnt, work) ----
@@ -332,21 +353,22 @@ __global__ void __launch_bounds__(kAdvanceThreads) advance_kernel(AdvanceArgs a)
     uint64_t W = s_block_w + pre_w + ex_w;
 #pragma unroll
     for (int r = 0; r < R; ++r) {
-        for (uint32_t t = nb[r]; t; t &= t - 1) {
-            const uint64_t v = (w0 + r) * 32 + (__ffs(t) - 1);
-            const uint64_t d = __ldg(a.deg32 + v);
-            a.queue[q] = (uint32_t)v;
-            bool done = false;
-            if (d >= 8ull * kTileWork) {  // long list: hand its tile writes to the whole block
-                const uint32_t slot = atomicAdd(&s_nhub, 1u);
-                if (slot < kHubCap) {
-                    s_hub[slot] = HubItem{q, W, d};
-                    done = true;
-                }
+        const uint32_t m = nb[r];
+        if (!m) continue;
+        const uint64_t v0 = (w0 + r) * 32;
+        DegWord dw;
+        if (m & (m - 1)) dw.load(a.deg32, w0 + r);
+#pragma unroll
+        for (int bb = 0; bb < 32; ++bb) {
+            if (m >> bb & 1) {
+                const uint64_t d = (m & (m - 1)) ? dw.at(bb) : __ldg(a.deg32 + v0 + bb);
+                a.queue[q] = (uint32_t)(v0 + bb);
+                // does a tile boundary fall inside [W, W + A + d)?
+                if (((W + kTileWork - 1) & ~(uint64_t)(kTileWork - 1)) < W + A + d)
+                    place_tiles(a.tiles, q, W, d, cl, s_hub, &s_nhub, kHubCap);
+                ++q;
+                W += A + d;
             }
-            if (!done) write_tiles(a.tiles, q, W, d, cl, 0, 1);
-            ++q;
-            W += A + d;
         }
     }
     __syncthreads();
