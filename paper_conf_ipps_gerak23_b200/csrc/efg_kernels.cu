@@ -234,27 +234,36 @@ __device__ __noinline__ void place_tiles(TileEntry *tiles, uint64_t q, uint64_t 
     write_tiles(tiles, q, W, d, cl, 0, 1);
 }
 
-// The 32 degrees of one bitmap word: eight 16-byte loads issued together.
-struct DegWord {
-    uint4 d[8];
-    __device__ __forceinline__ void load(const uint32_t *deg32, uint64_t word)
-    {
-        const uint4 *p = reinterpret_cast<const uint4 *>(deg32 + word * 32);
+// exact warp sum of a value < 2^48 with two 32-bit REDUX instructions
+__device__ __forceinline__ uint64_t warp_sum_small(uint64_t x)
+{
+    const uint32_t hi = __reduce_add_sync(FULL, (uint32_t)(x >> 16));
+    const uint32_t lo = __reduce_add_sync(FULL, (uint32_t)(x & 0xffff));
+    return ((uint64_t)hi << 16) + lo;
+}
+
+constexpr int kAdvGroup = 8;  // bitmap words whose degree loads are in flight together
+
+// Pop up to kAdvGroup set bits (word indices) from a warp-uniform mask.
+__device__ __forceinline__ int pop_words(uint32_t &mask, int (&j)[kAdvGroup])
+{
+    int n = 0;
 #pragma unroll
-        for (int i = 0; i < 8; ++i) d[i] = __ldg(p + i);
+    for (int u = 0; u < kAdvGroup; ++u) {
+        j[u] = 0;
+        if (mask) {
+            j[u] = __ffs(mask) - 1;
+            mask &= mask - 1;
+            n = u + 1;
+        }
     }
-    __device__ __forceinline__ uint32_t at(int b) const  // b is a compile-time constant after unrolling
-    {
-        const uint4 &x = d[b >> 2];
-        return (b & 3) == 0 ? x.x : (b & 3) == 1 ? x.y : (b & 3) == 2 ? x.z : x.w;
-    }
-};
+    return n;
+}
 
 __global__ void __launch_bounds__(kAdvanceThreads, 3) advance_kernel(AdvanceArgs a)
 {
     constexpr int NW = kAdvanceThreads / 32;
     constexpr int R = kAdvanceRounds;
-    static_assert(R == 4, "one uint4 of bitmap words per thread");
     constexpr int kHubCap = 256;
     __shared__ uint32_t s_wcnt[NW];
     __shared__ uint64_t s_wwork[NW];
@@ -266,48 +275,54 @@ __global__ void __launch_bounds__(kAdvanceThreads, 3) advance_kernel(AdvanceArgs
     const uint64_t b = blockIdx.x;
     const ChunkLen cl = make_chunk(a.k, a.kshift);
     const uint64_t A = kVertexWork;
-    const uint64_t w0 = b * (uint64_t)kAdvanceWords + (uint64_t)tid * R;  // first owned word
+    const uint32_t lt = (1u << lane) - 1;
+    // words of (warp, round r): rbase(r) + 0..31, lane j owns word rbase(r) + j
+    const uint64_t wbase = b * (uint64_t)kAdvanceWords + (uint64_t)wid * 32 * R;
 
     if (tid == 0) s_nhub = 0;
 
-    // ---- pass 1: new bits, depth, (count, work) of this thread's words ----
-    const uint4 xv = *reinterpret_cast<const uint4 *>(a.vis + w0);
-    const uint4 pv = *reinterpret_cast<const uint4 *>(a.prev + w0);
-    const uint32_t nb[R] = {xv.x & ~pv.x, xv.y & ~pv.y, xv.z & ~pv.z, xv.w & ~pv.w};
-    if (nb[0] | nb[1] | nb[2] | nb[3]) *reinterpret_cast<uint4 *>(a.prev + w0) = xv;
-    uint32_t cnt = 0;
-    uint64_t work = 0;
+    // ---- pass 1: new bits (a7), depth, per-word (count, work) via a1 ----
+    uint32_t nb[R], wc[R];
+    uint64_t ww[R];
 #pragma unroll
     for (int r = 0; r < R; ++r) {
-        const uint32_t m = nb[r];
-        if (!m) continue;
-        const uint64_t v0 = (w0 + r) * 32;
-        cnt += __popc(m);
-        if (m & (m - 1)) {  // >= 2 new vertices: all 32 degrees at once (a1)
-            DegWord dw;
-            dw.load(a.deg32, w0 + r);
+        const uint64_t rb = wbase + (uint64_t)r * 32;
+        const uint32_t x = a.vis[rb + lane], p = a.prev[rb + lane];
+        nb[r] = x & ~p;
+        if (nb[r]) a.prev[rb + lane] = x;
+        wc[r] = __popc(nb[r]);
+        ww[r] = 0;
+        uint32_t mask = __ballot_sync(FULL, nb[r] != 0);
+        while (mask) {
+            int j[kAdvGroup];
+            pop_words(mask, j);
+            uint32_t d[kAdvGroup], nbw[kAdvGroup];
 #pragma unroll
-            for (int bb = 0; bb < 32; ++bb) {
-                if (m >> bb & 1) {
-                    work += A + dw.at(bb);
-                    a.depth[v0 + bb] = a.depth_value;
-                }
+            for (int u = 0; u < kAdvGroup; ++u) {
+                nbw[u] = __shfl_sync(FULL, nb[r], j[u]);
+                // lanes past the popped words see j = 0 duplicates: drop them
+                if (u > 0 && j[u] == 0) nbw[u] = 0;
+                d[u] = (nbw[u] >> lane & 1) ? __ldg(a.deg32 + (rb + j[u]) * 32 + lane) : 0;
             }
-        } else {
-            const uint64_t v = v0 + (__ffs(m) - 1);
-            work += A + __ldg(a.deg32 + v);
-            a.depth[v] = a.depth_value;
+#pragma unroll
+            for (int u = 0; u < kAdvGroup; ++u) {
+                const bool bit = nbw[u] >> lane & 1;
+                if (bit) a.depth[(rb + j[u]) * 32 + lane] = a.depth_value;
+                const uint64_t s = warp_sum_small(bit ? A + d[u] : 0);
+                if (nbw[u] && (int)lane == j[u]) ww[r] = s;
+            }
         }
     }
-
-    // ---- a2: block scan of (cnt, work) ----
-    uint32_t wtot_c;
-    uint64_t wtot_w;
-    const uint32_t ex_c = warp_excl_u32(cnt, wtot_c);
-    const uint64_t ex_w = warp_excl_u64(work, wtot_w);
-    if (lane == 31) {
-        s_wcnt[wid] = wtot_c;
-        s_wwork[wid] = wtot_w;
+    // warp totals -> block scan
+    uint64_t tot_c = 0, tot_w = 0;
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+        tot_c += __reduce_add_sync(FULL, wc[r]);
+        tot_w += warp_sum_small(ww[r]);
+    }
+    if (lane == 0) {
+        s_wcnt[wid] = (uint32_t)tot_c;
+        s_wwork[wid] = tot_w;
     }
     __syncthreads();
     uint64_t pre_c = 0, pre_w = 0, blk_c = 0, blk_w = 0;
@@ -348,26 +363,43 @@ __global__ void __launch_bounds__(kAdvanceThreads, 3) advance_kernel(AdvanceArgs
     }
     __syncthreads();
 
-    // ---- pass 2: a7 queue + a3 tile table ----
-    uint64_t q = s_block_q + pre_c + ex_c;
-    uint64_t W = s_block_w + pre_w + ex_w;
+    // ---- pass 2: sorted queue (a7) + tile table (a3) ----
+    uint64_t run_c = s_block_q + pre_c, run_w = s_block_w + pre_w;
 #pragma unroll
     for (int r = 0; r < R; ++r) {
-        const uint32_t m = nb[r];
-        if (!m) continue;
-        const uint64_t v0 = (w0 + r) * 32;
-        DegWord dw;
-        if (m & (m - 1)) dw.load(a.deg32, w0 + r);
+        const uint64_t rb = wbase + (uint64_t)r * 32;
+        uint32_t tc;
+        uint64_t tw;
+        const uint64_t wq = run_c + warp_excl_u32(wc[r], tc);
+        const uint64_t wwp = run_w + warp_excl_u64(ww[r], tw);
+        run_c += tc;
+        run_w += tw;
+        uint32_t mask = __ballot_sync(FULL, nb[r] != 0);
+        while (mask) {
+            int j[kAdvGroup];
+            pop_words(mask, j);
+            uint32_t d[kAdvGroup], nbw[kAdvGroup];
 #pragma unroll
-        for (int bb = 0; bb < 32; ++bb) {
-            if (m >> bb & 1) {
-                const uint64_t d = (m & (m - 1)) ? dw.at(bb) : __ldg(a.deg32 + v0 + bb);
-                a.queue[q] = (uint32_t)(v0 + bb);
-                // does a tile boundary fall inside [W, W + A + d)?
-                if (((W + kTileWork - 1) & ~(uint64_t)(kTileWork - 1)) < W + A + d)
-                    place_tiles(a.tiles, q, W, d, cl, s_hub, &s_nhub, kHubCap);
-                ++q;
-                W += A + d;
+            for (int u = 0; u < kAdvGroup; ++u) {
+                nbw[u] = __shfl_sync(FULL, nb[r], j[u]);
+                if (u > 0 && j[u] == 0) nbw[u] = 0;
+                d[u] = (nbw[u] >> lane & 1) ? __ldg(a.deg32 + (rb + j[u]) * 32 + lane) : 0;
+            }
+#pragma unroll
+            for (int u = 0; u < kAdvGroup; ++u) {
+                const bool bit = nbw[u] >> lane & 1;
+                const uint64_t q0 = __shfl_sync(FULL, wq, j[u]);
+                const uint64_t w0 = __shfl_sync(FULL, wwp, j[u]);
+                uint64_t dummy;
+                const uint64_t wex = warp_excl_u64(bit ? A + d[u] : 0, dummy);
+                if (bit) {
+                    const uint64_t q = q0 + __popc(nbw[u] & lt);
+                    const uint64_t W = w0 + wex;
+                    a.queue[q] = (uint32_t)((rb + j[u]) * 32 + lane);
+                    // does a tile boundary fall inside [W, W + A + d)?
+                    if (((W + kTileWork - 1) & ~(uint64_t)(kTileWork - 1)) < W + A + d[u])
+                        place_tiles(a.tiles, q, W, d[u], cl, s_hub, &s_nhub, kHubCap);
+                }
             }
         }
     }
@@ -377,7 +409,7 @@ __global__ void __launch_bounds__(kAdvanceThreads, 3) advance_kernel(AdvanceArgs
         write_tiles(a.tiles, s_hub[h].q, s_hub[h].w, s_hub[h].d, cl, tid, kAdvanceThreads);
 }
 
-// --------------------------------------------------------------------------
+
 // --------------------------------------------------------------------------
 // expand_kernel: a4 + a5 + a6 (P:137-177 generalised, Alg. 1 lines 3-6)
 //
