@@ -185,6 +185,16 @@ efg_status efg_sssp(efg_graph *g, uint32_t source, float *dist, efg_stats *st);
 efg_status efg_pagerank(efg_graph *g, double damping, uint32_t iters, double *rank,
                         efg_stats *st);
 
+/* Options (efg_set_option). */
+#define EFG_OPT_LEVEL_LOOP 1 /* 0 (default): the BFS level loop runs on the device as one
+                              * CUDA graph with a conditional WHILE node (no host round trip
+                              * per level); 1: host-driven loop that reads the frontier size
+                              * each level and times every expand launch with CUDA events. */
+
+/* Set a per-handle option.  Errors: EFG_EINVAL (unknown option / value),
+ * EFG_ESTATE (host-only handle). */
+efg_status efg_set_option(efg_graph *g, int option, int64_t value);
+
 /* ---- multi-GPU: 1-D row partition, per-level exchange ---- */
 
 /* 128-byte opaque id (an ncclUniqueId).  Rank 0 creates it and the caller

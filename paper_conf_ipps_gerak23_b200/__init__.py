@@ -78,6 +78,11 @@ class Graph:
         check(lib.efg_build(n, src.size, _ptr(src), _ptr(dst), C.byref(o), C.byref(h)), "efg_build")
         return cls(h.value, stream)
 
+    def set_level_loop(self, host: bool) -> None:
+        """EFG_OPT_LEVEL_LOOP: False = device-side CUDA-graph loop (default),
+        True = host loop with per-level CUDA-event timing of the expand kernel."""
+        check(lib.efg_set_option(self._h, _abi.EFG_OPT_LEVEL_LOOP, 1 if host else 0), "efg_set_option")
+
     def free(self) -> None:
         if self._h:
             lib.efg_free(self._h)

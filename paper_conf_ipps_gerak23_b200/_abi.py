@@ -17,6 +17,7 @@ STATUS_NAMES = {0: "EFG_OK", 1: "EFG_EINVAL", 2: "EFG_ERANGE", 3: "EFG_ENOMEM", 
                 5: "EFG_ENCCL", 6: "EFG_ENOTSUP", 7: "EFG_ESTATE"}
 EFG_SYMMETRIZE, EFG_DEDUP, EFG_DROP_SELF_LOOPS = 0x1, 0x2, 0x4
 EFG_DEFAULT_FLAGS = 0x7
+EFG_OPT_LEVEL_LOOP = 1
 
 
 class BuildOpts(C.Structure):
@@ -55,6 +56,7 @@ SIGNATURES = [
     ("efg_bfs", C.c_int, [C.c_void_p, C.c_uint32, C.c_void_p, C.c_void_p, C.POINTER(Stats)]),
     ("efg_sssp", C.c_int, [C.c_void_p, C.c_uint32, C.c_void_p, C.POINTER(Stats)]),
     ("efg_pagerank", C.c_int, [C.c_void_p, C.c_double, C.c_uint32, C.c_void_p, C.POINTER(Stats)]),
+    ("efg_set_option", C.c_int, [C.c_void_p, C.c_int, C.c_int64]),
     ("efg_get_unique_id", C.c_int, [C.c_void_p]),
     ("efg_dist_init", C.c_int, [C.c_int, C.c_int, C.c_void_p, C.c_int, C.POINTER(C.c_void_p)]),
     ("efg_dist_free", None, [C.c_void_p]),

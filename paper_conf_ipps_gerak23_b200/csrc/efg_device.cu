@@ -1,0 +1,432 @@
+// efg_device.cu — device side of a handle: upload of the packed EFG, the
+// traversal workspace, and the level-synchronous driver.
+//
+// Per BFS level the driver runs three kernels (efg_kernels.cu):
+//   expand  (a4 a5 a6)  ->  compact (a7)  ->  plan (a1 a2 a3)
+// Two drivers share them:
+//   * graph mode (default): the level loop is one CUDA graph with a
+//     conditional WHILE node; plan_kernel's last block sets the condition
+//     (frontier non-empty) on the device, so a whole BFS costs one graph launch
+//     and no host round trip per level;
+//   * host mode (efg_set_option EFG_OPT_LEVEL_LOOP = 1): the host launches each
+//     level, reads the frontier size back, and brackets every expand launch
+//     with CUDA events (the per-kernel timing bench.py reports for the roofline).
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cstring>
+#include <string>
+#include <vector>
+
+#include "efg_internal.h"
+#include "efg_kernels.cuh"
+
+namespace efg {
+
+#define CUDA_TRY(expr)                                                                         \
+    do {                                                                                       \
+        cudaError_t _e = (expr);                                                               \
+        if (_e != cudaSuccess)                                                                 \
+            return set_error(EFG_ECUDA, std::string(#expr) + ": " + cudaGetErrorString(_e)); \
+    } while (0)
+
+#define EFG_TRY(expr)                \
+    do {                             \
+        efg_status _s = (expr);      \
+        if (_s != EFG_OK) return _s; \
+    } while (0)
+
+namespace {
+
+bool is_device_ptr(const void *p)
+{
+    cudaPointerAttributes at;
+    if (cudaPointerGetAttributes(&at, p) != cudaSuccess) {
+        cudaGetLastError();
+        return false;
+    }
+    return at.type == cudaMemoryTypeDevice || at.type == cudaMemoryTypeManaged;
+}
+
+template <typename T>
+efg_status dev_alloc(DeviceGraph &d, T **p, uint64_t count)
+{
+    const size_t bytes = std::max<uint64_t>(count, 1) * sizeof(T);
+    cudaError_t e = cudaMalloc(reinterpret_cast<void **>(p), bytes);
+    if (e != cudaSuccess) {
+        cudaGetLastError();
+        *p = nullptr;
+        return set_error(e == cudaErrorMemoryAllocation ? EFG_ENOMEM : EFG_ECUDA,
+                         std::string("cudaMalloc(") + std::to_string(bytes) + "): " + cudaGetErrorString(e));
+    }
+    d.device_bytes += bytes;
+    return EFG_OK;
+}
+
+int kshift_of(uint32_t k)
+{
+    if (k == 0 || (k & (k - 1))) return -1;
+    return __builtin_ctz(k);
+}
+
+cudaStream_t stream_of(const DeviceGraph &d) { return static_cast<cudaStream_t>(d.stream); }
+
+ExpandArgs expand_args(DeviceGraph &d, uint32_t *out)
+{
+    ExpandArgs a;
+    a.data = d.data;
+    a.rec = d.rec;
+    a.queue = d.queue;
+    a.tiles = d.tiles;
+    a.ctrl = d.ctrl;
+    a.vis = d.vis;
+    a.out = out;
+    a.stats = d.stats;
+    a.max_stats = kMaxLevelStats;
+    a.k = d.k;
+    a.kshift = kshift_of(d.k);
+    return a;
+}
+
+CompactArgs compact_args(DeviceGraph &d)
+{
+    CompactArgs a;
+    a.vis = d.vis;
+    a.prev = d.prev;
+    a.queue = d.queue;
+    a.ctrl = d.ctrl;
+    a.status = d.status;
+    a.nwords = d.nwords;
+    a.words_per_block = d.words_per_block;
+    return a;
+}
+
+PlanArgs plan_args(DeviceGraph &d, cudaGraphConditionalHandle cond)
+{
+    PlanArgs a;
+    a.queue = d.queue;
+    a.deg32 = d.deg32;
+    a.tiles = d.tiles;
+    a.ctrl = d.ctrl;
+    a.status = d.status + kMaxGrid;
+    a.stats = d.stats;
+    a.max_stats = kMaxLevelStats;
+    a.k = d.k;
+    a.kshift = kshift_of(d.k);
+    a.cond = cond;
+    return a;
+}
+
+efg_status launch_level_end(DeviceGraph &d, cudaGraphConditionalHandle cond, cudaStream_t s)
+{
+    CUDA_TRY(launch_compact(compact_args(d), (unsigned)((d.nwords + d.words_per_block - 1) / d.words_per_block), s));
+    CUDA_TRY(launch_plan(plan_args(d, cond), d.frontier_blocks, s));
+    return EFG_OK;
+}
+
+// Build (once per handle and mode) the graph: while (frontier) { expand; compact; plan }
+efg_status build_loop_graph(DeviceGraph &d, int mode)
+{
+    if (d.loop_exec[mode]) return EFG_OK;
+    cudaGraph_t g;
+    CUDA_TRY(cudaGraphCreate(&g, 0));
+    cudaGraphConditionalHandle cond;
+    CUDA_TRY(cudaGraphConditionalHandleCreate(&cond, g, 1, cudaGraphCondAssignDefault));
+    cudaGraphNodeParams cp = {};
+    cp.type = cudaGraphNodeTypeConditional;
+    cp.conditional.handle = cond;
+    cp.conditional.type = cudaGraphCondTypeWhile;
+    cp.conditional.size = 1;
+    cudaGraphNode_t node;
+    CUDA_TRY(cudaGraphAddNode(&node, g, nullptr, 0, &cp));
+    cudaGraph_t body = cp.conditional.phGraph_out[0];
+    cudaStream_t cs;
+    CUDA_TRY(cudaStreamCreateWithFlags(&cs, cudaStreamNonBlocking));
+    CUDA_TRY(cudaStreamBeginCaptureToGraph(cs, body, nullptr, nullptr, 0, cudaStreamCaptureModeRelaxed));
+    const int blocks = d.num_sms * expand_occupancy(mode);
+    cudaError_t e1 = launch_expand(mode, expand_args(d, nullptr), blocks, cs);
+    efg_status st = e1 == cudaSuccess ? launch_level_end(d, cond, cs) : EFG_ECUDA;
+    cudaGraph_t captured;
+    cudaError_t e2 = cudaStreamEndCapture(cs, &captured);
+    cudaStreamDestroy(cs);
+    if (e1 != cudaSuccess || st != EFG_OK || e2 != cudaSuccess) {
+        cudaGraphDestroy(g);
+        return set_error(EFG_ECUDA, std::string("loop graph capture failed: ") +
+                                        cudaGetErrorString(e1 != cudaSuccess ? e1 : e2));
+    }
+    cudaGraphExec_t exec;
+    CUDA_TRY(cudaGraphInstantiate(&exec, g, 0));
+    d.loop_graph[mode] = g;
+    d.loop_exec[mode] = exec;
+    return EFG_OK;
+}
+
+}  // namespace
+
+void device_free(DeviceGraph &d)
+{
+    if (d.device >= 0) cudaSetDevice(d.device);
+    for (int m = 0; m < 2; ++m) {
+        if (d.loop_exec[m]) cudaGraphExecDestroy(d.loop_exec[m]);
+        if (d.loop_graph[m]) cudaGraphDestroy(d.loop_graph[m]);
+    }
+    cudaFree(d.data);
+    cudaFree(d.rec);
+    cudaFree(d.deg32);
+    cudaFree(d.vlist);
+    cudaFree(d.weights);
+    cudaFree(d.vis);
+    cudaFree(d.prev);
+    cudaFree(d.queue);
+    cudaFree(d.tiles);
+    cudaFree(d.depth);
+    cudaFree(d.parent);
+    cudaFree(d.status);
+    cudaFree(d.stats);
+    cudaFree(d.ctrl);
+    cudaFree(d.fbuf);
+    cudaFree(d.dbuf);
+    if (d.ctrl_host) cudaFreeHost(d.ctrl_host);
+    if (d.stats_host) cudaFreeHost(d.stats_host);
+    d = DeviceGraph{};
+}
+
+efg_status device_upload(efg_graph *g, const efg_build_opts &o)
+{
+    DeviceGraph &d = g->dev;
+    const HostEFG &h = g->host;
+    CUDA_TRY(cudaSetDevice(o.device));
+    d.device = o.device;
+    d.stream = o.stream;
+    d.n = h.n;
+    d.k = h.k;
+    cudaStream_t s = stream_of(d);
+    cudaDeviceProp prop;
+    CUDA_TRY(cudaGetDeviceProperties(&prop, o.device));
+    d.num_sms = prop.multiProcessorCount;
+
+    // EF data, padded so 32-bit word reads past the last list stay in bounds
+    d.data_bytes = h.data.size();
+    const uint64_t padded = ((d.data_bytes + 64) + 15) & ~15ull;
+    EFG_TRY(dev_alloc(d, &d.data, padded));
+    CUDA_TRY(cudaMemsetAsync(d.data, 0, padded, s));
+    if (d.data_bytes) CUDA_TRY(cudaMemcpyAsync(d.data, h.data.data(), d.data_bytes, cudaMemcpyHostToDevice, s));
+
+    // bitmap geometry
+    const uint64_t words = (h.n + 31) / 32;
+    d.nwords = (words + kBitmapAlign - 1) / kBitmapAlign * kBitmapAlign;
+
+    // packed vertex records (one 16-byte load per frontier vertex) and degrees
+    std::vector<VRec> rec(h.n);
+    std::vector<uint32_t> deg(d.nwords * 32, 0);
+#pragma omp parallel for schedule(static)
+    for (int64_t v = 0; v < (int64_t)h.n; ++v) {
+        const uint64_t dv = h.vlist[v + 1] - h.vlist[v];
+        const uint32_t l = h.nlb[v];
+        const uint64_t size = h.offsets[v + 1] - h.offsets[v];
+        const uint64_t fwd = h.k ? 4 * (dv / h.k) : 0;
+        const uint64_t lower = (dv * l + 7) / 8;
+        VRec r;
+        r.off_l = (h.offsets[v] & kOffMask) | ((uint64_t)l << kOffBits);
+        r.deg = (uint32_t)dv;
+        r.ubytes = (uint32_t)(dv ? size - fwd - lower : 0);
+        rec[v] = r;
+        deg[v] = (uint32_t)dv;
+    }
+    EFG_TRY(dev_alloc(d, &d.rec, h.n));
+    CUDA_TRY(cudaMemcpyAsync(d.rec, rec.data(), h.n * sizeof(VRec), cudaMemcpyHostToDevice, s));
+    EFG_TRY(dev_alloc(d, &d.deg32, d.nwords * 32));
+    CUDA_TRY(cudaMemcpyAsync(d.deg32, deg.data(), d.nwords * 32 * 4, cudaMemcpyHostToDevice, s));
+    EFG_TRY(dev_alloc(d, &d.vlist, h.n + 1));
+    CUDA_TRY(cudaMemcpyAsync(d.vlist, h.vlist.data(), (h.n + 1) * 8, cudaMemcpyHostToDevice, s));
+    if (!h.weights.empty()) {
+        EFG_TRY(dev_alloc(d, &d.weights, h.m));
+        CUDA_TRY(cudaMemcpyAsync(d.weights, h.weights.data(), h.m * 4, cudaMemcpyHostToDevice, s));
+    }
+
+    // traversal workspace
+    EFG_TRY(dev_alloc(d, &d.vis, d.nwords));
+    EFG_TRY(dev_alloc(d, &d.prev, d.nwords));
+    EFG_TRY(dev_alloc(d, &d.queue, h.n));
+    d.max_tiles = (h.m + (uint64_t)kVertexWork * h.n) / kTileWork + 2;
+    EFG_TRY(dev_alloc(d, &d.tiles, d.max_tiles));
+    EFG_TRY(dev_alloc(d, &d.depth, h.n));
+    EFG_TRY(dev_alloc(d, &d.status, 2 * kMaxGrid));
+    CUDA_TRY(cudaMemsetAsync(d.status, 0, 2 * kMaxGrid * 8, s));
+    EFG_TRY(dev_alloc(d, &d.stats, kMaxLevelStats));
+    EFG_TRY(dev_alloc(d, &d.ctrl, 1));
+    CUDA_TRY(cudaMemsetAsync(d.ctrl, 0, sizeof(LevelCtrl), s));
+    CUDA_TRY(cudaMallocHost(reinterpret_cast<void **>(&d.ctrl_host), sizeof(LevelCtrl)));
+    CUDA_TRY(cudaMallocHost(reinterpret_cast<void **>(&d.stats_host), kMaxLevelStats * sizeof(LevelStat)));
+    // persistent grids of the frontier kernels: 2 blocks per SM, whole bitmap words
+    d.frontier_blocks = (unsigned)std::min<uint64_t>(2 * (uint64_t)d.num_sms, kMaxGrid);
+    const uint64_t per = (d.nwords + d.frontier_blocks - 1) / d.frontier_blocks;
+    d.words_per_block = (per + kFrontierThreads - 1) / kFrontierThreads * kFrontierThreads;
+    CUDA_TRY(cudaStreamSynchronize(s));
+    return EFG_OK;
+}
+
+// Start a traversal: reset the bitmaps, mark [v0, v1), run the level-0 frontier
+// kernels.  depth: device buffer receiving the level numbers.
+static efg_status start_traversal(DeviceGraph &d, uint64_t v0, uint64_t v1, int32_t *depth,
+                                  uint32_t *parent, uint32_t &launches)
+{
+    cudaStream_t s = stream_of(d);
+    CUDA_TRY(cudaMemsetAsync(d.vis, 0, d.nwords * 4, s));
+    CUDA_TRY(cudaMemsetAsync(d.prev, 0, d.nwords * 4, s));
+    InitArgs ia;
+    ia.ctrl = d.ctrl;
+    ia.vis = d.vis;
+    ia.depth = depth;
+    ia.parent = parent;
+    ia.v0 = v0;
+    ia.v1 = v1;
+    CUDA_TRY(launch_init(ia, s));
+    EFG_TRY(launch_level_end(d, 0, s));
+    launches += 3;
+    return EFG_OK;
+}
+
+efg_status device_decode(efg_graph *g, uint32_t v0, uint32_t v1, uint32_t *out)
+{
+    const HostEFG &h = g->host;
+    DeviceGraph &d = g->dev;
+    const uint64_t cnt = h.vlist[v1] - h.vlist[v0];
+    CUDA_TRY(cudaSetDevice(d.device));
+    cudaStream_t s = stream_of(d);
+    const bool out_dev = is_device_ptr(out);
+    uint32_t *od = out;
+    if (!out_dev) EFG_TRY(dev_alloc(d, &od, cnt));
+    efg_status st = EFG_OK;
+    uint32_t launches = 0;
+    do {
+        if ((st = start_traversal(d, v0, v1, d.depth, nullptr, launches)) != EFG_OK) break;
+        const int blocks = d.num_sms * expand_occupancy(kModeDecode);
+        cudaError_t e = launch_expand(kModeDecode, expand_args(d, od), blocks, s);
+        if (e == cudaSuccess && !out_dev) e = cudaMemcpyAsync(out, od, cnt * 4, cudaMemcpyDeviceToHost, s);
+        if (e == cudaSuccess) e = cudaStreamSynchronize(s);
+        if (e != cudaSuccess) st = set_error(EFG_ECUDA, std::string("efg_decode: ") + cudaGetErrorString(e));
+    } while (0);
+    if (!out_dev) {
+        cudaFree(od);
+        d.device_bytes -= std::max<uint64_t>(cnt, 1) * 4;
+    }
+    return st;
+}
+
+efg_status device_bfs(efg_graph *g, uint32_t source, int32_t *depth, uint32_t *parent, efg_stats *st)
+{
+    DeviceGraph &d = g->dev;
+    CUDA_TRY(cudaSetDevice(d.device));
+    cudaStream_t s = stream_of(d);
+    const bool depth_dev = is_device_ptr(depth);
+    int32_t *dd = depth_dev ? depth : d.depth;
+    uint32_t *pd = nullptr;
+    bool parent_dev = false;
+    if (parent) {
+        parent_dev = is_device_ptr(parent);
+        if (!parent_dev && !d.parent) EFG_TRY(dev_alloc(d, &d.parent, d.n));
+        pd = parent_dev ? parent : d.parent;
+    }
+    const int mode = parent ? kModeVisitParent : kModeVisit;
+    const bool graph_mode = d.level_loop == 0;
+    if (graph_mode) EFG_TRY(build_loop_graph(d, mode));
+
+    cudaEvent_t ev0, ev1;
+    CUDA_TRY(cudaEventCreate(&ev0));
+    CUDA_TRY(cudaEventCreate(&ev1));
+    std::vector<cudaEvent_t> lev;  // host mode: expand start/stop pairs
+    uint32_t launches = 0;
+
+    CUDA_TRY(cudaEventRecord(ev0, s));
+    CUDA_TRY(cudaMemsetAsync(dd, 0xFF, d.n * 4, s));
+    if (pd) CUDA_TRY(cudaMemsetAsync(pd, 0xFF, d.n * 4, s));
+    EFG_TRY(start_traversal(d, source, (uint64_t)source + 1, dd, pd, launches));
+
+    std::vector<uint64_t> lf, le;
+    std::vector<float> lms;
+    uint32_t levels = 0;
+    if (graph_mode) {
+        CUDA_TRY(cudaGraphLaunch(d.loop_exec[mode], s));
+        CUDA_TRY(cudaEventRecord(ev1, s));
+        CUDA_TRY(cudaMemcpyAsync(d.ctrl_host, d.ctrl, sizeof(LevelCtrl), cudaMemcpyDeviceToHost, s));
+        CUDA_TRY(cudaStreamSynchronize(s));
+        levels = d.ctrl_host->nlevels;
+        const uint32_t ns = std::min(levels, kMaxLevelStats);
+        if (ns) {
+            CUDA_TRY(cudaMemcpyAsync(d.stats_host, d.stats, ns * sizeof(LevelStat), cudaMemcpyDeviceToHost, s));
+            CUDA_TRY(cudaStreamSynchronize(s));
+        }
+        for (uint32_t i = 0; i < ns; ++i) {
+            lf.push_back(d.stats_host[i].nf);
+            le.push_back(d.stats_host[i].ne);
+            const LevelStat &x = d.stats_host[i];
+            lms.push_back(x.t1 > x.t0 ? (float)((double)(x.t1 - x.t0) * 1e-6) : 0.f);
+        }
+        launches += 3 * levels;
+    } else {
+        const int blocks = d.num_sms * expand_occupancy(mode);
+        for (;;) {
+            CUDA_TRY(cudaMemcpyAsync(d.ctrl_host, d.ctrl, sizeof(LevelCtrl), cudaMemcpyDeviceToHost, s));
+            CUDA_TRY(cudaStreamSynchronize(s));
+            const LevelCtrl c = *d.ctrl_host;
+            if (c.nf == 0) break;
+            lf.push_back(c.nf);
+            le.push_back(c.ne);
+            cudaEvent_t a, b;
+            CUDA_TRY(cudaEventCreate(&a));
+            CUDA_TRY(cudaEventCreate(&b));
+            lev.push_back(a);
+            lev.push_back(b);
+            CUDA_TRY(cudaEventRecord(a, s));
+            CUDA_TRY(launch_expand(mode, expand_args(d, nullptr), blocks, s));
+            CUDA_TRY(cudaEventRecord(b, s));
+            EFG_TRY(launch_level_end(d, 0, s));
+            launches += 3;
+            ++levels;
+        }
+        CUDA_TRY(cudaEventRecord(ev1, s));
+    }
+    if (!depth_dev) CUDA_TRY(cudaMemcpyAsync(depth, dd, d.n * 4, cudaMemcpyDeviceToHost, s));
+    if (parent && !parent_dev) CUDA_TRY(cudaMemcpyAsync(parent, pd, d.n * 4, cudaMemcpyDeviceToHost, s));
+    CUDA_TRY(cudaStreamSynchronize(s));
+
+    float total_ms = 0.f;
+    cudaEventElapsedTime(&total_ms, ev0, ev1);
+    if (!graph_mode) {
+        lms.assign(levels, 0.f);
+        for (uint32_t i = 0; i < levels; ++i) cudaEventElapsedTime(&lms[i], lev[2 * i], lev[2 * i + 1]);
+    }
+    for (auto e : lev) cudaEventDestroy(e);
+    cudaEventDestroy(ev0);
+    cudaEventDestroy(ev1);
+    if (st) {
+        uint64_t edges = 0, reached = 0;
+        float exp_ms = 0.f;
+        for (size_t i = 0; i < lf.size(); ++i) {
+            reached += lf[i];
+            edges += le[i];
+            exp_ms += lms[i];
+        }
+        if (graph_mode) {  // exact even past kMaxLevelStats levels
+            reached = d.ctrl_host->total_nf;
+            edges = d.ctrl_host->total_ne;
+        }
+        st->levels = levels;
+        st->edges_traversed = edges;
+        st->vertices_reached = reached;
+        st->device_ms = total_ms;
+        st->expand_ms = exp_ms;
+        st->expand_launches = levels;
+        st->kernel_launches = launches;
+        st->expand_bytes = 0;
+        for (uint32_t i = 0; i < std::min<uint32_t>((uint32_t)lf.size(), st->level_cap); ++i) {
+            if (st->level_frontier) st->level_frontier[i] = lf[i];
+            if (st->level_edges) st->level_edges[i] = le[i];
+            if (st->level_expand_ms) st->level_expand_ms[i] = lms[i];
+        }
+    }
+    return EFG_OK;
+}
+
+}  // namespace efg

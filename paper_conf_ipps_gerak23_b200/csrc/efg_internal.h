@@ -8,6 +8,8 @@
 #include <string>
 #include <vector>
 
+#include <cuda_runtime.h>
+
 #include "efg.h"
 
 namespace efg {
@@ -73,17 +75,33 @@ struct LevelCtrl {
     uint64_t ne;        // edges out of that frontier (E_L)
     uint64_t ntiles;    // ceil(nwork / kTileWork)
     uint64_t nwork;     // work units = ne + kVertexWork * nf
+    int32_t *depth;     // depth buffer of the current call
+    uint32_t *parent;   // parent buffer of the current call, or null
+    uint32_t level;     // depth assigned by the next compact
+    uint32_t xlevel;    // index of the level the next expand processes
+    uint32_t seq;       // tag of the cross-block prefix words of this level
+    uint32_t nlevels;   // levels expanded so far
+    uint64_t total_nf;  // sum of frontier sizes (= vertices reached)
+    uint64_t total_ne;  // sum of E_L (= edges traversed, reading C18)
 };
 
+// Per-level statistics written on the device (graph mode has no host loop).
+struct LevelStat {
+    uint64_t nf, ne;                 // frontier size and its edges
+    unsigned long long t0, t1;       // expand kernel start / end (%globaltimer, ns)
+};
+constexpr uint32_t kMaxLevelStats = 4096;
+
 constexpr int kExpandThreads = 128;          // 4 warps (static smem < 48 KB)
-constexpr int kAdvanceThreads = 256;         // 8 warps
-constexpr int kAdvanceRounds = 4;            // runs of 32 words per warp
-constexpr int kAdvanceWords = kAdvanceThreads * kAdvanceRounds;  // bitmap words per block
+constexpr int kFrontierThreads = 256;        // compact / plan kernels
+constexpr int kBitmapAlign = 1024;           // bitmap words are padded to a multiple of this
 // Step a3 partitions "work units" rather than bare edges: a frontier vertex
 // costs kVertexWork units (its record gather and list set-up) plus one per edge,
 // so a tile of kTileWork units holds at most kTileWork/kVertexWork short lists.
 constexpr uint32_t kTileWork = 2048;         // work units per warp tile (a3)
 constexpr uint32_t kVertexWork = 32;         // per-vertex overhead in work units
+
+constexpr unsigned kMaxGrid = 4096;
 
 struct DeviceGraph {
     int device = -1;
@@ -104,15 +122,20 @@ struct DeviceGraph {
     uint64_t max_tiles = 0;
     int32_t *depth = nullptr;          // internal depth (n)
     uint32_t *parent = nullptr;        // internal parent (n), lazily allocated
-    uint64_t *status = nullptr;        // decoupled look-back status, 2 parities x 2 values x nblk
-    uint64_t status_blocks = 0;
+    uint64_t *status = nullptr;        // cross-block prefix words: compact [kMaxGrid], plan [kMaxGrid]
+    LevelStat *stats = nullptr;        // per-level statistics (kMaxLevelStats)
+    unsigned frontier_blocks = 0;      // grid of compact / plan
+    uint64_t words_per_block = 0;
     LevelCtrl *ctrl = nullptr;         // device control block
     LevelCtrl *ctrl_host = nullptr;    // pinned mirror
     float *fbuf = nullptr;             // SSSP distance (n) lazily
     double *dbuf = nullptr;            // PageRank buffers lazily (3n)
     uint64_t device_bytes = 0;
     int num_sms = 148;
-    int expand_blocks = 0;             // persistent grid size
+    LevelStat *stats_host = nullptr;   // pinned mirror of stats
+    int level_loop = 0;                // 0 = CUDA graph (device loop), 1 = host loop + events
+    cudaGraph_t loop_graph[2] = {nullptr, nullptr};      // per mode (visit, visit+parent)
+    cudaGraphExec_t loop_exec[2] = {nullptr, nullptr};
 };
 
 }  // namespace efg
@@ -122,6 +145,14 @@ struct efg_graph {
     efg::DeviceGraph dev;
     bool on_device = false;
 };
+
+// device side (efg_device.cu)
+namespace efg {
+efg_status device_upload(efg_graph *g, const efg_build_opts &o);
+void device_free(DeviceGraph &d);
+efg_status device_decode(efg_graph *g, uint32_t v0, uint32_t v1, uint32_t *out);
+efg_status device_bfs(efg_graph *g, uint32_t source, int32_t *depth, uint32_t *parent, efg_stats *st);
+}  // namespace efg
 
 // error handling (efg_error.cpp)
 namespace efg {

@@ -1,12 +1,13 @@
 // efg_kernels.cu — hand-written sm_100a kernels of the EFG BFS hot path.
 //
-// Steps and where they live:
-//   a7 level end + a1 frontier materialisation/degree lookup + a2 exclusive scan
-//      + a3 load-balanced partition  -> advance_kernel (one pass over the
-//      visited bitmap; single-pass decoupled look-back scan; writes the sorted
-//      next-frontier queue and the edge-tile table)
+// Steps and where they live, per BFS level:
 //   a4 locate compressed bit ranges + a5 EF element decode + a6 visit
-//      -> expand_kernel (persistent, warp per edge tile)
+//      -> expand_kernel (persistent, warp per work tile)
+//   a7 level end: visited-bitmap diff -> sorted next frontier queue + depth
+//      -> compact_kernel (reduce-then-scan over the bitmap)
+//   a1 degree lookup + a2 exclusive scan of per-vertex work + a3 partition
+//      into tiles -> plan_kernel (reduce-then-scan over the queue)
+// init_kernel starts a traversal (source bit, per-call state).
 //
 // Paper anchors: Alg. 1 (§III-B), scans/searches (§III-C),
 // load-balanced partitioning (§VI-A, Fig. 4), single/partial/multi-list
@@ -31,6 +32,13 @@ constexpr int kWarps = kExpandThreads / 32;
 // warp / block primitives (§III-C: exclusive scan, bounded search)
 // --------------------------------------------------------------------------
 __device__ __forceinline__ uint32_t lane_id() { return threadIdx.x & 31; }
+
+__device__ __forceinline__ unsigned long long globaltimer()
+{
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    return t;
+}
 
 __device__ __forceinline__ uint32_t warp_excl_u32(uint32_t x, uint32_t &total)
 {
@@ -89,21 +97,8 @@ __device__ __forceinline__ uint32_t ld_u32_unaligned(const uint32_t *data32, uin
     return __funnelshift_r(lo, hi, (uint32_t)(byteoff & 3) * 8);
 }
 
-__device__ __forceinline__ void st_release_u64(uint64_t *p, uint64_t v)
-{
-    asm volatile("st.release.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
-}
 
-__device__ __forceinline__ uint64_t ld_acquire_u64(const uint64_t *p)
-{
-    uint64_t v;
-    asm volatile("ld.acquire.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
-    return v;
-}
 
-constexpr uint64_t kFlagAgg = 1ull << 62;
-constexpr uint64_t kFlagIncl = 2ull << 62;
-constexpr uint64_t kValMask = (1ull << 62) - 1;
 
 // Chunk length CH = k (forward-pointer quantum), or 2^40 when k = 0 (lists are
 // never split).  Divisions by CH use a shift when k is a power of two (the
@@ -122,71 +117,6 @@ __device__ __forceinline__ ChunkLen make_chunk(uint32_t k, int kshift)
     return c;
 }
 
-// Cross-block exclusive prefix for the advance scan (a2).  Every block
-// publishes its aggregate pair (frontier count, work) as two 64-bit words
-// flag | value (same flag in both, so no fence is needed: each value travels in
-// the same single-copy-atomic word as its flag).  A block then sums the
-// aggregates of ALL its predecessors directly, 32 lanes x several independent
-// loads per step: latency is a couple of L2 round trips regardless of the block
-// index, instead of a look-back chain that grows with the grid when every
-// block is resident at once.
-__device__ __forceinline__ uint64_t ld_relaxed_u64(const uint64_t *p)
-{
-    uint64_t v;
-    asm volatile("ld.relaxed.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
-    return v;
-}
-
-__device__ __forceinline__ void st_relaxed_u64(uint64_t *p, uint64_t v)
-{
-    asm volatile("st.relaxed.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
-}
-
-__device__ void prefix_of_block(const uint64_t *st, uint64_t b, uint64_t &ex_c, uint64_t &ex_w)
-{
-    const uint32_t lane = lane_id();
-    uint64_t c_acc = 0, w_acc = 0;
-    for (uint64_t base = 0; base < b; base += 32 * 4) {
-        uint64_t c[4], w[4];
-#pragma unroll
-        for (int u = 0; u < 4; ++u) {
-            const uint64_t idx = base + u * 32 + lane;
-            c[u] = kFlagAgg;
-            w[u] = kFlagAgg;
-            if (idx < b) {
-                c[u] = ld_relaxed_u64(st + 2 * idx);
-                w[u] = ld_relaxed_u64(st + 2 * idx + 1);
-            }
-        }
-#pragma unroll
-        for (int u = 0; u < 4; ++u) {
-            const uint64_t idx = base + u * 32 + lane;
-            while (idx < b && ((c[u] >> 62) == 0 || (w[u] >> 62) == 0)) {
-                c[u] = ld_relaxed_u64(st + 2 * idx);
-                w[u] = ld_relaxed_u64(st + 2 * idx + 1);
-            }
-            c_acc += c[u] & kValMask;
-            w_acc += w[u] & kValMask;
-        }
-    }
-    ex_c = warp_sum_u64(c_acc);
-    ex_w = warp_sum_u64(w_acc);
-}
-
-// --------------------------------------------------------------------------
-// advance_kernel: a7 + a1 + a2 + a3
-//   new = vis & ~prev per 32-vertex word; depth[new] = level; sorted queue of
-//   the new frontier; per-vertex degree (a1) scanned (a2) into work offsets
-//   W_v = sum over earlier frontier vertices of (kVertexWork + deg); tiles of
-//   kTileWork units -> first owned chunk (a3: the Fig. 4 maxle rule applied
-//   once per tile, with boundaries snapped to k-aligned chunk starts).
-//   Vertex v occupies work [W_v, W_v + kVertexWork + deg_v); its chunk 0
-//   starts at W_v, chunk c > 0 at W_v + kVertexWork + c*k.
-//   Layout: a block covers kAdvanceWords bitmap words; thread t owns
-//   kAdvanceRounds consecutive words (one 16-byte load per bitmap).  Degrees
-//   come from the compact deg32 array: a word with many new bits loads its 32
-//   degrees as eight 16-byte loads, a sparse word loads per bit.
-// --------------------------------------------------------------------------
 struct HubItem {
     uint64_t q, w, d;
 };
@@ -234,181 +164,248 @@ __device__ __noinline__ void place_tiles(TileEntry *tiles, uint64_t q, uint64_t 
     write_tiles(tiles, q, W, d, cl, 0, 1);
 }
 
-// exact warp sum of a value < 2^48 with two 32-bit REDUX instructions
-__device__ __forceinline__ uint64_t warp_sum_small(uint64_t x)
+// --------------------------------------------------------------------------
+// Cross-block exclusive prefix for the two frontier scans (a2, a7).  A block
+// publishes its aggregate as one 64-bit word tag << 40 | value (value < 2^40),
+// with tag = the per-launch sequence number, so no clearing pass and no fence
+// are needed (the value travels in the same single-copy-atomic word as its
+// tag).  The block then sums the aggregates of ALL its predecessors with every
+// load issued at once (grids are at most 2 x #SMs blocks), i.e. one or two L2
+// round trips instead of a look-back chain.
+// --------------------------------------------------------------------------
+__device__ __forceinline__ uint64_t ld_relaxed_u64(const uint64_t *p)
 {
-    const uint32_t hi = __reduce_add_sync(FULL, (uint32_t)(x >> 16));
-    const uint32_t lo = __reduce_add_sync(FULL, (uint32_t)(x & 0xffff));
-    return ((uint64_t)hi << 16) + lo;
+    uint64_t v;
+    asm volatile("ld.relaxed.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+    return v;
 }
 
-constexpr int kAdvGroup = 8;  // bitmap words whose degree loads are in flight together
-
-// Pop up to kAdvGroup set bits (word indices) from a warp-uniform mask.
-__device__ __forceinline__ int pop_words(uint32_t &mask, int (&j)[kAdvGroup])
+__device__ __forceinline__ void st_relaxed_u64(uint64_t *p, uint64_t v)
 {
-    int n = 0;
+    asm volatile("st.relaxed.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+
+constexpr int kTagShift = 40;
+constexpr uint64_t kTagVal = (1ull << kTagShift) - 1;
+
+// warp 0: publish `agg` for block b and return the sum over blocks < b
+__device__ uint64_t publish_and_prefix(uint64_t *st, uint32_t b, uint32_t tag, uint64_t agg)
+{
+    const uint32_t lane = lane_id();
+    const uint64_t t = (uint64_t)(tag & 0xffffffu);
+    if (lane == 0) st_relaxed_u64(st + b, (t << kTagShift) | agg);
+    uint64_t acc = 0;
+    for (uint32_t base = 0; base < b; base += 32 * 8) {
+        uint64_t w[8];
 #pragma unroll
-    for (int u = 0; u < kAdvGroup; ++u) {
-        j[u] = 0;
-        if (mask) {
-            j[u] = __ffs(mask) - 1;
-            mask &= mask - 1;
-            n = u + 1;
+        for (int u = 0; u < 8; ++u) {
+            const uint32_t idx = base + u * 32 + lane;
+            w[u] = idx < b ? ld_relaxed_u64(st + idx) : (t << kTagShift);
+        }
+#pragma unroll
+        for (int u = 0; u < 8; ++u) {
+            const uint32_t idx = base + u * 32 + lane;
+            while ((w[u] >> kTagShift) != t) w[u] = ld_relaxed_u64(st + idx);
+            acc += w[u] & kTagVal;
         }
     }
-    return n;
+    return warp_sum_u64(acc);
 }
 
-__global__ void __launch_bounds__(kAdvanceThreads, 3) advance_kernel(AdvanceArgs a)
+// block-wide exclusive scan of a u64 (256 threads); returns the block total in `total`
+template <int NT>
+__device__ __forceinline__ uint64_t block_excl_u64(uint64_t x, uint64_t &total, uint64_t *s_warp)
 {
-    constexpr int NW = kAdvanceThreads / 32;
-    constexpr int R = kAdvanceRounds;
+    const uint32_t lane = lane_id(), wid = threadIdx.x >> 5;
+    uint64_t wt;
+    const uint64_t ex = warp_excl_u64(x, wt);
+    if (lane == 31) s_warp[wid] = wt;
+    __syncthreads();
+    uint64_t pre = 0, tot = 0;
+#pragma unroll
+    for (int w = 0; w < NT / 32; ++w) {
+        const uint64_t v = s_warp[w];
+        if (w < (int)wid) pre += v;
+        tot += v;
+    }
+    __syncthreads();
+    total = tot;
+    return pre + ex;
+}
+
+__device__ __forceinline__ uint64_t block_sum_u64(uint64_t x, uint64_t *s_warp)
+{
+    uint64_t tot;
+    block_excl_u64<kFrontierThreads>(x, tot, s_warp);
+    return tot;
+}
+
+// --------------------------------------------------------------------------
+// init_kernel: per-call state (level 0, a fresh tag) and the start set:
+// BFS marks the source (Alg. 1 initial frontier), decode marks [v0, v1).
+// --------------------------------------------------------------------------
+__global__ void init_kernel(InitArgs a)
+{
+    if (blockIdx.x == 0 && threadIdx.x == 0) {
+        a.ctrl->depth = a.depth;
+        a.ctrl->parent = a.parent;
+        a.ctrl->level = 0;
+        a.ctrl->xlevel = 0;
+        a.ctrl->seq = a.ctrl->seq + 1;
+        a.ctrl->nlevels = 0;
+        a.ctrl->total_nf = 0;
+        a.ctrl->total_ne = 0;
+        if (a.parent) a.parent[a.v0] = (uint32_t)a.v0;
+    }
+    const uint64_t w0 = a.v0 >> 5, w1 = (a.v1 + 31) >> 5;
+    for (uint64_t w = w0 + blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; w < w1;
+         w += (uint64_t)gridDim.x * blockDim.x) {
+        uint32_t m = FULL;
+        if (w == (a.v0 >> 5)) m &= FULL << (a.v0 & 31);
+        if (w == ((a.v1 - 1) >> 5) && (a.v1 & 31)) m &= (1u << (a.v1 & 31)) - 1;
+        a.vis[w] |= m;
+    }
+}
+
+// --------------------------------------------------------------------------
+// compact_kernel: a7 level end.  new = vis & ~prev; the new vertices, in
+// increasing id order, become the next frontier queue (sorted for free, in
+// place of the paper's partial radix sort); depth[new] = level.
+// Reduce-then-scan over a persistent grid: pass 1 counts the block's word
+// range, the cross-block prefix places it, pass 2 re-reads the range 256 words
+// at a time, stages the new ids in shared memory and writes them coalesced.
+// --------------------------------------------------------------------------
+__global__ void __launch_bounds__(kFrontierThreads) compact_kernel(CompactArgs a)
+{
+    constexpr int NT = kFrontierThreads;
+    __shared__ uint64_t s_warp[NT / 32];
+    __shared__ uint64_t s_pre;
+    __shared__ uint32_t s_ids[NT * 32];
+
+    const uint32_t tid = threadIdx.x, b = blockIdx.x;
+    const LevelCtrl *ctrl = a.ctrl;
+    const uint32_t tag = ctrl->seq;
+    const int32_t level = (int32_t)ctrl->level;
+    int32_t *depth = ctrl->depth;
+    const uint64_t lo = (uint64_t)b * a.words_per_block;
+    const uint64_t hi = min(lo + a.words_per_block, a.nwords);
+
+    // pass 1: count
+    uint64_t cnt = 0;
+    for (uint64_t w = lo + tid; w < hi; w += NT) cnt += __popc(a.vis[w] & ~a.prev[w]);
+    const uint64_t blk = block_sum_u64(cnt, s_warp);
+    if (tid < 32) {
+        const uint64_t pre = publish_and_prefix(a.status, b, tag, blk);
+        if (tid == 0) {
+            s_pre = pre;
+            if (b == gridDim.x - 1) a.ctrl->nf = pre + blk;
+        }
+    }
+    __syncthreads();
+
+    // pass 2: queue + depth, 256 words per step
+    uint64_t base = s_pre;
+    for (uint64_t c0 = lo; c0 < hi; c0 += NT) {
+        const uint64_t w = c0 + tid;
+        uint32_t nb = 0;
+        if (w < hi) {
+            const uint32_t x = a.vis[w], p = a.prev[w];
+            nb = x & ~p;
+            if (nb) a.prev[w] = x;
+        }
+        uint64_t tot;
+        const uint64_t ex = block_excl_u64<NT>(__popc(nb), tot, s_warp);
+        uint32_t k = (uint32_t)ex;
+        for (uint32_t t = nb; t; t &= t - 1) s_ids[k++] = (uint32_t)(w * 32 + (__ffs(t) - 1));
+        __syncthreads();
+        for (uint32_t i = tid; i < tot; i += NT) {
+            const uint32_t v = s_ids[i];
+            a.queue[base + i] = v;
+            depth[v] = level;
+        }
+        base += tot;
+        __syncthreads();
+    }
+}
+
+// --------------------------------------------------------------------------
+// plan_kernel: a1 + a2 + a3.  For the sorted frontier queue: degree lookup
+// (a1), exclusive scan of the per-vertex work kVertexWork + deg (a2), and the
+// tile table (a3: each tile of kTileWork units gets its first chunk, the
+// Fig. 4 maxle rule applied once per tile).  Same reduce-then-scan scheme as
+// compact_kernel, over the frontier index range.  The last block publishes
+// the level totals, records per-level statistics and, in graph mode, sets the
+// loop condition (frontier non-empty).
+// --------------------------------------------------------------------------
+__global__ void __launch_bounds__(kFrontierThreads) plan_kernel(PlanArgs a)
+{
+    constexpr int NT = kFrontierThreads;
     constexpr int kHubCap = 256;
-    __shared__ uint32_t s_wcnt[NW];
-    __shared__ uint64_t s_wwork[NW];
-    __shared__ uint64_t s_block_q, s_block_w;
+    __shared__ uint64_t s_warp[NT / 32];
+    __shared__ uint64_t s_pre;
     __shared__ HubItem s_hub[kHubCap];
     __shared__ uint32_t s_nhub;
 
-    const uint32_t tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
-    const uint64_t b = blockIdx.x;
+    const uint32_t tid = threadIdx.x, b = blockIdx.x;
+    LevelCtrl *ctrl = a.ctrl;
+    const uint32_t tag = ctrl->seq;
+    const uint64_t nf = ctrl->nf;
     const ChunkLen cl = make_chunk(a.k, a.kshift);
     const uint64_t A = kVertexWork;
-    const uint32_t lt = (1u << lane) - 1;
-    // words of (warp, round r): rbase(r) + 0..31, lane j owns word rbase(r) + j
-    const uint64_t wbase = b * (uint64_t)kAdvanceWords + (uint64_t)wid * 32 * R;
-
+    const uint64_t per = (nf + gridDim.x - 1) / gridDim.x;
+    const uint64_t lo = min((uint64_t)b * per, nf), hi = min(lo + per, nf);
     if (tid == 0) s_nhub = 0;
 
-    // ---- pass 1: new bits (a7), depth, per-word (count, work) via a1 ----
-    uint32_t nb[R], wc[R];
-    uint64_t ww[R];
-#pragma unroll
-    for (int r = 0; r < R; ++r) {
-        const uint64_t rb = wbase + (uint64_t)r * 32;
-        const uint32_t x = a.vis[rb + lane], p = a.prev[rb + lane];
-        nb[r] = x & ~p;
-        if (nb[r]) a.prev[rb + lane] = x;
-        wc[r] = __popc(nb[r]);
-        ww[r] = 0;
-        uint32_t mask = __ballot_sync(FULL, nb[r] != 0);
-        while (mask) {
-            int j[kAdvGroup];
-            pop_words(mask, j);
-            uint32_t d[kAdvGroup], nbw[kAdvGroup];
-#pragma unroll
-            for (int u = 0; u < kAdvGroup; ++u) {
-                nbw[u] = __shfl_sync(FULL, nb[r], j[u]);
-                // lanes past the popped words see j = 0 duplicates: drop them
-                if (u > 0 && j[u] == 0) nbw[u] = 0;
-                d[u] = (nbw[u] >> lane & 1) ? __ldg(a.deg32 + (rb + j[u]) * 32 + lane) : 0;
-            }
-#pragma unroll
-            for (int u = 0; u < kAdvGroup; ++u) {
-                const bool bit = nbw[u] >> lane & 1;
-                if (bit) a.depth[(rb + j[u]) * 32 + lane] = a.depth_value;
-                const uint64_t s = warp_sum_small(bit ? A + d[u] : 0);
-                if (nbw[u] && (int)lane == j[u]) ww[r] = s;
-            }
-        }
-    }
-    // warp totals -> block scan
-    uint64_t tot_c = 0, tot_w = 0;
-#pragma unroll
-    for (int r = 0; r < R; ++r) {
-        tot_c += __reduce_add_sync(FULL, wc[r]);
-        tot_w += warp_sum_small(ww[r]);
-    }
-    if (lane == 0) {
-        s_wcnt[wid] = (uint32_t)tot_c;
-        s_wwork[wid] = tot_w;
-    }
-    __syncthreads();
-    uint64_t pre_c = 0, pre_w = 0, blk_c = 0, blk_w = 0;
-#pragma unroll
-    for (int w = 0; w < NW; ++w) {
-        if (w < (int)wid) {
-            pre_c += s_wcnt[w];
-            pre_w += s_wwork[w];
-        }
-        blk_c += s_wcnt[w];
-        blk_w += s_wwork[w];
-    }
-
-    // ---- a2 across blocks ----
-    uint64_t *st = a.status + (uint64_t)a.parity * 2 * a.nblocks;
-    if (wid == 0) {
-        if (lane == 0) {
-            // clear this block's slots of the other parity for the next launch
-            uint64_t *other = a.status + (uint64_t)(a.parity ^ 1) * 2 * a.nblocks;
-            other[2 * b] = 0;
-            other[2 * b + 1] = 0;
-            st_relaxed_u64(st + 2 * b, kFlagAgg | blk_c);
-            st_relaxed_u64(st + 2 * b + 1, kFlagAgg | blk_w);
-        }
-        uint64_t bq, bw;
-        prefix_of_block(st, b, bq, bw);
-        if (lane == 0) {
-            s_block_q = bq;
-            s_block_w = bw;
-            if (b == a.nblocks - 1) {
-                const uint64_t nf = bq + blk_c, nwork = bw + blk_w;
-                a.ctrl->nf = nf;
-                a.ctrl->nwork = nwork;
-                a.ctrl->ne = nwork - A * nf;
-                a.ctrl->ntiles = (nwork + kTileWork - 1) / kTileWork;
-            }
-        }
-    }
-    __syncthreads();
-
-    // ---- pass 2: sorted queue (a7) + tile table (a3) ----
-    uint64_t run_c = s_block_q + pre_c, run_w = s_block_w + pre_w;
-#pragma unroll
-    for (int r = 0; r < R; ++r) {
-        const uint64_t rb = wbase + (uint64_t)r * 32;
-        uint32_t tc;
-        uint64_t tw;
-        const uint64_t wq = run_c + warp_excl_u32(wc[r], tc);
-        const uint64_t wwp = run_w + warp_excl_u64(ww[r], tw);
-        run_c += tc;
-        run_w += tw;
-        uint32_t mask = __ballot_sync(FULL, nb[r] != 0);
-        while (mask) {
-            int j[kAdvGroup];
-            pop_words(mask, j);
-            uint32_t d[kAdvGroup], nbw[kAdvGroup];
-#pragma unroll
-            for (int u = 0; u < kAdvGroup; ++u) {
-                nbw[u] = __shfl_sync(FULL, nb[r], j[u]);
-                if (u > 0 && j[u] == 0) nbw[u] = 0;
-                d[u] = (nbw[u] >> lane & 1) ? __ldg(a.deg32 + (rb + j[u]) * 32 + lane) : 0;
-            }
-#pragma unroll
-            for (int u = 0; u < kAdvGroup; ++u) {
-                const bool bit = nbw[u] >> lane & 1;
-                const uint64_t q0 = __shfl_sync(FULL, wq, j[u]);
-                const uint64_t w0 = __shfl_sync(FULL, wwp, j[u]);
-                uint64_t dummy;
-                const uint64_t wex = warp_excl_u64(bit ? A + d[u] : 0, dummy);
-                if (bit) {
-                    const uint64_t q = q0 + __popc(nbw[u] & lt);
-                    const uint64_t W = w0 + wex;
-                    a.queue[q] = (uint32_t)((rb + j[u]) * 32 + lane);
-                    // does a tile boundary fall inside [W, W + A + d)?
-                    if (((W + kTileWork - 1) & ~(uint64_t)(kTileWork - 1)) < W + A + d[u])
-                        place_tiles(a.tiles, q, W, d[u], cl, s_hub, &s_nhub, kHubCap);
+    // pass 1: work of the block's range
+    uint64_t wk = 0;
+    for (uint64_t i = lo + tid; i < hi; i += NT) wk += A + __ldg(a.deg32 + a.queue[i]);
+    const uint64_t blk = block_sum_u64(wk, s_warp);
+    if (tid < 32) {
+        const uint64_t pre = publish_and_prefix(a.status, b, tag, blk);
+        if (tid == 0) {
+            s_pre = pre;
+            if (b == gridDim.x - 1) {
+                const uint64_t nwork = pre + blk;
+                const uint32_t lvl = ctrl->level;
+                ctrl->nwork = nwork;
+                ctrl->ne = nwork - A * nf;
+                ctrl->ntiles = (nwork + kTileWork - 1) / kTileWork;
+                ctrl->xlevel = lvl;
+                if (nf) {
+                    ctrl->nlevels = lvl + 1;
+                    ctrl->total_nf += nf;
+                    ctrl->total_ne += nwork - A * nf;
+                    if (a.stats && lvl < a.max_stats) {
+                        a.stats[lvl].nf = nf;
+                        a.stats[lvl].ne = nwork - A * nf;
+                        a.stats[lvl].t0 = ~0ull;
+                        a.stats[lvl].t1 = 0;
+                    }
                 }
+                if (a.cond) cudaGraphSetConditional(a.cond, nf ? 1u : 0u);
             }
         }
+    }
+    __syncthreads();
+
+    // pass 2: tiles
+    uint64_t run = s_pre;
+    for (uint64_t c0 = lo; c0 < hi; c0 += NT) {
+        const uint64_t i = c0 + tid;
+        uint64_t d = 0;
+        if (i < hi) d = __ldg(a.deg32 + a.queue[i]);
+        uint64_t tot;
+        const uint64_t W = run + block_excl_u64<NT>(i < hi ? A + d : 0, tot, s_warp);
+        // does a tile boundary fall inside [W, W + A + d)?
+        if (i < hi && ((W + kTileWork - 1) & ~(uint64_t)(kTileWork - 1)) < W + A + d)
+            place_tiles(a.tiles, i, W, d, cl, s_hub, &s_nhub, kHubCap);
+        run += tot;
     }
     __syncthreads();
     const uint32_t nhub = min(s_nhub, (uint32_t)kHubCap);
     for (uint32_t h = 0; h < nhub; ++h)
-        write_tiles(a.tiles, s_hub[h].q, s_hub[h].w, s_hub[h].d, cl, tid, kAdvanceThreads);
+        write_tiles(a.tiles, s_hub[h].q, s_hub[h].w, s_hub[h].d, cl, tid, NT);
 }
-
 
 // --------------------------------------------------------------------------
 // expand_kernel: a4 + a5 + a6 (P:137-177 generalised, Alg. 1 lines 3-6)
@@ -480,6 +477,15 @@ __global__ void __launch_bounds__(kExpandThreads, 8) expand_kernel(ExpandArgs a)
 
     const uint32_t lane = lane_id(), wid = threadIdx.x >> 5;
     const uint64_t ntiles = a.ctrl->ntiles, nf = a.ctrl->nf, nwork = a.ctrl->nwork;
+    const uint32_t xl = a.ctrl->xlevel;  // index of the level being expanded
+    uint32_t *parent = MODE == kModeVisitParent ? a.ctrl->parent : nullptr;
+    if (MODE != kModeDecode) {
+        if (threadIdx.x == 0 && a.stats && xl < a.max_stats) atomicMin(&a.stats[xl].t0, globaltimer());
+        if (blockIdx.x == 0 && threadIdx.x == 0) {
+            a.ctrl->level = xl + 1;  // depth of the vertices this launch discovers
+            a.ctrl->seq = a.ctrl->seq + 1;
+        }
+    }
     const uint32_t *data32 = reinterpret_cast<const uint32_t *>(a.data);
     const ChunkLen cl = make_chunk(a.k, a.kshift);
     const uint64_t CH = cl.ch;
@@ -672,7 +678,7 @@ __global__ void __launch_bounds__(kExpandThreads, 8) expand_kernel(ExpandArgs a)
                                         atomicOr(a.vis + (xs[u] >> 5), bit);  // line 4
                                     } else {
                                         const uint32_t old = atomicOr(a.vis + (xs[u] >> 5), bit);
-                                        if (!(old & bit)) a.out[xs[u]] = (uint32_t)m.aux;
+                                        if (!(old & bit)) parent[xs[u]] = (uint32_t)m.aux;
                                     }
                                 }
                             }
@@ -683,27 +689,10 @@ __global__ void __launch_bounds__(kExpandThreads, 8) expand_kernel(ExpandArgs a)
             }
         }
     }
+    if (MODE != kModeDecode && threadIdx.x == 0 && a.stats && xl < a.max_stats)
+        atomicMax(&a.stats[xl].t1, globaltimer());
 }
 
-
-__global__ void set_range_bits_kernel(uint32_t *vis, uint64_t v0, uint64_t v1)
-{
-    const uint64_t w0 = v0 >> 5, w1 = (v1 + 31) >> 5;
-    for (uint64_t w = w0 + blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; w < w1;
-         w += (uint64_t)gridDim.x * blockDim.x) {
-        uint32_t m = FULL;
-        if (w == (v0 >> 5)) m &= FULL << (v0 & 31);
-        if (w == ((v1 - 1) >> 5) && (v1 & 31)) m &= (1u << (v1 & 31)) - 1;
-        vis[w] |= m;
-    }
-}
-
-__global__ void fill_u32_kernel(uint32_t *p, uint32_t val, uint64_t n)
-{
-    for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n;
-         i += (uint64_t)gridDim.x * blockDim.x)
-        p[i] = val;
-}
 
 }  // namespace
 
@@ -740,26 +729,23 @@ cudaError_t launch_expand(int mode, const ExpandArgs &a, int blocks, cudaStream_
     return cudaGetLastError();
 }
 
-cudaError_t launch_advance(const AdvanceArgs &a, cudaStream_t s)
+cudaError_t launch_init(const InitArgs &a, cudaStream_t s)
 {
-    advance_kernel<<<(unsigned)a.nblocks, kAdvanceThreads, 0, s>>>(a);
+    const uint64_t words = ((a.v1 + 31) >> 5) - (a.v0 >> 5);
+    const unsigned blocks = (unsigned)std::max<uint64_t>(1, std::min<uint64_t>((words + 255) / 256, 4096));
+    init_kernel<<<blocks, 256, 0, s>>>(a);
     return cudaGetLastError();
 }
 
-cudaError_t launch_set_range_bits(uint32_t *vis, uint64_t v0, uint64_t v1, cudaStream_t s)
+cudaError_t launch_compact(const CompactArgs &a, unsigned blocks, cudaStream_t s)
 {
-    if (v1 <= v0) return cudaSuccess;
-    const uint64_t words = ((v1 + 31) >> 5) - (v0 >> 5);
-    const unsigned blocks = (unsigned)std::min<uint64_t>((words + 255) / 256, 4096);
-    set_range_bits_kernel<<<blocks, 256, 0, s>>>(vis, v0, v1);
+    compact_kernel<<<blocks, kFrontierThreads, 0, s>>>(a);
     return cudaGetLastError();
 }
 
-cudaError_t launch_fill_u32(uint32_t *p, uint32_t val, uint64_t n, cudaStream_t s)
+cudaError_t launch_plan(const PlanArgs &a, unsigned blocks, cudaStream_t s)
 {
-    if (!n) return cudaSuccess;
-    const unsigned blocks = (unsigned)std::min<uint64_t>((n + 255) / 256, 148 * 16);
-    fill_u32_kernel<<<blocks, 256, 0, s>>>(p, val, n);
+    plan_kernel<<<blocks, kFrontierThreads, 0, s>>>(a);
     return cudaGetLastError();
 }
 

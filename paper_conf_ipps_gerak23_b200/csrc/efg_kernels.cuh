@@ -18,35 +18,48 @@ struct ExpandArgs {
     const VRec *rec;           // packed vertex records
     const uint32_t *queue;     // frontier queue
     const TileEntry *tiles;    // tile table
-    const LevelCtrl *ctrl;     // nf, ne, ntiles of this level
+    LevelCtrl *ctrl;           // nf, ne, ntiles of this level; parent pointer; level
     uint32_t *vis;             // visited bitmap (modes 0, 1)
-    uint32_t *out;             // parent (mode 1) or decode output (mode 2)
+    uint32_t *out;             // decode output (mode 2)
+    LevelStat *stats;          // per-level statistics (device) or null
+    uint32_t max_stats;
     uint32_t k;                // forward-pointer quantum (chunk length); 0 = none
     int32_t kshift;            // log2(k) if k is a power of two, else -1
 };
 
-struct AdvanceArgs {
-    uint32_t *vis;             // visited bitmap
-    uint32_t *prev;            // visited bitmap after the previous advance
-    const VRec *rec;
-    const uint32_t *deg32;     // degrees (compact copy for the frontier step a1)
-    int32_t *depth;            // depth output (may be the caller's device buffer)
-    uint32_t *queue;           // next frontier (sorted by vertex id)
-    TileEntry *tiles;          // tile table of the next level
-    uint64_t *status;          // decoupled look-back status [2][2][nblocks]
-    LevelCtrl *ctrl;           // totals of the next level
-    uint64_t nwords;           // bitmap words
-    uint64_t nblocks;          // grid size
-    int32_t depth_value;       // depth assigned to newly discovered vertices
-    uint32_t parity;           // status parity of this launch
-    uint32_t k;                // chunk length (0 = whole lists)
-    int32_t kshift;            // log2(k) if k is a power of two, else -1
+struct InitArgs {
+    LevelCtrl *ctrl;
+    uint32_t *vis;
+    int32_t *depth;            // depth buffer of this call (device)
+    uint32_t *parent;          // parent buffer of this call (device) or null
+    uint64_t v0, v1;           // start set [v0, v1)
+};
+
+struct CompactArgs {
+    uint32_t *vis, *prev;      // visited bitmap now / at the previous level end
+    uint32_t *queue;           // out: next frontier, sorted
+    LevelCtrl *ctrl;           // in: level, seq, depth ptr; out: nf
+    uint64_t *status;          // cross-block prefix words (one per block)
+    uint64_t nwords, words_per_block;
+};
+
+struct PlanArgs {
+    const uint32_t *queue;
+    const uint32_t *deg32;
+    TileEntry *tiles;
+    LevelCtrl *ctrl;           // in: nf, level, seq; out: ne, nwork, ntiles, xlevel
+    uint64_t *status;
+    LevelStat *stats;
+    uint32_t max_stats;
+    uint32_t k;
+    int32_t kshift;
+    cudaGraphConditionalHandle cond;  // graph-mode loop condition, 0 = host loop
 };
 
 cudaError_t launch_expand(int mode, const ExpandArgs &a, int blocks, cudaStream_t s);
-cudaError_t launch_advance(const AdvanceArgs &a, cudaStream_t s);
-cudaError_t launch_set_range_bits(uint32_t *vis, uint64_t v0, uint64_t v1, cudaStream_t s);
-cudaError_t launch_fill_u32(uint32_t *p, uint32_t val, uint64_t n, cudaStream_t s);
+cudaError_t launch_init(const InitArgs &a, cudaStream_t s);
+cudaError_t launch_compact(const CompactArgs &a, unsigned blocks, cudaStream_t s);
+cudaError_t launch_plan(const PlanArgs &a, unsigned blocks, cudaStream_t s);
 int expand_occupancy(int mode);
 
 }  // namespace efg

@@ -214,3 +214,32 @@ def test_c2_rmat24_full_size(efg):
     for a, b in [(0, 64), (n // 2, n // 2 + 4096), (n - 5000, n)]:
         assert np.array_equal(g.decode(a, b), oe[ov[a]:ov[b]])
     g.free()
+
+
+def test_graph_and_host_level_loops_agree(efg):
+    n, src, dst = synth.rmat(13, 16, seed=7)
+    g = efg.Graph.build(n, src, dst)
+    ov, oe = oracle.csr_build(n, src, dst)
+    for s in (0, 3, 4000):
+        ref = oracle.bfs(ov, oe, s)
+        g.set_level_loop(False)
+        d1, _, st1 = g.bfs(s, stats=True)
+        g.set_level_loop(True)
+        d2, _, st2 = g.bfs(s, stats=True)
+        assert np.array_equal(d1, ref) and np.array_equal(d2, ref)
+        assert st1["levels"] == st2["levels"] == ref.max() + 1
+        assert np.array_equal(st1["level_edges"], st2["level_edges"])
+        assert st1["edges_traversed"] == st2["edges_traversed"]
+        assert st1["vertices_reached"] == (ref >= 0).sum()
+    g.free()
+
+
+def test_long_path_many_levels(efg):
+    # more levels than the per-level statistics buffer (graph-mode device loop)
+    n = 6000
+    src = np.arange(n - 1, dtype=np.uint32)
+    g = efg.Graph.build(n, src, src + 1)
+    d, _, st = g.bfs(0, stats=True, level_cap=16)
+    assert np.array_equal(d, np.arange(n))
+    assert st["levels"] == n and st["vertices_reached"] == n
+    g.free()
