@@ -51,6 +51,8 @@ def parse():
     p.add_argument("--config", type=int, default=2, help="BASELINE.json config index (1-based)")
     p.add_argument("--scale", type=int, default=None, help="override RMAT scale (debug only)")
     p.add_argument("--no-cpu-baseline", action="store_true")
+    p.add_argument("--reorder", default="degree", choices=["none", "degree"],
+                   help="EFG_REORDER_DEGREE relabelling at build time (results stay in input ids)")
     p.add_argument("--profile-levels", action="store_true", help="print per-level stats to stderr")
     return p.parse_args()
 
@@ -185,12 +187,16 @@ def main():
     stream = torch.cuda.Stream(device=dev)
 
     n, src, dst, gen_s = make_graph_edges(args.config, args.scale)
-    g = efg.Graph.build(n, src, dst, device=local, stream=stream.cuda_stream)
+    flags = efg.EFG_DEFAULT_FLAGS | (efg.EFG_REORDER_DEGREE if args.reorder == "degree" else 0)
+    g = efg.Graph.build(n, src, dst, device=local, stream=stream.cuda_stream, flags=flags)
     del src, dst
     info = g.info
     vlist, nlb, offsets, _ = g.export()
-    deg = np.diff(vlist)
-    sizes = np.diff(offsets).astype(np.int64)
+    perm = g.perm()  # stored id -> input id
+    deg = np.empty(n, np.int64)
+    deg[perm] = np.diff(vlist).astype(np.int64)       # input-id order
+    sizes = np.empty(n, np.int64)
+    sizes[perm] = np.diff(offsets).astype(np.int64)   # input-id order
 
     nsrc = args.warmup + args.steps
     all_srcs = synth.sources(n, nsrc * world, seed=1000 + args.config, nonisolated_mask=deg > 0)
@@ -309,6 +315,7 @@ def main():
             "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u32",
             "data": "synthetic",
             "config": {"workload": cfgname, "n": int(n), "m_directed": int(info["m"]),
+                       "reorder": args.reorder,
                        "sources_per_rank": args.steps, "fwd_quantum": int(info["fwd_quantum"]),
                        "efg_bytes_per_edge": (info["data_bytes"] + 17 * n) / info["m"],
                        "ef_data_bytes_per_edge": info["data_bytes"] / info["m"],

@@ -44,6 +44,12 @@ typedef enum efg_status {
 #define EFG_SYMMETRIZE 0x1u       /* add (d,s) for every input (s,d): "_sym" graphs  */
 #define EFG_DEDUP 0x2u            /* keep one copy of each directed (s,d)                   */
 #define EFG_DROP_SELF_LOOPS 0x4u  /* remove (v,v)                                           */
+#define EFG_REORDER_DEGREE 0x8u   /* relabel vertices by degree (descending, ties by id) before
+                                   * encoding: the reordering preprocessing of P:246-258 in its
+                                   * simplest form.  Traversal inputs/outputs (source, depth,
+                                   * parent, dist, rank) stay in INPUT ids; efg_export and
+                                   * efg_decode describe the relabelled graph, whose relabelling
+                                   * efg_export_perm returns. */
 #define EFG_DEFAULT_FLAGS (EFG_SYMMETRIZE | EFG_DEDUP | EFG_DROP_SELF_LOOPS)
 
 typedef struct efg_graph efg_graph; /* opaque: host EFG arrays + device copy */
@@ -126,6 +132,11 @@ efg_status efg_info(const efg_graph *g, efg_info_t *info);
  * owned row range (vertices outside it have empty lists). */
 efg_status efg_export(const efg_graph *g, uint64_t *vlist, uint8_t *num_lower_bits,
                       uint64_t *offsets, uint8_t *data);
+
+/* Copy the relabelling of an EFG_REORDER_DEGREE handle: old_of_new[i] = input id
+ * of stored vertex i (n entries, caller-owned host buffer).  Without the flag
+ * the identity is written. */
+efg_status efg_export_perm(const efg_graph *g, uint32_t *old_of_new);
 
 /*
  * efg_decode — GPU decode of the neighbour lists of vertices [v0, v1) into

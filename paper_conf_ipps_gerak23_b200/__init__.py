@@ -16,11 +16,11 @@ import ctypes as C
 import numpy as np
 
 from . import _abi
-from ._abi import (EFG_DEDUP, EFG_DEFAULT_FLAGS, EFG_DROP_SELF_LOOPS, EFG_SYMMETRIZE,  # noqa: F401
-                   EFGError, check, lib)
+from ._abi import (EFG_DEDUP, EFG_DEFAULT_FLAGS, EFG_DROP_SELF_LOOPS, EFG_REORDER_DEGREE,  # noqa: F401
+                   EFG_SYMMETRIZE, EFGError, check, lib)
 
 __all__ = ["Graph", "EFGError", "EFG_DEFAULT_FLAGS", "EFG_SYMMETRIZE", "EFG_DEDUP",
-           "EFG_DROP_SELF_LOOPS", "version", "partition"]
+           "EFG_DROP_SELF_LOOPS", "EFG_REORDER_DEGREE", "version", "partition"]
 
 
 def version() -> str:
@@ -107,6 +107,12 @@ class Graph:
     @property
     def m(self) -> int:
         return self.info["m"]
+
+    def perm(self) -> np.ndarray:
+        """old_of_new relabelling (identity unless built with EFG_REORDER_DEGREE)."""
+        p = np.empty(max(self.info["n"], 1), np.uint32)
+        check(lib.efg_export_perm(self._h, _ptr(p)), "efg_export_perm")
+        return p[:self.info["n"]]
 
     def export(self):
         """(vlist u64[n+1], num_lower_bits u8[n], offsets u64[n+1], data u8[]) — P:113."""

@@ -17,6 +17,7 @@ STATUS_NAMES = {0: "EFG_OK", 1: "EFG_EINVAL", 2: "EFG_ERANGE", 3: "EFG_ENOMEM", 
                 5: "EFG_ENCCL", 6: "EFG_ENOTSUP", 7: "EFG_ESTATE"}
 EFG_SYMMETRIZE, EFG_DEDUP, EFG_DROP_SELF_LOOPS = 0x1, 0x2, 0x4
 EFG_DEFAULT_FLAGS = 0x7
+EFG_REORDER_DEGREE = 0x8
 EFG_OPT_LEVEL_LOOP = 1
 
 
@@ -52,6 +53,7 @@ SIGNATURES = [
     ("efg_free", None, [C.c_void_p]),
     ("efg_info", C.c_int, [C.c_void_p, C.POINTER(Info)]),
     ("efg_export", C.c_int, [C.c_void_p, C.c_void_p, C.c_void_p, C.c_void_p, C.c_void_p]),
+    ("efg_export_perm", C.c_int, [C.c_void_p, C.c_void_p]),
     ("efg_decode", C.c_int, [C.c_void_p, C.c_uint32, C.c_uint32, C.c_void_p]),
     ("efg_bfs", C.c_int, [C.c_void_p, C.c_uint32, C.c_void_p, C.c_void_p, C.POINTER(Stats)]),
     ("efg_sssp", C.c_int, [C.c_void_p, C.c_uint32, C.c_void_p, C.POINTER(Stats)]),

@@ -125,6 +125,19 @@ extern "C" efg_status efg_export(const efg_graph *g, uint64_t *vlist, uint8_t *n
     return EFG_OK;
 }
 
+extern "C" efg_status efg_export_perm(const efg_graph *g, uint32_t *old_of_new)
+{
+    clear_error();
+    if (!g || !old_of_new) return set_error(EFG_EINVAL, "efg_export_perm: null argument");
+    const HostEFG &h = g->host;
+    if (h.old_of_new.empty()) {
+        for (uint64_t i = 0; i < h.n; ++i) old_of_new[i] = (uint32_t)i;
+    } else {
+        std::memcpy(old_of_new, h.old_of_new.data(), h.n * 4);
+    }
+    return EFG_OK;
+}
+
 extern "C" efg_status efg_decode(efg_graph *g, uint32_t v0, uint32_t v1, uint32_t *out)
 {
     clear_error();
@@ -142,7 +155,8 @@ extern "C" efg_status efg_bfs(efg_graph *g, uint32_t source, int32_t *depth, uin
     EFG_TRY(check_handle(g));
     if (source >= g->dev.n) return set_error(EFG_ERANGE, "efg_bfs: source >= n");
     if (!depth) return set_error(EFG_EINVAL, "efg_bfs: depth is NULL");
-    return device_bfs(g, source, depth, parent, st);
+    const uint32_t s = g->host.new_of_old.empty() ? source : g->host.new_of_old[source];
+    return device_bfs(g, s, depth, parent, st);
 }
 
 extern "C" efg_status efg_set_option(efg_graph *g, int option, int64_t value)

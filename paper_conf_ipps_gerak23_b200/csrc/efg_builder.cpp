@@ -154,6 +154,42 @@ efg_status build_host(uint64_t n, uint64_t m, const uint32_t *src, const uint32_
             }
             deg[v] = w;
         }
+        // optional relabelling by degree (descending, ties by id): the
+        // reordering preprocessing of P:246-258 / P:35 in its simplest form.
+        // Hubs get the smallest ids, which the expand kernel keeps in a
+        // shared-memory visited snapshot.  Results are reported in input ids.
+        if (o.flags & EFG_REORDER_DEGREE) {
+            uint64_t maxd = 0;
+#pragma omp parallel for reduction(max : maxd)
+            for (int64_t v = 0; v < (int64_t)n; ++v) maxd = std::max<uint64_t>(maxd, deg[v]);
+            std::vector<uint64_t> bucket(maxd + 2, 0);
+            for (uint64_t v = 0; v < n; ++v) bucket[maxd - deg[v]]++;
+            exclusive_scan_inplace(bucket.data(), maxd + 1);
+            out.old_of_new.resize(n);
+            out.new_of_old.resize(n);
+            for (uint64_t v = 0; v < n; ++v) {  // stable: ascending id within a degree
+                const uint64_t i = bucket[maxd - deg[v]]++;
+                out.old_of_new[i] = (uint32_t)v;
+                out.new_of_old[v] = (uint32_t)i;
+            }
+            std::vector<uint64_t> start2(n + 1, 0), deg2(n + 1, 0);
+            for (uint64_t i = 0; i < n; ++i) deg2[i] = deg[out.old_of_new[i]];
+            for (uint64_t i = 0; i < n; ++i) start2[i + 1] = start2[i] + deg2[i];
+            std::unique_ptr<uint64_t[]> tmp2(new uint64_t[start2[n] ? start2[n] : 1]);
+            const uint32_t *nof = out.new_of_old.data();
+#pragma omp parallel for schedule(dynamic, 512)
+            for (int64_t i = 0; i < (int64_t)n; ++i) {
+                const uint64_t v = out.old_of_new[i];
+                const uint64_t *a = tmp.get() + start[v];
+                uint64_t *b = tmp2.get() + start2[i];
+                for (uint64_t t = 0; t < deg2[i]; ++t)
+                    b[t] = ((uint64_t)nof[(uint32_t)(a[t] >> 32)] << 32) | (uint32_t)a[t];
+                std::sort(b, b + deg2[i]);
+            }
+            tmp.swap(tmp2);
+            start.swap(start2);
+            deg.swap(deg2);
+        }
         // partition: keep only the owned rows' lists
         const uint64_t lo = o.dist ? out.row_lo : 0, hi = o.dist ? out.row_hi : n;
         for (uint64_t v = 0; v < n; ++v)

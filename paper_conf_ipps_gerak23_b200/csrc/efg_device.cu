@@ -83,6 +83,7 @@ ExpandArgs expand_args(DeviceGraph &d, uint32_t *out)
     a.out = out;
     a.stats = d.stats;
     a.max_stats = kMaxLevelStats;
+    a.hot_words = (uint32_t)std::min<uint64_t>(kHotWords, d.nwords) & ~3u;
     a.k = d.k;
     a.kshift = kshift_of(d.k);
     return a;
@@ -94,6 +95,7 @@ CompactArgs compact_args(DeviceGraph &d)
     a.vis = d.vis;
     a.prev = d.prev;
     a.queue = d.queue;
+    a.idmap = d.old_of_new;
     a.ctrl = d.ctrl;
     a.status = d.status;
     a.nwords = d.nwords;
@@ -181,6 +183,8 @@ void device_free(DeviceGraph &d)
     cudaFree(d.tiles);
     cudaFree(d.depth);
     cudaFree(d.parent);
+    cudaFree(d.parent2);
+    cudaFree(d.old_of_new);
     cudaFree(d.status);
     cudaFree(d.stats);
     cudaFree(d.ctrl);
@@ -239,6 +243,10 @@ efg_status device_upload(efg_graph *g, const efg_build_opts &o)
     CUDA_TRY(cudaMemcpyAsync(d.deg32, deg.data(), d.nwords * 32 * 4, cudaMemcpyHostToDevice, s));
     EFG_TRY(dev_alloc(d, &d.vlist, h.n + 1));
     CUDA_TRY(cudaMemcpyAsync(d.vlist, h.vlist.data(), (h.n + 1) * 8, cudaMemcpyHostToDevice, s));
+    if (!h.old_of_new.empty()) {
+        EFG_TRY(dev_alloc(d, &d.old_of_new, h.n));
+        CUDA_TRY(cudaMemcpyAsync(d.old_of_new, h.old_of_new.data(), h.n * 4, cudaMemcpyHostToDevice, s));
+    }
     if (!h.weights.empty()) {
         EFG_TRY(dev_alloc(d, &d.weights, h.m));
         CUDA_TRY(cudaMemcpyAsync(d.weights, h.weights.data(), h.m * 4, cudaMemcpyHostToDevice, s));
@@ -321,12 +329,16 @@ efg_status device_bfs(efg_graph *g, uint32_t source, int32_t *depth, uint32_t *p
     cudaStream_t s = stream_of(d);
     const bool depth_dev = is_device_ptr(depth);
     int32_t *dd = depth_dev ? depth : d.depth;
-    uint32_t *pd = nullptr;
+    uint32_t *pd = nullptr;     // parent buffer the kernels write (stored ids)
+    uint32_t *pout = nullptr;   // parent in input ids on the device
     bool parent_dev = false;
+    const bool relabel = d.old_of_new != nullptr;
     if (parent) {
         parent_dev = is_device_ptr(parent);
-        if (!parent_dev && !d.parent) EFG_TRY(dev_alloc(d, &d.parent, d.n));
-        pd = parent_dev ? parent : d.parent;
+        if ((relabel || !parent_dev) && !d.parent) EFG_TRY(dev_alloc(d, &d.parent, d.n));
+        if (relabel && !parent_dev && !d.parent2) EFG_TRY(dev_alloc(d, &d.parent2, d.n));
+        pd = (parent_dev && !relabel) ? parent : d.parent;
+        pout = parent_dev ? parent : (relabel ? d.parent2 : d.parent);
     }
     const int mode = parent ? kModeVisitParent : kModeVisit;
     const bool graph_mode = d.level_loop == 0;
@@ -387,8 +399,9 @@ efg_status device_bfs(efg_graph *g, uint32_t source, int32_t *depth, uint32_t *p
         }
         CUDA_TRY(cudaEventRecord(ev1, s));
     }
+    if (parent && relabel) CUDA_TRY(launch_map_parent(pd, d.old_of_new, pout, d.n, s));
     if (!depth_dev) CUDA_TRY(cudaMemcpyAsync(depth, dd, d.n * 4, cudaMemcpyDeviceToHost, s));
-    if (parent && !parent_dev) CUDA_TRY(cudaMemcpyAsync(parent, pd, d.n * 4, cudaMemcpyDeviceToHost, s));
+    if (parent && !parent_dev) CUDA_TRY(cudaMemcpyAsync(parent, pout, d.n * 4, cudaMemcpyDeviceToHost, s));
     CUDA_TRY(cudaStreamSynchronize(s));
 
     float total_ms = 0.f;

@@ -27,6 +27,7 @@ struct HostEFG {
     std::vector<uint64_t> offsets;  // n+1  exclusive sum of per-vertex byte sizes
     std::vector<uint8_t> data;      // offsets[n] bytes (+ padding on device)
     std::vector<float> weights;     // m (CSR order) or empty
+    std::vector<uint32_t> old_of_new, new_of_old;  // EFG_REORDER_DEGREE relabelling (else empty)
     uint64_t fwd_bytes = 0, lower_bytes = 0, upper_bytes = 0, apriori_bits = 0;
     uint64_t row_lo = 0, row_hi = 0;
     double build_seconds = 0.0;
@@ -92,7 +93,10 @@ struct LevelStat {
 };
 constexpr uint32_t kMaxLevelStats = 4096;
 
-constexpr int kExpandThreads = 128;          // 4 warps (static smem < 48 KB)
+constexpr int kExpandThreads = 512;          // one CTA per SM, 16 warps
+constexpr int kExpandWarps = kExpandThreads / 32;
+constexpr int kExpandStage = 1024;           // elements of one 32-word step (<= 32*32)
+constexpr uint32_t kHotWords = 28 * 1024;    // 112 KB shared-memory visited snapshot = 917,504 ids
 constexpr int kFrontierThreads = 256;        // compact / plan kernels
 constexpr int kBitmapAlign = 1024;           // bitmap words are padded to a multiple of this
 // Step a3 partitions "work units" rather than bare edges: a frontier vertex
@@ -122,6 +126,8 @@ struct DeviceGraph {
     uint64_t max_tiles = 0;
     int32_t *depth = nullptr;          // internal depth (n)
     uint32_t *parent = nullptr;        // internal parent (n), lazily allocated
+    uint32_t *parent2 = nullptr;       // parent in input ids (reordered graphs), lazily
+    uint32_t *old_of_new = nullptr;    // EFG_REORDER_DEGREE relabelling (n) or null
     uint64_t *status = nullptr;        // cross-block prefix words: compact [kMaxGrid], plan [kMaxGrid]
     LevelStat *stats = nullptr;        // per-level statistics (kMaxLevelStats)
     unsigned frontier_blocks = 0;      // grid of compact / plan

@@ -26,7 +26,6 @@ namespace efg {
 namespace {
 
 constexpr uint32_t FULL = 0xffffffffu;
-constexpr int kWarps = kExpandThreads / 32;
 
 // --------------------------------------------------------------------------
 // warp / block primitives (§III-C: exclusive scan, bounded search)
@@ -321,7 +320,7 @@ __global__ void __launch_bounds__(kFrontierThreads) compact_kernel(CompactArgs a
         for (uint32_t i = tid; i < tot; i += NT) {
             const uint32_t v = s_ids[i];
             a.queue[base + i] = v;
-            depth[v] = level;
+            depth[a.idmap ? a.idmap[v] : v] = level;
         }
         base += tot;
         __syncthreads();
@@ -410,25 +409,31 @@ __global__ void __launch_bounds__(kFrontierThreads) plan_kernel(PlanArgs a)
 // --------------------------------------------------------------------------
 // expand_kernel: a4 + a5 + a6 (P:137-177 generalised, Alg. 1 lines 3-6)
 //
-// One warp per tile (persistent grid-stride over tiles).  A tile's work is a
-// run of "chunks": k-aligned pieces of frontier lists, so every chunk
-// starts right after a forward pointer and needs no select to find its first
-// bit.  Chunks are taken 32 at a time ("batch"; many short lists per warp: the
-// multi-list case).  The batch's upper-bit words are laid end to
-// end and processed 32 words per step (one aligned 32-bit word per lane,
-// coalesced; the next step's word is loaded before the current one is used):
-//   popcount + warp exclusive scan  -> rank of each word's first stop bit
-//                                      (the segmented scan of P:171-177: the
-//                                      segments are chunks, whose element
-//                                      prefix is subtracted)
-//   per lane, serially over its word -> select1(i) - i by ffs-and-clear, the
-//                                      lower bits from a bit buffer streamed
-//                                      over the lower section, x = hi<<l | lo,
-//                                      then the visits, kGroup probes in flight.
+// Persistent: one CTA of kExpandThreads per SM, one warp per work tile.  A
+// tile's work is a run of "chunks": k-aligned pieces of frontier lists
+// (P:157), so every chunk starts right after a forward pointer and needs no
+// select to find its first bit.  Chunks are taken 32 at a time ("batch"; many
+// short lists per warp: the multi-list case).  The batch's
+// upper-bit words are laid end to end and processed 32 words per step (one
+// aligned 32-bit word per lane, coalesced; the next step's word is loaded
+// before the current one is used):
+//   popcount + warp exclusive scan -> rank of each word's first stop bit (the
+//                                     segmented scan of P:171-177; segments are
+//                                     chunks, whose element prefix is subtracted)
+//   set-bit enumeration (ffs)       -> select1(i) - i per element, staged in
+//                                     shared memory by element slot (Alg. 2's
+//                                     "s_bytes/select" step without the LUT)
+//   balanced pass, 4 elements per lane in flight
+//                                   -> lower bits by a funnel shift of two
+//                                     coalesced words, x = hi * 2^l + lo,
+//                                     visit (Alg. 1 lines 3-4).
+// Visit: the first kHotWords*32 vertex ids (the highest-degree vertices when the
+// graph was built with EFG_REORDER_DEGREE) have a per-CTA shared-memory copy of
+// their visited bits, loaded at kernel start (a snapshot of the level start,
+// updated by this CTA's own discoveries).  A set bit there answers the probe
+// without touching L1/L2; otherwise the global bitmap is probed and the
+// atomicOr decides (stale reads are benign).
 // --------------------------------------------------------------------------
-
-constexpr int kGroup = 8;  // probes in flight per lane
-
 struct SlotGeom {
     uint64_t A0, A1, U0;  // absolute bit range of the chunk's upper bits; upper start
     uint32_t wb, eb;      // exclusive word / element prefix within the batch
@@ -436,9 +441,18 @@ struct SlotGeom {
 };
 
 struct SlotMeta {
-    uint64_t lbase_l;  // absolute bit address of the lower section | l << 58
-    int64_t rankoff;   // rank = rankoff + batch element index
-    uint64_t aux;      // parent: source vertex; decode: output index base
+    uint64_t lb;     // lower-bit address of batch element e: lb + e*l
+    uint32_t l;      // lower bits per element
+    uint32_t lmask;  // (1 << l) - 1
+    uint64_t aux;    // parent: source vertex; decode: output index base
+};
+static_assert(sizeof(SlotMeta) == 24, "SlotMeta layout");
+
+struct WarpSmem {
+    uint32_t hi[kExpandStage];  // select1(i) - i by batch-step element slot
+    uint8_t cs[kExpandStage];   // chunk slot of the element
+    SlotGeom geom[32];
+    SlotMeta meta[32];
 };
 
 struct WordLd {
@@ -469,29 +483,39 @@ __device__ __forceinline__ WordLd load_word(const uint32_t *data32, const SlotGe
     return r;
 }
 
+constexpr int kVisitBatch = 4;  // elements per lane in flight in the balanced pass
+
 template <int MODE>
-__global__ void __launch_bounds__(kExpandThreads, 8) expand_kernel(ExpandArgs a)
+__global__ void __launch_bounds__(kExpandThreads, 1) expand_kernel(ExpandArgs a)
 {
-    __shared__ SlotGeom s_geom[kWarps][32];
-    __shared__ SlotMeta s_meta[kWarps][32];
+    extern __shared__ __align__(16) uint8_t smem_raw[];
+    uint32_t *s_hot = reinterpret_cast<uint32_t *>(smem_raw);
+    WarpSmem *ws_all = reinterpret_cast<WarpSmem *>(smem_raw + kHotWords * 4);
 
     const uint32_t lane = lane_id(), wid = threadIdx.x >> 5;
+    WarpSmem &ws = ws_all[wid];
     const uint64_t ntiles = a.ctrl->ntiles, nf = a.ctrl->nf, nwork = a.ctrl->nwork;
     const uint32_t xl = a.ctrl->xlevel;  // index of the level being expanded
     uint32_t *parent = MODE == kModeVisitParent ? a.ctrl->parent : nullptr;
+    const uint32_t hot_limit = a.hot_words * 32;  // vertex ids below this use s_hot
     if (MODE != kModeDecode) {
         if (threadIdx.x == 0 && a.stats && xl < a.max_stats) atomicMin(&a.stats[xl].t0, globaltimer());
         if (blockIdx.x == 0 && threadIdx.x == 0) {
             a.ctrl->level = xl + 1;  // depth of the vertices this launch discovers
             a.ctrl->seq = a.ctrl->seq + 1;
         }
+        // level-start snapshot of the hot visited words
+        const uint4 *src = reinterpret_cast<const uint4 *>(a.vis);
+        uint4 *dst = reinterpret_cast<uint4 *>(s_hot);
+        for (uint32_t i = threadIdx.x; i < a.hot_words / 4; i += blockDim.x) dst[i] = src[i];
+        __syncthreads();
     }
     const uint32_t *data32 = reinterpret_cast<const uint32_t *>(a.data);
     const ChunkLen cl = make_chunk(a.k, a.kshift);
     const uint64_t CH = cl.ch;
     const uint64_t A = kVertexWork;
-    const uint64_t gw = (uint64_t)blockIdx.x * kWarps + wid;
-    const uint64_t nwarps = (uint64_t)gridDim.x * kWarps;
+    const uint64_t gw = (uint64_t)blockIdx.x * kExpandWarps + wid;
+    const uint64_t nwarps = (uint64_t)gridDim.x * kExpandWarps;
 
     for (uint64_t tile = gw; tile < ntiles; tile += nwarps) {
         const TileEntry te = a.tiles[tile];
@@ -569,7 +593,7 @@ __global__ void __launch_bounds__(kExpandThreads, 8) expand_kernel(ExpandArgs a)
             const uint32_t ebt = warp_excl_u32(nel, NE);
             (void)NE;
             if (valid) {
-                s_geom[wid][lane] = SlotGeom{A0, A1, U0, wb, ebt, r0};
+                ws.geom[lane] = SlotGeom{A0, A1, U0, wb, ebt, r0};
                 uint64_t aux = 0;
                 if (MODE == kModeVisitParent) aux = v_j;
                 if (MODE == kModeDecode) {
@@ -577,7 +601,12 @@ __global__ void __launch_bounds__(kExpandThreads, 8) expand_kernel(ExpandArgs a)
                     const uint64_t qv = fi + (uint64_t)j;
                     aux = Wv_j - A * qv + r0 - ebt;
                 }
-                s_meta[wid][lane] = SlotMeta{lbase | ((uint64_t)l << kOffBits), (int64_t)r0 - (int64_t)ebt, aux};
+                SlotMeta m;
+                m.lb = lbase + (r0 - (uint64_t)ebt) * l;  // modular: rank = r0 + (e - ebt)
+                m.l = l;
+                m.lmask = l ? (FULL >> (32 - l)) : 0u;
+                m.aux = aux;
+                ws.meta[lane] = m;
             }
             // state after this batch: continue after the last valid chunk
             {
@@ -599,92 +628,84 @@ __global__ void __launch_bounds__(kExpandThreads, 8) expand_kernel(ExpandArgs a)
             }
             __syncwarp();
 
-            // ---- a5 + a6: 32 upper-bit words per step, one word per lane ----
-            // Each lane decodes the elements whose stop bits lie in its word,
-            // serially: select1(i) - i by ffs-and-clear, the lower bits from a
-            // per-lane bit buffer streamed over the chunk's lower section, then
-            // the visit.  Lanes start at ranks given by the warp scan of the
-            // words' popcounts.
+            // ---- a5 + a6: 32 upper-bit words per step ----
             uint32_t run = 0;
-            WordLd nxt = load_word(data32, s_geom[wid], wb, lane, W);
+            WordLd nxt = load_word(data32, ws.geom, wb, lane, W);
             for (uint32_t g0 = 0; g0 < W; g0 += 32) {
                 const WordLd cur = nxt;
-                if (g0 + 32 < W) nxt = load_word(data32, s_geom[wid], wb, g0 + 32 + lane, W);
+                if (g0 + 32 < W) nxt = load_word(data32, ws.geom, wb, g0 + 32 + lane, W);
                 uint32_t tot;
                 const uint32_t ep = warp_excl_u32(__popc(cur.word), tot);
                 if (cur.word) {
-                    const SlotGeom &sg = s_geom[wid][cur.s];
-                    const SlotMeta m = s_meta[wid][cur.s];
-                    const uint64_t rank = sg.r0 + run + ep - sg.eb;         // rank of the first set bit
-                    uint32_t hb = (uint32_t)(cur.wi * 32 - sg.U0 - rank);  // hi = hb + p - jj
-                    const uint32_t ll = (uint32_t)(m.lbase_l >> kOffBits);
-                    const uint32_t lmask = ll ? (0xffffffffu >> (32 - ll)) : 0u;
-                    // lower-bit stream at bit lbase + rank*l (bit buffer `buf` holds nb bits)
-                    const uint64_t lpos = (m.lbase_l & kOffMask) + rank * ll;
-                    const uint32_t *lp = data32 + (lpos >> 5);
-                    uint64_t buf = 0;
-                    uint32_t nb = 64, pre = 0;
-                    if (ll) {
-                        const uint32_t sh = (uint32_t)(lpos & 31);
-                        buf = (((uint64_t)ldg_u32(lp + 1) << 32) | ldg_u32(lp)) >> sh;
-                        nb = 64 - sh;
-                        pre = ldg_u32(lp + 2);
-                        lp += 3;
-                    }
-                    uint64_t obase = m.aux + run + ep;  // decode: output index of the next element
-                    uint32_t w = cur.word;
+                    const SlotGeom &sg = ws.geom[cur.s];
+                    const uint64_t rank = sg.r0 + run + ep - sg.eb;  // rank of the first set bit
+                    uint32_t hb = (uint32_t)(cur.wi * 32 - sg.U0 - rank);  // hi = hb + p (hb -= 1 per bit)
+                    uint32_t w = cur.word, e = ep;
+                    const uint8_t sc = (uint8_t)cur.s;
                     while (w) {
-                        // decode up to kGroup elements, then resolve their probes together
-                        uint32_t xs[kGroup];
-                        uint32_t valid = 0;
+                        ws.hi[e] = hb + (__ffs(w) - 1);  // select1(i) - i
+                        ws.cs[e] = sc;
+                        w &= w - 1;
+                        --hb;
+                        ++e;
+                    }
+                }
+                __syncwarp();
+                for (uint32_t base = 0; base < tot; base += 32 * kVisitBatch) {
+                    uint32_t xv[kVisitBatch];
+                    uint64_t ax[kVisitBatch];
+                    bool ok[kVisitBatch];
 #pragma unroll
-                        for (int u = 0; u < kGroup; ++u) {
-                            xs[u] = 0;
-                            if (w) {
-                                const uint32_t p = __ffs(w) - 1;
-                                w &= w - 1;
-                                const uint32_t hi = hb + p;  // select1(i) - i
-                                hb -= 1;
-                                uint32_t lo = 0;
-                                if (ll) {
-                                    if (nb < ll) {
-                                        buf |= (uint64_t)pre << nb;
-                                        nb += 32;
-                                        pre = ldg_u32(lp++);
-                                    }
-                                    lo = (uint32_t)buf & lmask;
-                                    buf >>= ll;
-                                    nb -= ll;
-                                }
-                                xs[u] = (hi << ll) | lo;
-                                valid |= 1u << u;
+                    for (int u = 0; u < kVisitBatch; ++u) {
+                        const uint32_t e = base + u * 32 + lane;
+                        ok[u] = e < tot;
+                        xv[u] = 0;
+                        ax[u] = 0;
+                        if (ok[u]) {
+                            const uint32_t hi = ws.hi[e];
+                            const SlotMeta &m = ws.meta[ws.cs[e]];
+                            uint32_t lo = 0;
+                            if (m.l) {
+                                const uint64_t ba = m.lb + (uint64_t)(run + e) * m.l;
+                                const uint32_t *p = data32 + (ba >> 5);
+                                lo = __funnelshift_r(ldg_u32(p), ldg_u32(p + 1), (uint32_t)(ba & 31)) & m.lmask;
                             }
+                            xv[u] = (hi << m.l) | lo;  // (select1(i) - i) << l | lower[i]
+                            ax[u] = MODE == kModeDecode ? m.aux + run + e : m.aux;
                         }
-                        if (MODE == kModeDecode) {
+                    }
+                    if (MODE == kModeDecode) {
 #pragma unroll
-                            for (int u = 0; u < kGroup; ++u)
-                                if (valid >> u & 1) a.out[obase + u] = xs[u];
-                            obase += __popc(valid);
-                        } else {
-                            uint32_t ws[kGroup];
+                        for (int u = 0; u < kVisitBatch; ++u)
+                            if (ok[u]) a.out[ax[u]] = xv[u];
+                    } else {
+                        // Alg. 1 line 3: hot ids answer from shared memory
+                        bool need[kVisitBatch];
 #pragma unroll
-                            for (int u = 0; u < kGroup; ++u)  // Alg. 1 line 3: probes in flight together
-                                ws[u] = (valid >> u & 1) ? a.vis[xs[u] >> 5] : FULL;
+                        for (int u = 0; u < kVisitBatch; ++u) {
+                            need[u] = ok[u];
+                            if (ok[u] && xv[u] < hot_limit)
+                                need[u] = !((s_hot[xv[u] >> 5] >> (xv[u] & 31)) & 1);
+                        }
+                        uint32_t gwd[kVisitBatch];
 #pragma unroll
-                            for (int u = 0; u < kGroup; ++u) {
-                                const uint32_t bit = 1u << (xs[u] & 31);
-                                if (!(ws[u] & bit)) {  // stale reads are benign: the atomic decides
-                                    if (MODE == kModeVisit) {
-                                        atomicOr(a.vis + (xs[u] >> 5), bit);  // line 4
-                                    } else {
-                                        const uint32_t old = atomicOr(a.vis + (xs[u] >> 5), bit);
-                                        if (!(old & bit)) parent[xs[u]] = (uint32_t)m.aux;
-                                    }
+                        for (int u = 0; u < kVisitBatch; ++u) gwd[u] = need[u] ? a.vis[xv[u] >> 5] : FULL;
+#pragma unroll
+                        for (int u = 0; u < kVisitBatch; ++u) {
+                            const uint32_t bit = 1u << (xv[u] & 31);
+                            if (!(gwd[u] & bit)) {  // line 4 (stale reads are benign: the atomic decides)
+                                if (MODE == kModeVisit) {
+                                    atomicOr(a.vis + (xv[u] >> 5), bit);
+                                } else {
+                                    const uint32_t old = atomicOr(a.vis + (xv[u] >> 5), bit);
+                                    if (!(old & bit)) parent[xv[u]] = (uint32_t)ax[u];
                                 }
                             }
+                            if (need[u] && xv[u] < hot_limit) atomicOr(s_hot + (xv[u] >> 5), bit);
                         }
                     }
                 }
+                __syncwarp();
                 run += tot;
             }
         }
@@ -693,37 +714,60 @@ __global__ void __launch_bounds__(kExpandThreads, 8) expand_kernel(ExpandArgs a)
         atomicMax(&a.stats[xl].t1, globaltimer());
 }
 
+__global__ void map_parent_kernel(const uint32_t *pin, const uint32_t *old_of_new, uint32_t *pout, uint64_t n)
+{
+    for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x) {
+        const uint32_t p = pin[i];
+        pout[old_of_new[i]] = p == FULL ? FULL : old_of_new[p];
+    }
+}
 
 }  // namespace
 
+cudaError_t launch_map_parent(const uint32_t *pin, const uint32_t *old_of_new, uint32_t *pout, uint64_t n,
+                              cudaStream_t s)
+{
+    const unsigned blocks = (unsigned)std::max<uint64_t>(1, std::min<uint64_t>((n + 255) / 256, 148 * 16));
+    map_parent_kernel<<<blocks, 256, 0, s>>>(pin, old_of_new, pout, n);
+    return cudaGetLastError();
+}
+
+size_t expand_smem_bytes() { return (size_t)kHotWords * 4 + (size_t)kExpandWarps * sizeof(WarpSmem); }
+
+static cudaError_t expand_set_attrs()
+{
+    static bool done = false;
+    if (done) return cudaSuccess;
+    const int bytes = (int)expand_smem_bytes();
+    cudaError_t e = cudaFuncSetAttribute(expand_kernel<kModeVisit>, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes);
+    if (e == cudaSuccess)
+        e = cudaFuncSetAttribute(expand_kernel<kModeVisitParent>, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes);
+    if (e == cudaSuccess)
+        e = cudaFuncSetAttribute(expand_kernel<kModeDecode>, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes);
+    if (e == cudaSuccess) done = true;
+    return e;
+}
+
 int expand_occupancy(int mode)
 {
-    int nb = 0;
-    switch (mode) {
-    case kModeVisit:
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, expand_kernel<kModeVisit>, kExpandThreads, 0);
-        break;
-    case kModeVisitParent:
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, expand_kernel<kModeVisitParent>, kExpandThreads, 0);
-        break;
-    default:
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, expand_kernel<kModeDecode>, kExpandThreads, 0);
-        break;
-    }
-    return nb > 0 ? nb : 1;
+    (void)mode;
+    return 1;  // one CTA per SM (shared-memory resident hot bitmap)
 }
 
 cudaError_t launch_expand(int mode, const ExpandArgs &a, int blocks, cudaStream_t s)
 {
+    cudaError_t e = expand_set_attrs();
+    if (e != cudaSuccess) return e;
+    const size_t sm = expand_smem_bytes();
     switch (mode) {
     case kModeVisit:
-        expand_kernel<kModeVisit><<<blocks, kExpandThreads, 0, s>>>(a);
+        expand_kernel<kModeVisit><<<blocks, kExpandThreads, sm, s>>>(a);
         break;
     case kModeVisitParent:
-        expand_kernel<kModeVisitParent><<<blocks, kExpandThreads, 0, s>>>(a);
+        expand_kernel<kModeVisitParent><<<blocks, kExpandThreads, sm, s>>>(a);
         break;
     default:
-        expand_kernel<kModeDecode><<<blocks, kExpandThreads, 0, s>>>(a);
+        expand_kernel<kModeDecode><<<blocks, kExpandThreads, sm, s>>>(a);
         break;
     }
     return cudaGetLastError();

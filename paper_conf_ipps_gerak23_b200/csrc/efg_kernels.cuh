@@ -23,6 +23,7 @@ struct ExpandArgs {
     uint32_t *out;             // decode output (mode 2)
     LevelStat *stats;          // per-level statistics (device) or null
     uint32_t max_stats;
+    uint32_t hot_words;        // bitmap words with a shared-memory snapshot (multiple of 4)
     uint32_t k;                // forward-pointer quantum (chunk length); 0 = none
     int32_t kshift;            // log2(k) if k is a power of two, else -1
 };
@@ -38,6 +39,7 @@ struct InitArgs {
 struct CompactArgs {
     uint32_t *vis, *prev;      // visited bitmap now / at the previous level end
     uint32_t *queue;           // out: next frontier, sorted
+    const uint32_t *idmap;     // stored id -> input id for depth (EFG_REORDER_DEGREE) or null
     LevelCtrl *ctrl;           // in: level, seq, depth ptr; out: nf
     uint64_t *status;          // cross-block prefix words (one per block)
     uint64_t nwords, words_per_block;
@@ -61,5 +63,9 @@ cudaError_t launch_init(const InitArgs &a, cudaStream_t s);
 cudaError_t launch_compact(const CompactArgs &a, unsigned blocks, cudaStream_t s);
 cudaError_t launch_plan(const PlanArgs &a, unsigned blocks, cudaStream_t s);
 int expand_occupancy(int mode);
+size_t expand_smem_bytes();
+// pout[old_of_new[i]] = pin[i] == ~0u ? ~0u : old_of_new[pin[i]]  (parents back to input ids)
+cudaError_t launch_map_parent(const uint32_t *pin, const uint32_t *old_of_new, uint32_t *pout, uint64_t n,
+                              cudaStream_t s);
 
 }  // namespace efg

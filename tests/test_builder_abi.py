@@ -121,3 +121,31 @@ def test_partition_balanced_and_aligned():
         w = (np.diff(offsets).astype(np.float64) + 29.0)
         share = np.array([w[int(b[r]):int(b[r + 1])].sum() for r in range(world)])
         assert share.max() <= w.sum() / world + 64 * (w.max() + 29)
+
+
+def _degree_order(vlist):
+    """Expected EFG_REORDER_DEGREE relabelling: degree descending, ties by id."""
+    deg = np.diff(vlist).astype(np.int64)
+    n = deg.size
+    old_of_new = np.lexsort((np.arange(n), -deg)).astype(np.uint32)
+    new_of_old = np.empty(n, np.uint32)
+    new_of_old[old_of_new] = np.arange(n, dtype=np.uint32)
+    return old_of_new, new_of_old
+
+
+def test_reorder_degree_byte_identical_to_oracle_on_relabelled_graph():
+    import paper_conf_ipps_gerak23_b200 as efg
+    n, src, dst = synth.rmat(12, 16, seed=9)
+    g = efg.Graph.build(n, src, dst, device=-1,
+                        flags=efg.EFG_DEFAULT_FLAGS | efg.EFG_REORDER_DEGREE)
+    ov, oe = oracle.csr_build(n, src, dst)
+    old_of_new, new_of_old = _degree_order(ov)
+    assert np.array_equal(g.perm(), old_of_new)
+    rv, re_ = oracle.csr_build(n, new_of_old[src], new_of_old[dst])
+    oo, onlb, odata = oracle.efg_encode(rv, re_, 512)
+    vlist, nlb, offsets, data = g.export()
+    assert np.array_equal(vlist, rv) and np.array_equal(offsets, oo)
+    assert np.array_equal(nlb, onlb) and np.array_equal(data, odata)
+    # degrees are non-increasing in the stored order
+    assert np.all(np.diff(np.diff(vlist).astype(np.int64)) <= 0)
+    g.free()

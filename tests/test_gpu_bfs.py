@@ -243,3 +243,35 @@ def test_long_path_many_levels(efg):
     assert np.array_equal(d, np.arange(n))
     assert st["levels"] == n and st["vertices_reached"] == n
     g.free()
+
+
+def test_reorder_degree_bfs_in_input_ids(efg):
+    n, src, dst = synth.rmat(14, 16, seed=11)
+    g = efg.Graph.build(n, src, dst, flags=efg.EFG_DEFAULT_FLAGS | efg.EFG_REORDER_DEGREE)
+    ov, oe = oracle.csr_build(n, src, dst)
+    # decode describes the relabelled graph
+    p = g.perm()
+    new_of_old = np.empty(n, np.uint32)
+    new_of_old[p] = np.arange(n, dtype=np.uint32)
+    rv, re_ = oracle.csr_build(n, new_of_old[src], new_of_old[dst])
+    assert np.array_equal(g.decode(0, n), re_)
+    # traversal inputs and outputs are in input ids
+    _check_bfs(g, ov, oe, [0, 1, 5, n - 1, 4321])
+    for s in (0, 99):
+        d, par, _ = g.bfs(s, parent=True, stats=True)
+        assert np.array_equal(d, oracle.bfs(ov, oe, s))
+        assert par[s] == s
+        for v in np.flatnonzero(d > 0)[:2000]:
+            pv = int(par[v])
+            assert d[pv] == d[v] - 1 and v in oe[ov[pv]:ov[pv + 1]]
+    g.free()
+
+
+def test_hot_snapshot_boundary(efg):
+    # graph larger than the shared-memory hot range (917,504 ids): probes on both sides
+    n, src, dst = synth.rmat(20, 8, seed=12)
+    for flags in (efg.EFG_DEFAULT_FLAGS, efg.EFG_DEFAULT_FLAGS | efg.EFG_REORDER_DEGREE):
+        g = efg.Graph.build(n, src, dst, flags=flags)
+        ov, oe = oracle.csr_build(n, src, dst)
+        _check_bfs(g, ov, oe, [0, 917503, 917504, n - 1])
+        g.free()
