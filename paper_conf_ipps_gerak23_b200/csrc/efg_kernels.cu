@@ -420,14 +420,12 @@ __global__ void __launch_bounds__(kFrontierThreads) plan_kernel(PlanArgs a)
 //   popcount + warp exclusive scan -> rank of each word's first stop bit (the
 //                                     segmented scan of P:171-177; segments are
 //                                     chunks, whose element prefix is subtracted)
-//   element-balanced assignment     -> lane i decodes elements [i*T/32, (i+1)*T/32)
-//                                     of the step's T elements: its first word by
-//                                     binsearch_maxle over the word prefix (Fig. 4
-//                                     rule), the in-word start by clearing
-//                                     set bits, then serially select1(i) - i by
-//                                     ffs-and-clear and the lower bits from a bit
-//                                     buffer streamed over the lower section;
-//                                     x = hi << l | lo, visited kVisitBatch at a time.
+//   set-bit enumeration (ffs)       -> select1(i) - i per element, staged in
+//                                     shared memory by element slot (Alg. 2's
+//                                     select step, without its byte LUT)
+//   balanced pass, element e on lane e%32, kVisitBatch in flight, branch-free
+//                                   -> lower bits by a funnel shift of two
+//                                     coalesced words, x = hi << l | lo, visit.
 // Visit: the first hot_words*32 vertex ids (the highest-degree vertices when the
 // graph was built with EFG_REORDER_DEGREE) have a per-CTA shared-memory copy of
 // their visited bits, loaded at kernel start (a snapshot of the level start,
@@ -448,12 +446,11 @@ struct SlotMeta {
 };
 
 struct WarpSmem {
-    uint32_t wd[32];     // the step's upper words (masked)
-    uint32_t hb[32];     // per word: select1 - i of its first stop bit, minus its position
-    uint8_t ws[32];      // per word: chunk slot
+    uint32_t hi[kExpandStage];  // select1(i) - i by element slot of the step
+    uint8_t cs[kExpandStage];   // chunk slot of the element
     SlotGeom geom[32];
     SlotMeta meta[32];
-    uint64_t aux[32];    // parent: source vertex; decode: output index base
+    uint64_t aux[32];           // parent: source vertex; decode: output index base
 };
 
 struct WordLd {
@@ -483,33 +480,6 @@ __device__ __forceinline__ WordLd load_word(const uint32_t *data32, const SlotGe
     }
     return r;
 }
-
-// Lower-bits stream of one lane: `buf` holds nb >= 32 valid bits (l <= 31).
-struct LowerStream {
-    const uint32_t *lp;
-    uint64_t buf;
-    uint32_t nb;
-    __device__ __forceinline__ void init(const uint32_t *data32, uint64_t ba)
-    {
-        lp = data32 + (ba >> 5);
-        const uint32_t sh = (uint32_t)(ba & 31);
-        buf = (((uint64_t)ldg_u32(lp + 1) << 32) | ldg_u32(lp)) >> sh;
-        nb = 64 - sh;
-        lp += 2;
-    }
-    __device__ __forceinline__ uint32_t next(uint32_t l, uint32_t lmask)
-    {
-        const uint32_t lo = (uint32_t)buf & lmask;
-        buf >>= l;
-        nb -= l;
-        if (nb < 32) {
-            buf |= (uint64_t)ldg_u32(lp) << nb;
-            ++lp;
-            nb += 32;
-        }
-        return lo;
-    }
-};
 
 constexpr int kVisitBatch = 4;  // decoded elements per lane whose probes are in flight together
 
@@ -659,84 +629,69 @@ __global__ void __launch_bounds__(kExpandThreads, 1) expand_kernel(ExpandArgs a)
                 if (g0 + 32 < W) nxt = load_word(data32, ws.geom, wb, g0 + 32 + lane, W);
                 uint32_t tot;
                 const uint32_t ep = warp_excl_u32(__popc(cur.word), tot);
-                {
-                    uint32_t hbw = 0;
-                    if (cur.word) {
-                        const SlotGeom &sg = ws.geom[cur.s];
-                        const uint64_t rank = sg.r0 + run + ep - sg.eb;  // rank of the first set bit
-                        hbw = (uint32_t)(cur.wi * 32 - sg.U0 - rank);    // hi = hbw + p - (index in word)
-                    }
-                    ws.wd[lane] = cur.word;
-                    ws.hb[lane] = hbw;
-                    ws.ws[lane] = (uint8_t)cur.s;
+                // set-bit enumeration: select1(i) - i of every element, by slot
+                if (cur.word) {
+                    const SlotGeom &sg = ws.geom[cur.s];
+                    const uint64_t rank = sg.r0 + run + ep - sg.eb;  // rank of the first set bit
+                    uint32_t hb = (uint32_t)(cur.wi * 32 - sg.U0 - rank);  // hi = hb + p, hb -= 1 per bit
+                    uint32_t w = cur.word, e = ep;
+                    const uint8_t sc = (uint8_t)cur.s;
+                    do {
+                        ws.hi[e] = hb + (__ffs(w) - 1);
+                        ws.cs[e] = sc;
+                        w &= w - 1;
+                        --hb;
+                        ++e;
+                    } while (w);
                 }
                 __syncwarp();
-                // element-balanced assignment of the step's tot elements
-                const uint32_t e0 = (lane * tot) >> 5, e1 = ((lane + 1) * tot) >> 5;
-                int w = warp_maxle_u32(ep, e0);
-                const uint32_t k = e0 - __shfl_sync(FULL, ep, w);
-                if (e0 < e1) {
-                    uint32_t wd = ws.wd[w], hb = ws.hb[w] - k;
-                    for (uint32_t t = 0; t < k; ++t) wd &= wd - 1;
-                    int s = ws.ws[w];
-                    SlotMeta m = ws.meta[s];
-                    LowerStream ls;
-                    if (m.l) ls.init(data32, m.lb + (uint64_t)(run + e0) * m.l);
-                    for (uint32_t e = e0; e < e1; e += kVisitBatch) {
-                        uint32_t xv[kVisitBatch];
-                        uint32_t sv[kVisitBatch];
+                // balanced pass: element e on lane e % 32, kVisitBatch in flight,
+                // written branch-free (slots past the step are computed and masked)
+                for (uint32_t base = 0; base < tot; base += 32 * kVisitBatch) {
+                    uint32_t xv[kVisitBatch], sv[kVisitBatch];
+                    bool ok[kVisitBatch];
+#pragma unroll
+                    for (int u = 0; u < kVisitBatch; ++u) {
+                        const uint32_t e = base + u * 32 + lane;
+                        ok[u] = e < tot;
+                        const uint32_t es = ok[u] ? e : 0;
+                        const uint32_t hi = ws.hi[es];
+                        sv[u] = ws.cs[es];
+                        const SlotMeta m = ws.meta[sv[u]];
+                        const uint64_t ba = m.lb + (uint64_t)(run + es) * m.l;
+                        const uint32_t *p = data32 + (ba >> 5);
+                        const uint32_t lo =
+                            __funnelshift_r(ldg_u32(p), ldg_u32(p + 1), (uint32_t)(ba & 31)) & m.lmask;
+                        xv[u] = (hi << m.l) | lo;  // (select1(i) - i) << l | lower[i]
+                    }
+                    if (MODE == kModeDecode) {
+#pragma unroll
+                        for (int u = 0; u < kVisitBatch; ++u)
+                            if (ok[u]) a.out[ws.aux[sv[u]] + run + base + u * 32 + lane] = xv[u];
+                    } else {
+                        // Alg. 1 line 3: hot ids answer from shared memory
+                        bool need[kVisitBatch], hot[kVisitBatch];
 #pragma unroll
                         for (int u = 0; u < kVisitBatch; ++u) {
-                            xv[u] = 0;
-                            sv[u] = s;
-                            if (e + u < e1) {
-                                while (wd == 0) {  // next word of the step
-                                    ++w;
-                                    wd = ws.wd[w];
-                                    hb = ws.hb[w];
-                                    if (ws.ws[w] != s) {  // next chunk: restart the lower stream
-                                        s = ws.ws[w];
-                                        m = ws.meta[s];
-                                        if (m.l) ls.init(data32, m.lb + (uint64_t)(run + e + u) * m.l);
-                                    }
-                                }
-                                const uint32_t hi = hb + (__ffs(wd) - 1);  // select1(i) - i
-                                wd &= wd - 1;
-                                --hb;
-                                const uint32_t lo = m.l ? ls.next(m.l, m.lmask) : 0u;
-                                xv[u] = (hi << m.l) | lo;
-                                sv[u] = s;
-                            }
+                            hot[u] = ok[u] && xv[u] < hot_limit;
+                            const uint32_t hw = hot[u] ? s_hot[xv[u] >> 5] : 0u;
+                            need[u] = ok[u] && !((hw >> (xv[u] & 31)) & 1);
                         }
-                        if (MODE == kModeDecode) {
+                        uint32_t gwd[kVisitBatch];
 #pragma unroll
-                            for (int u = 0; u < kVisitBatch; ++u)
-                                if (e + u < e1) a.out[ws.aux[sv[u]] + run + e + u] = xv[u];
-                        } else {
-                            // Alg. 1 line 3: hot ids answer from shared memory
-                            bool need[kVisitBatch];
+                        for (int u = 0; u < kVisitBatch; ++u) gwd[u] = need[u] ? a.vis[xv[u] >> 5] : FULL;
 #pragma unroll
-                            for (int u = 0; u < kVisitBatch; ++u) {
-                                need[u] = e + u < e1;
-                                if (need[u] && xv[u] < hot_limit)
-                                    need[u] = !((s_hot[xv[u] >> 5] >> (xv[u] & 31)) & 1);
-                            }
-                            uint32_t gwd[kVisitBatch];
-#pragma unroll
-                            for (int u = 0; u < kVisitBatch; ++u) gwd[u] = need[u] ? a.vis[xv[u] >> 5] : FULL;
-#pragma unroll
-                            for (int u = 0; u < kVisitBatch; ++u) {
-                                const uint32_t bit = 1u << (xv[u] & 31);
-                                if (!(gwd[u] & bit)) {  // line 4 (stale reads are benign: the atomic decides)
-                                    if (MODE == kModeVisit) {
-                                        atomicOr(a.vis + (xv[u] >> 5), bit);
-                                    } else {
-                                        const uint32_t old = atomicOr(a.vis + (xv[u] >> 5), bit);
-                                        if (!(old & bit)) parent[xv[u]] = (uint32_t)ws.aux[sv[u]];
-                                    }
+                        for (int u = 0; u < kVisitBatch; ++u) {
+                            const uint32_t bit = 1u << (xv[u] & 31);
+                            if (!(gwd[u] & bit)) {  // line 4 (stale reads are benign: the atomic decides)
+                                if (MODE == kModeVisit) {
+                                    atomicOr(a.vis + (xv[u] >> 5), bit);
+                                } else {
+                                    const uint32_t old = atomicOr(a.vis + (xv[u] >> 5), bit);
+                                    if (!(old & bit)) parent[xv[u]] = (uint32_t)ws.aux[sv[u]];
                                 }
-                                if (need[u] && xv[u] < hot_limit) atomicOr(s_hot + (xv[u] >> 5), bit);
                             }
+                            if (need[u] && hot[u]) atomicOr(s_hot + (xv[u] >> 5), bit);
                         }
                     }
                 }
