@@ -93,9 +93,9 @@ struct LevelStat {
 };
 constexpr uint32_t kMaxLevelStats = 4096;
 
-constexpr int kExpandThreads = 512;          // one CTA per SM, 16 warps
+constexpr int kExpandThreads = 768;          // one CTA per SM, 24 warps
 constexpr int kExpandWarps = kExpandThreads / 32;
-constexpr int kExpandStage = 1024;           // elements of one 32-word step (<= 32*32)
+constexpr int kExpandStage = 512;            // elements of one 16-word step (<= 16*32)
 constexpr uint32_t kHotWords = 28 * 1024;    // 112 KB shared-memory visited snapshot = 917,504 ids
 constexpr int kFrontierThreads = 256;        // compact / plan kernels
 constexpr int kBitmapAlign = 1024;           // bitmap words are padded to a multiple of this

@@ -439,7 +439,7 @@ struct SlotGeom {
     uint64_t r0;          // rank of the chunk's first element in its list
 };
 
-struct SlotMeta {
+struct alignas(16) SlotMeta {
     uint64_t lb;     // lower-bit address of batch element e: lb + e*l (modular)
     uint32_t l;      // lower bits per element
     uint32_t lmask;  // (1 << l) - 1
@@ -479,6 +479,20 @@ __device__ __forceinline__ WordLd load_word(const uint32_t *data32, const SlotGe
         r.word = word;
     }
     return r;
+}
+
+// Lane l of a step handles the 16-bit half (l & 1) of batch word g0 + (l >> 1).
+__device__ __forceinline__ WordLd load_half(const uint32_t *data32, const SlotGeom *geom, uint32_t wb,
+                                            uint32_t lane, uint32_t g0, uint32_t W)
+{
+    WordLd r = load_word(data32, geom, wb, g0 + (lane >> 1), W);
+    r.word = (lane & 1) ? (r.word >> 16) : (r.word & 0xffffu);
+    return r;
+}
+
+__device__ __forceinline__ void prefetch_l2(const void *p)
+{
+    asm volatile("prefetch.global.L2 [%0];" ::"l"(p));
 }
 
 constexpr int kVisitBatch = 4;  // decoded elements per lane whose probes are in flight together
@@ -597,6 +611,12 @@ __global__ void __launch_bounds__(kExpandThreads, 1) expand_kernel(ExpandArgs a)
                 m.l = l;
                 m.lmask = l ? (FULL >> (32 - l)) : 0u;
                 ws.meta[lane] = m;
+                // pull the chunk's lower and upper bits toward L2 ahead of the word steps
+                {
+                    const uint64_t lb0 = (lbase + r0 * l) >> 3, lb1 = (lbase + (r0 + nel) * l + 7) >> 3;
+                    for (uint64_t q = lb0 & ~127ull; q < lb1; q += 128) prefetch_l2(a.data + q);
+                    for (uint64_t q = (A0 >> 3) & ~127ull; q < ((A1 + 7) >> 3); q += 128) prefetch_l2(a.data + q);
+                }
                 if (MODE == kModeVisitParent) ws.aux[lane] = v_j;
                 // decode: CSR position of the chunk's first element E_v + r0, E_v = W_v - A*q_v
                 if (MODE == kModeDecode) ws.aux[lane] = Wv_j - A * (fi + (uint64_t)j) + r0 - ebt;
@@ -621,19 +641,20 @@ __global__ void __launch_bounds__(kExpandThreads, 1) expand_kernel(ExpandArgs a)
             }
             __syncwarp();
 
-            // ---- a5 + a6: 32 upper-bit words per step ----
+            // ---- a5 + a6: 16 upper-bit words per step, one 16-bit half per lane ----
             uint32_t run = 0;
-            WordLd nxt = load_word(data32, ws.geom, wb, lane, W);
-            for (uint32_t g0 = 0; g0 < W; g0 += 32) {
+            WordLd nxt = load_half(data32, ws.geom, wb, lane, 0, W);
+            for (uint32_t g0 = 0; g0 < W; g0 += 16) {
                 const WordLd cur = nxt;
-                if (g0 + 32 < W) nxt = load_word(data32, ws.geom, wb, g0 + 32 + lane, W);
+                if (g0 + 16 < W) nxt = load_half(data32, ws.geom, wb, lane, g0 + 16, W);
                 uint32_t tot;
                 const uint32_t ep = warp_excl_u32(__popc(cur.word), tot);
                 // set-bit enumeration: select1(i) - i of every element, by slot
                 if (cur.word) {
                     const SlotGeom &sg = ws.geom[cur.s];
                     const uint64_t rank = sg.r0 + run + ep - sg.eb;  // rank of the first set bit
-                    uint32_t hb = (uint32_t)(cur.wi * 32 - sg.U0 - rank);  // hi = hb + p, hb -= 1 per bit
+                    // hi = hb + p (p = bit within the half), hb -= 1 per bit
+                    uint32_t hb = (uint32_t)(cur.wi * 32 + (lane & 1) * 16 - sg.U0 - rank);
                     uint32_t w = cur.word, e = ep;
                     const uint8_t sc = (uint8_t)cur.s;
                     do {
