@@ -53,7 +53,6 @@ typedef enum efg_status {
 #define EFG_DEFAULT_FLAGS (EFG_SYMMETRIZE | EFG_DEDUP | EFG_DROP_SELF_LOOPS)
 
 typedef struct efg_graph efg_graph; /* opaque: host EFG arrays + device copy */
-typedef struct efg_dist efg_dist;   /* opaque: multi-GPU communicator        */
 
 typedef struct efg_build_opts {
     /* Forward-pointer quantum k (§VI-C; k = 512 in the paper's
@@ -73,10 +72,11 @@ typedef struct efg_build_opts {
      * NULL = unweighted.  Weights of duplicate (s,d) pairs: the minimum is kept.
      * With EFG_SYMMETRIZE the reverse edge gets the same weight. */
     const float *weights;
-    /* Multi-GPU: NULL = the whole graph on `device`.  Otherwise this rank keeps
-     * the row range [row_lo, row_hi) chosen by efg_partition (1-D partition,
-     * SURVEY §8(e)); every rank passes the same edge list. */
-    efg_dist *dist;
+    /* 1-D row partition: when row_hi > row_lo this handle encodes
+     * and uploads only the lists of rows [row_lo, row_hi) (e.g. a range from
+     * efg_partition); all other vertices keep empty lists.  Every rank passes
+     * the same edge list.  0, 0 = the whole graph. */
+    uint64_t row_lo, row_hi;
 } efg_build_opts;
 
 /* Fill *o with the defaults above (k = 512, EFG_DEFAULT_FLAGS, device 0). */
@@ -206,23 +206,50 @@ efg_status efg_pagerank(efg_graph *g, double damping, uint32_t iters, double *ra
  * EFG_ESTATE (host-only handle). */
 efg_status efg_set_option(efg_graph *g, int option, int64_t value);
 
-/* ---- multi-GPU: 1-D row partition, per-level exchange ---- */
+/* ---- multi-GPU: 1-D row partition, per-level exchange ----
+ *
+ * One process per GPU; rank r's handle holds rows [bounds[r], bounds[r+1]).
+ * A partitioned BFS is driven level by level (all ranks in lock step):
+ *   efg_bfs_begin                 source, level 0
+ *   repeat:
+ *     efg_bfs_expand              decode + visit the rank's own frontier rows
+ *                                 (discoveries land in the rank's full-width
+ *                                 visited bitmap)
+ *     efg_xchg_pack               slice h of this rank's new bits -> send[h*S ..]
+ *     (caller) all-to-all         send -> recv   (e.g. torch.distributed over NCCL)
+ *     efg_xchg_reduce             OR of the P received slices -> mine[0..S)
+ *     (caller) all-gather         mine -> gathered[P*S]
+ *     efg_xchg_unpack             visited |= gathered (same global bitmap on all ranks)
+ *     efg_bfs_finish_level        next frontier = new owned vertices, depth of all
+ *                                 new vertices; returns the GLOBAL new count
+ *   until the global new count is 0;  efg_bfs_end.
+ * The library provides every computation; the caller only moves bytes.  S =
+ * slice length in 32-bit words (the largest owner range, see efg_xchg_geometry).
+ * All buffers are device pointers on the handle's device; calls are ordered on
+ * the handle's stream (efg_bfs_finish_level synchronises it).
+ */
 
-/* 128-byte opaque id (an ncclUniqueId).  Rank 0 creates it and the caller
- * broadcasts it (e.g. over torch.distributed) to every rank. */
-efg_status efg_get_unique_id(uint8_t id[128]);
+/* bounds[world+1] vertex boundaries (multiples of 64, bounds[world] = n).
+ * Writes the slice length S in 32-bit words (max over ranks). */
+efg_status efg_xchg_geometry(const efg_graph *g, int world, const uint64_t *bounds, uint64_t *slice_words);
 
-/* Create this rank's communicator (ranks 0..world-1, one GPU per rank). */
-efg_status efg_dist_init(int rank, int world, const uint8_t id[128], int device,
-                         efg_dist **out);
-void efg_dist_free(efg_dist *d);
+efg_status efg_bfs_begin(efg_graph *g, uint32_t source, int32_t *depth_device);
+efg_status efg_bfs_expand(efg_graph *g);
+efg_status efg_xchg_pack(efg_graph *g, int world, const uint64_t *bounds, uint64_t slice_words,
+                         uint32_t *send);
+efg_status efg_xchg_reduce(efg_graph *g, int world, uint64_t slice_words, const uint32_t *recv,
+                           uint32_t *mine);
+efg_status efg_xchg_unpack(efg_graph *g, int world, const uint64_t *bounds, uint64_t slice_words,
+                           const uint32_t *gathered);
+efg_status efg_bfs_finish_level(efg_graph *g, uint64_t *global_new);
+efg_status efg_bfs_end(efg_graph *g, efg_stats *st);
 
 /*
- * efg_partition — the 1-D row partition used by efg_build with opts->dist:
+ * efg_partition — the 1-D row partition (efg_build_opts.row_lo / row_hi):
  * rank r owns vertices [bounds[r], bounds[r+1]).  Boundaries balance
  * sum(offsets bytes) + 29 bytes per vertex and are multiples
  * of 64 (so bitmap words have one owner).  bounds: world+1 entries.
- * Host-only computation over the CSR degrees implied by (n, m, src, dst, flags).
+ * Host-only computation over the P:113 vlist/offsets arrays of the whole graph.
  */
 efg_status efg_partition(uint64_t n, const uint64_t *vlist, const uint64_t *offsets, int world,
                          uint64_t *bounds);

@@ -52,7 +52,8 @@ class Graph:
     # -- construction -----------------------------------------------------
     @classmethod
     def build(cls, n: int, src, dst, *, k: int = 512, flags: int = EFG_DEFAULT_FLAGS,
-              device: int = 0, stream: int | None = None, weights=None, n_threads: int = 0):
+              device: int = 0, stream: int | None = None, weights=None, n_threads: int = 0,
+              rows: tuple[int, int] | None = None):
         """efg_build: host edge arrays (uint32) -> EFG handle (uploaded to `device`).
 
         `stream` is a cudaStream_t as an int (e.g. ``torch.cuda.current_stream().cuda_stream``);
@@ -68,6 +69,8 @@ class Graph:
         o.device = device
         o.n_threads = n_threads
         o.stream = stream
+        if rows is not None:
+            o.row_lo, o.row_hi = int(rows[0]), int(rows[1])
         w = None
         if weights is not None:
             w = np.ascontiguousarray(weights, dtype=np.float32)
@@ -174,6 +177,46 @@ class Graph:
                   "level_edges": arrs[1][:min(L, level_cap)].copy(),
                   "level_expand_ms": arrs[2][:min(L, level_cap)].copy()}
         return depth, par, sd
+
+    # -- stepwise partitioned BFS (efg.h "multi-GPU"); device buffers only --
+    def xchg_geometry(self, bounds: np.ndarray) -> int:
+        b = np.ascontiguousarray(bounds, np.uint64)
+        S = C.c_uint64()
+        check(lib.efg_xchg_geometry(self._h, b.size - 1, _ptr(b), C.byref(S)), "efg_xchg_geometry")
+        return S.value
+
+    def bfs_begin(self, source: int, depth) -> None:
+        check(lib.efg_bfs_begin(self._h, source, _ptr(depth)), "efg_bfs_begin")
+
+    def bfs_expand(self) -> None:
+        check(lib.efg_bfs_expand(self._h), "efg_bfs_expand")
+
+    def xchg_pack(self, bounds: np.ndarray, S: int, send) -> None:
+        b = np.ascontiguousarray(bounds, np.uint64)
+        check(lib.efg_xchg_pack(self._h, b.size - 1, _ptr(b), S, _ptr(send)), "efg_xchg_pack")
+
+    def xchg_reduce(self, world: int, S: int, recv, mine) -> None:
+        check(lib.efg_xchg_reduce(self._h, world, S, _ptr(recv), _ptr(mine)), "efg_xchg_reduce")
+
+    def xchg_unpack(self, bounds: np.ndarray, S: int, gathered) -> None:
+        b = np.ascontiguousarray(bounds, np.uint64)
+        check(lib.efg_xchg_unpack(self._h, b.size - 1, _ptr(b), S, _ptr(gathered)), "efg_xchg_unpack")
+
+    def bfs_finish_level(self) -> int:
+        n = C.c_uint64()
+        check(lib.efg_bfs_finish_level(self._h, C.byref(n)), "efg_bfs_finish_level")
+        return n.value
+
+    def bfs_end(self, level_cap: int = 256) -> dict:
+        st = _abi.Stats()
+        st.level_cap = level_cap
+        lf, le = np.zeros(level_cap, np.uint64), np.zeros(level_cap, np.uint64)
+        st.level_frontier, st.level_edges = lf.ctypes.data, le.ctypes.data
+        check(lib.efg_bfs_end(self._h, C.byref(st)), "efg_bfs_end")
+        L = min(st.levels + 1, level_cap)
+        return {"levels": st.levels, "edges_traversed": st.edges_traversed,
+                "vertices_reached": st.vertices_reached, "level_frontier": lf[:L].copy(),
+                "level_edges": le[:L].copy()}
 
     def sssp(self, source: int, dist=None, stats: bool = False):
         n = self.info["n"]

@@ -24,7 +24,7 @@ EFG_OPT_LEVEL_LOOP = 1
 class BuildOpts(C.Structure):
     _fields_ = [("fwd_quantum", C.c_uint32), ("flags", C.c_uint32), ("device", C.c_int32),
                 ("n_threads", C.c_uint32), ("stream", C.c_void_p), ("weights", C.c_void_p),
-                ("dist", C.c_void_p)]
+                ("row_lo", C.c_uint64), ("row_hi", C.c_uint64)]
 
 
 class Info(C.Structure):
@@ -59,9 +59,14 @@ SIGNATURES = [
     ("efg_sssp", C.c_int, [C.c_void_p, C.c_uint32, C.c_void_p, C.POINTER(Stats)]),
     ("efg_pagerank", C.c_int, [C.c_void_p, C.c_double, C.c_uint32, C.c_void_p, C.POINTER(Stats)]),
     ("efg_set_option", C.c_int, [C.c_void_p, C.c_int, C.c_int64]),
-    ("efg_get_unique_id", C.c_int, [C.c_void_p]),
-    ("efg_dist_init", C.c_int, [C.c_int, C.c_int, C.c_void_p, C.c_int, C.POINTER(C.c_void_p)]),
-    ("efg_dist_free", None, [C.c_void_p]),
+    ("efg_xchg_geometry", C.c_int, [C.c_void_p, C.c_int, C.c_void_p, C.POINTER(C.c_uint64)]),
+    ("efg_bfs_begin", C.c_int, [C.c_void_p, C.c_uint32, C.c_void_p]),
+    ("efg_bfs_expand", C.c_int, [C.c_void_p]),
+    ("efg_xchg_pack", C.c_int, [C.c_void_p, C.c_int, C.c_void_p, C.c_uint64, C.c_void_p]),
+    ("efg_xchg_reduce", C.c_int, [C.c_void_p, C.c_int, C.c_uint64, C.c_void_p, C.c_void_p]),
+    ("efg_xchg_unpack", C.c_int, [C.c_void_p, C.c_int, C.c_void_p, C.c_uint64, C.c_void_p]),
+    ("efg_bfs_finish_level", C.c_int, [C.c_void_p, C.POINTER(C.c_uint64)]),
+    ("efg_bfs_end", C.c_int, [C.c_void_p, C.POINTER(Stats)]),
     ("efg_partition", C.c_int, [C.c_uint64, C.c_void_p, C.c_void_p, C.c_int, C.c_void_p]),
     ("efg_last_error", C.c_char_p, []),
     ("efg_version", C.c_char_p, []),

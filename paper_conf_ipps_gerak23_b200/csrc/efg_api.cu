@@ -60,7 +60,8 @@ extern "C" efg_status efg_build(uint64_t n, uint64_t m, const uint32_t *src, con
         efg_default_opts(&o);
     if (n == 0 || n > 0xFFFFFFFFull) return set_error(EFG_EINVAL, "efg_build: need 1 <= n <= 2^32-1");
     if (m && (!src || !dst)) return set_error(EFG_EINVAL, "efg_build: src/dst is NULL");
-    if (o.dist) return set_error(EFG_ENOTSUP, "efg_build: multi-GPU partition not built into this library");
+    if (o.row_hi > o.row_lo && (o.row_lo % 64 || (o.row_hi % 64 && o.row_hi < n)))
+        return set_error(EFG_EINVAL, "efg_build: row range bounds must be multiples of 64 (or n)");
     efg_graph *g = new (std::nothrow) efg_graph();
     if (!g) return set_error(EFG_ENOMEM, "efg_build: handle allocation failed");
     efg_status st = build_host(n, m, src, dst, o, g->host);
@@ -187,19 +188,77 @@ extern "C" efg_status efg_pagerank(efg_graph *g, double, uint32_t, double *, efg
     return set_error(EFG_ENOTSUP, "efg_pagerank: not implemented yet");
 }
 
-extern "C" efg_status efg_get_unique_id(uint8_t id[128])
+extern "C" efg_status efg_xchg_geometry(const efg_graph *g, int world, const uint64_t *bounds, uint64_t *slice_words)
 {
-    (void)id;
-    return set_error(EFG_ENOTSUP, "efg_get_unique_id: NCCL transport not built");
+    clear_error();
+    if (!g || !bounds || !slice_words || world < 1) return set_error(EFG_EINVAL, "efg_xchg_geometry: bad args");
+    uint64_t s = 0;
+    for (int r = 0; r < world; ++r) {
+        if (bounds[r + 1] < bounds[r] || bounds[r] % 64) return set_error(EFG_EINVAL, "efg_xchg_geometry: bounds");
+        const uint64_t w0 = bounds[r] / 32, w1 = (bounds[r + 1] + 31) / 32;
+        s = std::max<uint64_t>(s, w1 - w0);
+    }
+    *slice_words = s;
+    return EFG_OK;
 }
 
-extern "C" efg_status efg_dist_init(int, int, const uint8_t *, int, efg_dist **out)
+extern "C" efg_status efg_bfs_begin(efg_graph *g, uint32_t source, int32_t *depth_device)
 {
-    if (out) *out = nullptr;
-    return set_error(EFG_ENOTSUP, "efg_dist_init: NCCL transport not built");
+    clear_error();
+    EFG_TRY(check_handle(g));
+    if (source >= g->dev.n) return set_error(EFG_ERANGE, "efg_bfs_begin: source >= n");
+    if (!depth_device) return set_error(EFG_EINVAL, "efg_bfs_begin: depth is NULL");
+    const uint32_t s = g->host.new_of_old.empty() ? source : g->host.new_of_old[source];
+    return device_step_begin(g, s, depth_device);
 }
 
-extern "C" void efg_dist_free(efg_dist *) {}
+extern "C" efg_status efg_bfs_expand(efg_graph *g)
+{
+    clear_error();
+    EFG_TRY(check_handle(g));
+    return device_step_expand(g);
+}
+
+extern "C" efg_status efg_xchg_pack(efg_graph *g, int world, const uint64_t *bounds, uint64_t slice_words,
+                                    uint32_t *send)
+{
+    clear_error();
+    EFG_TRY(check_handle(g));
+    if (world < 1 || !bounds || !send) return set_error(EFG_EINVAL, "efg_xchg_pack: bad args");
+    return device_xchg(g, 0, world, bounds, slice_words, send, nullptr);
+}
+
+extern "C" efg_status efg_xchg_reduce(efg_graph *g, int world, uint64_t slice_words, const uint32_t *recv,
+                                      uint32_t *mine)
+{
+    clear_error();
+    EFG_TRY(check_handle(g));
+    if (world < 1 || !recv || !mine) return set_error(EFG_EINVAL, "efg_xchg_reduce: bad args");
+    return device_xchg(g, 1, world, nullptr, slice_words, mine, recv);
+}
+
+extern "C" efg_status efg_xchg_unpack(efg_graph *g, int world, const uint64_t *bounds, uint64_t slice_words,
+                                      const uint32_t *gathered)
+{
+    clear_error();
+    EFG_TRY(check_handle(g));
+    if (world < 1 || !bounds || !gathered) return set_error(EFG_EINVAL, "efg_xchg_unpack: bad args");
+    return device_xchg(g, 2, world, bounds, slice_words, nullptr, gathered);
+}
+
+extern "C" efg_status efg_bfs_finish_level(efg_graph *g, uint64_t *global_new)
+{
+    clear_error();
+    EFG_TRY(check_handle(g));
+    return device_step_finish(g, global_new);
+}
+
+extern "C" efg_status efg_bfs_end(efg_graph *g, efg_stats *st)
+{
+    clear_error();
+    EFG_TRY(check_handle(g));
+    return device_step_end(g, st);
+}
 
 extern "C" efg_status efg_partition(uint64_t n, const uint64_t *vlist, const uint64_t *offsets, int world,
                                     uint64_t *bounds)

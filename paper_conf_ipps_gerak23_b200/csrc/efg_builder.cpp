@@ -191,7 +191,8 @@ efg_status build_host(uint64_t n, uint64_t m, const uint32_t *src, const uint32_
             deg.swap(deg2);
         }
         // partition: keep only the owned rows' lists
-        const uint64_t lo = o.dist ? out.row_lo : 0, hi = o.dist ? out.row_hi : n;
+        const bool part = o.row_hi > o.row_lo;
+        const uint64_t lo = part ? std::min<uint64_t>(o.row_lo, n) : 0, hi = part ? std::min<uint64_t>(o.row_hi, n) : n;
         for (uint64_t v = 0; v < n; ++v)
             if (v < lo || v >= hi) deg[v] = 0;
         out.vlist.assign(deg.begin(), deg.end());

@@ -14,6 +14,7 @@
 #include <cuda_runtime.h>
 
 #include <algorithm>
+#include <cstddef>
 #include <cstring>
 #include <string>
 #include <vector>
@@ -100,6 +101,8 @@ CompactArgs compact_args(DeviceGraph &d)
     a.status = d.status;
     a.nwords = d.nwords;
     a.words_per_block = d.words_per_block;
+    a.own_lo_w = d.own_lo_w;
+    a.own_hi_w = d.own_hi_w;
     return a;
 }
 
@@ -187,6 +190,7 @@ void device_free(DeviceGraph &d)
     cudaFree(d.old_of_new);
     cudaFree(d.status);
     cudaFree(d.stats);
+    cudaFree(d.xchg_bounds);
     cudaFree(d.ctrl);
     cudaFree(d.fbuf);
     cudaFree(d.dbuf);
@@ -219,6 +223,8 @@ efg_status device_upload(efg_graph *g, const efg_build_opts &o)
     // bitmap geometry
     const uint64_t words = (h.n + 31) / 32;
     d.nwords = (words + kBitmapAlign - 1) / kBitmapAlign * kBitmapAlign;
+    d.own_lo_w = h.row_lo / 32;
+    d.own_hi_w = (h.row_hi + 31) / 32;
 
     // packed vertex records (one 16-byte load per frontier vertex) and degrees
     std::vector<VRec> rec(h.n);
@@ -439,6 +445,105 @@ efg_status device_bfs(efg_graph *g, uint32_t source, int32_t *depth, uint32_t *p
             if (st->level_expand_ms) st->level_expand_ms[i] = lms[i];
         }
     }
+    return EFG_OK;
+}
+
+// ---------------------------------------------------------------------------
+// Stepwise driver of the 1-D partitioned BFS (efg.h "multi-GPU").
+// ---------------------------------------------------------------------------
+efg_status device_step_begin(efg_graph *g, uint32_t source, int32_t *depth)
+{
+    DeviceGraph &d = g->dev;
+    CUDA_TRY(cudaSetDevice(d.device));
+    cudaStream_t s = stream_of(d);
+    if (!is_device_ptr(depth)) return set_error(EFG_EINVAL, "efg_bfs_begin: depth must be a device pointer");
+    d.step_levels = 0;
+    d.step_reached = d.step_edges = 0;
+    d.step_lf.clear();
+    d.step_le.clear();
+    CUDA_TRY(cudaMemsetAsync(depth, 0xFF, d.n * 4, s));
+    uint32_t launches = 0;
+    EFG_TRY(start_traversal(d, source, (uint64_t)source + 1, depth, nullptr, launches));
+    CUDA_TRY(cudaMemcpyAsync(d.ctrl_host, d.ctrl, sizeof(LevelCtrl), cudaMemcpyDeviceToHost, s));
+    CUDA_TRY(cudaStreamSynchronize(s));
+    d.step_lf.push_back(d.ctrl_host->nf);
+    d.step_le.push_back(d.ctrl_host->ne);
+    return EFG_OK;
+}
+
+efg_status device_step_expand(efg_graph *g)
+{
+    DeviceGraph &d = g->dev;
+    CUDA_TRY(cudaSetDevice(d.device));
+    const int blocks = d.num_sms * expand_occupancy(kModeVisit);
+    CUDA_TRY(launch_expand(kModeVisit, expand_args(d, nullptr), blocks, stream_of(d)));
+    ++d.step_levels;
+    return EFG_OK;
+}
+
+efg_status device_step_finish(efg_graph *g, uint64_t *global_new)
+{
+    DeviceGraph &d = g->dev;
+    CUDA_TRY(cudaSetDevice(d.device));
+    cudaStream_t s = stream_of(d);
+    EFG_TRY(launch_level_end(d, 0, s));
+    CUDA_TRY(cudaMemcpyAsync(d.ctrl_host, d.ctrl, sizeof(LevelCtrl), cudaMemcpyDeviceToHost, s));
+    CUDA_TRY(cudaStreamSynchronize(s));
+    const LevelCtrl c = *d.ctrl_host;
+    if (c.nnew) {
+        d.step_lf.push_back(c.nf);
+        d.step_le.push_back(c.ne);
+    }
+    if (global_new) *global_new = c.nnew;
+    return EFG_OK;
+}
+
+efg_status device_step_end(efg_graph *g, efg_stats *st)
+{
+    DeviceGraph &d = g->dev;
+    if (!st) return EFG_OK;
+    uint64_t reached = 0, edges = 0;
+    for (size_t i = 0; i < d.step_lf.size(); ++i) {
+        reached += d.step_lf[i];
+        edges += d.step_le[i];
+    }
+    std::memset(st, 0, offsetof(efg_stats, level_cap));
+    st->levels = d.step_levels;
+    st->edges_traversed = edges;      // this rank's rows
+    st->vertices_reached = reached;   // this rank's rows
+    st->expand_launches = d.step_levels;
+    for (uint32_t i = 0; i < std::min<uint32_t>((uint32_t)d.step_lf.size(), st->level_cap); ++i) {
+        if (st->level_frontier) st->level_frontier[i] = d.step_lf[i];
+        if (st->level_edges) st->level_edges[i] = d.step_le[i];
+    }
+    return EFG_OK;
+}
+
+efg_status device_xchg(efg_graph *g, int op, int world, const uint64_t *bounds, uint64_t slice_words,
+                       uint32_t *out, const uint32_t *in)
+{
+    DeviceGraph &d = g->dev;
+    CUDA_TRY(cudaSetDevice(d.device));
+    cudaStream_t s = stream_of(d);
+    if (op != 1) {
+        if ((uint64_t)world + 1 > d.xchg_bounds_cap) {
+            cudaFree(d.xchg_bounds);
+            d.xchg_bounds = nullptr;
+            EFG_TRY(dev_alloc(d, &d.xchg_bounds, (uint64_t)world + 1));
+            d.xchg_bounds_cap = (uint64_t)world + 1;
+        }
+        CUDA_TRY(cudaMemcpyAsync(d.xchg_bounds, bounds, (world + 1) * 8, cudaMemcpyHostToDevice, s));
+    }
+    XchgArgs a;
+    a.op = op;
+    a.world = world;
+    a.S = slice_words;
+    a.bounds = d.xchg_bounds;
+    a.vis = d.vis;
+    a.prev = d.prev;
+    a.out = out;
+    a.in = in;
+    CUDA_TRY(launch_xchg(a, s));
     return EFG_OK;
 }
 

@@ -82,6 +82,7 @@ struct LevelCtrl {
     uint32_t xlevel;    // index of the level the next expand processes
     uint32_t seq;       // tag of the cross-block prefix words of this level
     uint32_t nlevels;   // levels expanded so far
+    uint64_t nnew;      // vertices discovered in the last level (all rows; partitioned runs)
     uint64_t total_nf;  // sum of frontier sizes (= vertices reached)
     uint64_t total_ne;  // sum of E_L (= edges traversed, reading C18)
 };
@@ -142,6 +143,13 @@ struct DeviceGraph {
     int level_loop = 0;                // 0 = CUDA graph (device loop), 1 = host loop + events
     cudaGraph_t loop_graph[2] = {nullptr, nullptr};      // per mode (visit, visit+parent)
     cudaGraphExec_t loop_exec[2] = {nullptr, nullptr};
+    uint64_t own_lo_w = 0, own_hi_w = 0;   // bitmap words of the owned rows (queue filter)
+    uint64_t *xchg_bounds = nullptr;       // device copy of the partition bounds
+    uint64_t xchg_bounds_cap = 0;
+    // stepwise (partitioned) traversal state
+    uint32_t step_levels = 0;
+    uint64_t step_reached = 0, step_edges = 0;
+    std::vector<uint64_t> step_lf, step_le;
 };
 
 }  // namespace efg
@@ -158,6 +166,13 @@ efg_status device_upload(efg_graph *g, const efg_build_opts &o);
 void device_free(DeviceGraph &d);
 efg_status device_decode(efg_graph *g, uint32_t v0, uint32_t v1, uint32_t *out);
 efg_status device_bfs(efg_graph *g, uint32_t source, int32_t *depth, uint32_t *parent, efg_stats *st);
+efg_status device_step_begin(efg_graph *g, uint32_t source, int32_t *depth);
+efg_status device_step_expand(efg_graph *g);
+efg_status device_step_finish(efg_graph *g, uint64_t *global_new);
+efg_status device_step_end(efg_graph *g, efg_stats *st);
+// op 0 = pack (out = send), 1 = reduce (in = recv, out = mine), 2 = unpack (in = gathered)
+efg_status device_xchg(efg_graph *g, int op, int world, const uint64_t *bounds, uint64_t slice_words,
+                       uint32_t *out, const uint32_t *in);
 }  // namespace efg
 
 // error handling (efg_error.cpp)

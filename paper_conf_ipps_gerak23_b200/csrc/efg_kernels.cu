@@ -252,6 +252,7 @@ __global__ void init_kernel(InitArgs a)
         a.ctrl->xlevel = 0;
         a.ctrl->seq = a.ctrl->seq + 1;
         a.ctrl->nlevels = 0;
+        a.ctrl->nnew = 0;
         a.ctrl->total_nf = 0;
         a.ctrl->total_ne = 0;
         if (a.parent) a.parent[a.v0] = (uint32_t)a.v0;
@@ -289,10 +290,16 @@ __global__ void __launch_bounds__(kFrontierThreads) compact_kernel(CompactArgs a
     const uint64_t lo = (uint64_t)b * a.words_per_block;
     const uint64_t hi = min(lo + a.words_per_block, a.nwords);
 
-    // pass 1: count
-    uint64_t cnt = 0;
-    for (uint64_t w = lo + tid; w < hi; w += NT) cnt += __popc(a.vis[w] & ~a.prev[w]);
+    // pass 1: count (queue = owned words only; nnew = every row)
+    uint64_t cnt = 0, all = 0;
+    for (uint64_t w = lo + tid; w < hi; w += NT) {
+        const uint32_t c = __popc(a.vis[w] & ~a.prev[w]);
+        all += c;
+        if (w >= a.own_lo_w && w < a.own_hi_w) cnt += c;
+    }
     const uint64_t blk = block_sum_u64(cnt, s_warp);
+    const uint64_t blk_all = block_sum_u64(all, s_warp);
+    if (tid == 0 && blk_all) atomicAdd(reinterpret_cast<unsigned long long *>(&a.ctrl->nnew), blk_all);
     if (tid < 32) {
         const uint64_t pre = publish_and_prefix(a.status, b, tag, blk);
         if (tid == 0) {
@@ -312,10 +319,17 @@ __global__ void __launch_bounds__(kFrontierThreads) compact_kernel(CompactArgs a
             nb = x & ~p;
             if (nb) a.prev[w] = x;
         }
+        const bool own = w >= a.own_lo_w && w < a.own_hi_w;
+        if (!own)  // rows owned by another rank: depth only
+            for (uint32_t t = nb; t; t &= t - 1) {
+                const uint32_t v = (uint32_t)(w * 32 + (__ffs(t) - 1));
+                depth[a.idmap ? a.idmap[v] : v] = level;
+            }
+        const uint32_t nq = own ? nb : 0u;
         uint64_t tot;
-        const uint64_t ex = block_excl_u64<NT>(__popc(nb), tot, s_warp);
+        const uint64_t ex = block_excl_u64<NT>(__popc(nq), tot, s_warp);
         uint32_t k = (uint32_t)ex;
-        for (uint32_t t = nb; t; t &= t - 1) s_ids[k++] = (uint32_t)(w * 32 + (__ffs(t) - 1));
+        for (uint32_t t = nq; t; t &= t - 1) s_ids[k++] = (uint32_t)(w * 32 + (__ffs(t) - 1));
         __syncthreads();
         for (uint32_t i = tid; i < tot; i += NT) {
             const uint32_t v = s_ids[i];
@@ -324,6 +338,35 @@ __global__ void __launch_bounds__(kFrontierThreads) compact_kernel(CompactArgs a
         }
         base += tot;
         __syncthreads();
+    }
+}
+
+// --------------------------------------------------------------------------
+// Exchange kernels of the 1-D partitioned BFS.  Slices are the
+// owners' bitmap word ranges [bw[h], bw[h+1]), padded to S words.
+//   pack:   send[h*S + i] = (vis & ~prev)[bw[h] + i]      (this rank's new bits)
+//   reduce: mine[i] = OR_p recv[p*S + i]                    (owner ORs P slices)
+//   unpack: vis[bw[h] + i] |= gathered[h*S + i]            (global new bits)
+// --------------------------------------------------------------------------
+__global__ void xchg_kernel(XchgArgs a)
+{
+    const uint64_t total = (uint64_t)(a.op == 1 ? 1 : a.world) * a.S;
+    for (uint64_t t = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; t < total;
+         t += (uint64_t)gridDim.x * blockDim.x) {
+        if (a.op == 1) {
+            uint32_t m = 0;
+            for (int p = 0; p < a.world; ++p) m |= a.in[(uint64_t)p * a.S + t];
+            a.out[t] = m;
+            continue;
+        }
+        const int h = (int)(t / a.S);
+        const uint64_t i = t - (uint64_t)h * a.S;
+        const uint64_t w0 = a.bounds[h] / 32, w1 = (a.bounds[h + 1] + 31) / 32;
+        const uint64_t w = w0 + i;
+        if (a.op == 0)
+            a.out[t] = w < w1 ? (a.vis[w] & ~a.prev[w]) : 0u;
+        else if (w < w1 && a.in[t])
+            a.vis[w] |= a.in[t];
     }
 }
 
@@ -515,6 +558,7 @@ __global__ void __launch_bounds__(kExpandThreads, 1) expand_kernel(ExpandArgs a)
         if (blockIdx.x == 0 && threadIdx.x == 0) {
             a.ctrl->level = xl + 1;  // depth of the vertices this launch discovers
             a.ctrl->seq = a.ctrl->seq + 1;
+            a.ctrl->nnew = 0;
         }
         // level-start snapshot of the hot visited words
         const uint4 *src = reinterpret_cast<const uint4 *>(a.vis);
@@ -795,6 +839,14 @@ cudaError_t launch_init(const InitArgs &a, cudaStream_t s)
 cudaError_t launch_compact(const CompactArgs &a, unsigned blocks, cudaStream_t s)
 {
     compact_kernel<<<blocks, kFrontierThreads, 0, s>>>(a);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_xchg(const XchgArgs &a, cudaStream_t s)
+{
+    const uint64_t total = (uint64_t)(a.op == 1 ? 1 : a.world) * a.S;
+    const unsigned blocks = (unsigned)std::max<uint64_t>(1, std::min<uint64_t>((total + 255) / 256, 148 * 8));
+    xchg_kernel<<<blocks, 256, 0, s>>>(a);
     return cudaGetLastError();
 }
 

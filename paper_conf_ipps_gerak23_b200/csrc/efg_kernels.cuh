@@ -43,6 +43,18 @@ struct CompactArgs {
     LevelCtrl *ctrl;           // in: level, seq, depth ptr; out: nf
     uint64_t *status;          // cross-block prefix words (one per block)
     uint64_t nwords, words_per_block;
+    uint64_t own_lo_w, own_hi_w;  // owned bitmap words: only these enter the queue
+};
+
+struct XchgArgs {
+    int op;                        // 0 pack, 1 reduce, 2 unpack
+    int world;
+    uint64_t S;                    // slice words
+    const uint64_t *bounds;        // device copy of the vertex bounds (world+1)
+    uint32_t *vis;
+    const uint32_t *prev;
+    uint32_t *out;
+    const uint32_t *in;
 };
 
 struct PlanArgs {
@@ -62,6 +74,7 @@ cudaError_t launch_expand(int mode, const ExpandArgs &a, int blocks, cudaStream_
 cudaError_t launch_init(const InitArgs &a, cudaStream_t s);
 cudaError_t launch_compact(const CompactArgs &a, unsigned blocks, cudaStream_t s);
 cudaError_t launch_plan(const PlanArgs &a, unsigned blocks, cudaStream_t s);
+cudaError_t launch_xchg(const XchgArgs &a, cudaStream_t s);
 int expand_occupancy(int mode);
 size_t expand_smem_bytes();
 // pout[old_of_new[i]] = pin[i] == ~0u ? ~0u : old_of_new[pin[i]]  (parents back to input ids)

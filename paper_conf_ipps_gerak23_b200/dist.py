@@ -1,0 +1,113 @@
+"""1-D partitioned BFS across ranks: the per-level exchange.
+
+Every computation (expand, pack, OR-reduce, unpack, frontier compaction) runs
+in libefg.so on the rank's GPU; this module only moves bytes between ranks
+with torch.distributed (NCCL over NVLink on GPUs; gloo in the CPU tests).
+
+Per level (all ranks in lock step):
+    g.bfs_expand()                      decode + visit the rank's own rows
+    g.xchg_pack(bounds, S, send)        slice h of the rank's new bits -> send[h]
+    all_to_all(send -> recv)            rank h receives every rank's slice h
+    g.xchg_reduce(P, S, recv, mine)     OR of the P copies of slice h
+    all_gather(mine -> gathered)        every rank gets every owner's slice
+    g.xchg_unpack(bounds, S, gathered)  visited |= global new bits
+    g.bfs_finish_level()                next frontier = new owned vertices,
+                                        depth of all new vertices; global count
+The global new-vertex count is identical on every rank (same bitmap), so the
+loop ends on all ranks at the same level with no extra collective.
+"""
+from __future__ import annotations
+
+import numpy as np
+
+
+class TorchTransport:
+    """all_to_all / all_gather of equal slices with torch.distributed."""
+
+    def __init__(self, group=None):
+        import torch.distributed as dist
+        self.dist = dist
+        self.group = group
+
+    def all_to_all(self, send, recv):
+        self.dist.all_to_all_single(recv, send, group=self.group)
+
+    def all_gather(self, mine, gathered):
+        try:
+            self.dist.all_gather_into_tensor(gathered, mine, group=self.group)
+        except (RuntimeError, NotImplementedError):
+            world = self.dist.get_world_size(self.group)
+            parts = list(gathered.chunk(world))
+            self.dist.all_gather(parts, mine, group=self.group)
+
+
+def partition_bounds(vlist: np.ndarray, offsets: np.ndarray, world: int) -> np.ndarray:
+    from . import partition
+    return partition(vlist, offsets, world)
+
+
+def partitioned_bfs(g, source: int, depth, bounds: np.ndarray, transport, make_buffer):
+    """Run one BFS over the partitioned handles of all ranks.
+
+    g          this rank's Graph (built with rows=(bounds[r], bounds[r+1]))
+    depth      this rank's device int32 buffer (n); receives the full depth array
+    bounds     np.uint64[world+1] vertex boundaries (efg_partition)
+    transport  object with all_to_all(send, recv) and all_gather(mine, gathered)
+    make_buffer(nwords) -> device uint32/int32 tensor
+    Returns the list of global new-vertex counts per level.
+    """
+    world = bounds.size - 1
+    S = g.xchg_geometry(bounds)
+    send = make_buffer(world * S)
+    recv = make_buffer(world * S)
+    mine = make_buffer(S)
+    gathered = make_buffer(world * S)
+    g.bfs_begin(source, depth)
+    counts = [1]
+    while True:
+        g.bfs_expand()
+        g.xchg_pack(bounds, S, send)
+        transport.all_to_all(send, recv)
+        g.xchg_reduce(world, S, recv, mine)
+        transport.all_gather(mine, gathered)
+        g.xchg_unpack(bounds, S, gathered)
+        new = g.bfs_finish_level()
+        if new == 0:
+            break
+        counts.append(new)
+    return counts
+
+
+def simulated_partitioned_bfs(graphs, source: int, depths, bounds: np.ndarray, make_buffer):
+    """The same protocol with all `world` rank handles in one process (one GPU):
+    the all-to-all and all-gather become buffer copies.  Used by the GPU tests to
+    run the partitioned kernels without several GPUs."""
+    world = bounds.size - 1
+    S = graphs[0].xchg_geometry(bounds)
+    send = [make_buffer(world * S) for _ in range(world)]
+    recv = [make_buffer(world * S) for _ in range(world)]
+    mine = [make_buffer(S) for _ in range(world)]
+    gathered = make_buffer(world * S)
+    for g, d in zip(graphs, depths):
+        g.bfs_begin(source, d)
+    counts = [1]
+    while True:
+        for r, g in enumerate(graphs):
+            g.bfs_expand()
+            g.xchg_pack(bounds, S, send[r])
+        for r in range(world):          # all-to-all
+            for p in range(world):
+                recv[r][p * S:(p + 1) * S].copy_(send[p][r * S:(r + 1) * S])
+        for r, g in enumerate(graphs):
+            g.xchg_reduce(world, S, recv[r], mine[r])
+        for r in range(world):          # all-gather
+            gathered[r * S:(r + 1) * S].copy_(mine[r])
+        news = []
+        for g in graphs:
+            g.xchg_unpack(bounds, S, gathered)
+            news.append(g.bfs_finish_level())
+        assert len(set(news)) == 1, news
+        if news[0] == 0:
+            break
+        counts.append(news[0])
+    return counts

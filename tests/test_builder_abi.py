@@ -149,3 +149,19 @@ def test_reorder_degree_byte_identical_to_oracle_on_relabelled_graph():
     # degrees are non-increasing in the stored order
     assert np.all(np.diff(np.diff(vlist).astype(np.int64)) <= 0)
     g.free()
+
+
+def test_row_range_build_keeps_only_owned_lists():
+    import paper_conf_ipps_gerak23_b200 as efg
+    n, src, dst = synth.rmat(12, 8, seed=4)
+    whole = efg.Graph.build(n, src, dst, device=-1)
+    wv, wn, wo, wd = whole.export()
+    part = efg.Graph.build(n, src, dst, device=-1, rows=(1024, 2048))
+    pv, pn, po, pd = part.export()
+    deg_w, deg_p = np.diff(wv), np.diff(pv)
+    assert np.all(deg_p[:1024] == 0) and np.all(deg_p[2048:] == 0)
+    assert np.array_equal(deg_p[1024:2048], deg_w[1024:2048])
+    assert pd.tobytes() == wd[wo[1024]:wo[2048]].tobytes()
+    assert part.info["row_lo"] == 1024 and part.info["row_hi"] == 2048
+    with pytest.raises(efg.EFGError):
+        efg.Graph.build(n, src, dst, device=-1, rows=(100, 2048))

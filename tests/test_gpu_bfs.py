@@ -275,3 +275,31 @@ def test_hot_snapshot_boundary(efg):
         ov, oe = oracle.csr_build(n, src, dst)
         _check_bfs(g, ov, oe, [0, 917503, 917504, n - 1])
         g.free()
+
+
+@pytest.mark.parametrize("world", [1, 2, 3, 4])
+def test_partitioned_bfs_simulated_ranks(efg, world):
+    """the 1-D partitioned kernels (row-range handles, pack /
+    OR-reduce / unpack, owned-row frontiers) with the transport emulated in
+    one process; every rank's depth must equal the oracle's."""
+    import torch
+    from paper_conf_ipps_gerak23_b200.dist import simulated_partitioned_bfs
+    n, src, dst = synth.rmat(14, 16, seed=13)
+    ov, oe = oracle.csr_build(n, src, dst)
+    for flags in (efg.EFG_DEFAULT_FLAGS, efg.EFG_DEFAULT_FLAGS | efg.EFG_REORDER_DEGREE):
+        whole = efg.Graph.build(n, src, dst, flags=flags, device=-1)
+        vlist, _, offsets, _ = whole.export()
+        bounds = efg.partition(vlist, offsets, world)
+        whole.free()
+        graphs = [efg.Graph.build(n, src, dst, flags=flags,
+                                  rows=(int(bounds[r]), int(bounds[r + 1]))) for r in range(world)]
+        for s in (0, 3, 9999):
+            depths = [torch.empty(n, dtype=torch.int32, device="cuda") for _ in range(world)]
+            simulated_partitioned_bfs(graphs, s, depths, bounds,
+                                      lambda k: torch.zeros(k, dtype=torch.int32, device="cuda"))
+            torch.cuda.synchronize()
+            ref = oracle.bfs(ov, oe, s)
+            for d in depths:
+                assert np.array_equal(d.cpu().numpy(), ref)
+        for g in graphs:
+            g.free()
