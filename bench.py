@@ -51,6 +51,9 @@ def parse():
     p.add_argument("--config", type=int, default=2, help="BASELINE.json config index (1-based)")
     p.add_argument("--scale", type=int, default=None, help="override RMAT scale (debug only)")
     p.add_argument("--no-cpu-baseline", action="store_true")
+    p.add_argument("--mode", default="partition", choices=["partition", "replicas"],
+                   help="N > 1: 1-D partitioned BFS with a per-level NCCL exchange (SURVEY 8(e)), "
+                        "or independent replicas on disjoint sources")
     p.add_argument("--reorder", default="degree", choices=["none", "degree"],
                    help="EFG_REORDER_DEGREE relabelling at build time (results stay in input ids)")
     p.add_argument("--profile-levels", action="store_true", help="print per-level stats to stderr")
@@ -167,6 +170,89 @@ def run_reference(args, rank, world):
     print(json.dumps(line), flush=True)
 
 
+def run_partitioned(args, rank, world, local):
+    """N ranks, one BFS at a time over the 1-D row partition (strong scaling)."""
+    import torch
+    import torch.distributed as dist
+    import synth
+    import paper_conf_ipps_gerak23_b200 as efg
+    from paper_conf_ipps_gerak23_b200.dist import TorchTransport, partitioned_bfs
+
+    dev = torch.device("cuda", local)
+    stream = torch.cuda.Stream(device=dev)
+    n, src, dst, gen_s = make_graph_edges(args.config, args.scale)
+    flags = efg.EFG_DEFAULT_FLAGS | (efg.EFG_REORDER_DEGREE if args.reorder == "degree" else 0)
+    cdev = dev if dist.get_backend() == "nccl" else torch.device("cpu")
+    bounds = torch.zeros(world + 1, dtype=torch.int64, device=cdev)
+    deg_in = torch.zeros(n, dtype=torch.int64, device=cdev)
+    if rank == 0:  # byte-balanced partition of the whole graph (host-only handle)
+        whole = efg.Graph.build(n, src, dst, device=-1, flags=flags)
+        vl, _, of, _ = whole.export()
+        pm = whole.perm()
+        b = efg.partition(vl, of, world)
+        bounds.copy_(torch.from_numpy(b.astype(np.int64)))
+        d = np.empty(n, np.int64)
+        d[pm] = np.diff(vl).astype(np.int64)
+        deg_in.copy_(torch.from_numpy(d))
+        whole.free()
+    dist.broadcast(bounds, 0)
+    dist.broadcast(deg_in, 0)
+    b = bounds.cpu().numpy().astype(np.uint64)
+    deg = deg_in.cpu().numpy()
+    g = efg.Graph.build(n, src, dst, device=local, stream=stream.cuda_stream, flags=flags,
+                        rows=(int(b[rank]), int(b[rank + 1])))
+    del src, dst
+    srcs = synth.sources(n, args.warmup + args.steps, seed=1000 + args.config, nonisolated_mask=deg > 0)
+    depth = torch.empty(n, dtype=torch.int32, device=dev)
+    tr = TorchTransport(stage_on_host=dist.get_backend() != "nccl")
+    mk = lambda k: torch.zeros(k, dtype=torch.int32, device=dev)  # noqa: E731
+    with torch.cuda.stream(stream):
+        for s in srcs[:args.warmup]:
+            partitioned_bfs(g, int(s), depth, b, tr, mk)
+    torch.cuda.synchronize()
+    dist.barrier()
+    torch.cuda.synchronize()
+    clk = ClockSampler(local)
+    clk.start()
+    time.sleep(0.3)
+    e0 = torch.cuda.Event(enable_timing=True)
+    e1 = torch.cuda.Event(enable_timing=True)
+    edges = 0
+    e0.record(stream)
+    with torch.cuda.stream(stream):
+        for s in srcs[args.warmup:]:
+            partitioned_bfs(g, int(s), depth, b, tr, mk)
+            st = g.bfs_end()
+            edges += st["edges_traversed"]  # this rank's rows
+    e1.record(stream)
+    torch.cuda.synchronize()
+    clocks = clk.stop()
+    ms = e0.elapsed_time(e1)
+    t = torch.tensor([ms], dtype=torch.float64, device=cdev)
+    e = torch.tensor([edges], dtype=torch.float64, device=cdev)
+    dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    dist.all_reduce(e, op=dist.ReduceOp.SUM)
+    value = float(e.item()) / (float(t.item()) * 1e-3) / 1e9
+    if rank == 0:
+        cfgname = synth.CONFIGS[args.config]["name"] + (f"_scale{args.scale}" if args.scale else "")
+        line = {
+            "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": float(t.item()) / args.steps,
+            "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "u32",
+            "data": "synthetic",
+            "config": {"workload": cfgname, "n": int(n), "reorder": args.reorder,
+                       "parallelism": f"1-D row partition over {world} GPUs, per-level bitmap "
+                                      "exchange (all_to_all + OR + all_gather, NCCL)",
+                       "bounds": [int(x) for x in b],
+                       "l2_policy": "inputs larger than L2"},
+            "clocks": clocks, "gpu_launches": None,
+            "e2e": None, "cpu_baseline": None,
+        }
+        print(json.dumps(line), flush=True)
+    g.free()
+    dist.destroy_process_group()
+
+
 def main():
     args = parse()
     rank, world, local = dist_env()
@@ -180,8 +266,15 @@ def main():
 
     if world > 1:
         import torch.distributed as dist
+        backend = os.environ.get("EFG_DIST_BACKEND", "nccl")  # gloo: functional runs on 1 GPU
+        local = local % torch.cuda.device_count()
         torch.cuda.set_device(local)
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        if backend == "nccl":
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        else:
+            dist.init_process_group(backend)
+        if args.mode == "partition":
+            return run_partitioned(args, rank, world, local)
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
     stream = torch.cuda.Stream(device=dev)

@@ -22,17 +22,34 @@ import numpy as np
 
 
 class TorchTransport:
-    """all_to_all / all_gather of equal slices with torch.distributed."""
+    """all_to_all / all_gather of equal slices with torch.distributed.
 
-    def __init__(self, group=None):
+    stage_on_host=True copies device buffers through host memory (for the gloo
+    backend, e.g. several ranks sharing one GPU in a functional test)."""
+
+    def __init__(self, group=None, stage_on_host: bool = False):
         import torch.distributed as dist
         self.dist = dist
         self.group = group
+        self.host = stage_on_host
 
     def all_to_all(self, send, recv):
+        if self.host:
+            r = recv.cpu()
+            self.dist.all_to_all_single(r, send.cpu(), group=self.group)
+            recv.copy_(r)
+            return
         self.dist.all_to_all_single(recv, send, group=self.group)
 
     def all_gather(self, mine, gathered):
+        if self.host:
+            gh = gathered.cpu()
+            self._all_gather(mine.cpu(), gh)
+            gathered.copy_(gh)
+            return
+        self._all_gather(mine, gathered)
+
+    def _all_gather(self, mine, gathered):
         try:
             self.dist.all_gather_into_tensor(gathered, mine, group=self.group)
         except (RuntimeError, NotImplementedError):
