@@ -186,7 +186,7 @@ def run_partitioned(args, rank, world, local):
     bounds = torch.zeros(world + 1, dtype=torch.int64, device=cdev)
     deg_in = torch.zeros(n, dtype=torch.int64, device=cdev)
     if rank == 0:  # byte-balanced partition of the whole graph (host-only handle)
-        whole = efg.Graph.build(n, src, dst, device=-1, flags=flags)
+        whole = efg.Graph.build(n, src, dst, device=-1, flags=flags, n_threads=os.cpu_count() or 1)
         vl, _, of, _ = whole.export()
         pm = whole.perm()
         b = efg.partition(vl, of, world)
@@ -199,8 +199,9 @@ def run_partitioned(args, rank, world, local):
     dist.broadcast(deg_in, 0)
     b = bounds.cpu().numpy().astype(np.uint64)
     deg = deg_in.cpu().numpy()
+    nthr = max(1, (os.cpu_count() or 1) // world)
     g = efg.Graph.build(n, src, dst, device=local, stream=stream.cuda_stream, flags=flags,
-                        rows=(int(b[rank]), int(b[rank + 1])))
+                        rows=(int(b[rank]), int(b[rank + 1])), n_threads=nthr)
     del src, dst
     srcs = synth.sources(n, args.warmup + args.steps, seed=1000 + args.config, nonisolated_mask=deg > 0)
     depth = torch.empty(n, dtype=torch.int32, device=dev)

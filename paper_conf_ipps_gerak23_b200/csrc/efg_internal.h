@@ -129,6 +129,9 @@ struct DeviceGraph {
     uint32_t *parent = nullptr;        // internal parent (n), lazily allocated
     uint32_t *parent2 = nullptr;       // parent in input ids (reordered graphs), lazily
     uint32_t *old_of_new = nullptr;    // EFG_REORDER_DEGREE relabelling (n) or null
+    uint32_t *new_of_old = nullptr;    // its inverse (n) or null
+    int32_t *depth_st = nullptr;       // depth by stored id (relabelled graphs)
+    int32_t *step_depth = nullptr;     // stepwise traversal: caller's depth buffer
     uint64_t *status = nullptr;        // cross-block prefix words: compact [kMaxGrid], plan [kMaxGrid]
     LevelStat *stats = nullptr;        // per-level statistics (kMaxLevelStats)
     unsigned frontier_blocks = 0;      // grid of compact / plan

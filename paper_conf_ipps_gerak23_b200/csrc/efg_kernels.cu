@@ -271,73 +271,87 @@ __global__ void init_kernel(InitArgs a)
 // compact_kernel: a7 level end.  new = vis & ~prev; the new vertices, in
 // increasing id order, become the next frontier queue (sorted for free, in
 // place of the paper's partial radix sort); depth[new] = level.
-// Reduce-then-scan over a persistent grid: pass 1 counts the block's word
-// range, the cross-block prefix places it, pass 2 re-reads the range 256 words
-// at a time, stages the new ids in shared memory and writes them coalesced.
+// Reduce-then-scan over a persistent grid.  A block's word range is split into
+// one contiguous run per warp.  Pass 1 counts (coalesced word loads); the
+// cross-block prefix places the block, the per-warp counts place the warps;
+// pass 2 walks 32 words at a time: a warp scan of the popcounts gives each
+// word's queue offset and, word by word, lane b writes bit b's vertex, so the
+// queue and depth stores are coalesced.  No block barrier inside the loops.
 // --------------------------------------------------------------------------
 __global__ void __launch_bounds__(kFrontierThreads) compact_kernel(CompactArgs a)
 {
-    constexpr int NT = kFrontierThreads;
-    __shared__ uint64_t s_warp[NT / 32];
+    constexpr int NT = kFrontierThreads, NW = NT / 32;
+    __shared__ uint64_t s_warp[NW];
+    __shared__ uint64_t s_wcnt[NW];
     __shared__ uint64_t s_pre;
-    __shared__ uint32_t s_ids[NT * 32];
 
-    const uint32_t tid = threadIdx.x, b = blockIdx.x;
+    const uint32_t tid = threadIdx.x, lane = tid & 31, wid = tid >> 5, b = blockIdx.x;
     const LevelCtrl *ctrl = a.ctrl;
     const uint32_t tag = ctrl->seq;
     const int32_t level = (int32_t)ctrl->level;
     int32_t *depth = ctrl->depth;
     const uint64_t lo = (uint64_t)b * a.words_per_block;
     const uint64_t hi = min(lo + a.words_per_block, a.nwords);
+    const uint64_t per_w = (a.words_per_block + NW - 1) / NW;
+    const uint64_t wlo = min(lo + wid * per_w, hi), whi = min(wlo + per_w, hi);
 
     // pass 1: count (queue = owned words only; nnew = every row)
     uint64_t cnt = 0, all = 0;
-    for (uint64_t w = lo + tid; w < hi; w += NT) {
+    for (uint64_t w = wlo + lane; w < whi; w += 32) {
         const uint32_t c = __popc(a.vis[w] & ~a.prev[w]);
         all += c;
         if (w >= a.own_lo_w && w < a.own_hi_w) cnt += c;
     }
-    const uint64_t blk = block_sum_u64(cnt, s_warp);
-    const uint64_t blk_all = block_sum_u64(all, s_warp);
-    if (tid == 0 && blk_all) atomicAdd(reinterpret_cast<unsigned long long *>(&a.ctrl->nnew), blk_all);
-    if (tid < 32) {
+    cnt = warp_sum_u64(cnt);
+    all = warp_sum_u64(all);
+    if (lane == 0) {
+        s_wcnt[wid] = cnt;
+        s_warp[wid] = all;
+    }
+    __syncthreads();
+    if (wid == 0) {
+        const uint64_t bc = lane < NW ? s_wcnt[lane] : 0, ba = lane < NW ? s_warp[lane] : 0;
+        const uint64_t blk = warp_sum_u64(bc), blk_all = warp_sum_u64(ba);
+        if (lane == 0 && blk_all) atomicAdd(reinterpret_cast<unsigned long long *>(&a.ctrl->nnew), blk_all);
         const uint64_t pre = publish_and_prefix(a.status, b, tag, blk);
-        if (tid == 0) {
+        if (lane == 0) {
             s_pre = pre;
             if (b == gridDim.x - 1) a.ctrl->nf = pre + blk;
         }
     }
     __syncthreads();
-
-    // pass 2: queue + depth, 256 words per step
     uint64_t base = s_pre;
-    for (uint64_t c0 = lo; c0 < hi; c0 += NT) {
-        const uint64_t w = c0 + tid;
+    for (uint32_t w = 0; w < wid; ++w) base += s_wcnt[w];
+
+    // pass 2: queue + depth
+    const uint32_t lt = (1u << lane) - 1;
+    for (uint64_t w0 = wlo; w0 < whi; w0 += 32) {
+        const uint64_t w = w0 + lane;
         uint32_t nb = 0;
-        if (w < hi) {
+        if (w < whi) {
             const uint32_t x = a.vis[w], p = a.prev[w];
             nb = x & ~p;
             if (nb) a.prev[w] = x;
         }
         const bool own = w >= a.own_lo_w && w < a.own_hi_w;
-        if (!own)  // rows owned by another rank: depth only
-            for (uint32_t t = nb; t; t &= t - 1) {
-                const uint32_t v = (uint32_t)(w * 32 + (__ffs(t) - 1));
-                depth[a.idmap ? a.idmap[v] : v] = level;
-            }
         const uint32_t nq = own ? nb : 0u;
-        uint64_t tot;
-        const uint64_t ex = block_excl_u64<NT>(__popc(nq), tot, s_warp);
-        uint32_t k = (uint32_t)ex;
-        for (uint32_t t = nq; t; t &= t - 1) s_ids[k++] = (uint32_t)(w * 32 + (__ffs(t) - 1));
-        __syncthreads();
-        for (uint32_t i = tid; i < tot; i += NT) {
-            const uint32_t v = s_ids[i];
-            a.queue[base + i] = v;
-            depth[a.idmap ? a.idmap[v] : v] = level;
+        uint32_t tq;
+        const uint32_t off = warp_excl_u32(__popc(nq), tq);
+        uint32_t todo = __ballot_sync(FULL, nb != 0);
+        while (todo) {
+            const int j = __ffs(todo) - 1;
+            todo &= todo - 1;
+            const uint32_t nbw = __shfl_sync(FULL, nb, j);
+            const uint32_t nqw = __shfl_sync(FULL, nq, j);
+            const uint32_t offj = __shfl_sync(FULL, off, j);
+            if ((nbw >> lane) & 1) {
+                const uint32_t v = (uint32_t)((w0 + j) * 32 + lane);
+                if (a.depth_stored) a.depth_stored[v] = level;  // stored-id order (coalesced)
+                if (!a.depth_stored_only) depth[v] = level;
+                if (nqw) a.queue[base + offj + __popc(nqw & lt)] = v;
+            }
         }
-        base += tot;
-        __syncthreads();
+        base += tq;
     }
 }
 
@@ -381,14 +395,14 @@ __global__ void xchg_kernel(XchgArgs a)
 // --------------------------------------------------------------------------
 __global__ void __launch_bounds__(kFrontierThreads) plan_kernel(PlanArgs a)
 {
-    constexpr int NT = kFrontierThreads;
+    constexpr int NT = kFrontierThreads, NW = NT / 32;
     constexpr int kHubCap = 256;
-    __shared__ uint64_t s_warp[NT / 32];
+    __shared__ uint64_t s_wwork[NW];
     __shared__ uint64_t s_pre;
     __shared__ HubItem s_hub[kHubCap];
     __shared__ uint32_t s_nhub;
 
-    const uint32_t tid = threadIdx.x, b = blockIdx.x;
+    const uint32_t tid = threadIdx.x, lane = tid & 31, wid = tid >> 5, b = blockIdx.x;
     LevelCtrl *ctrl = a.ctrl;
     const uint32_t tag = ctrl->seq;
     const uint64_t nf = ctrl->nf;
@@ -396,15 +410,20 @@ __global__ void __launch_bounds__(kFrontierThreads) plan_kernel(PlanArgs a)
     const uint64_t A = kVertexWork;
     const uint64_t per = (nf + gridDim.x - 1) / gridDim.x;
     const uint64_t lo = min((uint64_t)b * per, nf), hi = min(lo + per, nf);
+    const uint64_t per_w = (per + NW - 1) / NW;
+    const uint64_t qlo = min(lo + wid * per_w, hi), qhi = min(qlo + per_w, hi);
     if (tid == 0) s_nhub = 0;
 
-    // pass 1: work of the block's range
+    // pass 1: work of the warp's range (a1 degree lookup)
     uint64_t wk = 0;
-    for (uint64_t i = lo + tid; i < hi; i += NT) wk += A + __ldg(a.deg32 + a.queue[i]);
-    const uint64_t blk = block_sum_u64(wk, s_warp);
-    if (tid < 32) {
+    for (uint64_t i = qlo + lane; i < qhi; i += 32) wk += A + __ldg(a.deg32 + a.queue[i]);
+    wk = warp_sum_u64(wk);
+    if (lane == 0) s_wwork[wid] = wk;
+    __syncthreads();
+    if (wid == 0) {
+        const uint64_t blk = warp_sum_u64(lane < NW ? s_wwork[lane] : 0);
         const uint64_t pre = publish_and_prefix(a.status, b, tag, blk);
-        if (tid == 0) {
+        if (lane == 0) {
             s_pre = pre;
             if (b == gridDim.x - 1) {
                 const uint64_t nwork = pre + blk;
@@ -429,17 +448,17 @@ __global__ void __launch_bounds__(kFrontierThreads) plan_kernel(PlanArgs a)
         }
     }
     __syncthreads();
-
-    // pass 2: tiles
     uint64_t run = s_pre;
-    for (uint64_t c0 = lo; c0 < hi; c0 += NT) {
-        const uint64_t i = c0 + tid;
-        uint64_t d = 0;
-        if (i < hi) d = __ldg(a.deg32 + a.queue[i]);
+    for (uint32_t w = 0; w < wid; ++w) run += s_wwork[w];
+
+    // pass 2: exclusive scan of the work (a2) and the tile table (a3)
+    for (uint64_t i0 = qlo; i0 < qhi; i0 += 32) {
+        const uint64_t i = i0 + lane;
+        const uint64_t d = i < qhi ? __ldg(a.deg32 + a.queue[i]) : 0;
         uint64_t tot;
-        const uint64_t W = run + block_excl_u64<NT>(i < hi ? A + d : 0, tot, s_warp);
+        const uint64_t W = run + warp_excl_u64(i < qhi ? A + d : 0, tot);
         // does a tile boundary fall inside [W, W + A + d)?
-        if (i < hi && ((W + kTileWork - 1) & ~(uint64_t)(kTileWork - 1)) < W + A + d)
+        if (i < qhi && ((W + kTileWork - 1) & ~(uint64_t)(kTileWork - 1)) < W + A + d)
             place_tiles(a.tiles, i, W, d, cl, s_hub, &s_nhub, kHubCap);
         run += tot;
     }
@@ -769,6 +788,14 @@ __global__ void __launch_bounds__(kExpandThreads, 1) expand_kernel(ExpandArgs a)
         atomicMax(&a.stats[xl].t1, globaltimer());
 }
 
+// depth_out[old_of_new[i]] = depth_stored[i] as a gather over input ids:
+// depth_out[v] = depth_stored[new_of_old[v]] (coalesced stores).
+__global__ void map_depth_kernel(const int32_t *stored, const uint32_t *new_of_old, int32_t *out, uint64_t n)
+{
+    for (uint64_t v = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; v < n; v += (uint64_t)gridDim.x * blockDim.x)
+        out[v] = stored[new_of_old[v]];
+}
+
 __global__ void map_parent_kernel(const uint32_t *pin, const uint32_t *old_of_new, uint32_t *pout, uint64_t n)
 {
     for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x) {
@@ -778,6 +805,14 @@ __global__ void map_parent_kernel(const uint32_t *pin, const uint32_t *old_of_ne
 }
 
 }  // namespace
+
+cudaError_t launch_map_depth(const int32_t *stored, const uint32_t *new_of_old, int32_t *out, uint64_t n,
+                             cudaStream_t s)
+{
+    const unsigned blocks = (unsigned)std::max<uint64_t>(1, std::min<uint64_t>((n + 255) / 256, 148 * 16));
+    map_depth_kernel<<<blocks, 256, 0, s>>>(stored, new_of_old, out, n);
+    return cudaGetLastError();
+}
 
 cudaError_t launch_map_parent(const uint32_t *pin, const uint32_t *old_of_new, uint32_t *pout, uint64_t n,
                               cudaStream_t s)

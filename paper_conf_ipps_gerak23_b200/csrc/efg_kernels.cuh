@@ -39,7 +39,8 @@ struct InitArgs {
 struct CompactArgs {
     uint32_t *vis, *prev;      // visited bitmap now / at the previous level end
     uint32_t *queue;           // out: next frontier, sorted
-    const uint32_t *idmap;     // stored id -> input id for depth (EFG_REORDER_DEGREE) or null
+    int32_t *depth_stored;     // depth by stored id (always written)
+    int depth_stored_only;     // 1: depth_stored is the only depth output (relabelled graphs)
     LevelCtrl *ctrl;           // in: level, seq, depth ptr; out: nf
     uint64_t *status;          // cross-block prefix words (one per block)
     uint64_t nwords, words_per_block;
@@ -78,6 +79,8 @@ cudaError_t launch_xchg(const XchgArgs &a, cudaStream_t s);
 int expand_occupancy(int mode);
 size_t expand_smem_bytes();
 // pout[old_of_new[i]] = pin[i] == ~0u ? ~0u : old_of_new[pin[i]]  (parents back to input ids)
+cudaError_t launch_map_depth(const int32_t *stored, const uint32_t *new_of_old, int32_t *out, uint64_t n,
+                             cudaStream_t s);
 cudaError_t launch_map_parent(const uint32_t *pin, const uint32_t *old_of_new, uint32_t *pout, uint64_t n,
                               cudaStream_t s);
 
