@@ -98,7 +98,7 @@ constexpr int kExpandThreads = 768;          // one CTA per SM, 24 warps
 constexpr int kExpandWarps = kExpandThreads / 32;
 constexpr int kExpandStage = 512;            // elements of one 16-word step (<= 16*32)
 constexpr uint32_t kHotWords = 28 * 1024;    // 112 KB shared-memory visited snapshot = 917,504 ids
-constexpr int kFrontierThreads = 256;        // compact / plan kernels
+constexpr int kFrontierThreads = 512;        // compact / plan kernels (16 warps)
 constexpr int kBitmapAlign = 1024;           // bitmap words are padded to a multiple of this
 // Step a3 partitions "work units" rather than bare edges: a frontier vertex
 // costs kVertexWork units (its record gather and list set-up) plus one per edge,

@@ -295,12 +295,21 @@ __global__ void __launch_bounds__(kFrontierThreads) compact_kernel(CompactArgs a
     const uint64_t per_w = (a.words_per_block + NW - 1) / NW;
     const uint64_t wlo = min(lo + wid * per_w, hi), whi = min(wlo + per_w, hi);
 
-    // pass 1: count (queue = owned words only; nnew = every row)
+    // pass 1: count (queue = owned words only; nnew = every row); 4 loads in flight
     uint64_t cnt = 0, all = 0;
-    for (uint64_t w = wlo + lane; w < whi; w += 32) {
-        const uint32_t c = __popc(a.vis[w] & ~a.prev[w]);
-        all += c;
-        if (w >= a.own_lo_w && w < a.own_hi_w) cnt += c;
+    for (uint64_t w0 = wlo + lane; w0 < whi; w0 += 128) {
+        uint32_t c[4];
+#pragma unroll
+        for (int u = 0; u < 4; ++u) {
+            const uint64_t w = w0 + 32 * u;
+            c[u] = w < whi ? __popc(a.vis[w] & ~a.prev[w]) : 0u;
+        }
+#pragma unroll
+        for (int u = 0; u < 4; ++u) {
+            const uint64_t w = w0 + 32 * u;
+            all += c[u];
+            if (w >= a.own_lo_w && w < a.own_hi_w) cnt += c[u];
+        }
     }
     cnt = warp_sum_u64(cnt);
     all = warp_sum_u64(all);
@@ -414,9 +423,16 @@ __global__ void __launch_bounds__(kFrontierThreads) plan_kernel(PlanArgs a)
     const uint64_t qlo = min(lo + wid * per_w, hi), qhi = min(qlo + per_w, hi);
     if (tid == 0) s_nhub = 0;
 
-    // pass 1: work of the warp's range (a1 degree lookup)
+    // pass 1: work of the warp's range (a1 degree lookup), 4 lookups in flight
     uint64_t wk = 0;
-    for (uint64_t i = qlo + lane; i < qhi; i += 32) wk += A + __ldg(a.deg32 + a.queue[i]);
+    for (uint64_t i0 = qlo + lane; i0 < qhi; i0 += 128) {
+        uint32_t q[4];
+#pragma unroll
+        for (int u = 0; u < 4; ++u) q[u] = i0 + 32 * u < qhi ? a.queue[i0 + 32 * u] : 0u;
+#pragma unroll
+        for (int u = 0; u < 4; ++u)
+            if (i0 + 32 * u < qhi) wk += A + __ldg(a.deg32 + q[u]);
+    }
     wk = warp_sum_u64(wk);
     if (lane == 0) s_wwork[wid] = wk;
     __syncthreads();
@@ -451,10 +467,13 @@ __global__ void __launch_bounds__(kFrontierThreads) plan_kernel(PlanArgs a)
     uint64_t run = s_pre;
     for (uint32_t w = 0; w < wid; ++w) run += s_wwork[w];
 
-    // pass 2: exclusive scan of the work (a2) and the tile table (a3)
+    // pass 2: exclusive scan of the work (a2) and the tile table (a3); the next
+    // 32 degrees are fetched while the current ones are scanned
+    uint32_t dn = qlo + lane < qhi ? __ldg(a.deg32 + a.queue[qlo + lane]) : 0u;
     for (uint64_t i0 = qlo; i0 < qhi; i0 += 32) {
         const uint64_t i = i0 + lane;
-        const uint64_t d = i < qhi ? __ldg(a.deg32 + a.queue[i]) : 0;
+        const uint64_t d = dn;
+        if (i0 + 32 < qhi) dn = i + 32 < qhi ? __ldg(a.deg32 + a.queue[i + 32]) : 0u;
         uint64_t tot;
         const uint64_t W = run + warp_excl_u64(i < qhi ? A + d : 0, tot);
         // does a tile boundary fall inside [W, W + A + d)?
