@@ -116,51 +116,33 @@ __device__ __forceinline__ ChunkLen make_chunk(uint32_t k, int kshift)
     return c;
 }
 
-struct HubItem {
-    uint64_t q, w, d;
-};
-
-__device__ __forceinline__ void write_tiles(TileEntry *tiles, uint64_t q, uint64_t W, uint64_t d,
-                                            const ChunkLen &cl, uint64_t w_begin, uint64_t w_step)
+// Entry of tile t whose boundary t*T falls inside vertex q's work range
+// [W, W + kVertexWork + d): the first chunk whose start is >= t*T (chunk 0
+// starts at W, chunk c > 0 at W + kVertexWork + c*k), or the next vertex.
+__device__ __forceinline__ TileEntry tile_entry(uint64_t t, uint64_t q, uint64_t W, uint64_t d,
+                                                const ChunkLen &cl)
 {
-    const uint64_t ch = cl.ch;
-    const uint64_t T = kTileWork, A = kVertexWork;
-    for (uint64_t t = (W + T - 1) / T + w_begin; t * T < W + A + d; t += w_step) {
-        const uint64_t o = t * T - W;
-        TileEntry te;
-        if (o == 0) {
-            te.fi = (uint32_t)q;
-            te.chunk = 0;
-            te.w = W;
-        } else {
-            uint64_t c = o > A ? cl.div(o - A + ch - 1) : 1;
-            if (c == 0) c = 1;
-            if (c * ch < d) {
-                te.fi = (uint32_t)q;
-                te.chunk = (uint32_t)c;
-                te.w = W + A + c * ch;
-            } else {
-                te.fi = (uint32_t)(q + 1);
-                te.chunk = 0;
-                te.w = W + A + d;
-            }
-        }
-        tiles[t] = te;
+    const uint64_t ch = cl.ch, A = kVertexWork;
+    const uint64_t o = t * kTileWork - W;
+    TileEntry te;
+    if (o == 0) {
+        te.fi = (uint32_t)q;
+        te.chunk = 0;
+        te.w = W;
+        return te;
     }
-}
-
-// Tile entries for one frontier vertex; long lists are queued for the whole block.
-__device__ __noinline__ void place_tiles(TileEntry *tiles, uint64_t q, uint64_t W, uint64_t d,
-                                         const ChunkLen &cl, HubItem *hub, uint32_t *nhub, uint32_t cap)
-{
-    if (d >= 8ull * kTileWork) {
-        const uint32_t slot = atomicAdd(nhub, 1u);
-        if (slot < cap) {
-            hub[slot] = HubItem{q, W, d};
-            return;
-        }
+    uint64_t c = o > A ? cl.div(o - A + ch - 1) : 1;
+    if (c == 0) c = 1;
+    if (c * ch < d) {
+        te.fi = (uint32_t)q;
+        te.chunk = (uint32_t)c;
+        te.w = W + A + c * ch;
+    } else {
+        te.fi = (uint32_t)(q + 1);
+        te.chunk = 0;
+        te.w = W + A + d;
     }
-    write_tiles(tiles, q, W, d, cl, 0, 1);
+    return te;
 }
 
 // --------------------------------------------------------------------------
@@ -405,11 +387,8 @@ __global__ void xchg_kernel(XchgArgs a)
 __global__ void __launch_bounds__(kFrontierThreads) plan_kernel(PlanArgs a)
 {
     constexpr int NT = kFrontierThreads, NW = NT / 32;
-    constexpr int kHubCap = 256;
     __shared__ uint64_t s_wwork[NW];
     __shared__ uint64_t s_pre;
-    __shared__ HubItem s_hub[kHubCap];
-    __shared__ uint32_t s_nhub;
 
     const uint32_t tid = threadIdx.x, lane = tid & 31, wid = tid >> 5, b = blockIdx.x;
     LevelCtrl *ctrl = a.ctrl;
@@ -421,7 +400,6 @@ __global__ void __launch_bounds__(kFrontierThreads) plan_kernel(PlanArgs a)
     const uint64_t lo = min((uint64_t)b * per, nf), hi = min(lo + per, nf);
     const uint64_t per_w = (per + NW - 1) / NW;
     const uint64_t qlo = min(lo + wid * per_w, hi), qhi = min(qlo + per_w, hi);
-    if (tid == 0) s_nhub = 0;
 
     // pass 1: work of the warp's range (a1 degree lookup), 4 lookups in flight
     uint64_t wk = 0;
@@ -476,15 +454,20 @@ __global__ void __launch_bounds__(kFrontierThreads) plan_kernel(PlanArgs a)
         if (i0 + 32 < qhi) dn = i + 32 < qhi ? __ldg(a.deg32 + a.queue[i + 32]) : 0u;
         uint64_t tot;
         const uint64_t W = run + warp_excl_u64(i < qhi ? A + d : 0, tot);
-        // does a tile boundary fall inside [W, W + A + d)?
-        if (i < qhi && ((W + kTileWork - 1) & ~(uint64_t)(kTileWork - 1)) < W + A + d)
-            place_tiles(a.tiles, i, W, d, cl, s_hub, &s_nhub, kHubCap);
+        // tiles whose boundary t*T falls inside [W, W + A + d): written by the
+        // whole warp, one vertex at a time (hubs span thousands of tiles)
+        const uint64_t t0 = (W + kTileWork - 1) / kTileWork;
+        const uint64_t t1 = i < qhi ? (W + A + d + kTileWork - 1) / kTileWork : t0;
+        uint32_t todo = __ballot_sync(FULL, t1 > t0);
+        while (todo) {
+            const int j = __ffs(todo) - 1;
+            todo &= todo - 1;
+            const uint64_t jq = i0 + j, jW = __shfl_sync(FULL, W, j), jd = __shfl_sync(FULL, d, j);
+            const uint64_t jt0 = __shfl_sync(FULL, t0, j), jt1 = __shfl_sync(FULL, t1, j);
+            for (uint64_t t = jt0 + lane; t < jt1; t += 32) a.tiles[t] = tile_entry(t, jq, jW, jd, cl);
+        }
         run += tot;
     }
-    __syncthreads();
-    const uint32_t nhub = min(s_nhub, (uint32_t)kHubCap);
-    for (uint32_t h = 0; h < nhub; ++h)
-        write_tiles(a.tiles, s_hub[h].q, s_hub[h].w, s_hub[h].d, cl, tid, NT);
 }
 
 // --------------------------------------------------------------------------
