@@ -352,7 +352,8 @@ def main():
             b = int(sizes[fr].sum()) + 21 * int(fr.sum())
             alg_bytes += b
             lvl_rows.append((s, L, int(fr.sum()), int(st["level_edges"][L]), b,
-                             float(st["level_expand_ms"][L]), float(stg["level_expand_ms"][L])))
+                             float(st["level_expand_ms"][L]), float(stg["level_expand_ms"][L]),
+                             float(st["level_end_ms"][L])))
         exp_ms += st["expand_ms"]
         exp_ms_gt += stg["expand_ms"]
         exp_launch += st["expand_launches"]
@@ -360,7 +361,7 @@ def main():
     achieved = alg_bytes / (exp_ms * 1e-3) / 1e9 if exp_ms > 0 else 0.0
     if args.profile_levels and rank == 0:
         for r in lvl_rows:
-            print("level src=%d L=%d |F|=%d E=%d bytes=%d expand_ms(ev)=%.4f (gt)=%.4f GB/s=%.1f" %
+            print("level src=%d L=%d |F|=%d E=%d bytes=%d expand_ms(ev)=%.4f (gt)=%.4f end_ms=%.4f GB/s=%.1f" %
                   (*r, r[4] / max(r[5], 1e-9) / 1e6), file=sys.stderr)
 
     # ---- e2e: through the C ABI with a pinned host depth buffer ----

@@ -161,6 +161,8 @@ typedef struct efg_stats {
     uint64_t *level_frontier;  /* in/out: |F_L| per level (level_cap entries)        */
     uint64_t *level_edges;     /* in/out: E_L = sum of frontier degrees per level    */
     float *level_expand_ms;    /* in/out: expand kernel time per level, or NULL      */
+    float *level_end_ms;       /* in/out: compact + plan time per level (host loop   *
+                                *         only, CUDA events), or NULL                */
 } efg_stats;
 
 /*

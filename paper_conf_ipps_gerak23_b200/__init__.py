@@ -158,10 +158,11 @@ class Graph:
             st = _abi.Stats()
             st.level_cap = level_cap
             arrs = (np.zeros(level_cap, np.uint64), np.zeros(level_cap, np.uint64),
-                    np.zeros(level_cap, np.float32))
+                    np.zeros(level_cap, np.float32), np.zeros(level_cap, np.float32))
             st.level_frontier = arrs[0].ctypes.data
             st.level_edges = arrs[1].ctypes.data
             st.level_expand_ms = arrs[2].ctypes.data
+            st.level_end_ms = arrs[3].ctypes.data
         check(lib.efg_bfs(self._h, source, _ptr(depth), _ptr(par),
                           C.byref(st) if st is not None else None), "efg_bfs")
         if not stats and par is None:
@@ -175,7 +176,8 @@ class Graph:
                   "kernel_launches": st.kernel_launches,
                   "level_frontier": arrs[0][:min(L, level_cap)].copy(),
                   "level_edges": arrs[1][:min(L, level_cap)].copy(),
-                  "level_expand_ms": arrs[2][:min(L, level_cap)].copy()}
+                  "level_expand_ms": arrs[2][:min(L, level_cap)].copy(),
+                  "level_end_ms": arrs[3][:min(L, level_cap)].copy()}
         return depth, par, sd
 
     # -- stepwise partitioned BFS (efg.h "multi-GPU"); device buffers only --

@@ -359,7 +359,7 @@ efg_status device_bfs(efg_graph *g, uint32_t source, int32_t *depth, uint32_t *p
     cudaEvent_t ev0, ev1;
     CUDA_TRY(cudaEventCreate(&ev0));
     CUDA_TRY(cudaEventCreate(&ev1));
-    std::vector<cudaEvent_t> lev;  // host mode: expand start/stop pairs
+    std::vector<cudaEvent_t> lev;  // host mode: expand start, expand end, level end
     uint32_t launches = 0;
 
     CUDA_TRY(cudaEventRecord(ev0, s));
@@ -406,10 +406,14 @@ efg_status device_bfs(efg_graph *g, uint32_t source, int32_t *depth, uint32_t *p
             CUDA_TRY(cudaEventCreate(&b));
             lev.push_back(a);
             lev.push_back(b);
+            cudaEvent_t c;
+            CUDA_TRY(cudaEventCreate(&c));
+            lev.push_back(c);
             CUDA_TRY(cudaEventRecord(a, s));
             CUDA_TRY(launch_expand(mode, expand_args(d, nullptr), blocks, s));
             CUDA_TRY(cudaEventRecord(b, s));
             EFG_TRY(launch_level_end(d, 0, s));
+            CUDA_TRY(cudaEventRecord(c, s));
             launches += 3;
             ++levels;
         }
@@ -423,9 +427,13 @@ efg_status device_bfs(efg_graph *g, uint32_t source, int32_t *depth, uint32_t *p
 
     float total_ms = 0.f;
     cudaEventElapsedTime(&total_ms, ev0, ev1);
+    std::vector<float> ems(levels, 0.f);
     if (!graph_mode) {
         lms.assign(levels, 0.f);
-        for (uint32_t i = 0; i < levels; ++i) cudaEventElapsedTime(&lms[i], lev[2 * i], lev[2 * i + 1]);
+        for (uint32_t i = 0; i < levels; ++i) {
+            cudaEventElapsedTime(&lms[i], lev[3 * i], lev[3 * i + 1]);
+            cudaEventElapsedTime(&ems[i], lev[3 * i + 1], lev[3 * i + 2]);
+        }
     }
     for (auto e : lev) cudaEventDestroy(e);
     cudaEventDestroy(ev0);
@@ -454,6 +462,7 @@ efg_status device_bfs(efg_graph *g, uint32_t source, int32_t *depth, uint32_t *p
             if (st->level_frontier) st->level_frontier[i] = lf[i];
             if (st->level_edges) st->level_edges[i] = le[i];
             if (st->level_expand_ms) st->level_expand_ms[i] = lms[i];
+            if (st->level_end_ms && i < ems.size()) st->level_end_ms[i] = ems[i];
         }
     }
     return EFG_OK;
