@@ -406,14 +406,14 @@ efg_status device_bfs(efg_graph *g, uint32_t source, int32_t *depth, uint32_t *p
             CUDA_TRY(cudaEventCreate(&b));
             lev.push_back(a);
             lev.push_back(b);
-            cudaEvent_t c;
-            CUDA_TRY(cudaEventCreate(&c));
-            lev.push_back(c);
+            cudaEvent_t ec;
+            CUDA_TRY(cudaEventCreate(&ec));
+            lev.push_back(ec);
             CUDA_TRY(cudaEventRecord(a, s));
             CUDA_TRY(launch_expand(mode, expand_args(d, nullptr), blocks, s));
             CUDA_TRY(cudaEventRecord(b, s));
             EFG_TRY(launch_level_end(d, 0, s));
-            CUDA_TRY(cudaEventRecord(c, s));
+            CUDA_TRY(cudaEventRecord(ec, s));
             launches += 3;
             ++levels;
         }
