@@ -15,6 +15,7 @@
 
 #include <algorithm>
 #include <cstddef>
+#include <cstdlib>
 #include <cstring>
 #include <string>
 #include <vector>
@@ -280,6 +281,8 @@ efg_status device_upload(efg_graph *g, const efg_build_opts &o)
     CUDA_TRY(cudaMallocHost(reinterpret_cast<void **>(&d.stats_host), kMaxLevelStats * sizeof(LevelStat)));
     // persistent grids of the frontier kernels: 2 blocks per SM, whole bitmap words
     d.frontier_blocks = (unsigned)std::min<uint64_t>(2 * (uint64_t)d.num_sms, kMaxGrid);
+    if (const char *e = std::getenv("EFG_FRONTIER_BLOCKS"))  // tuning knob (blocks of compact / plan)
+        d.frontier_blocks = (unsigned)std::max(1, std::min(atoi(e), (int)kMaxGrid));
     const uint64_t per = (d.nwords + d.frontier_blocks - 1) / d.frontier_blocks;
     d.words_per_block = (per + kFrontierThreads - 1) / kFrontierThreads * kFrontierThreads;
     CUDA_TRY(cudaStreamSynchronize(s));

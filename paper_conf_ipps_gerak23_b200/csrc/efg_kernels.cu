@@ -454,17 +454,19 @@ __global__ void __launch_bounds__(kFrontierThreads) plan_kernel(PlanArgs a)
         if (i0 + 32 < qhi) dn = i + 32 < qhi ? __ldg(a.deg32 + a.queue[i + 32]) : 0u;
         uint64_t tot;
         const uint64_t W = run + warp_excl_u64(i < qhi ? A + d : 0, tot);
-        // tiles whose boundary t*T falls inside [W, W + A + d): written by the
-        // whole warp, one vertex at a time (hubs span thousands of tiles)
-        const uint64_t t0 = (W + kTileWork - 1) / kTileWork;
-        const uint64_t t1 = i < qhi ? (W + A + d + kTileWork - 1) / kTileWork : t0;
-        uint32_t todo = __ballot_sync(FULL, t1 > t0);
-        while (todo) {
-            const int j = __ffs(todo) - 1;
-            todo &= todo - 1;
-            const uint64_t jq = i0 + j, jW = __shfl_sync(FULL, W, j), jd = __shfl_sync(FULL, d, j);
-            const uint64_t jt0 = __shfl_sync(FULL, t0, j), jt1 = __shfl_sync(FULL, t1, j);
-            for (uint64_t t = jt0 + lane; t < jt1; t += 32) a.tiles[t] = tile_entry(t, jq, jW, jd, cl);
+        // tiles whose boundary t*T falls in this group's work window
+        // [W_0, W_0 + tot): lanes take consecutive tiles, each finds its vertex
+        // by maxle over the group's W (Fig. 4 rule inside the warp)
+        const uint64_t wstart = __shfl_sync(FULL, W, 0);
+        const uint64_t tfirst = (wstart + kTileWork - 1) / kTileWork;
+        const uint64_t tend = (wstart + tot + kTileWork - 1) / kTileWork;
+        const uint32_t wrel = i < qhi ? (uint32_t)(W - wstart) : 0xffffffffu;  // < tot <= 2^32
+        for (uint64_t t0 = tfirst; t0 < tend; t0 += 32) {
+            const uint64_t t = t0 + lane;
+            const uint32_t key = t < tend ? (uint32_t)(t * kTileWork - wstart) : 0u;
+            const int j = warp_maxle_u32(wrel, key);
+            const uint64_t jW = __shfl_sync(FULL, W, j), jd = __shfl_sync(FULL, d, j);
+            if (t < tend) a.tiles[t] = tile_entry(t, i0 + j, jW, jd, cl);
         }
         run += tot;
     }
