@@ -174,18 +174,24 @@ extern "C" efg_status efg_set_option(efg_graph *g, int option, int64_t value)
     }
 }
 
-extern "C" efg_status efg_sssp(efg_graph *g, uint32_t, float *, efg_stats *)
+extern "C" efg_status efg_sssp(efg_graph *g, uint32_t source, float *dist, efg_stats *st)
 {
     clear_error();
     EFG_TRY(check_handle(g));
-    return set_error(EFG_ENOTSUP, "efg_sssp: not implemented yet");
+    if (source >= g->dev.n) return set_error(EFG_ERANGE, "efg_sssp: source >= n");
+    if (!dist) return set_error(EFG_EINVAL, "efg_sssp: dist is NULL");
+    if (!g->dev.weights && g->host.m) return set_error(EFG_EINVAL, "efg_sssp: graph built without weights");
+    const uint32_t s = g->host.new_of_old.empty() ? source : g->host.new_of_old[source];
+    return device_sssp(g, s, dist, st);
 }
 
-extern "C" efg_status efg_pagerank(efg_graph *g, double, uint32_t, double *, efg_stats *)
+extern "C" efg_status efg_pagerank(efg_graph *g, double damping, uint32_t iters, double *rank, efg_stats *st)
 {
     clear_error();
     EFG_TRY(check_handle(g));
-    return set_error(EFG_ENOTSUP, "efg_pagerank: not implemented yet");
+    if (!rank) return set_error(EFG_EINVAL, "efg_pagerank: rank is NULL");
+    if (!(damping >= 0.0 && damping <= 1.0)) return set_error(EFG_EINVAL, "efg_pagerank: damping outside [0,1]");
+    return device_pagerank(g, damping, iters, rank, st);
 }
 
 extern "C" efg_status efg_xchg_geometry(const efg_graph *g, int world, const uint64_t *bounds, uint64_t *slice_words)

@@ -84,6 +84,11 @@ ExpandArgs expand_args(DeviceGraph &d, uint32_t *out)
     a.vis = d.vis;
     a.out = out;
     a.stats = d.stats;
+    a.vlist = d.vlist;
+    a.weights = d.weights;
+    a.dist = d.fbuf;
+    a.rank = d.dbuf;
+    a.next = d.dbuf ? d.dbuf + d.n : nullptr;
     a.max_stats = kMaxLevelStats;
     a.hot_words = (uint32_t)std::min<uint64_t>(kHotWords, d.nwords) & ~3u;
     a.k = d.k;
@@ -91,13 +96,14 @@ ExpandArgs expand_args(DeviceGraph &d, uint32_t *out)
     return a;
 }
 
-CompactArgs compact_args(DeviceGraph &d)
+CompactArgs compact_args(DeviceGraph &d, bool consume = false)
 {
     CompactArgs a;
+    a.consume = consume ? 1 : 0;
     a.vis = d.vis;
     a.prev = d.prev;
     a.queue = d.queue;
-    a.depth_stored = d.old_of_new ? d.depth_st : nullptr;
+    a.depth_stored = (d.old_of_new && !consume) ? d.depth_st : nullptr;
     a.depth_stored_only = d.old_of_new ? 1 : 0;
     a.ctrl = d.ctrl;
     a.status = d.status;
@@ -124,9 +130,11 @@ PlanArgs plan_args(DeviceGraph &d, cudaGraphConditionalHandle cond)
     return a;
 }
 
-efg_status launch_level_end(DeviceGraph &d, cudaGraphConditionalHandle cond, cudaStream_t s)
+efg_status launch_level_end(DeviceGraph &d, cudaGraphConditionalHandle cond, cudaStream_t s,
+                            bool consume = false)
 {
-    CUDA_TRY(launch_compact(compact_args(d), (unsigned)((d.nwords + d.words_per_block - 1) / d.words_per_block), s));
+    CUDA_TRY(launch_compact(compact_args(d, consume),
+                            (unsigned)((d.nwords + d.words_per_block - 1) / d.words_per_block), s));
     CUDA_TRY(launch_plan(plan_args(d, cond), d.frontier_blocks, s));
     return EFG_OK;
 }
@@ -575,6 +583,123 @@ efg_status device_xchg(efg_graph *g, int op, int world, const uint64_t *bounds, 
     a.out = out;
     a.in = in;
     CUDA_TRY(launch_xchg(a, s));
+    return EFG_OK;
+}
+
+// ---------------------------------------------------------------------------
+// SSSP (§VI-F): frontier Bellman-Ford over the compressed graph.  The
+// relaxed vertices of an iteration are marked in the visited bitmap, which the
+// next compact consumes as the next frontier (and resets).
+// ---------------------------------------------------------------------------
+efg_status device_sssp(efg_graph *g, uint32_t source, float *dist, efg_stats *st)
+{
+    DeviceGraph &d = g->dev;
+    CUDA_TRY(cudaSetDevice(d.device));
+    cudaStream_t s = stream_of(d);
+    if (!d.fbuf) EFG_TRY(dev_alloc(d, &d.fbuf, d.n));
+    const bool dist_dev = is_device_ptr(dist);
+    uint32_t *out = dist_dev && !d.old_of_new ? reinterpret_cast<uint32_t *>(dist) : nullptr;
+    cudaEvent_t ev0, ev1;
+    CUDA_TRY(cudaEventCreate(&ev0));
+    CUDA_TRY(cudaEventCreate(&ev1));
+    CUDA_TRY(cudaEventRecord(ev0, s));
+    CUDA_TRY(launch_fill(reinterpret_cast<uint32_t *>(d.fbuf), 0x7F800000u, d.n, s));  // +inf
+    CUDA_TRY(cudaMemsetAsync(d.fbuf + source, 0, 4, s));
+    CUDA_TRY(cudaMemsetAsync(d.vis, 0, d.nwords * 4, s));
+    InitArgs ia;
+    ia.ctrl = d.ctrl;
+    ia.vis = d.vis;
+    ia.depth = nullptr;
+    ia.parent = nullptr;
+    ia.v0 = source;
+    ia.v1 = (uint64_t)source + 1;
+    CUDA_TRY(launch_init(ia, s));
+    EFG_TRY(launch_level_end(d, 0, s, true));
+    const int blocks = d.num_sms * expand_occupancy(kModeSssp);
+    uint32_t iters = 0;
+    uint64_t relax_edges = 0;
+    for (;;) {
+        CUDA_TRY(cudaMemcpyAsync(d.ctrl_host, d.ctrl, sizeof(LevelCtrl), cudaMemcpyDeviceToHost, s));
+        CUDA_TRY(cudaStreamSynchronize(s));
+        if (d.ctrl_host->nf == 0) break;
+        relax_edges += d.ctrl_host->ne;
+        CUDA_TRY(launch_expand(kModeSssp, expand_args(d, nullptr), blocks, s));
+        EFG_TRY(launch_level_end(d, 0, s, true));
+        ++iters;
+    }
+    uint32_t *dst = out;
+    if (!dst) {  // stage: relabel and / or copy to the host
+        if (!d.parent2) EFG_TRY(dev_alloc(d, &d.parent2, d.n));
+        dst = d.parent2;
+    }
+    if (d.old_of_new || dst != reinterpret_cast<uint32_t *>(d.fbuf))
+        CUDA_TRY(launch_gather32(reinterpret_cast<uint32_t *>(d.fbuf), d.new_of_old, dst, d.n, s));
+    CUDA_TRY(cudaEventRecord(ev1, s));
+    if (!dist_dev) CUDA_TRY(cudaMemcpyAsync(dist, dst, d.n * 4, cudaMemcpyDeviceToHost, s));
+    else if (dst != reinterpret_cast<uint32_t *>(dist))
+        CUDA_TRY(cudaMemcpyAsync(dist, dst, d.n * 4, cudaMemcpyDeviceToDevice, s));
+    CUDA_TRY(cudaStreamSynchronize(s));
+    float ms = 0.f;
+    cudaEventElapsedTime(&ms, ev0, ev1);
+    cudaEventDestroy(ev0);
+    cudaEventDestroy(ev1);
+    if (st) {
+        std::memset(st, 0, offsetof(efg_stats, level_cap));
+        st->levels = iters;
+        st->edges_traversed = relax_edges;
+        st->device_ms = ms;
+        st->expand_launches = iters;
+    }
+    return EFG_OK;
+}
+
+// ---------------------------------------------------------------------------
+// PageRank (§VI-F; 50 iterations P:201; reading C21): every vertex is
+// active; the frontier/tile plan of "all vertices" is built once and reused.
+// ---------------------------------------------------------------------------
+efg_status device_pagerank(efg_graph *g, double damping, uint32_t iters, double *rank, efg_stats *st)
+{
+    DeviceGraph &d = g->dev;
+    CUDA_TRY(cudaSetDevice(d.device));
+    cudaStream_t s = stream_of(d);
+    if (!d.dbuf) EFG_TRY(dev_alloc(d, &d.dbuf, 2 * d.n + 1));
+    double *r = d.dbuf, *next = d.dbuf + d.n, *dsum = d.dbuf + 2 * d.n;
+    const bool rank_dev = is_device_ptr(rank);
+    cudaEvent_t ev0, ev1;
+    CUDA_TRY(cudaEventCreate(&ev0));
+    CUDA_TRY(cudaEventCreate(&ev1));
+    CUDA_TRY(cudaEventRecord(ev0, s));
+    CUDA_TRY(launch_fill_f64(r, 1.0 / (double)d.n, d.n, s));
+    CUDA_TRY(cudaMemsetAsync(next, 0, d.n * 8, s));
+    uint32_t launches = 0;
+    EFG_TRY(start_traversal(d, 0, d.n, d.depth, nullptr, launches));  // frontier = every vertex
+    const int blocks = d.num_sms * expand_occupancy(kModePagerank);
+    for (uint32_t it = 0; it < iters; ++it) {
+        CUDA_TRY(cudaMemsetAsync(dsum, 0, 8, s));
+        CUDA_TRY(launch_pr_dangling(r, d.deg32, d.n, dsum, s));
+        CUDA_TRY(launch_expand(kModePagerank, expand_args(d, nullptr), blocks, s));
+        CUDA_TRY(launch_pr_update(r, next, d.n, damping, dsum, s));
+    }
+    // ranks back to input ids (next[] is free scratch now)
+    double *src = r;
+    if (d.old_of_new) {
+        CUDA_TRY(launch_gather64(r, d.new_of_old, next, d.n, s));
+        src = next;
+    }
+    CUDA_TRY(cudaEventRecord(ev1, s));
+    CUDA_TRY(cudaMemcpyAsync(rank, src, d.n * 8, rank_dev ? cudaMemcpyDeviceToDevice : cudaMemcpyDeviceToHost, s));
+    CUDA_TRY(cudaStreamSynchronize(s));
+    float ms = 0.f;
+    cudaEventElapsedTime(&ms, ev0, ev1);
+    cudaEventDestroy(ev0);
+    cudaEventDestroy(ev1);
+    if (st) {
+        std::memset(st, 0, offsetof(efg_stats, level_cap));
+        st->levels = iters;
+        st->edges_traversed = (uint64_t)iters * g->host.m;
+        st->device_ms = ms;
+        st->expand_launches = iters;
+    }
     return EFG_OK;
 }
 

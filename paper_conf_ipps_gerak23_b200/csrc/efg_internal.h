@@ -169,6 +169,8 @@ efg_status device_upload(efg_graph *g, const efg_build_opts &o);
 void device_free(DeviceGraph &d);
 efg_status device_decode(efg_graph *g, uint32_t v0, uint32_t v1, uint32_t *out);
 efg_status device_bfs(efg_graph *g, uint32_t source, int32_t *depth, uint32_t *parent, efg_stats *st);
+efg_status device_sssp(efg_graph *g, uint32_t source, float *dist, efg_stats *st);
+efg_status device_pagerank(efg_graph *g, double damping, uint32_t iters, double *rank, efg_stats *st);
 efg_status device_step_begin(efg_graph *g, uint32_t source, int32_t *depth);
 efg_status device_step_expand(efg_graph *g);
 efg_status device_step_finish(efg_graph *g, uint64_t *global_new);

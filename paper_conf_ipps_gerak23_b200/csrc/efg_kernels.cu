@@ -284,7 +284,7 @@ __global__ void __launch_bounds__(kFrontierThreads) compact_kernel(CompactArgs a
 #pragma unroll
         for (int u = 0; u < 4; ++u) {
             const uint64_t w = w0 + 32 * u;
-            c[u] = w < whi ? __popc(a.vis[w] & ~a.prev[w]) : 0u;
+            c[u] = w < whi ? __popc(a.consume ? a.vis[w] : (a.vis[w] & ~a.prev[w])) : 0u;
         }
 #pragma unroll
         for (int u = 0; u < 4; ++u) {
@@ -320,9 +320,15 @@ __global__ void __launch_bounds__(kFrontierThreads) compact_kernel(CompactArgs a
         const uint64_t w = w0 + lane;
         uint32_t nb = 0;
         if (w < whi) {
-            const uint32_t x = a.vis[w], p = a.prev[w];
-            nb = x & ~p;
-            if (nb) a.prev[w] = x;
+            const uint32_t x = a.vis[w];
+            if (a.consume) {  // SSSP: the relaxed set itself is the next frontier; reset it
+                nb = x;
+                if (x) a.vis[w] = 0;
+            } else {
+                const uint32_t p = a.prev[w];
+                nb = x & ~p;
+                if (nb) a.prev[w] = x;
+            }
         }
         const bool own = w >= a.own_lo_w && w < a.own_hi_w;
         const uint32_t nq = own ? nb : 0u;
@@ -338,7 +344,7 @@ __global__ void __launch_bounds__(kFrontierThreads) compact_kernel(CompactArgs a
             if ((nbw >> lane) & 1) {
                 const uint32_t v = (uint32_t)((w0 + j) * 32 + lane);
                 if (a.depth_stored) a.depth_stored[v] = level;  // stored-id order (coalesced)
-                if (!a.depth_stored_only) depth[v] = level;
+                if (!a.depth_stored_only && depth) depth[v] = level;
                 if (nqw) a.queue[base + offj + __popc(nqw & lt)] = v;
             }
         }
@@ -516,7 +522,9 @@ struct WarpSmem {
     uint8_t cs[kExpandStage];   // chunk slot of the element
     SlotGeom geom[32];
     SlotMeta meta[32];
-    uint64_t aux[32];           // parent: source vertex; decode: output index base
+    uint64_t aux[32];           // parent: source vertex; decode: output index base;
+                                // SSSP: weight index base; PageRank: share (double bits)
+    float aux2[32];             // SSSP: dist of the chunk's source vertex
 };
 
 struct WordLd {
@@ -576,6 +584,7 @@ __global__ void __launch_bounds__(kExpandThreads, 1) expand_kernel(ExpandArgs a)
     const uint32_t xl = a.ctrl->xlevel;  // index of the level being expanded
     uint32_t *parent = MODE == kModeVisitParent ? a.ctrl->parent : nullptr;
     const uint32_t hot_limit = a.hot_words * 32;  // vertex ids below this use s_hot
+    constexpr bool kBfs = MODE == kModeVisit || MODE == kModeVisitParent;
     if (MODE != kModeDecode) {
         if (threadIdx.x == 0 && a.stats && xl < a.max_stats) atomicMin(&a.stats[xl].t0, globaltimer());
         if (blockIdx.x == 0 && threadIdx.x == 0) {
@@ -583,6 +592,8 @@ __global__ void __launch_bounds__(kExpandThreads, 1) expand_kernel(ExpandArgs a)
             a.ctrl->seq = a.ctrl->seq + 1;
             a.ctrl->nnew = 0;
         }
+    }
+    if (kBfs) {
         // level-start snapshot of the hot visited words
         const uint4 *src = reinterpret_cast<const uint4 *>(a.vis);
         uint4 *dst = reinterpret_cast<uint4 *>(s_hot);
@@ -685,6 +696,14 @@ __global__ void __launch_bounds__(kExpandThreads, 1) expand_kernel(ExpandArgs a)
                     for (uint64_t q = (A0 >> 3) & ~127ull; q < ((A1 + 7) >> 3); q += 128) prefetch_l2(a.data + q);
                 }
                 if (MODE == kModeVisitParent) ws.aux[lane] = v_j;
+                if (MODE == kModeSssp) {  // weights are stored in CSR order: index vlist[u] + rank
+                    ws.aux[lane] = a.vlist[v_j] + r0 - ebt;
+                    ws.aux2[lane] = a.dist[v_j];
+                }
+                if (MODE == kModePagerank) {  // push r(u)/deg(u) along every edge
+                    const double share = a.rank[v_j] / (double)deg_j;
+                    ws.aux[lane] = (uint64_t)__double_as_longlong(share);
+                }
                 // decode: CSR position of the chunk's first element E_v + r0, E_v = W_v - A*q_v
                 if (MODE == kModeDecode) ws.aux[lane] = Wv_j - A * (fi + (uint64_t)j) + r0 - ebt;
             }
@@ -756,6 +775,30 @@ __global__ void __launch_bounds__(kExpandThreads, 1) expand_kernel(ExpandArgs a)
 #pragma unroll
                         for (int u = 0; u < kVisitBatch; ++u)
                             if (ok[u]) a.out[ws.aux[sv[u]] + run + base + u * 32 + lane] = xv[u];
+                    } else if (MODE == kModeSssp) {
+                        // relax: d' = fl32(dist(u) + w), single rounding (reading C20)
+                        float nd[kVisitBatch], cd[kVisitBatch];
+#pragma unroll
+                        for (int u = 0; u < kVisitBatch; ++u) {
+                            nd[u] = INFINITY;
+                            cd[u] = 0.f;
+                            if (ok[u]) {
+                                const float w = __ldg(a.weights + ws.aux[sv[u]] + run + base + u * 32 + lane);
+                                nd[u] = __fadd_rn(ws.aux2[sv[u]], w);
+                                cd[u] = a.dist[xv[u]];
+                            }
+                        }
+#pragma unroll
+                        for (int u = 0; u < kVisitBatch; ++u) {
+                            if (ok[u] && nd[u] < cd[u]) {  // non-negative floats order like their bits
+                                const int old = atomicMin(reinterpret_cast<int *>(a.dist) + xv[u], __float_as_int(nd[u]));
+                                if (__float_as_int(nd[u]) < old) atomicOr(a.vis + (xv[u] >> 5), 1u << (xv[u] & 31));
+                            }
+                        }
+                    } else if (MODE == kModePagerank) {
+#pragma unroll
+                        for (int u = 0; u < kVisitBatch; ++u)
+                            if (ok[u]) atomicAdd(a.next + xv[u], __longlong_as_double((long long)ws.aux[sv[u]]));
                     } else {
                         // Alg. 1 line 3: hot ids answer from shared memory
                         bool need[kVisitBatch], hot[kVisitBatch];
@@ -792,6 +835,52 @@ __global__ void __launch_bounds__(kExpandThreads, 1) expand_kernel(ExpandArgs a)
         atomicMax(&a.stats[xl].t1, globaltimer());
 }
 
+// PageRank (reading C21): D = sum of rank over degree-0 vertices; then
+// r'(v) = (1-d)/N + d * (next(v) + D/N), next(v) = 0.  fp64 throughout.
+__global__ void pr_dangling_kernel(const double *rank, const uint32_t *deg32, uint64_t n, double *dsum)
+{
+    double acc = 0.0;
+    for (uint64_t v = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; v < n; v += (uint64_t)gridDim.x * blockDim.x)
+        if (deg32[v] == 0) acc += rank[v];
+#pragma unroll
+    for (int d = 16; d; d >>= 1) acc += __shfl_xor_sync(FULL, acc, d);
+    if ((threadIdx.x & 31) == 0 && acc != 0.0) atomicAdd(dsum, acc);
+}
+
+__global__ void pr_update_kernel(double *rank, double *next, uint64_t n, double damping, const double *dsum)
+{
+    const double base = (1.0 - damping) / (double)n, dn = *dsum / (double)n;
+    for (uint64_t v = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; v < n; v += (uint64_t)gridDim.x * blockDim.x) {
+        rank[v] = base + damping * (next[v] + dn);
+        next[v] = 0.0;
+    }
+}
+
+__global__ void fill_kernel(uint32_t *p, uint32_t val, uint64_t n)
+{
+    for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x)
+        p[i] = val;
+}
+
+__global__ void fill_f64_kernel(double *p, double val, uint64_t n)
+{
+    for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x)
+        p[i] = val;
+}
+
+// out[v] = stored[new_of_old[v]] for 32- or 64-bit values (relabelled graphs)
+__global__ void gather32_kernel(const uint32_t *stored, const uint32_t *new_of_old, uint32_t *out, uint64_t n)
+{
+    for (uint64_t v = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; v < n; v += (uint64_t)gridDim.x * blockDim.x)
+        out[v] = stored[new_of_old ? new_of_old[v] : v];
+}
+
+__global__ void gather64_kernel(const double *stored, const uint32_t *new_of_old, double *out, uint64_t n)
+{
+    for (uint64_t v = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; v < n; v += (uint64_t)gridDim.x * blockDim.x)
+        out[v] = stored[new_of_old ? new_of_old[v] : v];
+}
+
 // depth_out[old_of_new[i]] = depth_stored[i] as a gather over input ids:
 // depth_out[v] = depth_stored[new_of_old[v]] (coalesced stores).
 __global__ void map_depth_kernel(const int32_t *stored, const uint32_t *new_of_old, int32_t *out, uint64_t n)
@@ -809,6 +898,47 @@ __global__ void map_parent_kernel(const uint32_t *pin, const uint32_t *old_of_ne
 }
 
 }  // namespace
+
+static unsigned grid_for(uint64_t n) { return (unsigned)std::max<uint64_t>(1, std::min<uint64_t>((n + 255) / 256, 148 * 16)); }
+
+cudaError_t launch_pr_dangling(const double *rank, const uint32_t *deg32, uint64_t n, double *dsum, cudaStream_t s)
+{
+    pr_dangling_kernel<<<grid_for(n), 256, 0, s>>>(rank, deg32, n, dsum);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_pr_update(double *rank, double *next, uint64_t n, double damping, const double *dsum,
+                             cudaStream_t s)
+{
+    pr_update_kernel<<<grid_for(n), 256, 0, s>>>(rank, next, n, damping, dsum);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_fill(uint32_t *p, uint32_t val, uint64_t n, cudaStream_t s)
+{
+    fill_kernel<<<grid_for(n), 256, 0, s>>>(p, val, n);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_fill_f64(double *p, double val, uint64_t n, cudaStream_t s)
+{
+    fill_f64_kernel<<<grid_for(n), 256, 0, s>>>(p, val, n);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_gather32(const uint32_t *stored, const uint32_t *new_of_old, uint32_t *out, uint64_t n,
+                            cudaStream_t s)
+{
+    gather32_kernel<<<grid_for(n), 256, 0, s>>>(stored, new_of_old, out, n);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_gather64(const double *stored, const uint32_t *new_of_old, double *out, uint64_t n,
+                            cudaStream_t s)
+{
+    gather64_kernel<<<grid_for(n), 256, 0, s>>>(stored, new_of_old, out, n);
+    return cudaGetLastError();
+}
 
 cudaError_t launch_map_depth(const int32_t *stored, const uint32_t *new_of_old, int32_t *out, uint64_t n,
                              cudaStream_t s)
@@ -838,6 +968,10 @@ static cudaError_t expand_set_attrs()
         e = cudaFuncSetAttribute(expand_kernel<kModeVisitParent>, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes);
     if (e == cudaSuccess)
         e = cudaFuncSetAttribute(expand_kernel<kModeDecode>, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes);
+    if (e == cudaSuccess)
+        e = cudaFuncSetAttribute(expand_kernel<kModeSssp>, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes);
+    if (e == cudaSuccess)
+        e = cudaFuncSetAttribute(expand_kernel<kModePagerank>, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes);
     if (e == cudaSuccess) done = true;
     return e;
 }
@@ -859,6 +993,12 @@ cudaError_t launch_expand(int mode, const ExpandArgs &a, int blocks, cudaStream_
         break;
     case kModeVisitParent:
         expand_kernel<kModeVisitParent><<<blocks, kExpandThreads, sm, s>>>(a);
+        break;
+    case kModeSssp:
+        expand_kernel<kModeSssp><<<blocks, kExpandThreads, sm, s>>>(a);
+        break;
+    case kModePagerank:
+        expand_kernel<kModePagerank><<<blocks, kExpandThreads, sm, s>>>(a);
         break;
     default:
         expand_kernel<kModeDecode><<<blocks, kExpandThreads, sm, s>>>(a);

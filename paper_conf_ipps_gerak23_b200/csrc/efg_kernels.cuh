@@ -11,6 +11,8 @@ enum ExpandMode : int {
     kModeVisit = 0,        // BFS: visited-bitmap probe + atomicOr (Alg. 1 lines 3-4)
     kModeVisitParent = 1,  // BFS with parents (winner of the atomicOr writes parent)
     kModeDecode = 2,       // efg_decode: store the decoded value in CSR order
+    kModeSssp = 3,         // SSSP relax: atomicMin on fp32 dist, mark relaxed vertices
+    kModePagerank = 4,     // PageRank push: next[v] += r(u)/deg(u)
 };
 
 struct ExpandArgs {
@@ -22,6 +24,11 @@ struct ExpandArgs {
     uint32_t *vis;             // visited bitmap (modes 0, 1)
     uint32_t *out;             // decode output (mode 2)
     LevelStat *stats;          // per-level statistics (device) or null
+    const uint64_t *vlist;     // SSSP: CSR offsets (weight index)
+    const float *weights;      // SSSP: weights in CSR order
+    float *dist;               // SSSP: distances (stored ids)
+    const double *rank;        // PageRank: current ranks (stored ids)
+    double *next;              // PageRank: accumulated pushes
     uint32_t max_stats;
     uint32_t hot_words;        // bitmap words with a shared-memory snapshot (multiple of 4)
     uint32_t k;                // forward-pointer quantum (chunk length); 0 = none
@@ -41,6 +48,7 @@ struct CompactArgs {
     uint32_t *queue;           // out: next frontier, sorted
     int32_t *depth_stored;     // depth by stored id (always written)
     int depth_stored_only;     // 1: depth_stored is the only depth output (relabelled graphs)
+    int consume;               // 1: frontier = vis itself, vis reset (SSSP relaxed set)
     LevelCtrl *ctrl;           // in: level, seq, depth ptr; out: nf
     uint64_t *status;          // cross-block prefix words (one per block)
     uint64_t nwords, words_per_block;
@@ -79,6 +87,15 @@ cudaError_t launch_xchg(const XchgArgs &a, cudaStream_t s);
 int expand_occupancy(int mode);
 size_t expand_smem_bytes();
 // pout[old_of_new[i]] = pin[i] == ~0u ? ~0u : old_of_new[pin[i]]  (parents back to input ids)
+cudaError_t launch_pr_dangling(const double *rank, const uint32_t *deg32, uint64_t n, double *dsum, cudaStream_t s);
+cudaError_t launch_pr_update(double *rank, double *next, uint64_t n, double damping, const double *dsum,
+                             cudaStream_t s);
+cudaError_t launch_fill(uint32_t *p, uint32_t val, uint64_t n, cudaStream_t s);
+cudaError_t launch_fill_f64(double *p, double val, uint64_t n, cudaStream_t s);
+cudaError_t launch_gather32(const uint32_t *stored, const uint32_t *new_of_old, uint32_t *out, uint64_t n,
+                            cudaStream_t s);
+cudaError_t launch_gather64(const double *stored, const uint32_t *new_of_old, double *out, uint64_t n,
+                            cudaStream_t s);
 cudaError_t launch_map_depth(const int32_t *stored, const uint32_t *new_of_old, int32_t *out, uint64_t n,
                              cudaStream_t s);
 cudaError_t launch_map_parent(const uint32_t *pin, const uint32_t *old_of_new, uint32_t *pout, uint64_t n,

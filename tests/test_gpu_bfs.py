@@ -303,3 +303,43 @@ def test_partitioned_bfs_simulated_ranks(efg, world):
                 assert np.array_equal(d.cpu().numpy(), ref)
         for g in graphs:
             g.free()
+
+
+@pytest.mark.parametrize("reorder", [False, True])
+def test_sssp_bit_exact_vs_dijkstra(efg, reorder):
+    """NEXT-1: fp32 frontier Bellman-Ford == fp32 Dijkstra bit for bit (C20)."""
+    n, src, dst = synth.rmat(13, 16, seed=21)
+    w_in = synth.weights(src, dst, seed=2000 + 1)
+    flags = efg.EFG_DEFAULT_FLAGS | (efg.EFG_REORDER_DEGREE if reorder else 0)
+    g = efg.Graph.build(n, src, dst, weights=w_in, flags=flags)
+    ov, oe = oracle.csr_build(n, src, dst)
+    u = np.repeat(np.arange(n, dtype=np.uint32), np.diff(ov).astype(np.int64))
+    w_csr = synth.weights(u, oe, seed=2000 + 1)  # symmetric pair function -> CSR-order weights
+    for s in (0, 17, 4000):
+        got = g.sssp(s)
+        ref = oracle.sssp(ov, oe, w_csr, s)
+        assert np.array_equal(got.view(np.uint32), ref.view(np.uint32)), s
+    g.free()
+
+
+def test_sssp_requires_weights(efg):
+    n, src, dst = synth.rmat(10, 8, seed=1)
+    g = efg.Graph.build(n, src, dst)
+    with pytest.raises(efg.EFGError):
+        g.sssp(0)
+    g.free()
+
+
+@pytest.mark.parametrize("reorder", [False, True])
+def test_pagerank_vs_fp64_oracle(efg, reorder):
+    """NEXT-2 (P:185, 50 iterations P:201): within 1e-6 relative L1 of the fp64 oracle."""
+    n, src, dst = synth.rmat(14, 16, seed=22)
+    flags = efg.EFG_DEFAULT_FLAGS | (efg.EFG_REORDER_DEGREE if reorder else 0)
+    g = efg.Graph.build(n, src, dst, flags=flags)
+    ov, oe = oracle.csr_build(n, src, dst)
+    got = g.pagerank(0.85, 50)
+    ref = oracle.pagerank(ov, oe, 0.85, 50)
+    rel = np.abs(got - ref).sum() / np.abs(ref).sum()
+    assert rel < 1e-6, rel
+    assert abs(got.sum() - 1.0) < 1e-9
+    g.free()
