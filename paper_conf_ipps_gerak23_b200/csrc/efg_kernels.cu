@@ -569,7 +569,7 @@ __device__ __forceinline__ void prefetch_l2(const void *p)
     asm volatile("prefetch.global.L2 [%0];" ::"l"(p));
 }
 
-constexpr int kVisitBatch = 4;  // decoded elements per lane whose probes are in flight together
+constexpr int kVisitBatch = 2;  // decoded elements per lane whose probes are in flight together
 
 template <int MODE>
 __global__ void __launch_bounds__(kExpandThreads, 1) expand_kernel(ExpandArgs a)
@@ -740,16 +740,21 @@ __global__ void __launch_bounds__(kExpandThreads, 1) expand_kernel(ExpandArgs a)
                     const SlotGeom &sg = ws.geom[cur.s];
                     const uint64_t rank = sg.r0 + run + ep - sg.eb;  // rank of the first set bit
                     // hi = hb + p (p = bit within the half), hb -= 1 per bit
-                    uint32_t hb = (uint32_t)(cur.wi * 32 + (lane & 1) * 16 - sg.U0 - rank);
-                    uint32_t w = cur.word, e = ep;
+                    // hi of the bit at position b with e = its slot: hbe + b - e
+                    const uint32_t hbe = (uint32_t)(cur.wi * 32 + (lane & 1) * 16 - sg.U0 - rank) + ep;
+                    const uint32_t w = cur.word;
                     const uint8_t sc = (uint8_t)cur.s;
-                    do {
-                        ws.hi[e] = hb + (__ffs(w) - 1);
-                        ws.cs[e] = sc;
-                        w &= w - 1;
-                        --hb;
-                        ++e;
-                    } while (w);
+                    uint32_t e = ep;
+                    // uniform 16-step scan of the half-word (no lane waits on the
+                    // densest half of the warp, unlike an ffs loop)
+#pragma unroll
+                    for (int b = 0; b < 16; ++b) {
+                        if ((w >> b) & 1) {
+                            ws.hi[e] = hbe + b - e;
+                            ws.cs[e] = sc;
+                            ++e;
+                        }
+                    }
                 }
                 __syncwarp();
                 // balanced pass: element e on lane e % 32, kVisitBatch in flight,
@@ -811,18 +816,23 @@ __global__ void __launch_bounds__(kExpandThreads, 1) expand_kernel(ExpandArgs a)
                         uint32_t gwd[kVisitBatch];
 #pragma unroll
                         for (int u = 0; u < kVisitBatch; ++u) gwd[u] = need[u] ? a.vis[xv[u] >> 5] : FULL;
+                        bool act = false;
 #pragma unroll
-                        for (int u = 0; u < kVisitBatch; ++u) {
-                            const uint32_t bit = 1u << (xv[u] & 31);
-                            if (!(gwd[u] & bit)) {  // line 4 (stale reads are benign: the atomic decides)
-                                if (MODE == kModeVisit) {
-                                    atomicOr(a.vis + (xv[u] >> 5), bit);
-                                } else {
-                                    const uint32_t old = atomicOr(a.vis + (xv[u] >> 5), bit);
-                                    if (!(old & bit)) parent[xv[u]] = (uint32_t)ws.aux[sv[u]];
+                        for (int u = 0; u < kVisitBatch; ++u) act |= need[u];
+                        if (__any_sync(FULL, act)) {  // most probes of a heavy level stop here
+#pragma unroll
+                            for (int u = 0; u < kVisitBatch; ++u) {
+                                const uint32_t bit = 1u << (xv[u] & 31);
+                                if (!(gwd[u] & bit)) {  // line 4 (stale reads are benign: the atomic decides)
+                                    if (MODE == kModeVisit) {
+                                        atomicOr(a.vis + (xv[u] >> 5), bit);
+                                    } else {
+                                        const uint32_t old = atomicOr(a.vis + (xv[u] >> 5), bit);
+                                        if (!(old & bit)) parent[xv[u]] = (uint32_t)ws.aux[sv[u]];
+                                    }
                                 }
+                                if (need[u] && hot[u]) atomicOr(s_hot + (xv[u] >> 5), bit);
                             }
-                            if (need[u] && hot[u]) atomicOr(s_hot + (xv[u] >> 5), bit);
                         }
                     }
                 }
