@@ -51,6 +51,7 @@ def parse():
     p.add_argument("--config", type=int, default=2, help="BASELINE.json config index (1-based)")
     p.add_argument("--scale", type=int, default=None, help="override RMAT scale (debug only)")
     p.add_argument("--no-cpu-baseline", action="store_true")
+    p.add_argument("--no-alt", action="store_true", help="skip the reorder=none comparison run")
     p.add_argument("--mode", default="partition", choices=["partition", "replicas"],
                    help="N > 1: 1-D partitioned BFS with a per-level NCCL exchange (SURVEY 8(e)), "
                         "or independent replicas on disjoint sources")
@@ -112,6 +113,19 @@ class ClockSampler:
                     reasons.add(nm)
         return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": smax,
                 "reasons": sorted(reasons), "samples": len(sm)}
+
+
+def load_traffic(workload: str, reorder: str):
+    """dram bytes per expand launch from the committed ncu capture of this
+    workload (profiles/r1_expand_traffic.json), or None."""
+    path = os.path.join(ROOT, "profiles", "r1_expand_traffic.json")
+    if not os.path.exists(path):
+        return None
+    with open(path) as f:
+        t = json.load(f)
+    if t.get("workload") != workload or t.get("reorder") != reorder:
+        return None
+    return t
 
 
 def load_peak():
@@ -383,6 +397,30 @@ def main():
         dist.all_reduce(e2e_e, op=dist.ReduceOp.SUM)
     e2e_val = float(e2e_e.item()) / float(e2e_t.item()) / 1e9
 
+    # ---- the same measurement without the degree relabelling (transparency) ----
+    alt = None
+    if world == 1 and args.reorder == "degree" and not args.no_alt:
+        n2, s2, d2, _ = make_graph_edges(args.config, args.scale)
+        g2 = efg.Graph.build(n2, s2, d2, device=local, stream=stream.cuda_stream)
+        del s2, d2
+        with torch.cuda.stream(stream):
+            for s in my[:args.warmup]:
+                g2.bfs(int(s), depth=depth)
+        torch.cuda.synchronize()
+        a0 = torch.cuda.Event(enable_timing=True)
+        a1 = torch.cuda.Event(enable_timing=True)
+        e_alt = 0
+        a0.record(stream)
+        with torch.cuda.stream(stream):
+            for s in my[args.warmup:]:
+                _, _, st2 = g2.bfs(int(s), depth=depth, stats=True)
+                e_alt += st2["edges_traversed"]
+        a1.record(stream)
+        torch.cuda.synchronize()
+        alt = {"reorder": "none", "value": e_alt / (a0.elapsed_time(a1) * 1e-3) / 1e9, "unit": UNIT,
+               "ef_data_bytes_per_edge": g2.info["data_bytes"] / g2.info["m"]}
+        g2.free()
+
     # ---- cpu baseline: the oracle on a bounded sample (rank 0, N=1 only) ----
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
@@ -404,6 +442,7 @@ def main():
 
     if rank == 0:
         cfgname = synth.CONFIGS[args.config]["name"] + (f"_scale{args.scale}" if args.scale else "")
+        trf = load_traffic(cfgname, args.reorder)
         line = {
             "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": float(t_tot.item()) / args.steps,
@@ -422,7 +461,11 @@ def main():
             "gpu_launches": launches,
             "roofline": {"bound": "hbm", "kernel": "expand_kernel (a4+a5+a6)",
                          "achieved": achieved, "peak": peak, "unit": "GB/s",
-                         "frac": achieved / peak, "traffic": None, "peak_source": peak_src,
+                         "frac": achieved / peak,
+                         "traffic": (trf or {}).get("dram_bytes_per_launch"),
+                         "traffic_source": (trf or {}).get("source"),
+                         "alg_bytes_per_launch": alg_bytes / max(exp_launch, 1),
+                         "peak_source": peak_src,
                          "expand_launches": exp_launch, "expand_ms_total": exp_ms,
                          "expand_ms_total_graph_mode_globaltimer": exp_ms_gt,
                          "expand_share_of_step": exp_ms_gt / ms if ms else None,
@@ -431,6 +474,7 @@ def main():
             "e2e": {"value": e2e_val, "unit": UNIT, "h2d_bytes_per_step": 4,
                     "d2h_bytes_per_step": 4 * n},
             "cpu_baseline": cpu,
+            "alt_no_reorder": alt,
         }
         print(json.dumps(line), flush=True)
     g.free()

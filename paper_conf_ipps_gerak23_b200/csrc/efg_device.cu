@@ -402,7 +402,7 @@ efg_status device_bfs(efg_graph *g, uint32_t source, int32_t *depth, uint32_t *p
             const LevelStat &x = d.stats_host[i];
             lms.push_back(x.t1 > x.t0 ? (float)((double)(x.t1 - x.t0) * 1e-6) : 0.f);
         }
-        launches += 3 * levels;
+        launches += 3 * levels + (relabel ? 1 : 0);
     } else {
         const int blocks = d.num_sms * expand_occupancy(mode);
         for (;;) {
@@ -428,7 +428,10 @@ efg_status device_bfs(efg_graph *g, uint32_t source, int32_t *depth, uint32_t *p
             launches += 3;
             ++levels;
         }
-        if (relabel) CUDA_TRY(launch_map_depth(d.depth_st, d.new_of_old, dd, d.n, s));
+        if (relabel) {
+            CUDA_TRY(launch_map_depth(d.depth_st, d.new_of_old, dd, d.n, s));
+            ++launches;
+        }
         CUDA_TRY(cudaEventRecord(ev1, s));
     }
     if (parent && relabel) CUDA_TRY(launch_map_parent(pd, d.old_of_new, pout, d.n, s));
