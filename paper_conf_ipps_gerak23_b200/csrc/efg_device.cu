@@ -225,6 +225,11 @@ efg_status device_upload(efg_graph *g, const efg_build_opts &o)
     CUDA_TRY(cudaGetDeviceProperties(&prop, o.device));
     d.num_sms = prop.multiProcessorCount;
 
+    // the expand kernel stages select1(i) - i (< 2 * degree) in 27 bits
+    for (uint64_t v = 0; v < h.n; ++v)
+        if (h.vlist[v + 1] - h.vlist[v] >= (1ull << 26))
+            return set_error(EFG_ENOTSUP, "efg_build: a vertex degree >= 2^26 is not supported on the device");
+
     // EF data, padded so 32-bit word reads past the last list stay in bounds
     d.data_bytes = h.data.size();
     const uint64_t padded = ((d.data_bytes + 64) + 15) & ~15ull;

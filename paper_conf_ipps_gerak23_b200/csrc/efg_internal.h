@@ -97,7 +97,7 @@ constexpr uint32_t kMaxLevelStats = 4096;
 constexpr int kExpandThreads = 1024;         // one CTA per SM, 32 warps
 constexpr int kExpandWarps = kExpandThreads / 32;
 constexpr int kExpandStage = 512;            // elements of one 16-word step (<= 16*32)
-constexpr uint32_t kHotWords = 19 * 1024;    // 76 KB shared-memory visited snapshot = 622,592 ids
+constexpr uint32_t kHotWords = 23 * 1024;    // 92 KB shared-memory visited snapshot = 753,664 ids
 constexpr int kFrontierThreads = 512;        // compact / plan kernels (16 warps)
 constexpr int kBitmapAlign = 1024;           // bitmap words are padded to a multiple of this
 // Step a3 partitions "work units" rather than bare edges: a frontier vertex

@@ -518,8 +518,9 @@ struct alignas(16) SlotMeta {
 };
 
 struct WarpSmem {
-    uint32_t hi[kExpandStage];  // select1(i) - i by element slot of the step
-    uint8_t cs[kExpandStage];   // chunk slot of the element
+    // per element of the step: (select1(i) - i) << 5 | chunk slot.  select1(i) - i
+    // = x >> l < 2 * deg, and degrees are < 2^26 (checked at build), so it fits.
+    uint32_t hs[kExpandStage];
     SlotGeom geom[32];
     SlotMeta meta[32];
     uint64_t aux[32];           // parent: source vertex; decode: output index base;
@@ -743,15 +744,14 @@ __global__ void __launch_bounds__(kExpandThreads, 1) expand_kernel(ExpandArgs a)
                     // hi of the bit at position b with e = its slot: hbe + b - e
                     const uint32_t hbe = (uint32_t)(cur.wi * 32 + (lane & 1) * 16 - sg.U0 - rank) + ep;
                     const uint32_t w = cur.word;
-                    const uint8_t sc = (uint8_t)cur.s;
+                    const uint32_t sc = (uint32_t)cur.s;
                     uint32_t e = ep;
                     // uniform 16-step scan of the half-word (no lane waits on the
                     // densest half of the warp, unlike an ffs loop)
 #pragma unroll
                     for (int b = 0; b < 16; ++b) {
                         if ((w >> b) & 1) {
-                            ws.hi[e] = hbe + b - e;
-                            ws.cs[e] = sc;
+                            ws.hs[e] = ((hbe + b - e) << 5) | sc;
                             ++e;
                         }
                     }
@@ -767,8 +767,9 @@ __global__ void __launch_bounds__(kExpandThreads, 1) expand_kernel(ExpandArgs a)
                         const uint32_t e = base + u * 32 + lane;
                         ok[u] = e < tot;
                         const uint32_t es = ok[u] ? e : 0;
-                        const uint32_t hi = ws.hi[es];
-                        sv[u] = ws.cs[es];
+                        const uint32_t hsv = ws.hs[es];
+                        const uint32_t hi = hsv >> 5;
+                        sv[u] = hsv & 31;
                         const SlotMeta m = ws.meta[sv[u]];
                         const uint64_t ba = m.lb + (uint64_t)(run + es) * m.l;
                         const uint32_t *p = data32 + (ba >> 5);
