@@ -77,12 +77,13 @@ ExpandArgs expand_args(DeviceGraph &d, uint32_t *out)
 {
     ExpandArgs a;
     a.data = d.data;
-    a.rec = d.rec;
-    a.queue = d.queue;
+    a.chunks = d.chunks;
     a.tiles = d.tiles;
+    a.deg32 = d.deg32;
     a.ctrl = d.ctrl;
     a.vis = d.vis;
     a.out = out;
+    a.out_base = 0;
     a.stats = d.stats;
     a.vlist = d.vlist;
     a.weights = d.weights;
@@ -92,7 +93,6 @@ ExpandArgs expand_args(DeviceGraph &d, uint32_t *out)
     a.max_stats = kMaxLevelStats;
     a.hot_words = (uint32_t)std::min<uint64_t>(kHotWords, d.nwords) & ~3u;
     a.k = d.k;
-    a.kshift = kshift_of(d.k);
     return a;
 }
 
@@ -102,6 +102,7 @@ CompactArgs compact_args(DeviceGraph &d, bool consume = false)
     a.consume = consume ? 1 : 0;
     a.vis = d.vis;
     a.prev = d.prev;
+    a.iso = d.iso;
     a.queue = d.queue;
     a.depth_stored = (d.old_of_new && !consume) ? d.depth_st : nullptr;
     a.depth_stored_only = d.old_of_new ? 1 : 0;
@@ -119,6 +120,9 @@ PlanArgs plan_args(DeviceGraph &d, cudaGraphConditionalHandle cond)
     PlanArgs a;
     a.queue = d.queue;
     a.deg32 = d.deg32;
+    a.rec = d.rec;
+    a.data = d.data;
+    a.chunks = d.chunks;
     a.tiles = d.tiles;
     a.ctrl = d.ctrl;
     a.status = d.status + kMaxGrid;
@@ -188,12 +192,14 @@ void device_free(DeviceGraph &d)
     cudaFree(d.data);
     cudaFree(d.rec);
     cudaFree(d.deg32);
+    cudaFree(d.iso);
     cudaFree(d.vlist);
     cudaFree(d.weights);
     cudaFree(d.vis);
     cudaFree(d.prev);
     cudaFree(d.queue);
     cudaFree(d.tiles);
+    cudaFree(d.chunks);
     cudaFree(d.depth);
     cudaFree(d.parent);
     cudaFree(d.parent2);
@@ -264,6 +270,15 @@ efg_status device_upload(efg_graph *g, const efg_build_opts &o)
     CUDA_TRY(cudaMemcpyAsync(d.rec, rec.data(), h.n * sizeof(VRec), cudaMemcpyHostToDevice, s));
     EFG_TRY(dev_alloc(d, &d.deg32, d.nwords * 32));
     CUDA_TRY(cudaMemcpyAsync(d.deg32, deg.data(), d.nwords * 32 * 4, cudaMemcpyHostToDevice, s));
+    {
+        std::vector<uint32_t> iso(d.nwords, 0);
+        for (uint64_t v = 0; v < d.nwords * 32; ++v)
+            // a row-range handle knows degrees of its own rows only (others may be probed)
+            if (v >= h.n || (v >= h.row_lo && v < h.row_hi && deg[v] == 0)) iso[v >> 5] |= 1u << (v & 31);
+        EFG_TRY(dev_alloc(d, &d.iso, d.nwords));
+        CUDA_TRY(cudaMemcpyAsync(d.iso, iso.data(), d.nwords * 4, cudaMemcpyHostToDevice, s));
+        CUDA_TRY(cudaStreamSynchronize(s));
+    }
     EFG_TRY(dev_alloc(d, &d.vlist, h.n + 1));
     CUDA_TRY(cudaMemcpyAsync(d.vlist, h.vlist.data(), (h.n + 1) * 8, cudaMemcpyHostToDevice, s));
     if (!h.old_of_new.empty()) {
@@ -282,11 +297,15 @@ efg_status device_upload(efg_graph *g, const efg_build_opts &o)
     EFG_TRY(dev_alloc(d, &d.vis, d.nwords));
     EFG_TRY(dev_alloc(d, &d.prev, d.nwords));
     EFG_TRY(dev_alloc(d, &d.queue, h.n));
-    d.max_tiles = (h.m + (uint64_t)kVertexWork * h.n) / kTileWork + 2;
-    EFG_TRY(dev_alloc(d, &d.tiles, d.max_tiles));
+    // a level has at most one chunk per frontier vertex plus one per k elements
+    const uint64_t rows = (h.row_hi > h.row_lo) ? h.row_hi - h.row_lo : h.n;
+    d.max_chunks = rows + (h.k ? h.m / h.k : 0) + 1;
+    d.max_tiles = (h.m + (uint64_t)kChunkWork * d.max_chunks) / kTileWork + 2;
+    EFG_TRY(dev_alloc(d, &d.tiles, d.max_tiles + 1));
+    EFG_TRY(dev_alloc(d, &d.chunks, d.max_chunks));
     EFG_TRY(dev_alloc(d, &d.depth, h.n));
-    EFG_TRY(dev_alloc(d, &d.status, 2 * kMaxGrid));
-    CUDA_TRY(cudaMemsetAsync(d.status, 0, 2 * kMaxGrid * 8, s));
+    EFG_TRY(dev_alloc(d, &d.status, 3 * kMaxGrid));
+    CUDA_TRY(cudaMemsetAsync(d.status, 0, 3 * kMaxGrid * 8, s));
     EFG_TRY(dev_alloc(d, &d.stats, kMaxLevelStats));
     EFG_TRY(dev_alloc(d, &d.ctrl, 1));
     CUDA_TRY(cudaMemsetAsync(d.ctrl, 0, sizeof(LevelCtrl), s));
@@ -338,7 +357,9 @@ efg_status device_decode(efg_graph *g, uint32_t v0, uint32_t v1, uint32_t *out)
     do {
         if ((st = start_traversal(d, v0, v1, d.depth, nullptr, launches)) != EFG_OK) break;
         const int blocks = d.num_sms * expand_occupancy(kModeDecode);
-        cudaError_t e = launch_expand(kModeDecode, expand_args(d, od), blocks, s);
+        ExpandArgs ea = expand_args(d, od);
+        ea.out_base = h.vlist[v0];
+        cudaError_t e = launch_expand(kModeDecode, ea, blocks, s);
         if (e == cudaSuccess && !out_dev) e = cudaMemcpyAsync(out, od, cnt * 4, cudaMemcpyDeviceToHost, s);
         if (e == cudaSuccess) e = cudaStreamSynchronize(s);
         if (e != cudaSuccess) st = set_error(EFG_ECUDA, std::string("efg_decode: ") + cudaGetErrorString(e));

@@ -62,20 +62,26 @@ static_assert(sizeof(VRec) == 16, "VRec must be 16 bytes");
 constexpr int kOffBits = 58;
 constexpr uint64_t kOffMask = (1ull << kOffBits) - 1;
 
-// Tile table entry (step a3): first chunk owned by an edge tile.
-struct alignas(16) TileEntry {
-    uint32_t fi;      // index into the frontier queue
-    uint32_t chunk;   // chunk index within that vertex's list
-    uint64_t w;       // work position of the chunk start (see kTileWork)
+// Chunk descriptor (step a1, written by plan_kernel, read by expand_kernel):
+// one k-aligned piece of a frontier vertex's list.  The expand
+// kernel derives the chunk's bit ranges from it and the forward pointers (a4).
+struct alignas(16) ChunkDesc {
+    uint64_t off_l;  // the list's VRec.off_l: byte offset in data (58 bits) | l << 58
+    uint32_t deg;    // list length
+    uint32_t ubytes; // upper-bits section bytes of the list
+    uint32_t v;      // source vertex (stored id)
+    uint32_t cc;     // chunk index within the list (rank of its first element r0 = cc*k)
+    uint32_t pad[2];
 };
-static_assert(sizeof(TileEntry) == 16, "TileEntry must be 16 bytes");
+static_assert(sizeof(ChunkDesc) == 32, "ChunkDesc must be 32 bytes");
 
 // Level control block (device), written by the advance kernel.
 struct LevelCtrl {
     uint64_t nf;        // frontier size for the next expand
     uint64_t ne;        // edges out of that frontier (E_L)
     uint64_t ntiles;    // ceil(nwork / kTileWork)
-    uint64_t nwork;     // work units = ne + kVertexWork * nf
+    uint64_t nwork;     // work units = ne + kChunkWork * nchunks
+    uint64_t nchunks;   // chunk descriptors of the level
     int32_t *depth;     // depth buffer of the current call
     uint32_t *parent;   // parent buffer of the current call, or null
     uint32_t level;     // depth assigned by the next compact
@@ -85,6 +91,8 @@ struct LevelCtrl {
     uint64_t nnew;      // vertices discovered in the last level (all rows; partitioned runs)
     uint64_t total_nf;  // sum of frontier sizes (= vertices reached)
     uint64_t total_ne;  // sum of E_L (= edges traversed, reading C18)
+    uint32_t vmin;      // compact: smallest vertex that is neither visited nor isolated (atomicMin)
+    uint32_t vpre;      // plan -> expand: every vertex below it is visited or isolated
 };
 
 // Per-level statistics written on the device (graph mode has no host loop).
@@ -94,17 +102,21 @@ struct LevelStat {
 };
 constexpr uint32_t kMaxLevelStats = 4096;
 
-constexpr int kExpandThreads = 1024;         // one CTA per SM, 32 warps
+// expand_kernel: one CTA per SM, kExpandWarps warps; each warp owns two
+// staging buffers (TMA double buffering) and a word-round workspace.
+constexpr int kExpandThreads = 512;
 constexpr int kExpandWarps = kExpandThreads / 32;
-constexpr int kExpandStage = 512;            // elements of one 16-word step (<= 16*32)
-constexpr uint32_t kHotWords = 23 * 1024;    // 92 KB shared-memory visited snapshot = 753,664 ids
+constexpr uint32_t kStageBytes = 4096;       // one staging buffer (>= the largest single chunk)
+constexpr uint32_t kUpperStageMax = 1024;    // larger upper-bit regions are read from global memory
+constexpr uint32_t kRoundWords = 128;        // upper-bit words decoded per round
+constexpr uint32_t kHotWords = 8 * 1024;     // 32 KB shared-memory visited snapshot = 262,144 ids
 constexpr int kFrontierThreads = 512;        // compact / plan kernels (16 warps)
 constexpr int kBitmapAlign = 1024;           // bitmap words are padded to a multiple of this
-// Step a3 partitions "work units" rather than bare edges: a frontier vertex
-// costs kVertexWork units (its record gather and list set-up) plus one per edge,
-// so a tile of kTileWork units holds at most kTileWork/kVertexWork short lists.
-constexpr uint32_t kTileWork = 2048;         // work units per warp tile (a3)
-constexpr uint32_t kVertexWork = 32;         // per-vertex overhead in work units
+// Step a3 partitions "work units" rather than bare edges: a chunk costs
+// kChunkWork units (descriptor, staging, set-up) plus one per element, so a
+// tile of kTileWork units holds at most kTileWork/kChunkWork chunks.
+constexpr uint32_t kTileWork = 2048;         // work units per tile (a3)
+constexpr uint32_t kChunkWork = 32;          // per-chunk overhead in work units
 
 constexpr unsigned kMaxGrid = 4096;
 
@@ -117,14 +129,17 @@ struct DeviceGraph {
     uint64_t data_bytes = 0;
     VRec *rec = nullptr;               // n records
     uint32_t *deg32 = nullptr;         // n degrees (padded to the bitmap size)
+    uint32_t *iso = nullptr;           // bitmap of the degree-0 vertices and the padding (nwords)
     uint64_t *vlist = nullptr;         // n+1 (SSSP weight indexing / decode)
     float *weights = nullptr;          // m or null
     // traversal workspace
     uint32_t *vis = nullptr;           // visited bitmap (nwords)
     uint32_t *prev = nullptr;          // visited bitmap at the end of the last level
     uint32_t *queue = nullptr;         // frontier queue (n)
-    TileEntry *tiles = nullptr;        // tile table (max_tiles)
+    uint32_t *tiles = nullptr;         // tile table: first chunk of each tile (max_tiles + 1)
     uint64_t max_tiles = 0;
+    ChunkDesc *chunks = nullptr;       // chunk descriptors of the level (max_chunks)
+    uint64_t max_chunks = 0;
     int32_t *depth = nullptr;          // internal depth (n)
     uint32_t *parent = nullptr;        // internal parent (n), lazily allocated
     uint32_t *parent2 = nullptr;       // parent in input ids (reordered graphs), lazily

@@ -116,35 +116,6 @@ __device__ __forceinline__ ChunkLen make_chunk(uint32_t k, int kshift)
     return c;
 }
 
-// Entry of tile t whose boundary t*T falls inside vertex q's work range
-// [W, W + kVertexWork + d): the first chunk whose start is >= t*T (chunk 0
-// starts at W, chunk c > 0 at W + kVertexWork + c*k), or the next vertex.
-__device__ __forceinline__ TileEntry tile_entry(uint64_t t, uint64_t q, uint64_t W, uint64_t d,
-                                                const ChunkLen &cl)
-{
-    const uint64_t ch = cl.ch, A = kVertexWork;
-    const uint64_t o = t * kTileWork - W;
-    TileEntry te;
-    if (o == 0) {
-        te.fi = (uint32_t)q;
-        te.chunk = 0;
-        te.w = W;
-        return te;
-    }
-    uint64_t c = o > A ? cl.div(o - A + ch - 1) : 1;
-    if (c == 0) c = 1;
-    if (c * ch < d) {
-        te.fi = (uint32_t)q;
-        te.chunk = (uint32_t)c;
-        te.w = W + A + c * ch;
-    } else {
-        te.fi = (uint32_t)(q + 1);
-        te.chunk = 0;
-        te.w = W + A + d;
-    }
-    return te;
-}
-
 // --------------------------------------------------------------------------
 // Cross-block exclusive prefix for the two frontier scans (a2, a7).  A block
 // publishes its aggregate as one 64-bit word tag << 40 | value (value < 2^40),
@@ -214,12 +185,6 @@ __device__ __forceinline__ uint64_t block_excl_u64(uint64_t x, uint64_t &total, 
     return pre + ex;
 }
 
-__device__ __forceinline__ uint64_t block_sum_u64(uint64_t x, uint64_t *s_warp)
-{
-    uint64_t tot;
-    block_excl_u64<kFrontierThreads>(x, tot, s_warp);
-    return tot;
-}
 
 // --------------------------------------------------------------------------
 // init_kernel: per-call state (level 0, a fresh tag) and the start set:
@@ -237,6 +202,8 @@ __global__ void init_kernel(InitArgs a)
         a.ctrl->nnew = 0;
         a.ctrl->total_nf = 0;
         a.ctrl->total_ne = 0;
+        a.ctrl->vmin = 0xffffffffu;
+        a.ctrl->vpre = 0;
         if (a.parent) a.parent[a.v0] = (uint32_t)a.v0;
     }
     const uint64_t w0 = a.v0 >> 5, w1 = (a.v1 + 31) >> 5;
@@ -279,12 +246,21 @@ __global__ void __launch_bounds__(kFrontierThreads) compact_kernel(CompactArgs a
 
     // pass 1: count (queue = owned words only; nnew = every row); 4 loads in flight
     uint64_t cnt = 0, all = 0;
+    uint32_t vmin = 0xffffffffu;  // smallest vertex of this warp's range that is neither visited nor isolated
     for (uint64_t w0 = wlo + lane; w0 < whi; w0 += 128) {
         uint32_t c[4];
 #pragma unroll
         for (int u = 0; u < 4; ++u) {
             const uint64_t w = w0 + 32 * u;
-            c[u] = w < whi ? __popc(a.consume ? a.vis[w] : (a.vis[w] & ~a.prev[w])) : 0u;
+            c[u] = 0;
+            if (w < whi) {
+                const uint32_t x = a.vis[w];
+                c[u] = __popc(a.consume ? x : (x & ~a.prev[w]));
+                if (!a.consume && vmin == 0xffffffffu) {
+                    const uint32_t un = ~(x | a.iso[w]);
+                    if (un) vmin = (uint32_t)(w * 32) + (__ffs(un) - 1);
+                }
+            }
         }
 #pragma unroll
         for (int u = 0; u < 4; ++u) {
@@ -295,9 +271,12 @@ __global__ void __launch_bounds__(kFrontierThreads) compact_kernel(CompactArgs a
     }
     cnt = warp_sum_u64(cnt);
     all = warp_sum_u64(all);
+#pragma unroll
+    for (int d = 16; d; d >>= 1) vmin = min(vmin, __shfl_xor_sync(FULL, vmin, d));
     if (lane == 0) {
         s_wcnt[wid] = cnt;
         s_warp[wid] = all;
+        if (vmin != 0xffffffffu) atomicMin(&a.ctrl->vmin, vmin);
     }
     __syncthreads();
     if (wid == 0) {
@@ -382,63 +361,85 @@ __global__ void xchg_kernel(XchgArgs a)
 }
 
 // --------------------------------------------------------------------------
-// plan_kernel: a1 + a2 + a3.  For the sorted frontier queue: degree lookup
-// (a1), exclusive scan of the per-vertex work kVertexWork + deg (a2), and the
-// tile table (a3: each tile of kTileWork units gets its first chunk, the
-// Fig. 4 maxle rule applied once per tile).  Same reduce-then-scan scheme as
-// compact_kernel, over the frontier index range.  The last block publishes
-// the level totals, records per-level statistics and, in graph mode, sets the
-// loop condition (frontier non-empty).
+// plan_kernel: a1 + a2 + a3 + a4.  For the sorted frontier queue:
+//   a1  degree lookup (pass 1: compact deg32; pass 2: the 16-byte record),
+//   a2  exclusive scans of the per-vertex chunk count and work
+//       (kChunkWork per chunk + one unit per element),
+//       one ChunkDesc per k-aligned chunk: the list's record and
+//       the chunk index, written by lanes over the group's chunks,
+//   a3  the tile table: tile t (work [tT, (t+1)T)) starts at the first chunk
+//       whose work position is >= tT (the Fig. 4 maxle rule, once per tile).
+// Same reduce-then-scan scheme as compact_kernel, over the frontier index
+// range.  The last block publishes the level totals, records per-level
+// statistics and, in graph mode, sets the loop condition (frontier non-empty).
 // --------------------------------------------------------------------------
 __global__ void __launch_bounds__(kFrontierThreads) plan_kernel(PlanArgs a)
 {
     constexpr int NT = kFrontierThreads, NW = NT / 32;
-    __shared__ uint64_t s_wwork[NW];
-    __shared__ uint64_t s_pre;
+    __shared__ uint64_t s_wwork[NW], s_wch[NW];
+    __shared__ uint64_t s_pre, s_cpre;
 
     const uint32_t tid = threadIdx.x, lane = tid & 31, wid = tid >> 5, b = blockIdx.x;
     LevelCtrl *ctrl = a.ctrl;
     const uint32_t tag = ctrl->seq;
     const uint64_t nf = ctrl->nf;
     const ChunkLen cl = make_chunk(a.k, a.kshift);
-    const uint64_t A = kVertexWork;
+    const uint64_t CH = cl.ch, CW = kChunkWork;
     const uint64_t per = (nf + gridDim.x - 1) / gridDim.x;
     const uint64_t lo = min((uint64_t)b * per, nf), hi = min(lo + per, nf);
     const uint64_t per_w = (per + NW - 1) / NW;
     const uint64_t qlo = min(lo + wid * per_w, hi), qhi = min(qlo + per_w, hi);
 
-    // pass 1: work of the warp's range (a1 degree lookup), 4 lookups in flight
-    uint64_t wk = 0;
+    // pass 1: chunks and work of the warp's range (a1 degree lookup), 4 lookups in flight
+    uint64_t wk = 0, ch = 0;
     for (uint64_t i0 = qlo + lane; i0 < qhi; i0 += 128) {
         uint32_t q[4];
 #pragma unroll
         for (int u = 0; u < 4; ++u) q[u] = i0 + 32 * u < qhi ? a.queue[i0 + 32 * u] : 0u;
 #pragma unroll
         for (int u = 0; u < 4; ++u)
-            if (i0 + 32 * u < qhi) wk += A + __ldg(a.deg32 + q[u]);
+            if (i0 + 32 * u < qhi) {
+                const uint64_t d = __ldg(a.deg32 + q[u]);
+                const uint64_t nch = d ? cl.div(d + CH - 1) : 0;
+                wk += nch * CW + d;
+                ch += nch;
+            }
     }
     wk = warp_sum_u64(wk);
-    if (lane == 0) s_wwork[wid] = wk;
+    ch = warp_sum_u64(ch);
+    if (lane == 0) {
+        s_wwork[wid] = wk;
+        s_wch[wid] = ch;
+    }
     __syncthreads();
     if (wid == 0) {
         const uint64_t blk = warp_sum_u64(lane < NW ? s_wwork[lane] : 0);
+        const uint64_t blkc = warp_sum_u64(lane < NW ? s_wch[lane] : 0);
         const uint64_t pre = publish_and_prefix(a.status, b, tag, blk);
+        const uint64_t cpre = publish_and_prefix(a.status + kMaxGrid, b, tag, blkc);
         if (lane == 0) {
             s_pre = pre;
+            s_cpre = cpre;
             if (b == gridDim.x - 1) {
-                const uint64_t nwork = pre + blk;
+                const uint64_t nwork = pre + blk, nchunks = cpre + blkc;
+                const uint64_t ne = nwork - CW * nchunks;
                 const uint32_t lvl = ctrl->level;
+                const uint64_t ntiles = (nwork + kTileWork - 1) / kTileWork;
                 ctrl->nwork = nwork;
-                ctrl->ne = nwork - A * nf;
-                ctrl->ntiles = (nwork + kTileWork - 1) / kTileWork;
+                ctrl->nchunks = nchunks;
+                ctrl->ne = ne;
+                ctrl->ntiles = ntiles;
                 ctrl->xlevel = lvl;
+                ctrl->vpre = ctrl->vmin;  // compact of this level end is complete (stream order)
+                ctrl->vmin = 0xffffffffu;
+                a.tiles[ntiles] = (uint32_t)nchunks;  // sentinel: end of the last tile
                 if (nf) {
                     ctrl->nlevels = lvl + 1;
                     ctrl->total_nf += nf;
-                    ctrl->total_ne += nwork - A * nf;
+                    ctrl->total_ne += ne;
                     if (a.stats && lvl < a.max_stats) {
                         a.stats[lvl].nf = nf;
-                        a.stats[lvl].ne = nwork - A * nf;
+                        a.stats[lvl].ne = ne;
                         a.stats[lvl].t0 = ~0ull;
                         a.stats[lvl].t1 = 0;
                     }
@@ -448,140 +449,201 @@ __global__ void __launch_bounds__(kFrontierThreads) plan_kernel(PlanArgs a)
         }
     }
     __syncthreads();
-    uint64_t run = s_pre;
-    for (uint32_t w = 0; w < wid; ++w) run += s_wwork[w];
+    uint64_t run = s_pre, crun = s_cpre;
+    for (uint32_t w = 0; w < wid; ++w) {
+        run += s_wwork[w];
+        crun += s_wch[w];
+    }
 
-    // pass 2: exclusive scan of the work (a2) and the tile table (a3); the next
-    // 32 degrees are fetched while the current ones are scanned
-    uint32_t dn = qlo + lane < qhi ? __ldg(a.deg32 + a.queue[qlo + lane]) : 0u;
+    // pass 2: 32 frontier vertices at a time (one per lane); the next group's
+    // queue entries are fetched while the current group is processed
+    uint32_t vn = qlo + lane < qhi ? a.queue[qlo + lane] : 0u;
     for (uint64_t i0 = qlo; i0 < qhi; i0 += 32) {
         const uint64_t i = i0 + lane;
-        const uint64_t d = dn;
-        if (i0 + 32 < qhi) dn = i + 32 < qhi ? __ldg(a.deg32 + a.queue[i + 32]) : 0u;
-        uint64_t tot;
-        const uint64_t W = run + warp_excl_u64(i < qhi ? A + d : 0, tot);
-        // tiles whose boundary t*T falls in this group's work window
-        // [W_0, W_0 + tot): lanes take consecutive tiles, each finds its vertex
+        const uint32_t v = vn;
+        if (i0 + 32 < qhi) vn = i + 32 < qhi ? a.queue[i + 32] : 0u;
+        uint64_t off_l = 0;
+        uint32_t d = 0, ub = 0;
+        if (i < qhi) {
+            const uint4 r = __ldg(reinterpret_cast<const uint4 *>(a.rec + v));
+            off_l = ((uint64_t)r.y << 32) | r.x;
+            d = r.z;
+            ub = r.w;
+        }
+        const uint32_t nch = d ? (uint32_t)cl.div((uint64_t)d + CH - 1) : 0u;
+        uint64_t totw;
+        const uint64_t W = run + warp_excl_u64((uint64_t)nch * CW + d, totw);
+        uint32_t totc;
+        const uint32_t cb = warp_excl_u32(nch, totc);
+
+        // a4: descriptors, lanes over the group's chunks (owner by maxle, C13)
+        for (uint32_t j0 = 0; j0 < totc; j0 += 32) {
+            const uint32_t j = j0 + lane;
+            const int o = warp_maxle_u32(i < qhi ? cb : 0xffffffffu, j);
+            const uint64_t ol = __shfl_sync(FULL, off_l, o);
+            const uint32_t od = __shfl_sync(FULL, d, o), oub = __shfl_sync(FULL, ub, o);
+            const uint32_t ov = __shfl_sync(FULL, v, o), ocb = __shfl_sync(FULL, cb, o);
+            if (j < totc) {
+                uint4 *dp = reinterpret_cast<uint4 *>(a.chunks + crun + j);
+                dp[0] = make_uint4((uint32_t)ol, (uint32_t)(ol >> 32), od, oub);
+                dp[1] = make_uint4(ov, j - ocb, 0u, 0u);
+            }
+        }
+
+        // a3: tiles whose boundary t*T falls in this group's work window
+        // [W_0, W_0 + totw): lanes take consecutive tiles, each finds its vertex
         // by maxle over the group's W (Fig. 4 rule inside the warp)
         const uint64_t wstart = __shfl_sync(FULL, W, 0);
         const uint64_t tfirst = (wstart + kTileWork - 1) / kTileWork;
-        const uint64_t tend = (wstart + tot + kTileWork - 1) / kTileWork;
-        const uint32_t wrel = i < qhi ? (uint32_t)(W - wstart) : 0xffffffffu;  // < tot <= 2^32
+        const uint64_t tend = (wstart + totw + kTileWork - 1) / kTileWork;
+        const uint32_t wrel = i < qhi ? (uint32_t)(W - wstart) : 0xffffffffu;  // < totw <= 2^32
         for (uint64_t t0 = tfirst; t0 < tend; t0 += 32) {
             const uint64_t t = t0 + lane;
             const uint32_t key = t < tend ? (uint32_t)(t * kTileWork - wstart) : 0u;
-            const int j = warp_maxle_u32(wrel, key);
-            const uint64_t jW = __shfl_sync(FULL, W, j), jd = __shfl_sync(FULL, d, j);
-            if (t < tend) a.tiles[t] = tile_entry(t, i0 + j, jW, jd, cl);
+            const int o = warp_maxle_u32(wrel, key);
+            const uint64_t oW = __shfl_sync(FULL, W, o);
+            const uint32_t onch = __shfl_sync(FULL, nch, o), ocb = __shfl_sync(FULL, cb, o);
+            if (t < tend) {
+                // chunk c of the owner starts at W + c*(CW + k); first chunk at or after t*T
+                const uint64_t rel = t * kTileWork - oW;
+                const uint64_t c = a.k ? (rel + CW + CH - 1) / (CW + CH) : (rel ? 1 : 0);
+                a.tiles[t] = (uint32_t)(crun + ocb + min(c, (uint64_t)onch));
+            }
         }
-        run += tot;
+        run += totw;
+        crun += totc;
     }
 }
 
 // --------------------------------------------------------------------------
 // expand_kernel: a4 + a5 + a6 (P:137-177 generalised, Alg. 1 lines 3-6)
 //
-// Persistent: one CTA of kExpandThreads per SM, one warp per work tile.  A
-// tile's work is a run of "chunks": k-aligned pieces of frontier lists
-// (P:157), so every chunk starts right after a forward pointer and needs no
-// select to find its first bit.  Chunks are taken 32 at a time ("batch"; many
-// short lists per warp: the multi-list case).  The batch's
-// upper-bit words are laid end to end and processed 32 words per step (one
-// aligned 32-bit word per lane, coalesced; the next step's word is loaded
-// before the current one is used):
-//   popcount + warp exclusive scan -> rank of each word's first stop bit (the
-//                                     segmented scan of P:171-177; segments are
-//                                     chunks, whose element prefix is subtracted)
-//   set-bit enumeration (ffs)       -> select1(i) - i per element, staged in
-//                                     shared memory by element slot (Alg. 2's
-//                                     select step, without its byte LUT)
-//   balanced pass, element e on lane e%32, kVisitBatch in flight, branch-free
-//                                   -> lower bits by a funnel shift of two
-//                                     coalesced words, x = hi << l | lo, visit.
-// Visit: the first hot_words*32 vertex ids (the highest-degree vertices when the
-// graph was built with EFG_REORDER_DEGREE) have a per-CTA shared-memory copy of
-// their visited bits, loaded at kernel start (a snapshot of the level start,
-// updated by this CTA's own discoveries).  A set bit there answers the probe
-// without touching L1/L2; otherwise the global bitmap is probed and the
-// atomicOr decides (stale reads are benign).
+// Persistent: one CTA of kExpandWarps warps per SM; a warp takes tiles
+// gw, gw + #warps, ...  A tile's chunks (plan_kernel descriptors) are cut into
+// batches of <= 32 chunks whose compressed bytes fit one staging buffer.  Per
+// batch the warp
+//   (producer)  a4: locates each chunk's bits from the forward pointers
+//               (Fig. 6: a chunk starts right after pointer cc-1, so
+//               no select is needed) and stages the lower fields and upper
+//               words into shared memory with TMA bulk copies (cp.async.bulk,
+//               completion on a per-buffer mbarrier), one batch ahead of the
+//               decoder (double buffering);
+//   (rounds)    lays the batch's upper-bit words end to end (kRoundWords per
+//               round), masks each chunk's first/last word and keeps the
+//               non-zero words as 16-byte records {word, hi base, lower-field
+//               base, l} with the popcount prefix of each (the rank of its
+//               first stop bit: the segmented scan of P:171-177, segments =
+//               chunks);
+//   (decode)    a5: splits the round's elements evenly over the lanes; a lane
+//               finds select1 of its first element once (maxle over the record
+//               prefix, Fig. 4 rule, then an in-word select) and walks its run
+//               serially: the next set bit (ffs) gives select1(i) - i, the lower
+//               field is a funnel shift of two shared-memory words, x = hi << l
+//               | lo; an exhausted word is refilled from the next record without
+//               a branch (every record has a set bit);
+//   (visit)     a6: kU elements per lane in flight: hot ids answer from a
+//               per-CTA shared-memory copy of their visited bits (a snapshot of
+//               the level start, updated by this CTA's discoveries), the others
+//               probe the global bitmap, and atomicOr decides (stale reads are
+//               benign, C16).
 // --------------------------------------------------------------------------
-struct SlotGeom {
-    uint64_t A0, A1, U0;  // absolute bit range of the chunk's upper bits; upper start
-    uint32_t wb, eb;      // exclusive word / element prefix within the batch
-    uint64_t r0;          // rank of the chunk's first element in its list
+struct SlotP {        // one chunk of the batch being decoded (shared memory)
+    uint32_t lsmb;    // shared-window bit address of element e's lower field = lsmb + e*l (mod 2^32)
+    uint32_t lflags;  // l | (A0 & 31) << 8 | ((A1 - 1) & 31) << 16 | staged-upper << 24
+    uint32_t HB;      // hi = 32*g + p - e + HB  (g batch word, p bit in word, e batch element)
+    uint32_t eb;      // first batch element of the chunk
+    uint32_t wb;      // first batch word of the chunk
+    uint32_t nwd;     // upper-bit words of the chunk
+    uint64_t usrc;    // staged: stage-area word index of batch word wb; else global word index
+    uint64_t aux;     // parent: v; decode / SSSP: CSR position of the chunk's first element; PR: share bits
+    float aux2;       // SSSP: dist of the chunk's source vertex
+    uint32_t pad;
 };
-
-struct alignas(16) SlotMeta {
-    uint64_t lb;     // lower-bit address of batch element e: lb + e*l (modular)
-    uint32_t l;      // lower bits per element
-    uint32_t lmask;  // (1 << l) - 1
-};
+static_assert(sizeof(SlotP) == 48, "SlotP");
 
 struct WarpSmem {
-    // per element of the step: (select1(i) - i) << 5 | chunk slot.  select1(i) - i
-    // = x >> l < 2 * deg, and degrees are < 2^26 (checked at build), so it fits.
-    uint32_t hs[kExpandStage];
-    SlotGeom geom[32];
-    SlotMeta meta[32];
-    uint64_t aux[32];           // parent: source vertex; decode: output index base;
-                                // SSSP: weight index base; PageRank: share (double bits)
-    float aux2[32];             // SSSP: dist of the chunk's source vertex
+    uint32_t stage[2][kStageBytes / 4];   // TMA staging buffers (16-byte aligned)
+    uint4 wrec[kRoundWords];              // non-zero words of the round: {word, 32g + HB, lsmb, l | slot << 8}
+    uint32_t wpre[kRoundWords];           // batch element index of each record's first stop bit
+    SlotP slot[32];
+    uint64_t mbar[2];
 };
 
-struct WordLd {
-    uint32_t word;
-    int s;
-    uint64_t wi;
-};
+constexpr size_t kExpandSmem = (size_t)kHotWords * 4 + (size_t)kExpandWarps * sizeof(WarpSmem);
+static_assert(kExpandSmem <= 232448, "expand kernel shared memory exceeds 227 KB");
+static_assert(sizeof(WarpSmem) % 16 == 0, "WarpSmem alignment");
 
-__device__ __forceinline__ WordLd load_word(const uint32_t *data32, const SlotGeom *geom,
-                                            uint32_t wb, uint32_t g, uint32_t W)
+__device__ __forceinline__ uint32_t smem_u32(const void *p)
 {
-    WordLd r;
-    r.s = warp_maxle_u32(wb, g);
-    r.word = 0;
-    r.wi = 0;
-    if (g < W) {
-        const SlotGeom &sg = geom[r.s];
-        const uint64_t w0 = sg.A0 >> 5, wl = (sg.A1 - 1) >> 5;
-        r.wi = w0 + (g - sg.wb);
-        uint32_t word = ldg_u32(data32 + r.wi);
-        if (r.wi == w0) word &= FULL << (uint32_t)(sg.A0 & 31);
-        if (r.wi == wl) {
-            const uint32_t hb = (uint32_t)(sg.A1 - wl * 32);  // 1..32 valid bits
-            if (hb < 32) word &= (1u << hb) - 1;
-        }
-        r.word = word;
+    return static_cast<uint32_t>(__cvta_generic_to_shared(p));
+}
+
+__device__ __forceinline__ void mbar_init(uint64_t *bar, uint32_t count)
+{
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count) : "memory");
+}
+
+__device__ __forceinline__ void mbar_arrive_expect_tx(uint64_t *bar, uint32_t bytes)
+{
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes)
+                 : "memory");
+}
+
+__device__ __forceinline__ void mbar_wait(uint64_t *bar, uint32_t parity)
+{
+    const uint32_t addr = smem_u32(bar);
+    uint32_t done = 0;
+    while (!done) {
+        asm volatile(
+            "{\n\t.reg .pred p;\n\t"
+            "mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n\t"
+            "selp.u32 %0, 1, 0, p;\n\t}"
+            : "=r"(done)
+            : "r"(addr), "r"(parity)
+            : "memory");
     }
-    return r;
 }
 
-// Lane l of a step handles the 16-bit half (l & 1) of batch word g0 + (l >> 1).
-__device__ __forceinline__ WordLd load_half(const uint32_t *data32, const SlotGeom *geom, uint32_t wb,
-                                            uint32_t lane, uint32_t g0, uint32_t W)
+__device__ __forceinline__ uint32_t lds_u32(uint32_t addr)
 {
-    WordLd r = load_word(data32, geom, wb, g0 + (lane >> 1), W);
-    r.word = (lane & 1) ? (r.word >> 16) : (r.word & 0xffffu);
-    return r;
+    uint32_t v;
+    asm volatile("ld.shared.u32 %0, [%1];" : "=r"(v) : "r"(addr));
+    return v;
 }
 
-__device__ __forceinline__ void prefetch_l2(const void *p)
+// TMA bulk copy global -> shared (16-byte aligned addresses, size a multiple of 16)
+__device__ __forceinline__ void bulk_g2s(void *dst, const void *src, uint32_t bytes, uint64_t *bar)
 {
-    asm volatile("prefetch.global.L2 [%0];" ::"l"(p));
+    asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
+                 ::"r"(smem_u32(dst)), "l"(src), "r"(bytes), "r"(smem_u32(bar))
+                 : "memory");
 }
 
-constexpr int kVisitBatch = 2;  // decoded elements per lane whose probes are in flight together
+__device__ __forceinline__ void fence_proxy_async()
+{
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+}
+
+// Producer output of one batch: per lane = per chunk slot (registers), plus
+// the batch totals (warp-uniform).
+struct Batch {
+    uint32_t cnt, ne, nw, buf;   // chunks, elements, upper words, staging buffer
+    uint32_t lsmb, lflags, HB, eb, wb, nwd, v, cc;
+    uint64_t usrc;
+};
+
+constexpr int kU = 4;  // elements per lane whose probes are in flight together
 
 template <int MODE>
 __global__ void __launch_bounds__(kExpandThreads, 1) expand_kernel(ExpandArgs a)
 {
-    extern __shared__ __align__(16) uint8_t smem_raw[];
-    uint32_t *s_hot = reinterpret_cast<uint32_t *>(smem_raw);
-    WarpSmem *ws_all = reinterpret_cast<WarpSmem *>(smem_raw + kHotWords * 4);
+    extern __shared__ __align__(128) uint8_t smem_raw[];
+    WarpSmem *ws_all = reinterpret_cast<WarpSmem *>(smem_raw);
+    uint32_t *s_hot = reinterpret_cast<uint32_t *>(smem_raw + (size_t)kExpandWarps * sizeof(WarpSmem));
 
     const uint32_t lane = lane_id(), wid = threadIdx.x >> 5;
     WarpSmem &ws = ws_all[wid];
-    const uint64_t ntiles = a.ctrl->ntiles, nf = a.ctrl->nf, nwork = a.ctrl->nwork;
+    const uint64_t ntiles = a.ctrl->ntiles;
     const uint32_t xl = a.ctrl->xlevel;  // index of the level being expanded
     uint32_t *parent = MODE == kModeVisitParent ? a.ctrl->parent : nullptr;
     const uint32_t hot_limit = a.hot_words * 32;  // vertex ids below this use s_hot
@@ -594,253 +656,337 @@ __global__ void __launch_bounds__(kExpandThreads, 1) expand_kernel(ExpandArgs a)
             a.ctrl->nnew = 0;
         }
     }
+    if (lane == 0) {
+        mbar_init(&ws.mbar[0], 1);
+        mbar_init(&ws.mbar[1], 1);
+    }
     if (kBfs) {
         // level-start snapshot of the hot visited words
         const uint4 *src = reinterpret_cast<const uint4 *>(a.vis);
         uint4 *dst = reinterpret_cast<uint4 *>(s_hot);
         for (uint32_t i = threadIdx.x; i < a.hot_words / 4; i += blockDim.x) dst[i] = src[i];
-        __syncthreads();
     }
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    __syncthreads();
+
+    const uint8_t *data = a.data;
     const uint32_t *data32 = reinterpret_cast<const uint32_t *>(a.data);
-    const ChunkLen cl = make_chunk(a.k, a.kshift);
-    const uint64_t CH = cl.ch;
-    const uint64_t A = kVertexWork;
+    const uint32_t *st32 = &ws.stage[0][0];
+    const uint32_t sbits = smem_u32(st32) * 8;  // shared-window bit address of the staging area
+    const uint32_t vpre = kBfs ? a.ctrl->vpre : 0u;  // ids below it are visited (or never probed)
     const uint64_t gw = (uint64_t)blockIdx.x * kExpandWarps + wid;
     const uint64_t nwarps = (uint64_t)gridDim.x * kExpandWarps;
+    const uint64_t CH = a.k ? a.k : (1ull << 40);
 
-    for (uint64_t tile = gw; tile < ntiles; tile += nwarps) {
-        const TileEntry te = a.tiles[tile];
-        uint64_t fi = te.fi, c0 = te.chunk, P = te.w;
-        const uint64_t Pend = min((tile + 1) * (uint64_t)kTileWork, nwork);
+    // producer cursor: chunks [cnext, cend) of the current tile
+    uint64_t tile = gw;
+    uint64_t cnext = 0, cend = 0;
+    if (tile < ntiles) {
+        cnext = a.tiles[tile];
+        cend = a.tiles[tile + 1];
+    }
+    uint32_t phase = 0;  // bit b: parity of the next wait on buffer b
+    uint32_t nbuf = 0;   // buffer of the next produced batch
 
-        while (P < Pend && fi < nf) {
-            // ---- a1 (gather): up to 32 frontier vertices, one per lane ----
-            const uint64_t fv = fi + lane;
-            uint32_t v = 0, deg = 0, ubytes = 0;
-            uint64_t offl = 0;
-            if (fv < nf) {
-                v = a.queue[fv];
-                const uint4 r = __ldg(reinterpret_cast<const uint4 *>(a.rec + v));
-                offl = ((uint64_t)r.y << 32) | r.x;
-                deg = r.z;
-                ubytes = r.w;
+    // ---- producer: descriptors -> chunk bit ranges (a4) -> staged bytes ----
+    auto produce = [&](Batch &B) -> bool {
+        while (cnext >= cend) {
+            tile += nwarps;
+            if (tile >= ntiles) return false;
+            cnext = a.tiles[tile];
+            cend = a.tiles[tile + 1];
+        }
+        const uint64_t c = cnext + lane;
+        const bool valid = c < cend;
+        uint64_t lb = 0, A0 = 0, A1 = 0;
+        uint32_t l = 0, nel = 0, hib = 0, v = 0, cc = 0;
+        if (valid) {
+            const uint4 *dp = reinterpret_cast<const uint4 *>(a.chunks + c);
+            const uint4 d0 = dp[0], d1 = dp[1];
+            const uint64_t offl = ((uint64_t)d0.y << 32) | d0.x;
+            const uint64_t off = offl & kOffMask;
+            const uint32_t deg = d0.z, ubytes = d0.w;
+            l = (uint32_t)(offl >> kOffBits);
+            v = d1.x;
+            cc = d1.y;
+            const uint64_t F = a.k ? (uint64_t)deg / a.k : 0;           // forward pointers (C8)
+            const uint64_t Lb = ((uint64_t)deg * l + 7) >> 3;            // lower section bytes
+            const uint64_t lbase = (off + 4 * F) * 8;
+            const uint64_t U0 = (off + 4 * F + Lb) * 8;
+            const uint64_t r0 = (uint64_t)cc * CH;
+            const uint64_t r1 = min(r0 + CH, (uint64_t)deg);
+            // chunk cc starts right after element r0-1, whose stop bit is
+            // fwd[cc-1] + r0 - 1; it ends after element r1-1 (C14)
+            hib = cc ? ld_u32_unaligned(data32, off + 4 * (uint64_t)(cc - 1)) : 0u;
+            const uint64_t b1 = r1 < deg ? (uint64_t)ld_u32_unaligned(data32, off + 4 * (uint64_t)cc) + r1
+                                         : 8ull * ubytes;
+            nel = (uint32_t)(r1 - r0);
+            lb = lbase + r0 * l;
+            A0 = U0 + (cc ? (uint64_t)hib + r0 : 0);
+            A1 = U0 + b1;
+        }
+        // byte ranges: lower fields [lg0, lg1) (+8 bytes for the two-word window),
+        // upper words [ug0, ug1), both 16-byte aligned supersets
+        uint64_t lg0 = 0, lg1 = 0, ug0 = 0, ug1 = 0;
+        uint32_t bytes = 0, lsz = 0;
+        bool ustage = false, merged = false;
+        uint32_t nwd = 0;
+        if (valid) {
+            if (l) {
+                lg0 = (lb >> 3) & ~15ull;
+                lg1 = ((((lb + (uint64_t)nel * l - 1) >> 5) * 4 + 8) + 15) & ~15ull;
             }
-            const uint64_t first = lane == 0 ? c0 : 0;
-            const uint64_t nch = deg ? cl.div(deg + CH - 1) : 0;
-            const uint32_t nrem = (uint32_t)(nch > first ? nch - first : 0);
-            // work still ahead of this vertex (from its first remaining chunk on)
-            const uint64_t wrem = fv < nf ? (first == 0 ? A + deg : deg - first * CH) : 0;
-            uint32_t totc;
-            const uint32_t cb = warp_excl_u32(nrem, totc);
-            uint64_t totw;
-            const uint64_t wbv = warp_excl_u64(wrem, totw);
-            // W_v of each vertex (work position of its chunk 0)
-            const uint64_t Wv = P + wbv - (first ? A + first * CH : 0);
-            if (totc == 0) {  // 32 empty lists
-                fi += 32;
-                c0 = 0;
-                P += totw;
-                continue;
+            ug0 = ((A0 >> 5) * 4) & ~15ull;
+            ug1 = ((((A1 - 1) >> 5) * 4 + 4) + 15) & ~15ull;
+            nwd = (uint32_t)(((A1 - 1) >> 5) - (A0 >> 5) + 1);
+            ustage = ug1 - ug0 <= kUpperStageMax;
+            merged = l && ustage && ug0 >= lg0 && ug0 <= lg1 + 16;
+            lsz = (uint32_t)(lg1 - lg0);
+            bytes = merged ? (uint32_t)(max(lg1, ug1) - lg0) : lsz + (ustage ? (uint32_t)(ug1 - ug0) : 0u);
+        }
+        uint32_t tb;
+        const uint32_t sb = warp_excl_u32(bytes, tb);
+        const bool fits = valid && sb + bytes <= kStageBytes;
+        B.cnt = __popc(__ballot_sync(FULL, fits));  // a prefix of the lanes; >= 1 (one chunk always fits)
+        const uint32_t buf = nbuf;
+        B.buf = buf;
+        nbuf ^= 1;
+        uint32_t tot_e, tot_w, tot_b;
+        B.eb = warp_excl_u32(fits ? nel : 0u, tot_e);
+        B.wb = warp_excl_u32(fits ? nwd : 0u, tot_w);
+        warp_excl_u32(fits ? bytes : 0u, tot_b);
+        B.ne = tot_e;
+        B.nw = tot_w;
+        B.nwd = nwd;
+        B.v = v;
+        B.cc = cc;
+        const uint32_t base = buf * kStageBytes + sb;  // stage-area byte offset of this chunk
+        const uint32_t lsm = sbits + (l ? base * 8 + (uint32_t)(lb - lg0 * 8) : buf * kStageBytes * 8);
+        B.lsmb = lsm - B.eb * l;
+        B.lflags = l | ((uint32_t)(A0 & 31) << 8) | ((uint32_t)((A1 - 1) & 31) << 16) | (ustage ? 1u << 24 : 0u);
+        B.HB = hib - 32u * B.wb - (uint32_t)(A0 & 31) + B.eb;
+        if (ustage) {
+            const uint32_t ub = merged ? base + (uint32_t)(ug0 - lg0) : base + lsz;
+            B.usrc = (ub + (uint32_t)((A0 >> 5) * 4 - ug0)) >> 2;
+        } else {
+            B.usrc = A0 >> 5;
+        }
+        cnext += B.cnt;
+        // stage (the buffer was last read by the decoder two batches ago)
+        __syncwarp();
+        if (lane == 0) mbar_arrive_expect_tx(&ws.mbar[buf], tot_b);
+        __syncwarp();
+        if (fits) {
+            fence_proxy_async();
+            uint8_t *dst = reinterpret_cast<uint8_t *>(&ws.stage[0][0]) + base;
+            if (merged) {
+                bulk_g2s(dst, data + lg0, bytes, &ws.mbar[buf]);
+            } else {
+                if (lsz) bulk_g2s(dst, data + lg0, lsz, &ws.mbar[buf]);
+                if (ustage) bulk_g2s(dst + lsz, data + ug0, (uint32_t)(ug1 - ug0), &ws.mbar[buf]);
             }
+        }
+        return true;
+    };
 
-            // ---- chunk slot t = lane -> owning vertex lane j (maxle, C13) ----
-            const int j = warp_maxle_u32(cb, lane);
-            const uint32_t deg_j = __shfl_sync(FULL, deg, j);
-            const uint64_t offl_j = __shfl_sync(FULL, offl, j);
-            const uint32_t ub_j = __shfl_sync(FULL, ubytes, j);
-            const uint32_t cb_j = __shfl_sync(FULL, cb, j);
-            const uint64_t Wv_j = __shfl_sync(FULL, Wv, j);
-            const uint32_t v_j = __shfl_sync(FULL, v, j);
-            const uint64_t nch_j = __shfl_sync(FULL, nch, j);
-            const uint64_t cc = (j == 0 ? c0 : 0) + (lane - cb_j);
-            const uint64_t r0 = cc * CH;
-            const uint64_t cstart = Wv_j + (cc ? A + cc * CH : 0);
-            const bool valid = lane < totc && cstart < Pend;
-            const uint32_t count = __popc(__ballot_sync(FULL, valid));
-            if (count == 0) break;
+    Batch cur, nxt;
+    bool have = produce(cur);
+    while (have) {
+        // slot table of the current batch (its producer registers are about to be reused)
+        const uint32_t cnt = cur.cnt, NW = cur.nw, buf = cur.buf;
+        if (lane < cnt) {
+            SlotP sp;
+            sp.lsmb = cur.lsmb;
+            sp.lflags = cur.lflags;
+            sp.HB = cur.HB;
+            sp.eb = cur.eb;
+            sp.wb = cur.wb;
+            sp.nwd = cur.nwd;
+            sp.usrc = cur.usrc;
+            sp.aux = 0;
+            sp.aux2 = 0.f;
+            sp.pad = 0;
+            const uint64_t r0 = (uint64_t)cur.cc * CH;
+            if (MODE == kModeVisitParent) sp.aux = cur.v;
+            if (MODE == kModeDecode) sp.aux = a.vlist[cur.v] + r0 - a.out_base;
+            if (MODE == kModeSssp) {
+                sp.aux = a.vlist[cur.v] + r0;
+                sp.aux2 = a.dist[cur.v];
+            }
+            if (MODE == kModePagerank) {  // push r(u)/deg(u) along every edge
+                const double share = a.rank[cur.v] / (double)a.deg32[cur.v];
+                sp.aux = (uint64_t)__double_as_longlong(share);
+            }
+            ws.slot[lane] = sp;
+        }
+        const uint32_t cwb = lane < cnt ? cur.wb : 0xffffffffu;  // slot word starts, for maxle
+        // stage the next batch while this one is decoded
+        have = produce(nxt);
+        __syncwarp();
+        mbar_wait(&ws.mbar[buf], (phase >> buf) & 1);
+        phase ^= 1u << buf;
 
-            // ---- a4: bit ranges of the chunk (forward pointers) ----
-            uint32_t nwd = 0, nel = 0;
-            uint64_t A0 = 0, A1 = 0, U0 = 0, lbase = 0;
-            uint32_t l = 0;
-            if (valid) {
-                const uint64_t off = offl_j & kOffMask;
-                l = (uint32_t)(offl_j >> kOffBits);
-                const uint64_t F = a.k ? cl.div(deg_j) : 0;
-                const uint64_t L = ((uint64_t)deg_j * l + 7) >> 3;
-                lbase = (off + 4 * F) * 8;
-                U0 = (off + 4 * F + L) * 8;
-                const uint64_t r1 = min(r0 + CH, (uint64_t)deg_j);
-                nel = (uint32_t)(r1 - r0);
-                const uint64_t b0 = cc ? (uint64_t)ld_u32_unaligned(data32, off + 4 * (cc - 1)) + r0 : 0;
-                const uint64_t b1 = r1 < deg_j ? (uint64_t)ld_u32_unaligned(data32, off + 4 * cc) + r1
-                                               : 8ull * ub_j;
-                A0 = U0 + b0;
-                A1 = U0 + b1;
-                nwd = (uint32_t)(((A1 - 1) >> 5) - (A0 >> 5) + 1);
-            }
-            uint32_t W, NE;
-            const uint32_t wb = warp_excl_u32(nwd, W);
-            const uint32_t ebt = warp_excl_u32(nel, NE);
-            (void)NE;
-            if (valid) {
-                ws.geom[lane] = SlotGeom{A0, A1, U0, wb, ebt, r0};
-                SlotMeta m;
-                m.lb = lbase + (r0 - (uint64_t)ebt) * l;  // modular: rank = r0 + (e - ebt)
-                m.l = l;
-                m.lmask = l ? (FULL >> (32 - l)) : 0u;
-                ws.meta[lane] = m;
-                // pull the chunk's lower and upper bits toward L2 ahead of the word steps
-                {
-                    const uint64_t lb0 = (lbase + r0 * l) >> 3, lb1 = (lbase + (r0 + nel) * l + 7) >> 3;
-                    for (uint64_t q = lb0 & ~127ull; q < lb1; q += 128) prefetch_l2(a.data + q);
-                    for (uint64_t q = (A0 >> 3) & ~127ull; q < ((A1 + 7) >> 3); q += 128) prefetch_l2(a.data + q);
+        uint32_t Er0 = 0;  // batch element index at the round start
+        for (uint32_t ga = 0; ga < NW; ga += kRoundWords) {
+            const uint32_t nw = min(kRoundWords, NW - ga);
+            // ---- round words: mask, popcount prefix, non-zero records ----
+            uint32_t run = Er0, nrec = 0;
+#pragma unroll
+            for (uint32_t j = 0; j < kRoundWords / 32; ++j) {
+                if (j * 32 >= nw) break;
+                const uint32_t gl = j * 32 + lane;
+                const uint32_t g = ga + gl;
+                const int sl = warp_maxle_u32(cwb, gl < nw ? g : 0u);
+                uint32_t wd = 0;
+                const SlotP &sp = ws.slot[sl];
+                if (gl < nw) {
+                    const uint64_t idx = sp.usrc + (g - sp.wb);
+                    wd = (sp.lflags >> 24) ? st32[idx] : ldg_u32(data32 + idx);
+                    if (g == sp.wb) wd &= FULL << ((sp.lflags >> 8) & 31);
+                    if (g == sp.wb + sp.nwd - 1) wd &= FULL >> (31 - ((sp.lflags >> 16) & 31));
                 }
-                if (MODE == kModeVisitParent) ws.aux[lane] = v_j;
-                if (MODE == kModeSssp) {  // weights are stored in CSR order: index vlist[u] + rank
-                    ws.aux[lane] = a.vlist[v_j] + r0 - ebt;
-                    ws.aux2[lane] = a.dist[v_j];
+                uint32_t tot;
+                const uint32_t ex = warp_excl_u32(__popc(wd), tot);
+                const uint32_t nzm = __ballot_sync(FULL, wd != 0);
+                if (wd) {
+                    const uint32_t k = nrec + __popc(nzm & ((1u << lane) - 1));
+                    ws.wrec[k] = make_uint4(wd, 32 * g + sp.HB, sp.lsmb, (sp.lflags & 63) | ((uint32_t)sl << 8));
+                    ws.wpre[k] = run + ex;
                 }
-                if (MODE == kModePagerank) {  // push r(u)/deg(u) along every edge
-                    const double share = a.rank[v_j] / (double)deg_j;
-                    ws.aux[lane] = (uint64_t)__double_as_longlong(share);
-                }
-                // decode: CSR position of the chunk's first element E_v + r0, E_v = W_v - A*q_v
-                if (MODE == kModeDecode) ws.aux[lane] = Wv_j - A * (fi + (uint64_t)j) + r0 - ebt;
-            }
-            // state after this batch: continue after the last valid chunk
-            {
-                const int tl = (int)count - 1;
-                const uint64_t last_cc = __shfl_sync(FULL, cc, tl);
-                const uint64_t last_nch = __shfl_sync(FULL, nch_j, tl);
-                const int last_j = __shfl_sync(FULL, j, tl);
-                const uint64_t last_W = __shfl_sync(FULL, Wv_j, tl);
-                const uint32_t last_deg = __shfl_sync(FULL, deg_j, tl);
-                if (last_cc + 1 < last_nch) {
-                    fi += last_j;
-                    c0 = last_cc + 1;
-                    P = last_W + A + c0 * CH;
-                } else {
-                    fi += last_j + 1;
-                    c0 = 0;
-                    P = last_W + A + last_deg;
-                }
+                run += tot;
+                nrec += __popc(nzm);
             }
             __syncwarp();
+            const uint32_t Er1 = run;
+            const uint32_t NEr = Er1 - Er0;
+            uint32_t e = Er0 + (uint32_t)(((uint64_t)lane * NEr) >> 5);
+            const uint32_t e1 = Er0 + (uint32_t)(((uint64_t)(lane + 1) * NEr) >> 5);
+            if (e < e1) {
+                // ---- lane start: record of element e (maxle) + in-word select ----
+                uint32_t k = 0;
+#pragma unroll
+                for (uint32_t step = kRoundWords / 2; step; step >>= 1)
+                    if (k + step < nrec && ws.wpre[k + step] <= e) k += step;
+                uint4 r = ws.wrec[k];
+                uint32_t w = r.x;
+                const uint32_t kk = e - ws.wpre[k];
+                if (kk) w &= FULL << __fns(w, 0, (int)kk + 1);
+                uint32_t hbw = r.y, lsmb = r.z, l = r.w & 63, lmask = (1u << l) - 1, sl = r.w >> 8;
 
-            // ---- a5 + a6: 16 upper-bit words per step, one 16-bit half per lane ----
-            uint32_t run = 0;
-            WordLd nxt = load_half(data32, ws.geom, wb, lane, 0, W);
-            for (uint32_t g0 = 0; g0 < W; g0 += 16) {
-                const WordLd cur = nxt;
-                if (g0 + 16 < W) nxt = load_half(data32, ws.geom, wb, lane, g0 + 16, W);
-                uint32_t tot;
-                const uint32_t ep = warp_excl_u32(__popc(cur.word), tot);
-                // set-bit enumeration: select1(i) - i of every element, by slot
-                if (cur.word) {
-                    const SlotGeom &sg = ws.geom[cur.s];
-                    const uint64_t rank = sg.r0 + run + ep - sg.eb;  // rank of the first set bit
-                    // hi = hb + p (p = bit within the half), hb -= 1 per bit
-                    // hi of the bit at position b with e = its slot: hbe + b - e
-                    const uint32_t hbe = (uint32_t)(cur.wi * 32 + (lane & 1) * 16 - sg.U0 - rank) + ep;
-                    const uint32_t w = cur.word;
-                    const uint32_t sc = (uint32_t)cur.s;
-                    uint32_t e = ep;
-                    // uniform 16-step scan of the half-word (no lane waits on the
-                    // densest half of the warp, unlike an ffs loop)
-#pragma unroll
-                    for (int b = 0; b < 16; ++b) {
-                        if ((w >> b) & 1) {
-                            ws.hs[e] = ((hbe + b - e) << 5) | sc;
-                            ++e;
-                        }
+                // one element: next stop bit -> select1(i) - i, lower field, value
+                auto decode = [&](uint32_t &x, uint32_t &slot_of) {
+                    if (w == 0) {  // next record (always has a stop bit)
+                        ++k;
+                        r = ws.wrec[k];
+                        w = r.x;
+                        hbw = r.y;
+                        lsmb = r.z;
+                        l = r.w & 63;
+                        lmask = (1u << l) - 1;
+                        sl = r.w >> 8;
                     }
-                }
-                __syncwarp();
-                // balanced pass: element e on lane e % 32, kVisitBatch in flight,
-                // written branch-free (slots past the step are computed and masked)
-                for (uint32_t base = 0; base < tot; base += 32 * kVisitBatch) {
-                    uint32_t xv[kVisitBatch], sv[kVisitBatch];
-                    bool ok[kVisitBatch];
-#pragma unroll
-                    for (int u = 0; u < kVisitBatch; ++u) {
-                        const uint32_t e = base + u * 32 + lane;
-                        ok[u] = e < tot;
-                        const uint32_t es = ok[u] ? e : 0;
-                        const uint32_t hsv = ws.hs[es];
-                        const uint32_t hi = hsv >> 5;
-                        sv[u] = hsv & 31;
-                        const SlotMeta m = ws.meta[sv[u]];
-                        const uint64_t ba = m.lb + (uint64_t)(run + es) * m.l;
-                        const uint32_t *p = data32 + (ba >> 5);
-                        const uint32_t lo =
-                            __funnelshift_r(ldg_u32(p), ldg_u32(p + 1), (uint32_t)(ba & 31)) & m.lmask;
-                        xv[u] = (hi << m.l) | lo;  // (select1(i) - i) << l | lower[i]
-                    }
+                    const uint32_t p = __ffs(w) - 1;
+                    w &= w - 1;
+                    const uint32_t hi = hbw + p - e;  // select1(i) - i
+                    const uint32_t la = lsmb + e * l;
+                    const uint32_t ad = (la >> 3) & ~3u;
+                    const uint32_t lo = __funnelshift_r(lds_u32(ad), lds_u32(ad + 4), la & 31) & lmask;
+                    x = (hi << l) | lo;  // (select1(i) - i) << l | lower[i]
+                    slot_of = sl;
+                    ++e;
+                };
+
+                auto visit = [&](const uint32_t (&xv)[kU], const uint32_t (&sv)[kU], const uint32_t (&ev)[kU],
+                                 int cntu) {
                     if (MODE == kModeDecode) {
 #pragma unroll
-                        for (int u = 0; u < kVisitBatch; ++u)
-                            if (ok[u]) a.out[ws.aux[sv[u]] + run + base + u * 32 + lane] = xv[u];
+                        for (int u = 0; u < kU; ++u)
+                            if (u < cntu) a.out[ws.slot[sv[u]].aux + (ev[u] - ws.slot[sv[u]].eb)] = xv[u];
                     } else if (MODE == kModeSssp) {
                         // relax: d' = fl32(dist(u) + w), single rounding (reading C20)
-                        float nd[kVisitBatch], cd[kVisitBatch];
+                        float nd[kU], cd[kU];
 #pragma unroll
-                        for (int u = 0; u < kVisitBatch; ++u) {
+                        for (int u = 0; u < kU; ++u) {
                             nd[u] = INFINITY;
                             cd[u] = 0.f;
-                            if (ok[u]) {
-                                const float w = __ldg(a.weights + ws.aux[sv[u]] + run + base + u * 32 + lane);
-                                nd[u] = __fadd_rn(ws.aux2[sv[u]], w);
+                            if (u < cntu) {
+                                const SlotP &sp = ws.slot[sv[u]];
+                                nd[u] = __fadd_rn(sp.aux2, __ldg(a.weights + sp.aux + (ev[u] - sp.eb)));
                                 cd[u] = a.dist[xv[u]];
                             }
                         }
 #pragma unroll
-                        for (int u = 0; u < kVisitBatch; ++u) {
-                            if (ok[u] && nd[u] < cd[u]) {  // non-negative floats order like their bits
+                        for (int u = 0; u < kU; ++u) {
+                            if (u < cntu && nd[u] < cd[u]) {  // non-negative floats order like their bits
                                 const int old = atomicMin(reinterpret_cast<int *>(a.dist) + xv[u], __float_as_int(nd[u]));
                                 if (__float_as_int(nd[u]) < old) atomicOr(a.vis + (xv[u] >> 5), 1u << (xv[u] & 31));
                             }
                         }
                     } else if (MODE == kModePagerank) {
 #pragma unroll
-                        for (int u = 0; u < kVisitBatch; ++u)
-                            if (ok[u]) atomicAdd(a.next + xv[u], __longlong_as_double((long long)ws.aux[sv[u]]));
+                        for (int u = 0; u < kU; ++u)
+                            if (u < cntu)
+                                atomicAdd(a.next + xv[u], __longlong_as_double((long long)ws.slot[sv[u]].aux));
                     } else {
                         // Alg. 1 line 3: hot ids answer from shared memory
-                        bool need[kVisitBatch], hot[kVisitBatch];
+                        // ids below vpre are known visited without a memory access
+                        bool need[kU];
 #pragma unroll
-                        for (int u = 0; u < kVisitBatch; ++u) {
-                            hot[u] = ok[u] && xv[u] < hot_limit;
-                            const uint32_t hw = hot[u] ? s_hot[xv[u] >> 5] : 0u;
-                            need[u] = ok[u] && !((hw >> (xv[u] & 31)) & 1);
+                        for (int u = 0; u < kU; ++u) {
+                            const uint32_t hw = (xv[u] >= vpre && xv[u] < hot_limit) ? s_hot[xv[u] >> 5] : 0u;
+                            need[u] = u < cntu && xv[u] >= vpre && !((hw >> (xv[u] & 31)) & 1);
                         }
-                        uint32_t gwd[kVisitBatch];
+                        uint32_t gv[kU];
 #pragma unroll
-                        for (int u = 0; u < kVisitBatch; ++u) gwd[u] = need[u] ? a.vis[xv[u] >> 5] : FULL;
-                        bool act = false;
+                        for (int u = 0; u < kU; ++u) gv[u] = need[u] ? a.vis[xv[u] >> 5] : FULL;
+                        bool miss = false;
 #pragma unroll
-                        for (int u = 0; u < kVisitBatch; ++u) act |= need[u];
-                        if (__any_sync(FULL, act)) {  // most probes of a heavy level stop here
+                        for (int u = 0; u < kU; ++u) miss |= !((gv[u] >> (xv[u] & 31)) & 1);
+                        if (!__any_sync(__activemask(), miss)) return;  // most probes of a heavy level end here
 #pragma unroll
-                            for (int u = 0; u < kVisitBatch; ++u) {
-                                const uint32_t bit = 1u << (xv[u] & 31);
-                                if (!(gwd[u] & bit)) {  // line 4 (stale reads are benign: the atomic decides)
-                                    if (MODE == kModeVisit) {
-                                        atomicOr(a.vis + (xv[u] >> 5), bit);
-                                    } else {
-                                        const uint32_t old = atomicOr(a.vis + (xv[u] >> 5), bit);
-                                        if (!(old & bit)) parent[xv[u]] = (uint32_t)ws.aux[sv[u]];
-                                    }
+                        for (int u = 0; u < kU; ++u) {
+                            const uint32_t bit = 1u << (xv[u] & 31);
+                            if (!(gv[u] & bit)) {  // line 4 (the atomic decides)
+                                if (MODE == kModeVisit) {
+                                    atomicOr(a.vis + (xv[u] >> 5), bit);
+                                } else {
+                                    const uint32_t old = atomicOr(a.vis + (xv[u] >> 5), bit);
+                                    if (!(old & bit)) parent[xv[u]] = (uint32_t)ws.slot[sv[u]].aux;
                                 }
-                                if (need[u] && hot[u]) atomicOr(s_hot + (xv[u] >> 5), bit);
+                                if (xv[u] < hot_limit) atomicOr(s_hot + (xv[u] >> 5), bit);
                             }
                         }
                     }
+                };
+
+                // main loop: kU elements per step, no per-element guards
+                while (e + kU <= e1) {
+                    uint32_t xv[kU], sv[kU], ev[kU];
+#pragma unroll
+                    for (int u = 0; u < kU; ++u) {
+                        ev[u] = e;
+                        decode(xv[u], sv[u]);
+                    }
+                    visit(xv, sv, ev, kU);
                 }
-                __syncwarp();
-                run += tot;
+                // tail: < kU elements
+                if (e < e1) {
+                    uint32_t xv[kU], sv[kU], ev[kU];
+                    const int cntu = (int)(e1 - e);
+#pragma unroll
+                    for (int u = 0; u < kU; ++u) {
+                        xv[u] = 0;
+                        sv[u] = 0;
+                        ev[u] = e;
+                        if (u < cntu) decode(xv[u], sv[u]);
+                    }
+                    visit(xv, sv, ev, cntu);
+                }
             }
+            __syncwarp();
+            Er0 = Er1;
         }
+        cur = nxt;
     }
     if (MODE != kModeDecode && threadIdx.x == 0 && a.stats && xl < a.max_stats)
         atomicMax(&a.stats[xl].t1, globaltimer());
@@ -967,7 +1113,7 @@ cudaError_t launch_map_parent(const uint32_t *pin, const uint32_t *old_of_new, u
     return cudaGetLastError();
 }
 
-size_t expand_smem_bytes() { return (size_t)kHotWords * 4 + (size_t)kExpandWarps * sizeof(WarpSmem); }
+size_t expand_smem_bytes() { return kExpandSmem; }
 
 static cudaError_t expand_set_attrs()
 {

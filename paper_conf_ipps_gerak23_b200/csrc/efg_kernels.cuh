@@ -17,12 +17,13 @@ enum ExpandMode : int {
 
 struct ExpandArgs {
     const uint8_t *data;       // EF data (device, 4-byte aligned, padded)
-    const VRec *rec;           // packed vertex records
-    const uint32_t *queue;     // frontier queue
-    const TileEntry *tiles;    // tile table
+    const ChunkDesc *chunks;   // chunk descriptors of the level (plan_kernel)
+    const uint32_t *tiles;     // tile table: first chunk of tile t (ntiles + 1 entries)
+    const uint32_t *deg32;     // degrees (PageRank share)
     LevelCtrl *ctrl;           // nf, ne, ntiles of this level; parent pointer; level
     uint32_t *vis;             // visited bitmap (modes 0, 1)
-    uint32_t *out;             // decode output (mode 2)
+    uint32_t *out;             // decode output (mode 2): CSR positions minus out_base
+    uint64_t out_base;
     LevelStat *stats;          // per-level statistics (device) or null
     const uint64_t *vlist;     // SSSP: CSR offsets (weight index)
     const float *weights;      // SSSP: weights in CSR order
@@ -32,7 +33,6 @@ struct ExpandArgs {
     uint32_t max_stats;
     uint32_t hot_words;        // bitmap words with a shared-memory snapshot (multiple of 4)
     uint32_t k;                // forward-pointer quantum (chunk length); 0 = none
-    int32_t kshift;            // log2(k) if k is a power of two, else -1
 };
 
 struct InitArgs {
@@ -45,6 +45,7 @@ struct InitArgs {
 
 struct CompactArgs {
     uint32_t *vis, *prev;      // visited bitmap now / at the previous level end
+    const uint32_t *iso;       // degree-0 vertices (never probed): count as visited for vpre
     uint32_t *queue;           // out: next frontier, sorted
     int32_t *depth_stored;     // depth by stored id (always written)
     int depth_stored_only;     // 1: depth_stored is the only depth output (relabelled graphs)
@@ -69,9 +70,12 @@ struct XchgArgs {
 struct PlanArgs {
     const uint32_t *queue;
     const uint32_t *deg32;
-    TileEntry *tiles;
-    LevelCtrl *ctrl;           // in: nf, level, seq; out: ne, nwork, ntiles, xlevel
-    uint64_t *status;
+    const VRec *rec;
+    const uint8_t *data;       // EF data (forward pointers)
+    ChunkDesc *chunks;         // out: chunk descriptors
+    uint32_t *tiles;           // out: first chunk of each tile (+ sentinel)
+    LevelCtrl *ctrl;           // in: nf, level, seq; out: ne, nwork, nchunks, ntiles, xlevel
+    uint64_t *status;          // two cross-block prefix regions (work, chunks) of kMaxGrid words
     LevelStat *stats;
     uint32_t max_stats;
     uint32_t k;
