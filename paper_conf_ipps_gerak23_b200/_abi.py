@@ -10,7 +10,8 @@ import ctypes as C
 import os
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libefg.so")
+# EFG_LIB: an alternative build of the same library (tuning experiments only)
+LIB_PATH = os.environ.get("EFG_LIB") or os.path.join(_HERE, "libefg.so")
 
 EFG_OK, EFG_EINVAL, EFG_ERANGE, EFG_ENOMEM, EFG_ECUDA, EFG_ENCCL, EFG_ENOTSUP, EFG_ESTATE = range(8)
 STATUS_NAMES = {0: "EFG_OK", 1: "EFG_EINVAL", 2: "EFG_ERANGE", 3: "EFG_ENOMEM", 4: "EFG_ECUDA",

@@ -104,18 +104,37 @@ constexpr uint32_t kMaxLevelStats = 4096;
 
 // expand_kernel: one CTA per SM, kExpandWarps warps; each warp owns two
 // staging buffers (TMA double buffering) and a word-round workspace.
-constexpr int kExpandThreads = 512;
+#ifndef EFG_EXPAND_THREADS
+#define EFG_EXPAND_THREADS 768
+#endif
+constexpr int kExpandThreads = EFG_EXPAND_THREADS;
 constexpr int kExpandWarps = kExpandThreads / 32;
-constexpr uint32_t kStageBytes = 4096;       // one staging buffer (>= the largest single chunk)
-constexpr uint32_t kUpperStageMax = 1024;    // larger upper-bit regions are read from global memory
-constexpr uint32_t kRoundWords = 128;        // upper-bit words decoded per round
-constexpr uint32_t kHotWords = 8 * 1024;     // 32 KB shared-memory visited snapshot = 262,144 ids
+#ifndef EFG_STAGE_BYTES
+#define EFG_STAGE_BYTES 2560
+#endif
+constexpr uint32_t kStageBytes = EFG_STAGE_BYTES;       // one staging buffer (>= the largest single chunk)
+// upper-bit regions larger than this are read from global memory; a chunk's
+// lower fields take at most 512*23/8 + 24 bytes (n*2^l <= u < 2^32), so one
+// chunk always fits a staging buffer
+constexpr uint32_t kUpperStageMax = (kStageBytes - 1536 - 64) < 1024 ? ((kStageBytes - 1536 - 64) & ~15u) : 1024u;
+static_assert(kStageBytes >= 2048, "staging buffer too small for one chunk");
+#ifndef EFG_ROUND_WORDS
+#define EFG_ROUND_WORDS 64
+#endif
+constexpr uint32_t kRoundWords = EFG_ROUND_WORDS;        // upper-bit words decoded per round
+#ifndef EFG_HOT_WORDS
+#define EFG_HOT_WORDS 1024
+#endif
+constexpr uint32_t kHotWords = EFG_HOT_WORDS;     // 4 KB shared-memory visited snapshot = 32,768 ids (vpre covers the rest)
 constexpr int kFrontierThreads = 512;        // compact / plan kernels (16 warps)
 constexpr int kBitmapAlign = 1024;           // bitmap words are padded to a multiple of this
 // Step a3 partitions "work units" rather than bare edges: a chunk costs
 // kChunkWork units (descriptor, staging, set-up) plus one per element, so a
 // tile of kTileWork units holds at most kTileWork/kChunkWork chunks.
-constexpr uint32_t kTileWork = 2048;         // work units per tile (a3)
+#ifndef EFG_TILE_WORK
+#define EFG_TILE_WORK 2048
+#endif
+constexpr uint32_t kTileWork = EFG_TILE_WORK;         // work units per tile (a3)
 constexpr uint32_t kChunkWork = 32;          // per-chunk overhead in work units
 
 constexpr unsigned kMaxGrid = 4096;

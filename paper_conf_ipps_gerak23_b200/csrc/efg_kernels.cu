@@ -457,15 +457,23 @@ __global__ void __launch_bounds__(kFrontierThreads) plan_kernel(PlanArgs a)
 
     // pass 2: 32 frontier vertices at a time (one per lane); the next group's
     // queue entries are fetched while the current group is processed
+    // software pipeline: records of group g+1 and queue entries of group g+2 are
+    // in flight while group g is processed
     uint32_t vn = qlo + lane < qhi ? a.queue[qlo + lane] : 0u;
+    uint4 rn = make_uint4(0, 0, 0, 0);
+    if (qlo + lane < qhi) rn = __ldg(reinterpret_cast<const uint4 *>(a.rec + vn));
+    uint32_t vnn = qlo + 32 + lane < qhi ? a.queue[qlo + 32 + lane] : 0u;
     for (uint64_t i0 = qlo; i0 < qhi; i0 += 32) {
         const uint64_t i = i0 + lane;
         const uint32_t v = vn;
-        if (i0 + 32 < qhi) vn = i + 32 < qhi ? a.queue[i + 32] : 0u;
+        const uint4 r = rn;
+        vn = vnn;
+        rn = make_uint4(0, 0, 0, 0);
+        if (i + 32 < qhi) rn = __ldg(reinterpret_cast<const uint4 *>(a.rec + vn));
+        vnn = i + 64 < qhi ? a.queue[i + 64] : 0u;
         uint64_t off_l = 0;
         uint32_t d = 0, ub = 0;
         if (i < qhi) {
-            const uint4 r = __ldg(reinterpret_cast<const uint4 *>(a.rec + v));
             off_l = ((uint64_t)r.y << 32) | r.x;
             d = r.z;
             ub = r.w;
@@ -632,7 +640,13 @@ struct Batch {
     uint64_t usrc;
 };
 
-constexpr int kU = 4;  // elements per lane whose probes are in flight together
+// largest power of two below kRoundWords: the maxle search over a round's records
+constexpr uint32_t kSearchStep = kRoundWords <= 1 ? 0u : (1u << (31 - __builtin_clz(kRoundWords - 1)));
+
+#ifndef EFG_KU
+#define EFG_KU 4
+#endif
+constexpr int kU = EFG_KU;  // elements per lane whose probes are in flight together
 
 template <int MODE>
 __global__ void __launch_bounds__(kExpandThreads, 1) expand_kernel(ExpandArgs a)
@@ -865,7 +879,7 @@ __global__ void __launch_bounds__(kExpandThreads, 1) expand_kernel(ExpandArgs a)
                 // ---- lane start: record of element e (maxle) + in-word select ----
                 uint32_t k = 0;
 #pragma unroll
-                for (uint32_t step = kRoundWords / 2; step; step >>= 1)
+                for (uint32_t step = kSearchStep; step; step >>= 1)
                     if (k + step < nrec && ws.wpre[k + step] <= e) k += step;
                 uint4 r = ws.wrec[k];
                 uint32_t w = r.x;

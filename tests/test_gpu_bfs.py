@@ -268,12 +268,12 @@ def test_reorder_degree_bfs_in_input_ids(efg):
 
 
 def test_hot_snapshot_boundary(efg):
-    # graph larger than the shared-memory hot range (917,504 ids): probes on both sides
+    # graph larger than the shared-memory hot range (32,768 ids): probes on both sides
     n, src, dst = synth.rmat(20, 8, seed=12)
     for flags in (efg.EFG_DEFAULT_FLAGS, efg.EFG_DEFAULT_FLAGS | efg.EFG_REORDER_DEGREE):
         g = efg.Graph.build(n, src, dst, flags=flags)
         ov, oe = oracle.csr_build(n, src, dst)
-        _check_bfs(g, ov, oe, [0, 917503, 917504, n - 1])
+        _check_bfs(g, ov, oe, [0, 32767, 32768, 917504, n - 1])
         g.free()
 
 
