@@ -123,9 +123,9 @@ static_assert(kStageBytes >= 2048, "staging buffer too small for one chunk");
 #endif
 constexpr uint32_t kRoundWords = EFG_ROUND_WORDS;        // upper-bit words decoded per round
 #ifndef EFG_HOT_WORDS
-#define EFG_HOT_WORDS 1024
+#define EFG_HOT_WORDS 4
 #endif
-constexpr uint32_t kHotWords = EFG_HOT_WORDS;     // 4 KB shared-memory visited snapshot = 32,768 ids (vpre covers the rest)
+constexpr uint32_t kHotWords = EFG_HOT_WORDS;     // > 4: shared-memory visited snapshot of the first 32*kHotWords ids (off: vpre covers the visited prefix)
 constexpr int kFrontierThreads = 512;        // compact / plan kernels (16 warps)
 constexpr int kBitmapAlign = 1024;           // bitmap words are padded to a multiple of this
 // Step a3 partitions "work units" rather than bare edges: a chunk costs

@@ -41,12 +41,15 @@ __device__ __forceinline__ unsigned long long globaltimer()
 
 __device__ __forceinline__ uint32_t warp_excl_u32(uint32_t x, uint32_t &total)
 {
+    // Kogge-Stone scan; the shuffle's in-range predicate guards the add (no compare)
     uint32_t inc = x;
 #pragma unroll
-    for (int d = 1; d < 32; d <<= 1) {
-        const uint32_t y = __shfl_up_sync(FULL, inc, d);
-        if ((int)lane_id() >= d) inc += y;
-    }
+    for (int d = 1; d < 32; d <<= 1)
+        asm volatile("{\n\t.reg .u32 t;\n\t.reg .pred p;\n\t"
+                     "shfl.sync.up.b32 t|p, %0, %1, 0, -1;\n\t"
+                     "@p add.u32 %0, %0, t;\n\t}"
+                     : "+r"(inc)
+                     : "r"(d));
     total = __shfl_sync(FULL, inc, 31);
     return inc - x;
 }
@@ -619,6 +622,38 @@ __device__ __forceinline__ uint32_t lds_u32(uint32_t addr)
     return v;
 }
 
+// leading zeros of a non-zero word in one instruction (bfind.shiftamt)
+__device__ __forceinline__ uint32_t clz_nz(uint32_t x)
+{
+    uint32_t d;
+    asm("bfind.shiftamt.u32 %0, %1;" : "=r"(d) : "r"(x));
+    return d;
+}
+
+// funnel shift right with the shift amount taken mod 32 (no masking instruction)
+__device__ __forceinline__ uint32_t shf_r_wrap(uint32_t lo, uint32_t hi, uint32_t sh)
+{
+    uint32_t d;
+    asm("shf.r.wrap.b32 %0, %1, %2, %3;" : "=r"(d) : "r"(lo), "r"(hi), "r"(sh));
+    return d;
+}
+
+// position (0..31) of the set bit of rank kk (0-based, kk < popc(w)) of w:
+// five popcount halvings (the in-word part of select1)
+__device__ __forceinline__ uint32_t select_in_word(uint32_t w, uint32_t kk)
+{
+    uint32_t pos = 0;
+#pragma unroll
+    for (uint32_t sh = 16; sh; sh >>= 1) {
+        const uint32_t c = __popc(w & ((1u << sh) - 1));
+        const bool up = kk >= c;
+        kk -= up ? c : 0u;
+        w = up ? w >> sh : w;
+        pos += up ? sh : 0u;
+    }
+    return pos;
+}
+
 // TMA bulk copy global -> shared (16-byte aligned addresses, size a multiple of 16)
 __device__ __forceinline__ void bulk_g2s(void *dst, const void *src, uint32_t bytes, uint64_t *bar)
 {
@@ -642,6 +677,8 @@ struct Batch {
 
 // largest power of two below kRoundWords: the maxle search over a round's records
 constexpr uint32_t kSearchStep = kRoundWords <= 1 ? 0u : (1u << (31 - __builtin_clz(kRoundWords - 1)));
+
+constexpr bool kUseHot = kHotWords > 4;  // shared-memory visited snapshot compiled in
 
 #ifndef EFG_KU
 #define EFG_KU 4
@@ -674,7 +711,7 @@ __global__ void __launch_bounds__(kExpandThreads, 1) expand_kernel(ExpandArgs a)
         mbar_init(&ws.mbar[0], 1);
         mbar_init(&ws.mbar[1], 1);
     }
-    if (kBfs) {
+    if (kBfs && kUseHot) {
         // level-start snapshot of the hot visited words
         const uint4 *src = reinterpret_cast<const uint4 *>(a.vis);
         uint4 *dst = reinterpret_cast<uint4 *>(s_hot);
@@ -691,6 +728,8 @@ __global__ void __launch_bounds__(kExpandThreads, 1) expand_kernel(ExpandArgs a)
     const uint64_t gw = (uint64_t)blockIdx.x * kExpandWarps + wid;
     const uint64_t nwarps = (uint64_t)gridDim.x * kExpandWarps;
     const uint64_t CH = a.k ? a.k : (1ull << 40);
+    const bool kpow2 = a.k && !(a.k & (a.k - 1));
+    const uint32_t kshift = kpow2 ? (uint32_t)__ffs(a.k) - 1 : 0u;
 
     // producer cursor: chunks [cnext, cend) of the current tile
     uint64_t tile = gw;
@@ -723,7 +762,7 @@ __global__ void __launch_bounds__(kExpandThreads, 1) expand_kernel(ExpandArgs a)
             l = (uint32_t)(offl >> kOffBits);
             v = d1.x;
             cc = d1.y;
-            const uint64_t F = a.k ? (uint64_t)deg / a.k : 0;           // forward pointers (C8)
+            const uint64_t F = a.k ? (kpow2 ? (uint64_t)(deg >> kshift) : (uint64_t)deg / a.k) : 0;  // forward pointers (C8)
             const uint64_t Lb = ((uint64_t)deg * l + 7) >> 3;            // lower section bytes
             const uint64_t lbase = (off + 4 * F) * 8;
             const uint64_t U0 = (off + 4 * F + Lb) * 8;
@@ -765,10 +804,10 @@ __global__ void __launch_bounds__(kExpandThreads, 1) expand_kernel(ExpandArgs a)
         const uint32_t buf = nbuf;
         B.buf = buf;
         nbuf ^= 1;
-        uint32_t tot_e, tot_w, tot_b;
+        uint32_t tot_e, tot_w;
         B.eb = warp_excl_u32(fits ? nel : 0u, tot_e);
         B.wb = warp_excl_u32(fits ? nwd : 0u, tot_w);
-        warp_excl_u32(fits ? bytes : 0u, tot_b);
+        const uint32_t tot_b = __shfl_sync(FULL, sb + bytes, B.cnt - 1);  // bytes of the fitting prefix
         B.ne = tot_e;
         B.nw = tot_w;
         B.nwd = nwd;
@@ -864,7 +903,7 @@ __global__ void __launch_bounds__(kExpandThreads, 1) expand_kernel(ExpandArgs a)
                 const uint32_t nzm = __ballot_sync(FULL, wd != 0);
                 if (wd) {
                     const uint32_t k = nrec + __popc(nzm & ((1u << lane) - 1));
-                    ws.wrec[k] = make_uint4(wd, 32 * g + sp.HB, sp.lsmb, (sp.lflags & 63) | ((uint32_t)sl << 8));
+                    ws.wrec[k] = make_uint4(__brev(wd), 32 * g + sp.HB, sp.lsmb, (sp.lflags & 63) | ((uint32_t)sl << 8));
                     ws.wpre[k] = run + ex;
                 }
                 run += tot;
@@ -881,32 +920,29 @@ __global__ void __launch_bounds__(kExpandThreads, 1) expand_kernel(ExpandArgs a)
 #pragma unroll
                 for (uint32_t step = kSearchStep; step; step >>= 1)
                     if (k + step < nrec && ws.wpre[k + step] <= e) k += step;
+                // records hold bit-reversed words: the lowest remaining stop bit is the
+                // leading one (clz), so no bit reversal per element
                 uint4 r = ws.wrec[k];
-                uint32_t w = r.x;
                 const uint32_t kk = e - ws.wpre[k];
-                if (kk) w &= FULL << __fns(w, 0, (int)kk + 1);
-                uint32_t hbw = r.y, lsmb = r.z, l = r.w & 63, lmask = (1u << l) - 1, sl = r.w >> 8;
+                if (kk) r.x &= FULL >> select_in_word(__brev(r.x), kk);  // drop kk stop bits
+                uint32_t l = r.w & 63, lmask = (1u << l) - 1;
 
                 // one element: next stop bit -> select1(i) - i, lower field, value
                 auto decode = [&](uint32_t &x, uint32_t &slot_of) {
-                    if (w == 0) {  // next record (always has a stop bit)
+                    if (r.x == 0) {  // next record (always has a stop bit)
                         ++k;
                         r = ws.wrec[k];
-                        w = r.x;
-                        hbw = r.y;
-                        lsmb = r.z;
                         l = r.w & 63;
                         lmask = (1u << l) - 1;
-                        sl = r.w >> 8;
                     }
-                    const uint32_t p = __ffs(w) - 1;
-                    w &= w - 1;
-                    const uint32_t hi = hbw + p - e;  // select1(i) - i
-                    const uint32_t la = lsmb + e * l;
+                    const uint32_t p = clz_nz(r.x);
+                    r.x ^= 0x80000000u >> p;
+                    const uint32_t hi = r.y + p - e;  // select1(i) - i
+                    const uint32_t la = r.z + e * l;
                     const uint32_t ad = (la >> 3) & ~3u;
-                    const uint32_t lo = __funnelshift_r(lds_u32(ad), lds_u32(ad + 4), la & 31) & lmask;
+                    const uint32_t lo = shf_r_wrap(lds_u32(ad), lds_u32(ad + 4), la) & lmask;
                     x = (hi << l) | lo;  // (select1(i) - i) << l | lower[i]
-                    slot_of = sl;
+                    slot_of = r.w >> 8;
                     ++e;
                 };
 
@@ -947,15 +983,19 @@ __global__ void __launch_bounds__(kExpandThreads, 1) expand_kernel(ExpandArgs a)
                         bool need[kU];
 #pragma unroll
                         for (int u = 0; u < kU; ++u) {
-                            const uint32_t hw = (xv[u] >= vpre && xv[u] < hot_limit) ? s_hot[xv[u] >> 5] : 0u;
-                            need[u] = u < cntu && xv[u] >= vpre && !((hw >> (xv[u] & 31)) & 1);
+                            need[u] = u < cntu && xv[u] >= vpre;
+                            if (kUseHot) {
+                                const uint32_t hw = (need[u] && xv[u] < hot_limit) ? s_hot[xv[u] >> 5] : 0u;
+                                need[u] = need[u] && !((hw >> (xv[u] & 31)) & 1);
+                            }
                         }
                         uint32_t gv[kU];
 #pragma unroll
                         for (int u = 0; u < kU; ++u) gv[u] = need[u] ? a.vis[xv[u] >> 5] : FULL;
-                        bool miss = false;
+                        uint32_t hit = 1;
 #pragma unroll
-                        for (int u = 0; u < kU; ++u) miss |= !((gv[u] >> (xv[u] & 31)) & 1);
+                        for (int u = 0; u < kU; ++u) hit &= shf_r_wrap(gv[u], gv[u], xv[u]);
+                        const bool miss = !(hit & 1);
                         if (!__any_sync(__activemask(), miss)) return;  // most probes of a heavy level end here
 #pragma unroll
                         for (int u = 0; u < kU; ++u) {
@@ -967,7 +1007,7 @@ __global__ void __launch_bounds__(kExpandThreads, 1) expand_kernel(ExpandArgs a)
                                     const uint32_t old = atomicOr(a.vis + (xv[u] >> 5), bit);
                                     if (!(old & bit)) parent[xv[u]] = (uint32_t)ws.slot[sv[u]].aux;
                                 }
-                                if (xv[u] < hot_limit) atomicOr(s_hot + (xv[u] >> 5), bit);
+                                if (kUseHot && xv[u] < hot_limit) atomicOr(s_hot + (xv[u] >> 5), bit);
                             }
                         }
                     }
