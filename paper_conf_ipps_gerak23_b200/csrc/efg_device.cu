@@ -1,11 +1,11 @@
 // efg_device.cu — device side of a handle: upload of the packed EFG, the
 // traversal workspace, and the level-synchronous driver.
 //
-// Per BFS level the driver runs three kernels (efg_kernels.cu):
-//   expand  (a4 a5 a6)  ->  compact (a7)  ->  plan (a1 a2 a3)
+// Per BFS level the driver runs two kernels (efg_kernels.cu):
+//   expand  (a4 a5 a6)  ->  frontier (a7, then the next level's a1 a2 a3 a4)
 // Two drivers share them:
 //   * graph mode (default): the level loop is one CUDA graph with a
-//     conditional WHILE node; plan_kernel's last block sets the condition
+//     conditional WHILE node; frontier_kernel's last block sets the condition
 //     (frontier non-empty) on the device, so a whole BFS costs one graph launch
 //     and no host round trip per level;
 //   * host mode (efg_set_option EFG_OPT_LEVEL_LOOP = 1): the host launches each
@@ -14,6 +14,7 @@
 #include <cuda_runtime.h>
 
 #include <algorithm>
+#include <cstdio>
 #include <cstddef>
 #include <cstdlib>
 #include <cstring>
@@ -96,18 +97,29 @@ ExpandArgs expand_args(DeviceGraph &d, uint32_t *out)
     return a;
 }
 
-CompactArgs compact_args(DeviceGraph &d, bool consume = false)
+FrontierArgs frontier_args(DeviceGraph &d, cudaGraphConditionalHandle cond, bool consume = false)
 {
-    CompactArgs a;
+    FrontierArgs a;
     a.consume = consume ? 1 : 0;
     a.vis = d.vis;
     a.prev = d.prev;
     a.iso = d.iso;
-    a.queue = d.queue;
     a.depth_stored = (d.old_of_new && !consume) ? d.depth_st : nullptr;
     a.depth_stored_only = d.old_of_new ? 1 : 0;
+    a.deg32 = d.deg32;
+    a.rec = d.rec;
+    a.chunks = d.chunks;
+    a.tiles = d.tiles;
     a.ctrl = d.ctrl;
     a.status = d.status;
+    a.barrier = reinterpret_cast<unsigned long long *>(d.status + 3 * kMaxGrid);
+    a.big = d.big;
+    a.trace = d.trace;
+    a.stats = d.stats;
+    a.max_stats = kMaxLevelStats;
+    a.k = d.k;
+    a.kshift = kshift_of(d.k);
+    a.cond = cond;
     a.nwords = d.nwords;
     a.words_per_block = d.words_per_block;
     a.own_lo_w = d.own_lo_w;
@@ -115,35 +127,16 @@ CompactArgs compact_args(DeviceGraph &d, bool consume = false)
     return a;
 }
 
-PlanArgs plan_args(DeviceGraph &d, cudaGraphConditionalHandle cond)
-{
-    PlanArgs a;
-    a.queue = d.queue;
-    a.deg32 = d.deg32;
-    a.rec = d.rec;
-    a.data = d.data;
-    a.chunks = d.chunks;
-    a.tiles = d.tiles;
-    a.ctrl = d.ctrl;
-    a.status = d.status + kMaxGrid;
-    a.stats = d.stats;
-    a.max_stats = kMaxLevelStats;
-    a.k = d.k;
-    a.kshift = kshift_of(d.k);
-    a.cond = cond;
-    return a;
-}
-
+// level end + next plan: one launch (every block resident, see frontier_kernel)
 efg_status launch_level_end(DeviceGraph &d, cudaGraphConditionalHandle cond, cudaStream_t s,
                             bool consume = false)
 {
-    CUDA_TRY(launch_compact(compact_args(d, consume),
-                            (unsigned)((d.nwords + d.words_per_block - 1) / d.words_per_block), s));
-    CUDA_TRY(launch_plan(plan_args(d, cond), d.frontier_blocks, s));
+    CUDA_TRY(launch_frontier(frontier_args(d, cond, consume),
+                             (unsigned)((d.nwords + d.words_per_block - 1) / d.words_per_block), s));
     return EFG_OK;
 }
 
-// Build (once per handle and mode) the graph: while (frontier) { expand; compact; plan }
+// Build (once per handle and mode) the graph: while (frontier) { expand; frontier }
 efg_status build_loop_graph(DeviceGraph &d, int mode)
 {
     if (d.loop_exec[mode]) return EFG_OK;
@@ -197,7 +190,6 @@ void device_free(DeviceGraph &d)
     cudaFree(d.weights);
     cudaFree(d.vis);
     cudaFree(d.prev);
-    cudaFree(d.queue);
     cudaFree(d.tiles);
     cudaFree(d.chunks);
     cudaFree(d.depth);
@@ -207,6 +199,8 @@ void device_free(DeviceGraph &d)
     cudaFree(d.new_of_old);
     cudaFree(d.depth_st);
     cudaFree(d.status);
+    cudaFree(d.big);
+    cudaFree(d.trace);
     cudaFree(d.stats);
     cudaFree(d.xchg_bounds);
     cudaFree(d.ctrl);
@@ -296,7 +290,6 @@ efg_status device_upload(efg_graph *g, const efg_build_opts &o)
     // traversal workspace
     EFG_TRY(dev_alloc(d, &d.vis, d.nwords));
     EFG_TRY(dev_alloc(d, &d.prev, d.nwords));
-    EFG_TRY(dev_alloc(d, &d.queue, h.n));
     // a level has at most one chunk per frontier vertex plus one per k elements
     const uint64_t rows = (h.row_hi > h.row_lo) ? h.row_hi - h.row_lo : h.n;
     d.max_chunks = rows + (h.k ? h.m / h.k : 0) + 1;
@@ -304,8 +297,16 @@ efg_status device_upload(efg_graph *g, const efg_build_opts &o)
     EFG_TRY(dev_alloc(d, &d.tiles, d.max_tiles + 1));
     EFG_TRY(dev_alloc(d, &d.chunks, d.max_chunks));
     EFG_TRY(dev_alloc(d, &d.depth, h.n));
-    EFG_TRY(dev_alloc(d, &d.status, 3 * kMaxGrid));
-    CUDA_TRY(cudaMemsetAsync(d.status, 0, 3 * kMaxGrid * 8, s));
+    EFG_TRY(dev_alloc(d, &d.status, 3 * kMaxGrid + 1));  // + the grid-barrier counter
+    CUDA_TRY(cudaMemsetAsync(d.status, 0, (3 * kMaxGrid + 1) * 8, s));
+    if (std::getenv("EFG_FRONTIER_TRACE")) EFG_TRY(dev_alloc(d, &d.trace, 8 * kMaxGrid));
+    // lists planned grid-wide: more than one chunk (deg > k) or more than one
+    // tile of work (deg > kTileWork - kChunkWork)
+    {
+        const uint64_t q = h.k ? std::min<uint64_t>(h.k, kTileWork - kChunkWork) : kTileWork - kChunkWork;
+        d.max_big = std::min<uint64_t>(rows, h.m / q + 1);
+        EFG_TRY(dev_alloc(d, &d.big, d.max_big));
+    }
     EFG_TRY(dev_alloc(d, &d.stats, kMaxLevelStats));
     EFG_TRY(dev_alloc(d, &d.ctrl, 1));
     CUDA_TRY(cudaMemsetAsync(d.ctrl, 0, sizeof(LevelCtrl), s));
@@ -317,6 +318,12 @@ efg_status device_upload(efg_graph *g, const efg_build_opts &o)
         d.frontier_blocks = (unsigned)std::max(1, std::min(atoi(e), (int)kMaxGrid));
     const uint64_t per = (d.nwords + d.frontier_blocks - 1) / d.frontier_blocks;
     d.words_per_block = (per + kFrontierThreads - 1) / kFrontierThreads * kFrontierThreads;
+    // frontier_kernel blocks wait on their predecessors: the whole grid must be resident
+    const uint64_t grid = (d.nwords + d.words_per_block - 1) / d.words_per_block;
+    const int occ = frontier_occupancy();
+    if (occ <= 0 || grid > (uint64_t)occ * d.num_sms)
+        return set_error(EFG_ECUDA, "frontier_kernel grid (" + std::to_string(grid) + " blocks) exceeds the resident limit (" +
+                                        std::to_string(occ) + " per SM)");
     CUDA_TRY(cudaStreamSynchronize(s));
     return EFG_OK;
 }
@@ -338,7 +345,7 @@ static efg_status start_traversal(DeviceGraph &d, uint64_t v0, uint64_t v1, int3
     ia.v1 = v1;
     CUDA_TRY(launch_init(ia, s));
     EFG_TRY(launch_level_end(d, 0, s));
-    launches += 3;
+    launches += 2;
     return EFG_OK;
 }
 
@@ -428,7 +435,7 @@ efg_status device_bfs(efg_graph *g, uint32_t source, int32_t *depth, uint32_t *p
             const LevelStat &x = d.stats_host[i];
             lms.push_back(x.t1 > x.t0 ? (float)((double)(x.t1 - x.t0) * 1e-6) : 0.f);
         }
-        launches += 3 * levels + (relabel ? 1 : 0);
+        launches += 2 * levels + (relabel ? 1 : 0);
     } else {
         const int blocks = d.num_sms * expand_occupancy(mode);
         for (;;) {
@@ -451,7 +458,21 @@ efg_status device_bfs(efg_graph *g, uint32_t source, int32_t *depth, uint32_t *p
             CUDA_TRY(cudaEventRecord(b, s));
             EFG_TRY(launch_level_end(d, 0, s));
             CUDA_TRY(cudaEventRecord(ec, s));
-            launches += 3;
+            launches += 2;
+            if (d.trace) {  // debug: phase end times of frontier_kernel, max over blocks (us after the first start)
+                const unsigned nb = (unsigned)((d.nwords + d.words_per_block - 1) / d.words_per_block);
+                std::vector<unsigned long long> t(8 * nb);
+                CUDA_TRY(cudaMemcpyAsync(t.data(), d.trace, t.size() * 8, cudaMemcpyDeviceToHost, s));
+                CUDA_TRY(cudaStreamSynchronize(s));
+                unsigned long long t0 = ~0ull, mx[8] = {0};
+                for (unsigned b = 0; b < nb; ++b) {
+                    t0 = std::min(t0, t[8 * b]);
+                    for (int p = 0; p < 8; ++p) mx[p] = std::max(mx[p], t[8 * b + p]);
+                }
+                fprintf(stderr, "frontier-trace L=%u nf=%llu:", levels, (unsigned long long)0);
+                for (int p = 0; p < 8; ++p) fprintf(stderr, " %.1f", (double)(mx[p] - t0) * 1e-3);
+                fprintf(stderr, "\n");
+            }
             ++levels;
         }
         if (relabel) {

@@ -62,7 +62,7 @@ static_assert(sizeof(VRec) == 16, "VRec must be 16 bytes");
 constexpr int kOffBits = 58;
 constexpr uint64_t kOffMask = (1ull << kOffBits) - 1;
 
-// Chunk descriptor (step a1, written by plan_kernel, read by expand_kernel):
+// Chunk descriptor (step a1, written by frontier_kernel, read by expand_kernel):
 // one k-aligned piece of a frontier vertex's list.  The expand
 // kernel derives the chunk's bit ranges from it and the forward pointers (a4).
 struct alignas(16) ChunkDesc {
@@ -84,16 +84,28 @@ struct LevelCtrl {
     uint64_t nchunks;   // chunk descriptors of the level
     int32_t *depth;     // depth buffer of the current call
     uint32_t *parent;   // parent buffer of the current call, or null
-    uint32_t level;     // depth assigned by the next compact
+    uint32_t level;     // depth assigned by the next frontier_kernel
     uint32_t xlevel;    // index of the level the next expand processes
     uint32_t seq;       // tag of the cross-block prefix words of this level
     uint32_t nlevels;   // levels expanded so far
     uint64_t nnew;      // vertices discovered in the last level (all rows; partitioned runs)
     uint64_t total_nf;  // sum of frontier sizes (= vertices reached)
     uint64_t total_ne;  // sum of E_L (= edges traversed, reading C18)
-    uint32_t vmin;      // compact: smallest vertex that is neither visited nor isolated (atomicMin)
-    uint32_t vpre;      // plan -> expand: every vertex below it is visited or isolated
+    uint32_t vmin2[2];  // frontier_kernel of level L: smallest vertex neither visited nor isolated, in
+                        // slot L & 1 (atomicMin); the expand of level L reads it as its visited prefix
+    uint32_t nbig2[2];  // frontier_kernel of level L: BigList entries appended (slot L & 1)
 };
+
+// A frontier list whose chunk descriptors and tile boundaries are written by
+// the whole grid rather than by the warp that planned it (frontier_kernel):
+// lists of more than one chunk or more than one tile of work.
+struct BigList {
+    uint64_t W;       // work position of the list's first unit
+    uint64_t cstart;  // index of its first chunk descriptor
+    uint64_t off_l;   // VRec.off_l
+    uint32_t deg, ubytes, v, nch;
+};
+static_assert(sizeof(BigList) == 40, "BigList");
 
 // Per-level statistics written on the device (graph mode has no host loop).
 struct LevelStat {
@@ -126,7 +138,7 @@ constexpr uint32_t kRoundWords = EFG_ROUND_WORDS;        // upper-bit words deco
 #define EFG_HOT_WORDS 4
 #endif
 constexpr uint32_t kHotWords = EFG_HOT_WORDS;     // > 4: shared-memory visited snapshot of the first 32*kHotWords ids (off: vpre covers the visited prefix)
-constexpr int kFrontierThreads = 512;        // compact / plan kernels (16 warps)
+constexpr int kFrontierThreads = 512;        // frontier_kernel (16 warps)
 constexpr int kBitmapAlign = 1024;           // bitmap words are padded to a multiple of this
 // Step a3 partitions "work units" rather than bare edges: a chunk costs
 // kChunkWork units (descriptor, staging, set-up) plus one per element, so a
@@ -154,7 +166,6 @@ struct DeviceGraph {
     // traversal workspace
     uint32_t *vis = nullptr;           // visited bitmap (nwords)
     uint32_t *prev = nullptr;          // visited bitmap at the end of the last level
-    uint32_t *queue = nullptr;         // frontier queue (n)
     uint32_t *tiles = nullptr;         // tile table: first chunk of each tile (max_tiles + 1)
     uint64_t max_tiles = 0;
     ChunkDesc *chunks = nullptr;       // chunk descriptors of the level (max_chunks)
@@ -166,9 +177,12 @@ struct DeviceGraph {
     uint32_t *new_of_old = nullptr;    // its inverse (n) or null
     int32_t *depth_st = nullptr;       // depth by stored id (relabelled graphs)
     int32_t *step_depth = nullptr;     // stepwise traversal: caller's depth buffer
-    uint64_t *status = nullptr;        // cross-block prefix words: compact [kMaxGrid], plan [kMaxGrid]
+    uint64_t *status = nullptr;        // frontier_kernel: 3 x [kMaxGrid] per-block aggregates + barrier counter
+    BigList *big = nullptr;
+    unsigned long long *trace = nullptr;  // debug: frontier_kernel phase timestamps            // frontier_kernel: multi-chunk / multi-tile lists of a level
+    uint64_t max_big = 0;
     LevelStat *stats = nullptr;        // per-level statistics (kMaxLevelStats)
-    unsigned frontier_blocks = 0;      // grid of compact / plan
+    unsigned frontier_blocks = 0;      // grid of frontier_kernel
     uint64_t words_per_block = 0;
     LevelCtrl *ctrl = nullptr;         // device control block
     LevelCtrl *ctrl_host = nullptr;    // pinned mirror
@@ -180,7 +194,7 @@ struct DeviceGraph {
     int level_loop = 0;                // 0 = CUDA graph (device loop), 1 = host loop + events
     cudaGraph_t loop_graph[2] = {nullptr, nullptr};      // per mode (visit, visit+parent)
     cudaGraphExec_t loop_exec[2] = {nullptr, nullptr};
-    uint64_t own_lo_w = 0, own_hi_w = 0;   // bitmap words of the owned rows (queue filter)
+    uint64_t own_lo_w = 0, own_hi_w = 0;   // bitmap words of the owned rows (frontier filter)
     uint64_t *xchg_bounds = nullptr;       // device copy of the partition bounds
     uint64_t xchg_bounds_cap = 0;
     // stepwise (partitioned) traversal state

@@ -3,10 +3,10 @@
 // Steps and where they live, per BFS level:
 //   a4 locate compressed bit ranges + a5 EF element decode + a6 visit
 //      -> expand_kernel (persistent, warp per work tile)
-//   a7 level end: visited-bitmap diff -> sorted next frontier queue + depth
-//      -> compact_kernel (reduce-then-scan over the bitmap)
-//   a1 degree lookup + a2 exclusive scan of per-vertex work + a3 partition
-//      into tiles -> plan_kernel (reduce-then-scan over the queue)
+//   a7 level end: visited-bitmap diff -> sorted next frontier queue + depth,
+//   fused with the next level's a1 degree lookup + a2 exclusive scan of
+//   per-vertex work + a3 partition into tiles + a4 chunk descriptors
+//      -> frontier_kernel (reduce-then-scan over the bitmap)
 // init_kernel starts a traversal (source bit, per-call state).
 //
 // Paper anchors: Alg. 1 (§III-B), scans/searches (§III-C),
@@ -119,15 +119,7 @@ __device__ __forceinline__ ChunkLen make_chunk(uint32_t k, int kshift)
     return c;
 }
 
-// --------------------------------------------------------------------------
-// Cross-block exclusive prefix for the two frontier scans (a2, a7).  A block
-// publishes its aggregate as one 64-bit word tag << 40 | value (value < 2^40),
-// with tag = the per-launch sequence number, so no clearing pass and no fence
-// are needed (the value travels in the same single-copy-atomic word as its
-// tag).  The block then sums the aggregates of ALL its predecessors with every
-// load issued at once (grids are at most 2 x #SMs blocks), i.e. one or two L2
-// round trips instead of a look-back chain.
-// --------------------------------------------------------------------------
+// relaxed gpu-scope accesses (cross-block words of the persistent frontier grid)
 __device__ __forceinline__ uint64_t ld_relaxed_u64(const uint64_t *p)
 {
     uint64_t v;
@@ -135,36 +127,16 @@ __device__ __forceinline__ uint64_t ld_relaxed_u64(const uint64_t *p)
     return v;
 }
 
+__device__ __forceinline__ uint32_t ld_relaxed_u32(const uint32_t *p)
+{
+    uint32_t v;
+    asm volatile("ld.relaxed.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+    return v;
+}
+
 __device__ __forceinline__ void st_relaxed_u64(uint64_t *p, uint64_t v)
 {
     asm volatile("st.relaxed.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
-}
-
-constexpr int kTagShift = 40;
-constexpr uint64_t kTagVal = (1ull << kTagShift) - 1;
-
-// warp 0: publish `agg` for block b and return the sum over blocks < b
-__device__ uint64_t publish_and_prefix(uint64_t *st, uint32_t b, uint32_t tag, uint64_t agg)
-{
-    const uint32_t lane = lane_id();
-    const uint64_t t = (uint64_t)(tag & 0xffffffu);
-    if (lane == 0) st_relaxed_u64(st + b, (t << kTagShift) | agg);
-    uint64_t acc = 0;
-    for (uint32_t base = 0; base < b; base += 32 * 8) {
-        uint64_t w[8];
-#pragma unroll
-        for (int u = 0; u < 8; ++u) {
-            const uint32_t idx = base + u * 32 + lane;
-            w[u] = idx < b ? ld_relaxed_u64(st + idx) : (t << kTagShift);
-        }
-#pragma unroll
-        for (int u = 0; u < 8; ++u) {
-            const uint32_t idx = base + u * 32 + lane;
-            while ((w[u] >> kTagShift) != t) w[u] = ld_relaxed_u64(st + idx);
-            acc += w[u] & kTagVal;
-        }
-    }
-    return warp_sum_u64(acc);
 }
 
 // block-wide exclusive scan of a u64 (256 threads); returns the block total in `total`
@@ -205,8 +177,10 @@ __global__ void init_kernel(InitArgs a)
         a.ctrl->nnew = 0;
         a.ctrl->total_nf = 0;
         a.ctrl->total_ne = 0;
-        a.ctrl->vmin = 0xffffffffu;
-        a.ctrl->vpre = 0;
+        a.ctrl->vmin2[0] = FULL;
+        a.ctrl->vmin2[1] = FULL;
+        a.ctrl->nbig2[0] = 0;
+        a.ctrl->nbig2[1] = 0;
         if (a.parent) a.parent[a.v0] = (uint32_t)a.v0;
     }
     const uint64_t w0 = a.v0 >> 5, w1 = (a.v1 + 31) >> 5;
@@ -216,121 +190,6 @@ __global__ void init_kernel(InitArgs a)
         if (w == (a.v0 >> 5)) m &= FULL << (a.v0 & 31);
         if (w == ((a.v1 - 1) >> 5) && (a.v1 & 31)) m &= (1u << (a.v1 & 31)) - 1;
         a.vis[w] |= m;
-    }
-}
-
-// --------------------------------------------------------------------------
-// compact_kernel: a7 level end.  new = vis & ~prev; the new vertices, in
-// increasing id order, become the next frontier queue (sorted for free, in
-// place of the paper's partial radix sort); depth[new] = level.
-// Reduce-then-scan over a persistent grid.  A block's word range is split into
-// one contiguous run per warp.  Pass 1 counts (coalesced word loads); the
-// cross-block prefix places the block, the per-warp counts place the warps;
-// pass 2 walks 32 words at a time: a warp scan of the popcounts gives each
-// word's queue offset and, word by word, lane b writes bit b's vertex, so the
-// queue and depth stores are coalesced.  No block barrier inside the loops.
-// --------------------------------------------------------------------------
-__global__ void __launch_bounds__(kFrontierThreads) compact_kernel(CompactArgs a)
-{
-    constexpr int NT = kFrontierThreads, NW = NT / 32;
-    __shared__ uint64_t s_warp[NW];
-    __shared__ uint64_t s_wcnt[NW];
-    __shared__ uint64_t s_pre;
-
-    const uint32_t tid = threadIdx.x, lane = tid & 31, wid = tid >> 5, b = blockIdx.x;
-    const LevelCtrl *ctrl = a.ctrl;
-    const uint32_t tag = ctrl->seq;
-    const int32_t level = (int32_t)ctrl->level;
-    int32_t *depth = ctrl->depth;
-    const uint64_t lo = (uint64_t)b * a.words_per_block;
-    const uint64_t hi = min(lo + a.words_per_block, a.nwords);
-    const uint64_t per_w = (a.words_per_block + NW - 1) / NW;
-    const uint64_t wlo = min(lo + wid * per_w, hi), whi = min(wlo + per_w, hi);
-
-    // pass 1: count (queue = owned words only; nnew = every row); 4 loads in flight
-    uint64_t cnt = 0, all = 0;
-    uint32_t vmin = 0xffffffffu;  // smallest vertex of this warp's range that is neither visited nor isolated
-    for (uint64_t w0 = wlo + lane; w0 < whi; w0 += 128) {
-        uint32_t c[4];
-#pragma unroll
-        for (int u = 0; u < 4; ++u) {
-            const uint64_t w = w0 + 32 * u;
-            c[u] = 0;
-            if (w < whi) {
-                const uint32_t x = a.vis[w];
-                c[u] = __popc(a.consume ? x : (x & ~a.prev[w]));
-                if (!a.consume && vmin == 0xffffffffu) {
-                    const uint32_t un = ~(x | a.iso[w]);
-                    if (un) vmin = (uint32_t)(w * 32) + (__ffs(un) - 1);
-                }
-            }
-        }
-#pragma unroll
-        for (int u = 0; u < 4; ++u) {
-            const uint64_t w = w0 + 32 * u;
-            all += c[u];
-            if (w >= a.own_lo_w && w < a.own_hi_w) cnt += c[u];
-        }
-    }
-    cnt = warp_sum_u64(cnt);
-    all = warp_sum_u64(all);
-#pragma unroll
-    for (int d = 16; d; d >>= 1) vmin = min(vmin, __shfl_xor_sync(FULL, vmin, d));
-    if (lane == 0) {
-        s_wcnt[wid] = cnt;
-        s_warp[wid] = all;
-        if (vmin != 0xffffffffu) atomicMin(&a.ctrl->vmin, vmin);
-    }
-    __syncthreads();
-    if (wid == 0) {
-        const uint64_t bc = lane < NW ? s_wcnt[lane] : 0, ba = lane < NW ? s_warp[lane] : 0;
-        const uint64_t blk = warp_sum_u64(bc), blk_all = warp_sum_u64(ba);
-        if (lane == 0 && blk_all) atomicAdd(reinterpret_cast<unsigned long long *>(&a.ctrl->nnew), blk_all);
-        const uint64_t pre = publish_and_prefix(a.status, b, tag, blk);
-        if (lane == 0) {
-            s_pre = pre;
-            if (b == gridDim.x - 1) a.ctrl->nf = pre + blk;
-        }
-    }
-    __syncthreads();
-    uint64_t base = s_pre;
-    for (uint32_t w = 0; w < wid; ++w) base += s_wcnt[w];
-
-    // pass 2: queue + depth
-    const uint32_t lt = (1u << lane) - 1;
-    for (uint64_t w0 = wlo; w0 < whi; w0 += 32) {
-        const uint64_t w = w0 + lane;
-        uint32_t nb = 0;
-        if (w < whi) {
-            const uint32_t x = a.vis[w];
-            if (a.consume) {  // SSSP: the relaxed set itself is the next frontier; reset it
-                nb = x;
-                if (x) a.vis[w] = 0;
-            } else {
-                const uint32_t p = a.prev[w];
-                nb = x & ~p;
-                if (nb) a.prev[w] = x;
-            }
-        }
-        const bool own = w >= a.own_lo_w && w < a.own_hi_w;
-        const uint32_t nq = own ? nb : 0u;
-        uint32_t tq;
-        const uint32_t off = warp_excl_u32(__popc(nq), tq);
-        uint32_t todo = __ballot_sync(FULL, nb != 0);
-        while (todo) {
-            const int j = __ffs(todo) - 1;
-            todo &= todo - 1;
-            const uint32_t nbw = __shfl_sync(FULL, nb, j);
-            const uint32_t nqw = __shfl_sync(FULL, nq, j);
-            const uint32_t offj = __shfl_sync(FULL, off, j);
-            if ((nbw >> lane) & 1) {
-                const uint32_t v = (uint32_t)((w0 + j) * 32 + lane);
-                if (a.depth_stored) a.depth_stored[v] = level;  // stored-id order (coalesced)
-                if (!a.depth_stored_only && depth) depth[v] = level;
-                if (nqw) a.queue[base + offj + __popc(nqw & lt)] = v;
-            }
-        }
-        base += tq;
     }
 }
 
@@ -364,173 +223,435 @@ __global__ void xchg_kernel(XchgArgs a)
 }
 
 // --------------------------------------------------------------------------
-// plan_kernel: a1 + a2 + a3 + a4.  For the sorted frontier queue:
-//   a1  degree lookup (pass 1: compact deg32; pass 2: the 16-byte record),
-//   a2  exclusive scans of the per-vertex chunk count and work
-//       (kChunkWork per chunk + one unit per element),
-//       one ChunkDesc per k-aligned chunk: the list's record and
-//       the chunk index, written by lanes over the group's chunks,
+// frontier_kernel: the level end (a7) fused with the next level's plan
+// (a1 + a2 + a3 + a4), one launch per level.
+//
+//   a7  new = vis & ~prev: the new vertices, in increasing id order, become
+//       the next frontier queue (sorted for free, in place of the paper's
+//       partial radix sort); depth[new] = level;
+//   a1  degree lookup (compact deg32 of each new vertex, then its 16-byte
+//       record);
+//   a2  exclusive scans of the per-vertex chunk count and work (kChunkWork
+//       per k-aligned chunk + one unit per element);
+//   a4  one ChunkDesc per k-aligned chunk;
 //   a3  the tile table: tile t (work [tT, (t+1)T)) starts at the first chunk
 //       whose work position is >= tT (the Fig. 4 maxle rule, once per tile).
-// Same reduce-then-scan scheme as compact_kernel, over the frontier index
-// range.  The last block publishes the level totals, records per-level
-// statistics and, in graph mode, sets the loop condition (frontier non-empty).
+//
+// Persistent grid (every block resident: blocks wait on each other).  Phases:
+//   1   a warp counts the new vertices of its bitmap word run, their work and
+//       chunks (degree loads coalesced: lanes over the bits of a word);
+//       the per-block aggregates are published, a grid barrier, then each
+//       block sums its predecessors' (one warp per aggregate) and per-warp
+//       sums place every warp;
+//   2a  the warp writes its queue segment, depth, prev and, per queue entry,
+//       the exclusive work and chunk prefixes (warp scans over the bits of
+//       each word);
+//   --  grid barrier;
+//   2b  32-entry groups of the whole queue, grid-stride (balanced however the
+//       new vertices cluster in id space): a list of one chunk writes its
+//       descriptor and at most one tile boundary; longer lists are appended
+//       to a BigList table;
+//   --  grid barrier;
+//   3   one BigList per warp: its descriptors and tile boundaries (lanes over
+//       chunks / tiles), so hub lists are spread over the grid.
+// The visited prefix (smallest vertex neither visited nor of degree 0) is
+// reduced into ctrl->vmin2[level & 1], which the next expand reads; the
+// other slot is reset for the following level end.
 // --------------------------------------------------------------------------
-__global__ void __launch_bounds__(kFrontierThreads) plan_kernel(PlanArgs a)
+// Grid-wide barrier of a persistent grid (every block resident): a 64-bit
+// arrival counter that only grows (each barrier adds gridDim.x), release on
+// arrival, acquire while polling with a short back-off.
+__device__ __forceinline__ void grid_barrier(unsigned long long *count)
+{
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        __threadfence();
+        unsigned long long old;
+        asm volatile("atom.add.release.gpu.global.u64 %0, [%1], 1;" : "=l"(old) : "l"(count) : "memory");
+        const unsigned long long target = (old / gridDim.x + 1) * gridDim.x;
+        for (;;) {
+            unsigned long long cur;
+            asm volatile("ld.acquire.gpu.global.u64 %0, [%1];" : "=l"(cur) : "l"(count) : "memory");
+            if (cur >= target) break;
+            __nanosleep(32);
+        }
+        __threadfence();
+    }
+    __syncthreads();
+}
+
+// sums of the published per-block aggregates over blocks [0, b) and over all
+// blocks (warp-wide; every lane gets both); 8 loads per lane in flight
+__device__ __forceinline__ void sum_published(const uint64_t *agg, uint32_t b, uint64_t &pre, uint64_t &tot)
+{
+    uint64_t p = 0, t = 0;
+    for (uint32_t i0 = 0; i0 < gridDim.x; i0 += 256) {
+        uint64_t v[8];
+#pragma unroll
+        for (int u = 0; u < 8; ++u) {
+            const uint32_t i = i0 + u * 32 + lane_id();
+            v[u] = i < gridDim.x ? __ldcg(agg + i) : 0;
+        }
+#pragma unroll
+        for (int u = 0; u < 8; ++u) {
+            const uint32_t i = i0 + u * 32 + lane_id();
+            t += v[u];
+            p += i < b ? v[u] : 0;
+        }
+    }
+    pre = warp_sum_u64(p);
+    tot = warp_sum_u64(t);
+}
+
+// exclusive warp scans of N independent u32 values per lane, interleaved (N
+// shuffle chains in flight instead of one)
+template <int N>
+__device__ __forceinline__ void warp_excl_u32_n(uint32_t (&x)[N], uint32_t (&total)[N])
+{
+    uint32_t inc[N];
+#pragma unroll
+    for (int i = 0; i < N; ++i) inc[i] = x[i];
+#pragma unroll
+    for (int d = 1; d < 32; d <<= 1) {
+#pragma unroll
+        for (int i = 0; i < N; ++i) {
+            const uint32_t y = __shfl_up_sync(FULL, inc[i], d);
+            if ((int)lane_id() >= d) inc[i] += y;
+        }
+    }
+#pragma unroll
+    for (int i = 0; i < N; ++i) {
+        total[i] = __shfl_sync(FULL, inc[i], 31);
+        x[i] = inc[i] - x[i];
+    }
+}
+
+__global__ void __launch_bounds__(kFrontierThreads, 2) frontier_kernel(FrontierArgs a)
 {
     constexpr int NT = kFrontierThreads, NW = NT / 32;
-    __shared__ uint64_t s_wwork[NW], s_wch[NW];
-    __shared__ uint64_t s_pre, s_cpre;
+    __shared__ uint64_t s_q[NW], s_wk[NW], s_ch[NW], s_all[NW];
+    __shared__ uint64_t s_pre[3], s_tot[3];
 
     const uint32_t tid = threadIdx.x, lane = tid & 31, wid = tid >> 5, b = blockIdx.x;
+#define FTRACE(p)                                                      \
+    do {                                                               \
+        if (a.trace && tid == 0) a.trace[b * 8 + (p)] = globaltimer(); \
+    } while (0)
+    FTRACE(0);
     LevelCtrl *ctrl = a.ctrl;
-    const uint32_t tag = ctrl->seq;
-    const uint64_t nf = ctrl->nf;
+    const uint32_t level = ctrl->level;
+    int32_t *depth = ctrl->depth;
+    if (b == 0 && tid == 0) {  // slots of the next level end
+        ctrl->vmin2[(level & 1) ^ 1] = FULL;
+        ctrl->nbig2[(level & 1) ^ 1] = 0;
+    }
     const ChunkLen cl = make_chunk(a.k, a.kshift);
     const uint64_t CH = cl.ch, CW = kChunkWork;
-    const uint64_t per = (nf + gridDim.x - 1) / gridDim.x;
-    const uint64_t lo = min((uint64_t)b * per, nf), hi = min(lo + per, nf);
-    const uint64_t per_w = (per + NW - 1) / NW;
-    const uint64_t qlo = min(lo + wid * per_w, hi), qhi = min(qlo + per_w, hi);
+    // warp gw owns the 32-word groups gw, gw + G, ... of the bitmap (round
+    // robin: a dense id range, e.g. relabelled hubs, is spread over the grid);
+    // its queue segment is contiguous, in group order
+    const uint32_t G = gridDim.x * NW;
+    const uint32_t gw = b * NW + wid;
+    const uint64_t WG = 32ull * G;  // words between a warp's groups
+    const uint32_t lt = (1u << lane) - 1;
+    constexpr int kB = 8;  // pass 1: non-empty words whose degree loads are in flight together
 
-    // pass 1: chunks and work of the warp's range (a1 degree lookup), 4 lookups in flight
-    uint64_t wk = 0, ch = 0;
-    for (uint64_t i0 = qlo + lane; i0 < qhi; i0 += 128) {
-        uint32_t q[4];
+    // ---- 1: count, work and chunks of the warp's new (owned) vertices ----
+    uint32_t cq = 0, all = 0, ch = 0;  // lane partials
+    uint64_t wk = 0;
+    uint32_t vmin = FULL;  // smallest vertex of this warp's range that is neither visited nor isolated
+    for (uint64_t w0 = 32ull * gw; w0 < a.nwords; w0 += WG) {
+        const uint64_t w = w0 + lane;
+        uint32_t nb = 0, nq = 0;
+        if (w < a.nwords) {
+            const uint32_t x = a.vis[w];
+            nb = a.consume ? x : (x & ~a.prev[w]);
+            if (!a.consume && vmin == FULL) {
+                const uint32_t un = ~(x | a.iso[w]);
+                if (un) vmin = (uint32_t)(w * 32) + (__ffs(un) - 1);
+            }
+            nq = (w >= a.own_lo_w && w < a.own_hi_w) ? nb : 0u;
+        }
+        all += __popc(nb);
+        cq += __popc(nq);
+        // a1: degrees of the new vertices, lanes over the bits of each non-empty
+        // word (one coalesced 128-byte load per word)
+        uint32_t todo = __ballot_sync(FULL, nq != 0);
+        while (todo) {
+            uint32_t dv[kB];
 #pragma unroll
-        for (int u = 0; u < 4; ++u) q[u] = i0 + 32 * u < qhi ? a.queue[i0 + 32 * u] : 0u;
+            for (int u = 0; u < kB; ++u) {
+                dv[u] = 0;
+                if (todo) {
+                    const int j = __ffs(todo) - 1;
+                    todo &= todo - 1;
+                    const uint32_t bits = __shfl_sync(FULL, nq, j);
+                    if ((bits >> lane) & 1) dv[u] = __ldg(a.deg32 + (w0 + j) * 32 + lane);
+                }
+            }
 #pragma unroll
-        for (int u = 0; u < 4; ++u)
-            if (i0 + 32 * u < qhi) {
-                const uint64_t d = __ldg(a.deg32 + q[u]);
-                const uint64_t nch = d ? cl.div(d + CH - 1) : 0;
-                wk += nch * CW + d;
+            for (int u = 0; u < kB; ++u) {
+                const uint32_t d = dv[u];
+                const uint32_t nch = d ? (uint32_t)cl.div((uint64_t)d + CH - 1) : 0u;
+                wk += (uint64_t)nch * CW + d;
                 ch += nch;
             }
+        }
     }
+    const uint64_t cqw = warp_sum_u64(cq), allw = warp_sum_u64(all), chw = warp_sum_u64(ch);
     wk = warp_sum_u64(wk);
-    ch = warp_sum_u64(ch);
+#pragma unroll
+    for (int d = 16; d; d >>= 1) vmin = min(vmin, __shfl_xor_sync(FULL, vmin, d));
     if (lane == 0) {
-        s_wwork[wid] = wk;
-        s_wch[wid] = ch;
+        s_q[wid] = cqw;
+        s_all[wid] = allw;
+        s_wk[wid] = wk;
+        s_ch[wid] = chw;
+        if (vmin != FULL) atomicMin(&ctrl->vmin2[level & 1], vmin);
     }
     __syncthreads();
-    if (wid == 0) {
-        const uint64_t blk = warp_sum_u64(lane < NW ? s_wwork[lane] : 0);
-        const uint64_t blkc = warp_sum_u64(lane < NW ? s_wch[lane] : 0);
-        const uint64_t pre = publish_and_prefix(a.status, b, tag, blk);
-        const uint64_t cpre = publish_and_prefix(a.status + kMaxGrid, b, tag, blkc);
+    FTRACE(1);
+    // publish the block's aggregates (queue entries, work units, chunks),
+    // barrier, then every block sums its predecessors' (region r by warp r)
+    if (wid < 3) {
+        const uint64_t *src = wid == 0 ? s_q : (wid == 1 ? s_wk : s_ch);
+        const uint64_t agg = warp_sum_u64(lane < NW ? src[lane] : 0);
+        if (lane == 0) st_relaxed_u64(a.status + wid * kMaxGrid + b, agg);
+    } else if (wid == 3) {
+        const uint64_t blk_all = warp_sum_u64(lane < NW ? s_all[lane] : 0);
+        if (lane == 0 && blk_all) atomicAdd(reinterpret_cast<unsigned long long *>(&ctrl->nnew), blk_all);
+    }
+    grid_barrier(a.barrier);
+    if (wid < 3) {
+        uint64_t pre, tot;
+        sum_published(a.status + wid * kMaxGrid, b, pre, tot);
         if (lane == 0) {
-            s_pre = pre;
-            s_cpre = cpre;
-            if (b == gridDim.x - 1) {
-                const uint64_t nwork = pre + blk, nchunks = cpre + blkc;
-                const uint64_t ne = nwork - CW * nchunks;
-                const uint32_t lvl = ctrl->level;
-                const uint64_t ntiles = (nwork + kTileWork - 1) / kTileWork;
-                ctrl->nwork = nwork;
-                ctrl->nchunks = nchunks;
-                ctrl->ne = ne;
-                ctrl->ntiles = ntiles;
-                ctrl->xlevel = lvl;
-                ctrl->vpre = ctrl->vmin;  // compact of this level end is complete (stream order)
-                ctrl->vmin = 0xffffffffu;
-                a.tiles[ntiles] = (uint32_t)nchunks;  // sentinel: end of the last tile
-                if (nf) {
-                    ctrl->nlevels = lvl + 1;
-                    ctrl->total_nf += nf;
-                    ctrl->total_ne += ne;
-                    if (a.stats && lvl < a.max_stats) {
-                        a.stats[lvl].nf = nf;
-                        a.stats[lvl].ne = ne;
-                        a.stats[lvl].t0 = ~0ull;
-                        a.stats[lvl].t1 = 0;
+            s_pre[wid] = pre;
+            s_tot[wid] = tot;
+        }
+    }
+    __syncthreads();
+    const uint64_t nf = s_tot[0];
+    if (b == gridDim.x - 1 && tid == 0) {  // level totals
+        const uint64_t nwork = s_tot[1], nchunks = s_tot[2];
+        const uint64_t ne = nwork - CW * nchunks;
+        const uint64_t ntiles = (nwork + kTileWork - 1) / kTileWork;
+        ctrl->nf = nf;
+        ctrl->nwork = nwork;
+        ctrl->nchunks = nchunks;
+        ctrl->ne = ne;
+        ctrl->ntiles = ntiles;
+        ctrl->xlevel = level;
+        a.tiles[ntiles] = (uint32_t)nchunks;  // sentinel: end of the last tile
+        if (nf) {
+            ctrl->nlevels = level + 1;
+            ctrl->total_nf += nf;
+            ctrl->total_ne += ne;
+            if (a.stats && level < a.max_stats) {
+                a.stats[level].nf = nf;
+                a.stats[level].ne = ne;
+                a.stats[level].t0 = ~0ull;
+                a.stats[level].t1 = 0;
+            }
+        }
+        if (a.cond) cudaGraphSetConditional(a.cond, nf ? 1u : 0u);
+    }
+    FTRACE(2);
+    uint64_t run = s_pre[1];
+    uint32_t crun = (uint32_t)s_pre[2];  // chunks of a level < 2^32 (n + m/k)
+    for (uint32_t w = 0; w < wid; ++w) {
+        run += s_wk[w];
+        crun += (uint32_t)s_ch[w];
+    }
+
+    // ---- 2: depth, prev and the plan of the warp's new vertices, word by
+    // word (lanes over bits): record loads (a1), work / chunk prefixes (a2),
+    // descriptors (a4) and tile boundaries (a3) of single-chunk lists; longer
+    // lists go to the BigList table (phase 3) ----
+    const bool narrow = a.k == 0 || a.k >= 32;  // per-lane work < 2^27: 32-bit scans
+    constexpr int kS = 2;                         // non-empty words planned together
+    for (uint64_t w0 = 32ull * gw; w0 < a.nwords; w0 += WG) {
+        const uint64_t w = w0 + lane;
+        uint32_t nb = 0;
+        if (w < a.nwords) {
+            const uint32_t x = a.vis[w];
+            if (a.consume) {  // SSSP: the relaxed set itself is the next frontier; reset it
+                nb = x;
+                if (x) a.vis[w] = 0;
+            } else {
+                const uint32_t p = a.prev[w];
+                nb = x & ~p;
+                if (nb) a.prev[w] = x;
+            }
+        }
+        const bool own = w >= a.own_lo_w && w < a.own_hi_w;
+        const uint32_t nq = own ? nb : 0u;
+        uint32_t todo = __ballot_sync(FULL, nb != 0);
+        while (todo) {
+            uint32_t jw[kS], bq[kS], wl[kS], nc[kS];
+            uint4 rv[kS];
+#pragma unroll
+            for (int u = 0; u < kS; ++u) {
+                jw[u] = 32;
+                bq[u] = 0;
+                rv[u] = make_uint4(0, 0, 0, 0);
+                if (todo) {
+                    const int j = __ffs(todo) - 1;
+                    todo &= todo - 1;
+                    jw[u] = j;
+                    bq[u] = __shfl_sync(FULL, nq, j);
+                    const uint32_t bb = __shfl_sync(FULL, nb, j);
+                    const uint32_t v = (uint32_t)((w0 + j) * 32 + lane);
+                    if ((bq[u] >> lane) & 1) rv[u] = __ldg(reinterpret_cast<const uint4 *>(a.rec + v));
+                    if ((bb >> lane) & 1) {
+                        if (a.depth_stored) a.depth_stored[v] = (int32_t)level;  // stored-id order (coalesced)
+                        if (!a.depth_stored_only && depth) depth[v] = (int32_t)level;
                     }
                 }
-                if (a.cond) cudaGraphSetConditional(a.cond, nf ? 1u : 0u);
+            }
+            // per-list work nch*CW + d < 2^31.1 (deg < 2^26); the 32-lane sums fit
+            // 32 bits when k >= 32 (< 2^27 per list), else the work is scanned
+            // as (w >> 5, w & 31)
+            uint32_t wlo[kS], wt[kS], wtlo[kS], ct[kS];
+#pragma unroll
+            for (int u = 0; u < kS; ++u) {
+                const uint32_t d = rv[u].z;
+                nc[u] = d ? (uint32_t)cl.div((uint64_t)d + CH - 1) : 0u;
+                const uint32_t wv = nc[u] * (uint32_t)CW + d;
+                wl[u] = narrow ? wv : wv >> 5;
+                wlo[u] = narrow ? 0u : wv & 31;
+            }
+            warp_excl_u32_n<kS>(wl, wt);
+            if (!narrow) warp_excl_u32_n<kS>(wlo, wtlo);
+            uint32_t cex[kS];
+            bool one = true;  // every list of these words is one chunk (or empty)
+#pragma unroll
+            for (int u = 0; u < kS; ++u) {
+                one = one && nc[u] <= 1;
+                cex[u] = nc[u];
+            }
+            if (__all_sync(FULL, one)) {
+#pragma unroll
+                for (int u = 0; u < kS; ++u) {
+                    const uint32_t hm = __ballot_sync(FULL, nc[u] != 0);
+                    ct[u] = __popc(hm);
+                    cex[u] = __popc(hm & lt);
+                }
+            } else {
+                warp_excl_u32_n<kS>(cex, ct);
+            }
+#pragma unroll
+            for (int u = 0; u < kS; ++u) {
+                if (!bq[u]) continue;  // warp-uniform
+                const bool mine = (bq[u] >> lane) & 1;
+                const uint32_t d = rv[u].z, ub = rv[u].w, nch = nc[u];
+                const uint64_t off_l = ((uint64_t)rv[u].y << 32) | rv[u].x;
+                const uint64_t W = run + (narrow ? (uint64_t)wl[u] : ((uint64_t)wl[u] << 5) + wlo[u]);
+                const uint32_t C = crun + cex[u];
+                const uint64_t wlen = (uint64_t)nch * CW + d;
+                const bool big = mine && (nch > 1 || wlen > kTileWork);
+                if (mine && !big) {
+                    if (nch == 1) {  // a4: the list's only chunk
+                        uint4 *dp = reinterpret_cast<uint4 *>(a.chunks + C);
+                        dp[0] = make_uint4(rv[u].x, rv[u].y, d, ub);
+                        dp[1] = make_uint4((uint32_t)((w0 + jw[u]) * 32 + lane), 0u, 0u, 0u);
+                    }
+                    // a3: a tile boundary t*T inside [W, W + wlen) starts at this chunk or the next
+                    const uint64_t t = (W + kTileWork - 1) / kTileWork;
+                    if (t * kTileWork < W + wlen) a.tiles[t] = C + (t * kTileWork > W ? 1u : 0u);
+                }
+                const uint32_t bm = __ballot_sync(FULL, big);
+                if (bm) {
+                    uint32_t base = 0;
+                    if (lane == 0) base = atomicAdd(&ctrl->nbig2[level & 1], (uint32_t)__popc(bm));
+                    base = __shfl_sync(FULL, base, 0);
+                    if (big) {
+                        BigList bl;
+                        bl.W = W;
+                        bl.cstart = C;
+                        bl.off_l = off_l;
+                        bl.deg = d;
+                        bl.ubytes = ub;
+                        bl.v = (uint32_t)((w0 + jw[u]) * 32 + lane);
+                        bl.nch = nch;
+                        a.big[base + __popc(bm & lt)] = bl;
+                    }
+                }
+                run += narrow ? (uint64_t)wt[u] : ((uint64_t)wt[u] << 5) + wtlo[u];
+                crun += ct[u];
             }
         }
     }
-    __syncthreads();
-    uint64_t run = s_pre, crun = s_cpre;
-    for (uint32_t w = 0; w < wid; ++w) {
-        run += s_wwork[w];
-        crun += s_wch[w];
-    }
+    FTRACE(5);
+    grid_barrier(a.barrier);
+    FTRACE(6);
 
-    // pass 2: 32 frontier vertices at a time (one per lane); the next group's
-    // queue entries are fetched while the current group is processed
-    // software pipeline: records of group g+1 and queue entries of group g+2 are
-    // in flight while group g is processed
-    uint32_t vn = qlo + lane < qhi ? a.queue[qlo + lane] : 0u;
-    uint4 rn = make_uint4(0, 0, 0, 0);
-    if (qlo + lane < qhi) rn = __ldg(reinterpret_cast<const uint4 *>(a.rec + vn));
-    uint32_t vnn = qlo + 32 + lane < qhi ? a.queue[qlo + 32 + lane] : 0u;
-    for (uint64_t i0 = qlo; i0 < qhi; i0 += 32) {
-        const uint64_t i = i0 + lane;
-        const uint32_t v = vn;
-        const uint4 r = rn;
-        vn = vnn;
-        rn = make_uint4(0, 0, 0, 0);
-        if (i + 32 < qhi) rn = __ldg(reinterpret_cast<const uint4 *>(a.rec + vn));
-        vnn = i + 64 < qhi ? a.queue[i + 64] : 0u;
-        uint64_t off_l = 0;
-        uint32_t d = 0, ub = 0;
-        if (i < qhi) {
-            off_l = ((uint64_t)r.y << 32) | r.x;
-            d = r.z;
-            ub = r.w;
+    // ---- 3: the long lists, one per lane (lists of > 8 chunks or tiles: one
+    // per warp, lanes over chunks / tiles): descriptors and the tile
+    // boundaries of the list's window (Fig. 4 rule) ----
+    const uint32_t nbig = ld_relaxed_u32(&ctrl->nbig2[level & 1]);
+    const bool udiv = a.k && CW + CH < (1ull << 31);  // 32-bit chunk division (rel < 2^31.1 - CW - CH)
+    const uint32_t CWH = (uint32_t)(CW + CH);
+    auto tile_chunk = [&](uint32_t rel, uint32_t nch) -> uint32_t {
+        // chunk c of a list starts at W + c*(CW + k): first chunk at or after W + rel
+        uint32_t c = rel ? 1u : 0u;
+        if (udiv && nch > 1) c = min((rel + CWH - 1) / CWH, nch);
+        return c;
+    };
+    for (uint64_t e0 = (uint64_t)gw * 32; e0 < nbig; e0 += 32ull * G) {
+        const uint64_t e = e0 + lane;
+        uint64_t W = 0, cs = 0, off_l = 0;
+        uint32_t d = 0, ub = 0, v = 0, nch = 0;
+        if (e < nbig) {
+            const BigList *bp = a.big + e;
+            W = __ldcg(&bp->W);
+            cs = __ldcg(&bp->cstart);
+            off_l = __ldcg(&bp->off_l);
+            d = __ldcg(&bp->deg);
+            ub = __ldcg(&bp->ubytes);
+            v = __ldcg(&bp->v);
+            nch = __ldcg(&bp->nch);
         }
-        const uint32_t nch = d ? (uint32_t)cl.div((uint64_t)d + CH - 1) : 0u;
-        uint64_t totw;
-        const uint64_t W = run + warp_excl_u64((uint64_t)nch * CW + d, totw);
-        uint32_t totc;
-        const uint32_t cb = warp_excl_u32(nch, totc);
-
-        // a4: descriptors, lanes over the group's chunks (owner by maxle, C13)
-        for (uint32_t j0 = 0; j0 < totc; j0 += 32) {
-            const uint32_t j = j0 + lane;
-            const int o = warp_maxle_u32(i < qhi ? cb : 0xffffffffu, j);
-            const uint64_t ol = __shfl_sync(FULL, off_l, o);
+        const uint64_t wl = (uint64_t)nch * CW + d;
+        const uint64_t t_lo = (W + kTileWork - 1) / kTileWork, t_hi = (W + wl + kTileWork - 1) / kTileWork;
+        const bool huge = nch > 8 || t_hi - t_lo > 8;
+        if (!huge) {
+            for (uint32_t j = 0; j < nch; ++j) {
+                uint4 *dp = reinterpret_cast<uint4 *>(a.chunks + cs + j);
+                dp[0] = make_uint4((uint32_t)off_l, (uint32_t)(off_l >> 32), d, ub);
+                dp[1] = make_uint4(v, j, 0u, 0u);
+            }
+            for (uint64_t t = t_lo; t < t_hi; ++t)
+                a.tiles[t] = (uint32_t)(cs + tile_chunk((uint32_t)(t * kTileWork - W), nch));
+        }
+        uint32_t hm = __ballot_sync(FULL, huge);
+        while (hm) {
+            const int o = __ffs(hm) - 1;
+            hm &= hm - 1;
+            const uint64_t oW = __shfl_sync(FULL, W, o), ocs = __shfl_sync(FULL, cs, o);
+            const uint64_t ooff = __shfl_sync(FULL, off_l, o);
             const uint32_t od = __shfl_sync(FULL, d, o), oub = __shfl_sync(FULL, ub, o);
-            const uint32_t ov = __shfl_sync(FULL, v, o), ocb = __shfl_sync(FULL, cb, o);
-            if (j < totc) {
-                uint4 *dp = reinterpret_cast<uint4 *>(a.chunks + crun + j);
-                dp[0] = make_uint4((uint32_t)ol, (uint32_t)(ol >> 32), od, oub);
-                dp[1] = make_uint4(ov, j - ocb, 0u, 0u);
+            const uint32_t ov = __shfl_sync(FULL, v, o), onch = __shfl_sync(FULL, nch, o);
+            for (uint32_t j = lane; j < onch; j += 32) {
+                uint4 *dp = reinterpret_cast<uint4 *>(a.chunks + ocs + j);
+                dp[0] = make_uint4((uint32_t)ooff, (uint32_t)(ooff >> 32), od, oub);
+                dp[1] = make_uint4(ov, j, 0u, 0u);
             }
+            const uint64_t owl = (uint64_t)onch * CW + od;
+            const uint64_t ot_lo = (oW + kTileWork - 1) / kTileWork, ot_hi = (oW + owl + kTileWork - 1) / kTileWork;
+            for (uint64_t t = ot_lo + lane; t < ot_hi; t += 32)
+                a.tiles[t] = (uint32_t)(ocs + tile_chunk((uint32_t)(t * kTileWork - oW), onch));
         }
-
-        // a3: tiles whose boundary t*T falls in this group's work window
-        // [W_0, W_0 + totw): lanes take consecutive tiles, each finds its vertex
-        // by maxle over the group's W (Fig. 4 rule inside the warp)
-        const uint64_t wstart = __shfl_sync(FULL, W, 0);
-        const uint64_t tfirst = (wstart + kTileWork - 1) / kTileWork;
-        const uint64_t tend = (wstart + totw + kTileWork - 1) / kTileWork;
-        const uint32_t wrel = i < qhi ? (uint32_t)(W - wstart) : 0xffffffffu;  // < totw <= 2^32
-        for (uint64_t t0 = tfirst; t0 < tend; t0 += 32) {
-            const uint64_t t = t0 + lane;
-            const uint32_t key = t < tend ? (uint32_t)(t * kTileWork - wstart) : 0u;
-            const int o = warp_maxle_u32(wrel, key);
-            const uint64_t oW = __shfl_sync(FULL, W, o);
-            const uint32_t onch = __shfl_sync(FULL, nch, o), ocb = __shfl_sync(FULL, cb, o);
-            if (t < tend) {
-                // chunk c of the owner starts at W + c*(CW + k); first chunk at or after t*T
-                const uint64_t rel = t * kTileWork - oW;
-                const uint64_t c = a.k ? (rel + CW + CH - 1) / (CW + CH) : (rel ? 1 : 0);
-                a.tiles[t] = (uint32_t)(crun + ocb + min(c, (uint64_t)onch));
-            }
-        }
-        run += totw;
-        crun += totc;
     }
+    FTRACE(7);
+#undef FTRACE
 }
 
 // --------------------------------------------------------------------------
 // expand_kernel: a4 + a5 + a6 (P:137-177 generalised, Alg. 1 lines 3-6)
 //
 // Persistent: one CTA of kExpandWarps warps per SM; a warp takes tiles
-// gw, gw + #warps, ...  A tile's chunks (plan_kernel descriptors) are cut into
+// gw, gw + #warps, ...  A tile's chunks (frontier_kernel descriptors) are cut into
 // batches of <= 32 chunks whose compressed bytes fit one staging buffer.  Per
 // batch the warp
 //   (producer)  a4: locates each chunk's bits from the forward pointers
@@ -724,7 +845,7 @@ __global__ void __launch_bounds__(kExpandThreads, 1) expand_kernel(ExpandArgs a)
     const uint32_t *data32 = reinterpret_cast<const uint32_t *>(a.data);
     const uint32_t *st32 = &ws.stage[0][0];
     const uint32_t sbits = smem_u32(st32) * 8;  // shared-window bit address of the staging area
-    const uint32_t vpre = kBfs ? a.ctrl->vpre : 0u;  // ids below it are visited (or never probed)
+    const uint32_t vpre = kBfs ? a.ctrl->vmin2[xl & 1] : 0u;  // ids below it are visited (or never probed)
     const uint64_t gw = (uint64_t)blockIdx.x * kExpandWarps + wid;
     const uint64_t nwarps = (uint64_t)gridDim.x * kExpandWarps;
     const uint64_t CH = a.k ? a.k : (1ull << 40);
@@ -1226,9 +1347,19 @@ cudaError_t launch_init(const InitArgs &a, cudaStream_t s)
     return cudaGetLastError();
 }
 
-cudaError_t launch_compact(const CompactArgs &a, unsigned blocks, cudaStream_t s)
+int frontier_occupancy()
 {
-    compact_kernel<<<blocks, kFrontierThreads, 0, s>>>(a);
+    int nb = 0;
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, frontier_kernel, kFrontierThreads, 0) != cudaSuccess) {
+        cudaGetLastError();
+        return 0;
+    }
+    return nb;
+}
+
+cudaError_t launch_frontier(const FrontierArgs &a, unsigned blocks, cudaStream_t s)
+{
+    frontier_kernel<<<blocks, kFrontierThreads, 0, s>>>(a);
     return cudaGetLastError();
 }
 
@@ -1240,10 +1371,5 @@ cudaError_t launch_xchg(const XchgArgs &a, cudaStream_t s)
     return cudaGetLastError();
 }
 
-cudaError_t launch_plan(const PlanArgs &a, unsigned blocks, cudaStream_t s)
-{
-    plan_kernel<<<blocks, kFrontierThreads, 0, s>>>(a);
-    return cudaGetLastError();
-}
 
 }  // namespace efg

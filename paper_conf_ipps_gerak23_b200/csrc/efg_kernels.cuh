@@ -17,7 +17,7 @@ enum ExpandMode : int {
 
 struct ExpandArgs {
     const uint8_t *data;       // EF data (device, 4-byte aligned, padded)
-    const ChunkDesc *chunks;   // chunk descriptors of the level (plan_kernel)
+    const ChunkDesc *chunks;   // chunk descriptors of the level (frontier_kernel)
     const uint32_t *tiles;     // tile table: first chunk of tile t (ntiles + 1 entries)
     const uint32_t *deg32;     // degrees (PageRank share)
     LevelCtrl *ctrl;           // nf, ne, ntiles of this level; parent pointer; level
@@ -43,19 +43,6 @@ struct InitArgs {
     uint64_t v0, v1;           // start set [v0, v1)
 };
 
-struct CompactArgs {
-    uint32_t *vis, *prev;      // visited bitmap now / at the previous level end
-    const uint32_t *iso;       // degree-0 vertices (never probed): count as visited for vpre
-    uint32_t *queue;           // out: next frontier, sorted
-    int32_t *depth_stored;     // depth by stored id (always written)
-    int depth_stored_only;     // 1: depth_stored is the only depth output (relabelled graphs)
-    int consume;               // 1: frontier = vis itself, vis reset (SSSP relaxed set)
-    LevelCtrl *ctrl;           // in: level, seq, depth ptr; out: nf
-    uint64_t *status;          // cross-block prefix words (one per block)
-    uint64_t nwords, words_per_block;
-    uint64_t own_lo_w, own_hi_w;  // owned bitmap words: only these enter the queue
-};
-
 struct XchgArgs {
     int op;                        // 0 pack, 1 reduce, 2 unpack
     int world;
@@ -67,26 +54,34 @@ struct XchgArgs {
     const uint32_t *in;
 };
 
-struct PlanArgs {
-    const uint32_t *queue;
-    const uint32_t *deg32;
-    const VRec *rec;
-    const uint8_t *data;       // EF data (forward pointers)
+struct FrontierArgs {           // level end (a7) + next level plan (a1-a4), one launch
+    uint32_t *vis, *prev;      // visited bitmap now / at the previous level end
+    const uint32_t *iso;       // degree-0 vertices (never probed): count as visited for the visited prefix
+    int32_t *depth_stored;     // depth by stored id (relabelled graphs)
+    int depth_stored_only;     // 1: depth_stored is the only depth output (relabelled graphs)
+    int consume;               // 1: frontier = vis itself, vis reset (SSSP relaxed set)
+    const uint32_t *deg32;     // degrees (pass 1)
+    const VRec *rec;           // vertex records (pass 2)
     ChunkDesc *chunks;         // out: chunk descriptors
     uint32_t *tiles;           // out: first chunk of each tile (+ sentinel)
-    LevelCtrl *ctrl;           // in: nf, level, seq; out: ne, nwork, nchunks, ntiles, xlevel
-    uint64_t *status;          // two cross-block prefix regions (work, chunks) of kMaxGrid words
+    LevelCtrl *ctrl;           // in: level, seq, depth ptr; out: nf, ne, nwork, nchunks, ntiles, xlevel, vmin2
+    uint64_t *status;          // three per-block aggregate regions of kMaxGrid words
+    unsigned long long *barrier;  // grid-barrier arrival counter (grows by gridDim.x per barrier)
+    BigList *big;              // scratch: lists planned by the whole grid
+    unsigned long long *trace; // debug (EFG_FRONTIER_TRACE): per block, 8 phase timestamps, or null
     LevelStat *stats;
     uint32_t max_stats;
     uint32_t k;
     int32_t kshift;
     cudaGraphConditionalHandle cond;  // graph-mode loop condition, 0 = host loop
+    uint64_t nwords, words_per_block;
+    uint64_t own_lo_w, own_hi_w;  // owned bitmap words: only these enter the frontier
 };
 
 cudaError_t launch_expand(int mode, const ExpandArgs &a, int blocks, cudaStream_t s);
 cudaError_t launch_init(const InitArgs &a, cudaStream_t s);
-cudaError_t launch_compact(const CompactArgs &a, unsigned blocks, cudaStream_t s);
-cudaError_t launch_plan(const PlanArgs &a, unsigned blocks, cudaStream_t s);
+cudaError_t launch_frontier(const FrontierArgs &a, unsigned blocks, cudaStream_t s);
+int frontier_occupancy();  // resident frontier_kernel blocks per SM (its grid must fit: blocks spin on predecessors)
 cudaError_t launch_xchg(const XchgArgs &a, cudaStream_t s);
 int expand_occupancy(int mode);
 size_t expand_smem_bytes();

@@ -1,4 +1,5 @@
 #!/bin/bash
-# quick GPU iteration: parity tests + bench on C2 (used via gpurun)
-timeout 600 python -m pytest tests -m "gpu and not slow" -x -q 2>&1 | tail -3
-timeout 600 python bench.py --steps 10 --warmup 3 --no-cpu-baseline --profile-levels 2>&1 | grep -E "L=[23] |metric|passed|failed|Error" | tail -14
+# quick GPU iteration: build, parity tests + bench on C2 (used via gpurun)
+python -c "import __graft_entry__ as g; g.build()" > gpurun_out/build_quick.log 2>&1 || { tail -20 gpurun_out/build_quick.log; exit 1; }
+timeout 900 python -m pytest tests -m "gpu" -x -q 2>&1 | tail -15
+timeout 600 python bench.py --steps 10 --warmup 3 --no-cpu-baseline --profile-levels 2>&1 | tail -30
