@@ -58,6 +58,8 @@ def parse():
     p.add_argument("--reorder", default="degree", choices=["none", "degree"],
                    help="EFG_REORDER_DEGREE relabelling at build time (results stay in input ids)")
     p.add_argument("--profile-levels", action="store_true", help="print per-level stats to stderr")
+    p.add_argument("--no-pagerank", action="store_true",
+                   help="skip the PageRank measurement (BASELINE configs[1]: BFS and PageRank)")
     return p.parse_args()
 
 
@@ -421,6 +423,49 @@ def main():
                "ef_data_bytes_per_edge": g2.info["data_bytes"] / g2.info["m"]}
         g2.free()
 
+    # ---- the same BFS without the visited-prefix skip (EFG_OPT_PREFIX_SKIP = 0):
+    # every element decoded and probed, as in the paper's expansion ----
+    alt_ns = None
+    if world == 1:
+        g.set_prefix_skip(False)
+        with torch.cuda.stream(stream):
+            for s in my[:args.warmup]:
+                g.bfs(int(s), depth=depth)
+        torch.cuda.synchronize()
+        a0 = torch.cuda.Event(enable_timing=True)
+        a1 = torch.cuda.Event(enable_timing=True)
+        e_ns = 0
+        a0.record(stream)
+        with torch.cuda.stream(stream):
+            for s, _ in stats:
+                _, _, st3 = g.bfs(s, depth=depth, stats=True)
+                e_ns += st3["edges_traversed"]
+        a1.record(stream)
+        torch.cuda.synchronize()
+        g.set_prefix_skip(True)
+        alt_ns = {"prefix_skip": False, "value": e_ns / (a0.elapsed_time(a1) * 1e-3) / 1e9, "unit": UNIT}
+
+    # ---- PageRank over the same EFG (BASELINE configs[1] "BFS and PageRank"):
+    # 50 push iterations, fp64 accumulation (reading C21) ----
+    pr = None
+    if world == 1 and not args.no_pagerank:
+        rank_d = torch.empty(n, dtype=torch.float64, device=dev)
+        with torch.cuda.stream(stream):
+            g.pagerank(0.85, 50, rank=rank_d)  # warm-up (builds the all-vertex plan once)
+        torch.cuda.synchronize()
+        p0 = torch.cuda.Event(enable_timing=True)
+        p1 = torch.cuda.Event(enable_timing=True)
+        p0.record(stream)
+        with torch.cuda.stream(stream):
+            g.pagerank(0.85, 50, rank=rank_d)
+        p1.record(stream)
+        torch.cuda.synchronize()
+        pms = p0.elapsed_time(p1)
+        rs = float(rank_d.sum().item())
+        pr = {"iters": 50, "damping": 0.85, "ms": pms, "ms_per_iter": pms / 50,
+              "gteps": 50 * int(info["m"]) / (pms * 1e-3) / 1e9, "unit": "GTEPS (edges pushed / s)",
+              "rank_sum": rs, "accumulate": "fp64 atomicAdd (push, P:185)"}
+
     # ---- cpu baseline: the oracle on a bounded sample (rank 0, N=1 only) ----
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
@@ -475,6 +520,8 @@ def main():
                     "d2h_bytes_per_step": 4 * n},
             "cpu_baseline": cpu,
             "alt_no_reorder": alt,
+            "alt_no_prefix_skip": alt_ns,
+            "pagerank": pr,
         }
         print(json.dumps(line), flush=True)
     g.free()

@@ -203,6 +203,13 @@ efg_status efg_pagerank(efg_graph *g, double damping, uint32_t iters, double *ra
                               * CUDA graph with a conditional WHILE node (no host round trip
                               * per level); 1: host-driven loop that reads the frontier size
                               * each level and times every expand launch with CUDA events. */
+#define EFG_OPT_PREFIX_SKIP 2 /* 1 (default): BFS expand drops upper-bit words whose elements
+                               * are all below the visited prefix vpre (every id < vpre is
+                               * visited or has no in-edge; lists are sorted, so such words
+                               * form a prefix of each list): those ids are neither decoded
+                               * nor probed; their bytes are still staged.  0: every element
+                               * is decoded and probed (the paper's expansion, Alg. 1).
+                               * Results are identical either way. */
 
 /* Set a per-handle option.  Errors: EFG_EINVAL (unknown option / value),
  * EFG_ESTATE (host-only handle). */

@@ -86,6 +86,11 @@ class Graph:
         True = host loop with per-level CUDA-event timing of the expand kernel."""
         check(lib.efg_set_option(self._h, _abi.EFG_OPT_LEVEL_LOOP, 1 if host else 0), "efg_set_option")
 
+    def set_prefix_skip(self, on: bool) -> None:
+        """EFG_OPT_PREFIX_SKIP: True (default) = BFS skips upper-bit words whose ids are
+        all below the visited prefix; False = decode and probe every element."""
+        check(lib.efg_set_option(self._h, _abi.EFG_OPT_PREFIX_SKIP, 1 if on else 0), "efg_set_option")
+
     def free(self) -> None:
         if self._h:
             lib.efg_free(self._h)

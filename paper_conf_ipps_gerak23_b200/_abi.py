@@ -20,6 +20,7 @@ EFG_SYMMETRIZE, EFG_DEDUP, EFG_DROP_SELF_LOOPS = 0x1, 0x2, 0x4
 EFG_DEFAULT_FLAGS = 0x7
 EFG_REORDER_DEGREE = 0x8
 EFG_OPT_LEVEL_LOOP = 1
+EFG_OPT_PREFIX_SKIP = 2
 
 
 class BuildOpts(C.Structure):

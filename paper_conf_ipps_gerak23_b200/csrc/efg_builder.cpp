@@ -190,6 +190,15 @@ efg_status build_host(uint64_t n, uint64_t m, const uint32_t *src, const uint32_
             start.swap(start2);
             deg.swap(deg2);
         }
+        // vertices with an in-edge (any row, before the partition trim): only
+        // these can ever be probed, so the others count as visited for the
+        // expand kernel's visited prefix (for symmetric graphs: degree > 0)
+        out.has_in.assign(n, 0);
+#pragma omp parallel for schedule(dynamic, 4096)
+        for (int64_t v = 0; v < (int64_t)n; ++v) {
+            const uint64_t *a = tmp.get() + start[v];
+            for (uint64_t t = 0; t < deg[v]; ++t) out.has_in[(uint32_t)(a[t] >> 32)] = 1;  // benign same-value race
+        }
         // partition: keep only the owned rows' lists
         const bool part = o.row_hi > o.row_lo;
         const uint64_t lo = part ? std::min<uint64_t>(o.row_lo, n) : 0, hi = part ? std::min<uint64_t>(o.row_hi, n) : n;

@@ -94,6 +94,7 @@ ExpandArgs expand_args(DeviceGraph &d, uint32_t *out)
     a.max_stats = kMaxLevelStats;
     a.hot_words = (uint32_t)std::min<uint64_t>(kHotWords, d.nwords) & ~3u;
     a.k = d.k;
+    a.pskip = d.prefix_skip ? 1u : 0u;
     return a;
 }
 
@@ -175,13 +176,20 @@ efg_status build_loop_graph(DeviceGraph &d, int mode)
 
 }  // namespace
 
-void device_free(DeviceGraph &d)
+void device_drop_graphs(DeviceGraph &d)
 {
     if (d.device >= 0) cudaSetDevice(d.device);
     for (int m = 0; m < 2; ++m) {
         if (d.loop_exec[m]) cudaGraphExecDestroy(d.loop_exec[m]);
         if (d.loop_graph[m]) cudaGraphDestroy(d.loop_graph[m]);
+        d.loop_exec[m] = nullptr;
+        d.loop_graph[m] = nullptr;
     }
+}
+
+void device_free(DeviceGraph &d)
+{
+    device_drop_graphs(d);
     cudaFree(d.data);
     cudaFree(d.rec);
     cudaFree(d.deg32);
@@ -266,9 +274,10 @@ efg_status device_upload(efg_graph *g, const efg_build_opts &o)
     CUDA_TRY(cudaMemcpyAsync(d.deg32, deg.data(), d.nwords * 32 * 4, cudaMemcpyHostToDevice, s));
     {
         std::vector<uint32_t> iso(d.nwords, 0);
+        // never probed: padding ids and vertices without an in-edge (directed
+        // sinks are probed although their out-degree is 0)
         for (uint64_t v = 0; v < d.nwords * 32; ++v)
-            // a row-range handle knows degrees of its own rows only (others may be probed)
-            if (v >= h.n || (v >= h.row_lo && v < h.row_hi && deg[v] == 0)) iso[v >> 5] |= 1u << (v & 31);
+            if (v >= h.n || !h.has_in[v]) iso[v >> 5] |= 1u << (v & 31);
         EFG_TRY(dev_alloc(d, &d.iso, d.nwords));
         CUDA_TRY(cudaMemcpyAsync(d.iso, iso.data(), d.nwords * 4, cudaMemcpyHostToDevice, s));
         CUDA_TRY(cudaStreamSynchronize(s));

@@ -28,6 +28,7 @@ struct HostEFG {
     std::vector<uint8_t> data;      // offsets[n] bytes (+ padding on device)
     std::vector<float> weights;     // m (CSR order) or empty
     std::vector<uint32_t> old_of_new, new_of_old;  // EFG_REORDER_DEGREE relabelling (else empty)
+    std::vector<uint8_t> has_in;    // n: vertex has an in-edge (stored ids; all rows)
     uint64_t fwd_bytes = 0, lower_bytes = 0, upper_bytes = 0, apriori_bits = 0;
     uint64_t row_lo = 0, row_hi = 0;
     double build_seconds = 0.0;
@@ -192,6 +193,7 @@ struct DeviceGraph {
     int num_sms = 148;
     LevelStat *stats_host = nullptr;   // pinned mirror of stats
     int level_loop = 0;                // 0 = CUDA graph (device loop), 1 = host loop + events
+    int prefix_skip = 1;               // EFG_OPT_PREFIX_SKIP
     cudaGraph_t loop_graph[2] = {nullptr, nullptr};      // per mode (visit, visit+parent)
     cudaGraphExec_t loop_exec[2] = {nullptr, nullptr};
     uint64_t own_lo_w = 0, own_hi_w = 0;   // bitmap words of the owned rows (frontier filter)
@@ -214,6 +216,7 @@ struct efg_graph {
 // device side (efg_device.cu)
 namespace efg {
 efg_status device_upload(efg_graph *g, const efg_build_opts &o);
+void device_drop_graphs(DeviceGraph &d);  // captured level loops (rebuilt on next use)
 void device_free(DeviceGraph &d);
 efg_status device_decode(efg_graph *g, uint32_t v0, uint32_t v1, uint32_t *out);
 efg_status device_bfs(efg_graph *g, uint32_t source, int32_t *depth, uint32_t *parent, efg_stats *st);

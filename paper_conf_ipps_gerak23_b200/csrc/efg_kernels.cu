@@ -846,6 +846,7 @@ __global__ void __launch_bounds__(kExpandThreads, 1) expand_kernel(ExpandArgs a)
     const uint32_t *st32 = &ws.stage[0][0];
     const uint32_t sbits = smem_u32(st32) * 8;  // shared-window bit address of the staging area
     const uint32_t vpre = kBfs ? a.ctrl->vmin2[xl & 1] : 0u;  // ids below it are visited (or never probed)
+    const bool pskip = kBfs && a.pskip && vpre != 0;              // warp-uniform
     const uint64_t gw = (uint64_t)blockIdx.x * kExpandWarps + wid;
     const uint64_t nwarps = (uint64_t)gridDim.x * kExpandWarps;
     const uint64_t CH = a.k ? a.k : (1ull << 40);
@@ -1003,8 +1004,12 @@ __global__ void __launch_bounds__(kExpandThreads, 1) expand_kernel(ExpandArgs a)
         uint32_t Er0 = 0;  // batch element index at the round start
         for (uint32_t ga = 0; ga < NW; ga += kRoundWords) {
             const uint32_t nw = min(kRoundWords, NW - ga);
-            // ---- round words: mask, popcount prefix, non-zero records ----
-            uint32_t run = Er0, nrec = 0;
+            // ---- round words: mask, popcount prefix, records ----
+            // BFS prefix skip: a word whose stop bits all have a high part
+            // below vpre >> l holds only ids below the visited prefix (lists
+            // are sorted): no record, so those elements are neither decoded
+            // nor probed (their bytes are staged all the same)
+            uint32_t run = Er0, krun = 0, nrec = 0;
 #pragma unroll
             for (uint32_t j = 0; j < kRoundWords / 32; ++j) {
                 if (j * 32 >= nw) break;
@@ -1019,51 +1024,65 @@ __global__ void __launch_bounds__(kExpandThreads, 1) expand_kernel(ExpandArgs a)
                     if (g == sp.wb) wd &= FULL << ((sp.lflags >> 8) & 31);
                     if (g == sp.wb + sp.nwd - 1) wd &= FULL >> (31 - ((sp.lflags >> 16) & 31));
                 }
+                const uint32_t pc = __popc(wd);
                 uint32_t tot;
-                const uint32_t ex = warp_excl_u32(__popc(wd), tot);
-                const uint32_t nzm = __ballot_sync(FULL, wd != 0);
-                if (wd) {
-                    const uint32_t k = nrec + __popc(nzm & ((1u << lane) - 1));
-                    ws.wrec[k] = make_uint4(__brev(wd), 32 * g + sp.HB, sp.lsmb, (sp.lflags & 63) | ((uint32_t)sl << 8));
-                    ws.wpre[k] = run + ex;
+                const uint32_t ex = warp_excl_u32(pc, tot);
+                const uint32_t l = sp.lflags & 63;
+                // stop bit at p, j-th of the record: high part hb + p - j = select1(i) - i
+                const uint32_t hb = 32 * g + sp.HB - (run + ex);
+                bool keep = wd != 0;
+                uint32_t kex = ex, ktot = tot;  // kept-element prefix (= all without the skip)
+                if (pskip) {
+                    keep = keep && hb + (31 - __clz(wd)) - (pc - 1) >= (vpre >> l);
+                    kex = warp_excl_u32(keep ? pc : 0u, ktot);
+                }
+                const uint32_t km = __ballot_sync(FULL, keep);
+                if (keep) {
+                    const uint32_t k = nrec + __popc(km & ((1u << lane) - 1));
+                    ws.wrec[k] = make_uint4(__brev(wd), hb, sp.lsmb + (run + ex) * l, l | ((uint32_t)sl << 8));
+                    ws.wpre[k] = krun + kex;
                 }
                 run += tot;
-                nrec += __popc(nzm);
+                krun += ktot;
+                nrec += __popc(km);
             }
             __syncwarp();
             const uint32_t Er1 = run;
-            const uint32_t NEr = Er1 - Er0;
-            uint32_t e = Er0 + (uint32_t)(((uint64_t)lane * NEr) >> 5);
-            const uint32_t e1 = Er0 + (uint32_t)(((uint64_t)(lane + 1) * NEr) >> 5);
-            if (e < e1) {
-                // ---- lane start: record of element e (maxle) + in-word select ----
+            const uint32_t NK = krun;  // kept elements of the round
+            uint32_t c = (uint32_t)(((uint64_t)lane * NK) >> 5);
+            const uint32_t c1 = (uint32_t)(((uint64_t)(lane + 1) * NK) >> 5);
+            if (c < c1) {
+                // ---- lane start: record of kept element c (maxle) + in-word select ----
                 uint32_t k = 0;
 #pragma unroll
                 for (uint32_t step = kSearchStep; step; step >>= 1)
-                    if (k + step < nrec && ws.wpre[k + step] <= e) k += step;
+                    if (k + step < nrec && ws.wpre[k + step] <= c) k += step;
                 // records hold bit-reversed words: the lowest remaining stop bit is the
                 // leading one (clz), so no bit reversal per element
                 uint4 r = ws.wrec[k];
-                const uint32_t kk = e - ws.wpre[k];
-                if (kk) r.x &= FULL >> select_in_word(__brev(r.x), kk);  // drop kk stop bits
+                uint32_t j = c - ws.wpre[k];  // rank of the lane's first element in its record
+                if (j) r.x &= FULL >> select_in_word(__brev(r.x), j);  // drop j stop bits
                 uint32_t l = r.w & 63, lmask = (1u << l) - 1;
+                uint32_t e = Er0 + c;  // batch element index (modes without the skip keep every record)
 
                 // one element: next stop bit -> select1(i) - i, lower field, value
                 auto decode = [&](uint32_t &x, uint32_t &slot_of) {
                     if (r.x == 0) {  // next record (always has a stop bit)
                         ++k;
                         r = ws.wrec[k];
+                        j = 0;
                         l = r.w & 63;
                         lmask = (1u << l) - 1;
                     }
                     const uint32_t p = clz_nz(r.x);
                     r.x ^= 0x80000000u >> p;
-                    const uint32_t hi = r.y + p - e;  // select1(i) - i
-                    const uint32_t la = r.z + e * l;
+                    const uint32_t hi = r.y + p - j;  // select1(i) - i
+                    const uint32_t la = r.z + j * l;
                     const uint32_t ad = (la >> 3) & ~3u;
                     const uint32_t lo = shf_r_wrap(lds_u32(ad), lds_u32(ad + 4), la) & lmask;
                     x = (hi << l) | lo;  // (select1(i) - i) << l | lower[i]
                     slot_of = r.w >> 8;
+                    ++j;
                     ++e;
                 };
 
@@ -1135,7 +1154,7 @@ __global__ void __launch_bounds__(kExpandThreads, 1) expand_kernel(ExpandArgs a)
                 };
 
                 // main loop: kU elements per step, no per-element guards
-                while (e + kU <= e1) {
+                for (; c + kU <= c1; c += kU) {
                     uint32_t xv[kU], sv[kU], ev[kU];
 #pragma unroll
                     for (int u = 0; u < kU; ++u) {
@@ -1145,9 +1164,9 @@ __global__ void __launch_bounds__(kExpandThreads, 1) expand_kernel(ExpandArgs a)
                     visit(xv, sv, ev, kU);
                 }
                 // tail: < kU elements
-                if (e < e1) {
+                if (c < c1) {
                     uint32_t xv[kU], sv[kU], ev[kU];
-                    const int cntu = (int)(e1 - e);
+                    const int cntu = (int)(c1 - c);
 #pragma unroll
                     for (int u = 0; u < kU; ++u) {
                         xv[u] = 0;

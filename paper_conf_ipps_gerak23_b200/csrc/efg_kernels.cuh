@@ -33,6 +33,7 @@ struct ExpandArgs {
     uint32_t max_stats;
     uint32_t hot_words;        // bitmap words with a shared-memory snapshot (multiple of 4)
     uint32_t k;                // forward-pointer quantum (chunk length); 0 = none
+    uint32_t pskip;            // BFS: skip upper words whose ids are all below the visited prefix
 };
 
 struct InitArgs {

@@ -149,6 +149,47 @@ def test_directed_graph(efg):
     g.free()
 
 
+def test_directed_sink_below_visited_prefix(efg):
+    """A directed sink (out-degree 0, but an in-edge) with a smaller id than
+    every unvisited non-sink vertex must still be probed: the visited prefix
+    counts only vertices without in-edges as never probed."""
+    flags = efg.EFG_DEDUP | efg.EFG_DROP_SELF_LOOPS
+    src = np.array([1, 1, 2], np.uint32)
+    dst = np.array([0, 2, 1], np.uint32)
+    g = efg.Graph.build(3, src, dst, flags=flags)
+    ov, oe = oracle.csr_build(3, src, dst, symmetrize=False)
+    _check_bfs(g, ov, oe, [1, 2])
+    g.free()
+    # many sinks at the low ids, sources among the high ids
+    rng = np.random.default_rng(7)
+    n = 4096
+    s = rng.integers(n // 2, n, 40000).astype(np.uint32)
+    d = rng.integers(0, n, 40000).astype(np.uint32)
+    g = efg.Graph.build(n, s, d, flags=flags)
+    ov, oe = oracle.csr_build(n, s, d, symmetrize=False)
+    _check_bfs(g, ov, oe, [n // 2, n - 1, 3000])
+    g.free()
+
+
+@pytest.mark.parametrize("reorder", [False, True])
+def test_prefix_skip_on_off_identical(efg, reorder):
+    """EFG_OPT_PREFIX_SKIP only drops work on ids below the visited prefix:
+    depths with and without it equal the oracle's."""
+    n, src, dst = synth.rmat(14, 16, seed=11)
+    flags = efg.EFG_DEFAULT_FLAGS | (efg.EFG_REORDER_DEGREE if reorder else 0)
+    g = efg.Graph.build(n, src, dst, flags=flags)
+    ov, oe = oracle.csr_build(n, src, dst)
+    deg = np.diff(ov)
+    srcs = synth.sources(n, 6, 77, deg > 0)
+    for on in (False, True, False):
+        g.set_prefix_skip(on)
+        _check_bfs(g, ov, oe, srcs)
+        g.set_level_loop(True)
+        _check_bfs(g, ov, oe, srcs[:2])
+        g.set_level_loop(False)
+    g.free()
+
+
 def test_random_graphs_many_shapes(efg):
     rng = np.random.default_rng(21)
     for t in range(25):
