@@ -216,6 +216,7 @@ efg_status build_host(uint64_t n, uint64_t m, const uint32_t *src, const uint32_
         // ---- pass 1: a-priori sizes -> offsets ----
         if (weighted) out.weights.resize(out.m);
         out.nlb.assign(n, 0);
+        out.umax.assign(n, 0);
         out.offsets.assign(n + 1, 0);
         uint64_t fb = 0, lb = 0, ub = 0, ab = 0;
 #pragma omp parallel for schedule(dynamic, 1024) reduction(+ : fb, lb, ub, ab)
@@ -226,6 +227,7 @@ efg_status build_host(uint64_t n, uint64_t m, const uint32_t *src, const uint32_
             const uint32_t u = (uint32_t)(a[d - 1] >> 32);
             const ListGeom g = list_geom(d, u, k);
             out.nlb[v] = (uint8_t)g.l;
+            out.umax[v] = u;
             out.offsets[v] = g.fwd + g.lower + g.upper;
             fb += g.fwd;
             lb += g.lower;

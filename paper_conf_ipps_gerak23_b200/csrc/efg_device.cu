@@ -107,12 +107,14 @@ FrontierArgs frontier_args(DeviceGraph &d, cudaGraphConditionalHandle cond, bool
     a.iso = d.iso;
     a.old_of_new = d.old_of_new;
     a.deg32 = d.deg32;
+    a.umax = d.umax;
+    a.lskip = (d.prefix_skip && !consume) ? 1u : 0u;
     a.rec = d.rec;
     a.chunks = d.chunks;
     a.tiles = d.tiles;
     a.ctrl = d.ctrl;
     a.status = d.status;
-    a.barrier = reinterpret_cast<unsigned long long *>(d.status + 3 * kMaxGrid);
+    a.barrier = reinterpret_cast<unsigned long long *>(d.status + 4 * kMaxGrid);
     a.big = d.big;
     a.trace = d.trace;
     a.stats = d.stats;
@@ -192,6 +194,7 @@ void device_free(DeviceGraph &d)
     cudaFree(d.data);
     cudaFree(d.rec);
     cudaFree(d.deg32);
+    cudaFree(d.umax);
     cudaFree(d.iso);
     cudaFree(d.vlist);
     cudaFree(d.weights);
@@ -270,6 +273,9 @@ efg_status device_upload(efg_graph *g, const efg_build_opts &o)
     CUDA_TRY(cudaMemcpyAsync(d.rec, rec.data(), h.n * sizeof(VRec), cudaMemcpyHostToDevice, s));
     EFG_TRY(dev_alloc(d, &d.deg32, d.nwords * 32));
     CUDA_TRY(cudaMemcpyAsync(d.deg32, deg.data(), d.nwords * 32 * 4, cudaMemcpyHostToDevice, s));
+    EFG_TRY(dev_alloc(d, &d.umax, d.nwords * 32));
+    CUDA_TRY(cudaMemsetAsync(d.umax, 0, d.nwords * 32 * 4, s));
+    CUDA_TRY(cudaMemcpyAsync(d.umax, h.umax.data(), h.n * 4, cudaMemcpyHostToDevice, s));
     {
         std::vector<uint32_t> iso(d.nwords, 0);
         // never probed: padding ids and vertices without an in-edge (directed
@@ -303,8 +309,8 @@ efg_status device_upload(efg_graph *g, const efg_build_opts &o)
     EFG_TRY(dev_alloc(d, &d.tiles, d.max_tiles + 1));
     EFG_TRY(dev_alloc(d, &d.chunks, d.max_chunks));
     EFG_TRY(dev_alloc(d, &d.depth, h.n));
-    EFG_TRY(dev_alloc(d, &d.status, 3 * kMaxGrid + 1));  // + the grid-barrier counter
-    CUDA_TRY(cudaMemsetAsync(d.status, 0, (3 * kMaxGrid + 1) * 8, s));
+    EFG_TRY(dev_alloc(d, &d.status, 4 * kMaxGrid + 1));  // + the grid-barrier counter
+    CUDA_TRY(cudaMemsetAsync(d.status, 0, (4 * kMaxGrid + 1) * 8, s));
     if (std::getenv("EFG_FRONTIER_TRACE")) EFG_TRY(dev_alloc(d, &d.trace, 8 * kMaxGrid));
     // lists planned grid-wide: more than one chunk (deg > k) or more than one
     // tile of work (deg > kTileWork - kChunkWork)

@@ -29,6 +29,7 @@ struct HostEFG {
     std::vector<float> weights;     // m (CSR order) or empty
     std::vector<uint32_t> old_of_new, new_of_old;  // EFG_REORDER_DEGREE relabelling (else empty)
     std::vector<uint8_t> has_in;    // n: vertex has an in-edge (stored ids; all rows)
+    std::vector<uint32_t> umax;     // n: largest neighbour (list's last element, P:218 u), 0 if empty
     uint64_t fwd_bytes = 0, lower_bytes = 0, upper_bytes = 0, apriori_bits = 0;
     uint64_t row_lo = 0, row_hi = 0;
     double build_seconds = 0.0;
@@ -95,6 +96,7 @@ struct LevelCtrl {
     uint32_t vmin2[2];  // frontier_kernel of level L: smallest vertex neither visited nor isolated, in
                         // slot L & 1 (atomicMin); the expand of level L reads it as its visited prefix
     uint32_t nbig2[2];  // frontier_kernel of level L: BigList entries appended (slot L & 1)
+    uint32_t vpre_used; // visited prefix the last BFS expand used (0: none); lower bound for the next level end
 };
 
 // A frontier list whose chunk descriptors and tile boundaries are written by
@@ -161,6 +163,7 @@ struct DeviceGraph {
     uint64_t data_bytes = 0;
     VRec *rec = nullptr;               // n records
     uint32_t *deg32 = nullptr;         // n degrees (padded to the bitmap size)
+    uint32_t *umax = nullptr;          // n largest neighbour per list (padded to the bitmap size)
     uint32_t *iso = nullptr;           // bitmap of the degree-0 vertices and the padding (nwords)
     uint64_t *vlist = nullptr;         // n+1 (SSSP weight indexing / decode)
     float *weights = nullptr;          // m or null
@@ -177,7 +180,7 @@ struct DeviceGraph {
     uint32_t *old_of_new = nullptr;    // EFG_REORDER_DEGREE relabelling (n) or null
     uint32_t *new_of_old = nullptr;    // its inverse (n) or null
     int32_t *step_depth = nullptr;     // stepwise traversal: caller's depth buffer
-    uint64_t *status = nullptr;        // frontier_kernel: 3 x [kMaxGrid] per-block aggregates + barrier counter
+    uint64_t *status = nullptr;        // frontier_kernel: 4 x [kMaxGrid] per-block aggregates + barrier counter
     BigList *big = nullptr;
     unsigned long long *trace = nullptr;  // debug: frontier_kernel phase timestamps            // frontier_kernel: multi-chunk / multi-tile lists of a level
     uint64_t max_big = 0;

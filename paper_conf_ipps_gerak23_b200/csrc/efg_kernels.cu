@@ -142,6 +142,7 @@ __global__ void init_kernel(InitArgs a)
         a.ctrl->vmin2[1] = FULL;
         a.ctrl->nbig2[0] = 0;
         a.ctrl->nbig2[1] = 0;
+        a.ctrl->vpre_used = 0;
         if (a.parent) a.parent[a.v0] = (uint32_t)a.v0;
     }
     const uint64_t w0 = a.v0 >> 5, w1 = (a.v1 + 31) >> 5;
@@ -290,8 +291,8 @@ __device__ __forceinline__ void warp_excl_u32_n(uint32_t (&x)[N], uint32_t (&tot
 __global__ void __launch_bounds__(kFrontierThreads, 2) frontier_kernel(FrontierArgs a)
 {
     constexpr int NT = kFrontierThreads, NW = NT / 32;
-    __shared__ uint64_t s_q[NW], s_wk[NW], s_ch[NW], s_all[NW];
-    __shared__ uint64_t s_pre[3], s_tot[3];
+    __shared__ uint64_t s_q[NW], s_wk[NW], s_ch[NW], s_sk[NW], s_all[NW];
+    __shared__ uint64_t s_pre[4], s_tot[4];
 
     const uint32_t tid = threadIdx.x, lane = tid & 31, wid = tid >> 5, b = blockIdx.x;
 #define FTRACE(p)                                                      \
@@ -318,8 +319,13 @@ __global__ void __launch_bounds__(kFrontierThreads, 2) frontier_kernel(FrontierA
     constexpr int kB = 8;  // pass 1: non-empty words whose degree loads are in flight together
 
     // ---- 1: count, work and chunks of the warp's new (owned) vertices ----
+    // BFS list skip: a list whose largest neighbour is below the visited
+    // prefix the last expand used (a lower bound of the next one) cannot
+    // discover anything: it is neither planned nor expanded (its degree still
+    // counts in the level's edges, reading C18)
+    const uint32_t vlow = a.lskip ? ctrl->vpre_used : 0u;
     uint32_t cq = 0, all = 0, ch = 0;  // lane partials
-    uint64_t wk = 0;
+    uint64_t wk = 0, sk = 0;
     uint32_t vmin = FULL;  // smallest vertex of this warp's range that is neither visited nor isolated
     for (uint64_t w0 = 32ull * gw; w0 < a.nwords; w0 += WG) {
         const uint64_t w = w0 + lane;
@@ -339,20 +345,28 @@ __global__ void __launch_bounds__(kFrontierThreads, 2) frontier_kernel(FrontierA
         // word (one coalesced 128-byte load per word)
         uint32_t todo = __ballot_sync(FULL, nq != 0);
         while (todo) {
-            uint32_t dv[kB];
+            uint32_t dv[kB], uv[kB];
 #pragma unroll
             for (int u = 0; u < kB; ++u) {
                 dv[u] = 0;
+                uv[u] = 0;
                 if (todo) {
                     const int j = __ffs(todo) - 1;
                     todo &= todo - 1;
                     const uint32_t bits = __shfl_sync(FULL, nq, j);
-                    if ((bits >> lane) & 1) dv[u] = __ldg(a.deg32 + (w0 + j) * 32 + lane);
+                    if ((bits >> lane) & 1) {
+                        dv[u] = __ldg(a.deg32 + (w0 + j) * 32 + lane);
+                        if (vlow) uv[u] = __ldg(a.umax + (w0 + j) * 32 + lane);
+                    }
                 }
             }
 #pragma unroll
             for (int u = 0; u < kB; ++u) {
                 const uint32_t d = dv[u];
+                if (uv[u] < vlow) {  // skipped list (vlow = 0: never)
+                    sk += d;
+                    continue;
+                }
                 const uint32_t nch = d ? (uint32_t)cl.div((uint64_t)d + CH - 1) : 0u;
                 wk += (uint64_t)nch * CW + d;
                 ch += nch;
@@ -361,6 +375,7 @@ __global__ void __launch_bounds__(kFrontierThreads, 2) frontier_kernel(FrontierA
     }
     const uint64_t cqw = warp_sum_u64(cq), allw = warp_sum_u64(all), chw = warp_sum_u64(ch);
     wk = warp_sum_u64(wk);
+    sk = warp_sum_u64(sk);
 #pragma unroll
     for (int d = 16; d; d >>= 1) vmin = min(vmin, __shfl_xor_sync(FULL, vmin, d));
     if (lane == 0) {
@@ -368,22 +383,24 @@ __global__ void __launch_bounds__(kFrontierThreads, 2) frontier_kernel(FrontierA
         s_all[wid] = allw;
         s_wk[wid] = wk;
         s_ch[wid] = chw;
+        s_sk[wid] = sk;
         if (vmin != FULL) atomicMin(&ctrl->vmin2[level & 1], vmin);
     }
     __syncthreads();
     FTRACE(1);
-    // publish the block's aggregates (queue entries, work units, chunks),
-    // barrier, then every block sums its predecessors' (region r by warp r)
-    if (wid < 3) {
-        const uint64_t *src = wid == 0 ? s_q : (wid == 1 ? s_wk : s_ch);
+    // publish the block's aggregates (frontier vertices, work units, chunks,
+    // skipped-list edges), barrier, then every block sums its predecessors'
+    // (region r by warp r)
+    if (wid < 4) {
+        const uint64_t *src = wid == 0 ? s_q : (wid == 1 ? s_wk : (wid == 2 ? s_ch : s_sk));
         const uint64_t agg = warp_sum_u64(lane < NW ? src[lane] : 0);
         if (lane == 0) st_relaxed_u64(a.status + wid * kMaxGrid + b, agg);
-    } else if (wid == 3) {
+    } else if (wid == 4) {
         const uint64_t blk_all = warp_sum_u64(lane < NW ? s_all[lane] : 0);
         if (lane == 0 && blk_all) atomicAdd(reinterpret_cast<unsigned long long *>(&ctrl->nnew), blk_all);
     }
     grid_barrier(a.barrier);
-    if (wid < 3) {
+    if (wid < 4) {
         uint64_t pre, tot;
         sum_published(a.status + wid * kMaxGrid, b, pre, tot);
         if (lane == 0) {
@@ -395,7 +412,7 @@ __global__ void __launch_bounds__(kFrontierThreads, 2) frontier_kernel(FrontierA
     const uint64_t nf = s_tot[0];
     if (b == gridDim.x - 1 && tid == 0) {  // level totals
         const uint64_t nwork = s_tot[1], nchunks = s_tot[2];
-        const uint64_t ne = nwork - CW * nchunks;
+        const uint64_t ne = nwork - CW * nchunks + s_tot[3];  // every frontier list's edges
         const uint64_t ntiles = (nwork + kTileWork - 1) / kTileWork;
         ctrl->nf = nf;
         ctrl->nwork = nwork;
@@ -463,7 +480,10 @@ __global__ void __launch_bounds__(kFrontierThreads, 2) frontier_kernel(FrontierA
                     bq[u] = __shfl_sync(FULL, nq, j);
                     const uint32_t bb = __shfl_sync(FULL, nb, j);
                     const uint32_t v = (uint32_t)((w0 + j) * 32 + lane);
-                    if ((bq[u] >> lane) & 1) rv[u] = __ldg(reinterpret_cast<const uint4 *>(a.rec + v));
+                    if ((bq[u] >> lane) & 1) {
+                        rv[u] = __ldg(reinterpret_cast<const uint4 *>(a.rec + v));
+                        if (vlow && __ldg(a.umax + v) < vlow) rv[u] = make_uint4(0, 0, 0, 0);  // skipped list
+                    }
                     // depth in input ids (relabelled graphs: one scattered store per vertex
                     // into the L2-resident depth array, instead of a gather pass at the end)
                     if (((bb >> lane) & 1) && depth) depth[a.old_of_new ? __ldg(a.old_of_new + v) : v] = (int32_t)level;
@@ -807,6 +827,7 @@ __global__ void __launch_bounds__(kExpandThreads, 1) expand_kernel(ExpandArgs a)
     const uint32_t sbits = smem_u32(st32) * 8;  // shared-window bit address of the staging area
     const uint32_t vpre = kBfs ? a.ctrl->vmin2[xl & 1] : 0u;  // ids below it are visited (or never probed)
     const bool pskip = kBfs && a.pskip && vpre != 0;              // warp-uniform
+    if (blockIdx.x == 0 && threadIdx.x == 0) a.ctrl->vpre_used = pskip ? vpre : 0u;
     const uint64_t gw = (uint64_t)blockIdx.x * kExpandWarps + wid;
     const uint64_t nwarps = (uint64_t)gridDim.x * kExpandWarps;
     const uint64_t CH = a.k ? a.k : (1ull << 40);

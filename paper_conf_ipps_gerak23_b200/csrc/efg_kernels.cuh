@@ -61,11 +61,13 @@ struct FrontierArgs {           // level end (a7) + next level plan (a1-a4), one
     const uint32_t *old_of_new;  // relabelled graphs: input id of each stored id (depth is written in input ids), else null
     int consume;               // 1: frontier = vis itself, vis reset (SSSP relaxed set)
     const uint32_t *deg32;     // degrees (pass 1)
+    const uint32_t *umax;      // largest neighbour of each list
+    uint32_t lskip;            // BFS: lists whose largest neighbour is below ctrl->vpre_used are not planned
     const VRec *rec;           // vertex records (pass 2)
     ChunkDesc *chunks;         // out: chunk descriptors
     uint32_t *tiles;           // out: first chunk of each tile (+ sentinel)
     LevelCtrl *ctrl;           // in: level, seq, depth ptr; out: nf, ne, nwork, nchunks, ntiles, xlevel, vmin2
-    uint64_t *status;          // three per-block aggregate regions of kMaxGrid words
+    uint64_t *status;          // four per-block aggregate regions of kMaxGrid words
     unsigned long long *barrier;  // grid-barrier arrival counter (grows by gridDim.x per barrier)
     BigList *big;              // scratch: lists planned by the whole grid
     unsigned long long *trace; // debug (EFG_FRONTIER_TRACE): per block, 8 phase timestamps, or null
