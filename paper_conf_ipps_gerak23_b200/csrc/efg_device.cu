@@ -105,7 +105,8 @@ FrontierArgs frontier_args(DeviceGraph &d, cudaGraphConditionalHandle cond, bool
     a.vis = d.vis;
     a.prev = d.prev;
     a.iso = d.iso;
-    a.old_of_new = d.old_of_new;
+    a.depth_stored = (d.old_of_new && !consume) ? d.depth_st : nullptr;
+    a.depth_stored_only = d.old_of_new ? 1 : 0;
     a.deg32 = d.deg32;
     a.umax = d.umax;
     a.lskip = (d.prefix_skip && !consume) ? 1u : 0u;
@@ -207,6 +208,7 @@ void device_free(DeviceGraph &d)
     cudaFree(d.parent2);
     cudaFree(d.old_of_new);
     cudaFree(d.new_of_old);
+    cudaFree(d.depth_st);
     cudaFree(d.status);
     cudaFree(d.big);
     cudaFree(d.trace);
@@ -293,6 +295,7 @@ efg_status device_upload(efg_graph *g, const efg_build_opts &o)
         CUDA_TRY(cudaMemcpyAsync(d.old_of_new, h.old_of_new.data(), h.n * 4, cudaMemcpyHostToDevice, s));
         EFG_TRY(dev_alloc(d, &d.new_of_old, h.n));
         CUDA_TRY(cudaMemcpyAsync(d.new_of_old, h.new_of_old.data(), h.n * 4, cudaMemcpyHostToDevice, s));
+        EFG_TRY(dev_alloc(d, &d.depth_st, h.n));
     }
     if (!h.weights.empty()) {
         EFG_TRY(dev_alloc(d, &d.weights, h.m));
@@ -419,7 +422,10 @@ efg_status device_bfs(efg_graph *g, uint32_t source, int32_t *depth, uint32_t *p
     uint32_t launches = 0;
 
     CUDA_TRY(cudaEventRecord(ev0, s));
-    CUDA_TRY(cudaMemsetAsync(dd, 0xFF, d.n * 4, s));  // unreached: -1 (frontier_kernel writes input ids)
+    if (relabel)
+        CUDA_TRY(cudaMemsetAsync(d.depth_st, 0xFF, d.n * 4, s));  // gathered into dd at the end
+    else
+        CUDA_TRY(cudaMemsetAsync(dd, 0xFF, d.n * 4, s));
     if (pd) CUDA_TRY(cudaMemsetAsync(pd, 0xFF, d.n * 4, s));
     EFG_TRY(start_traversal(d, source, (uint64_t)source + 1, dd, pd, launches));
 
@@ -428,6 +434,7 @@ efg_status device_bfs(efg_graph *g, uint32_t source, int32_t *depth, uint32_t *p
     uint32_t levels = 0;
     if (graph_mode) {
         CUDA_TRY(cudaGraphLaunch(d.loop_exec[mode], s));
+        if (relabel) CUDA_TRY(launch_map_depth(d.depth_st, d.new_of_old, dd, d.n, s));
         CUDA_TRY(cudaEventRecord(ev1, s));
         CUDA_TRY(cudaMemcpyAsync(d.ctrl_host, d.ctrl, sizeof(LevelCtrl), cudaMemcpyDeviceToHost, s));
         CUDA_TRY(cudaStreamSynchronize(s));
@@ -443,7 +450,7 @@ efg_status device_bfs(efg_graph *g, uint32_t source, int32_t *depth, uint32_t *p
             const LevelStat &x = d.stats_host[i];
             lms.push_back(x.t1 > x.t0 ? (float)((double)(x.t1 - x.t0) * 1e-6) : 0.f);
         }
-        launches += 2 * levels;
+        launches += 2 * levels + (relabel ? 1 : 0);
     } else {
         const int blocks = d.num_sms * expand_occupancy(mode);
         for (;;) {
@@ -482,6 +489,10 @@ efg_status device_bfs(efg_graph *g, uint32_t source, int32_t *depth, uint32_t *p
                 fprintf(stderr, "\n");
             }
             ++levels;
+        }
+        if (relabel) {
+            CUDA_TRY(launch_map_depth(d.depth_st, d.new_of_old, dd, d.n, s));
+            ++launches;
         }
         CUDA_TRY(cudaEventRecord(ev1, s));
     }
@@ -547,7 +558,10 @@ efg_status device_step_begin(efg_graph *g, uint32_t source, int32_t *depth)
     d.step_lf.clear();
     d.step_le.clear();
     d.step_depth = depth;
-    CUDA_TRY(cudaMemsetAsync(depth, 0xFF, d.n * 4, s));
+    if (d.old_of_new)
+        CUDA_TRY(cudaMemsetAsync(d.depth_st, 0xFF, d.n * 4, s));
+    else
+        CUDA_TRY(cudaMemsetAsync(depth, 0xFF, d.n * 4, s));
     uint32_t launches = 0;
     EFG_TRY(start_traversal(d, source, (uint64_t)source + 1, depth, nullptr, launches));
     CUDA_TRY(cudaMemcpyAsync(d.ctrl_host, d.ctrl, sizeof(LevelCtrl), cudaMemcpyDeviceToHost, s));
@@ -576,6 +590,10 @@ efg_status device_step_finish(efg_graph *g, uint64_t *global_new)
     CUDA_TRY(cudaMemcpyAsync(d.ctrl_host, d.ctrl, sizeof(LevelCtrl), cudaMemcpyDeviceToHost, s));
     CUDA_TRY(cudaStreamSynchronize(s));
     const LevelCtrl c = *d.ctrl_host;
+    if (c.nnew == 0 && d.old_of_new) {  // traversal over: depth back to input ids
+        CUDA_TRY(launch_map_depth(d.depth_st, d.new_of_old, d.step_depth, d.n, s));
+        CUDA_TRY(cudaStreamSynchronize(s));
+    }
     if (c.nnew) {
         d.step_lf.push_back(c.nf);
         d.step_le.push_back(c.ne);

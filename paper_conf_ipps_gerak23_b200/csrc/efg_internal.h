@@ -179,6 +179,7 @@ struct DeviceGraph {
     uint32_t *parent2 = nullptr;       // parent in input ids (reordered graphs), lazily
     uint32_t *old_of_new = nullptr;    // EFG_REORDER_DEGREE relabelling (n) or null
     uint32_t *new_of_old = nullptr;    // its inverse (n) or null
+    int32_t *depth_st = nullptr;       // depth by stored id (relabelled graphs)
     int32_t *step_depth = nullptr;     // stepwise traversal: caller's depth buffer
     uint64_t *status = nullptr;        // frontier_kernel: 4 x [kMaxGrid] per-block aggregates + barrier counter
     BigList *big = nullptr;

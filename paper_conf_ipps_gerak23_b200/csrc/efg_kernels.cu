@@ -54,6 +54,18 @@ __device__ __forceinline__ uint32_t warp_excl_u32(uint32_t x, uint32_t &total)
     return inc - x;
 }
 
+__device__ __forceinline__ uint64_t warp_excl_u64(uint64_t x, uint64_t &total)
+{
+    uint64_t inc = x;
+#pragma unroll
+    for (int d = 1; d < 32; d <<= 1) {
+        const uint64_t y = __shfl_up_sync(FULL, inc, d);
+        if ((int)lane_id() >= d) inc += y;
+    }
+    total = __shfl_sync(FULL, inc, 31);
+    return inc - x;
+}
+
 __device__ __forceinline__ uint64_t warp_sum_u64(uint64_t x)
 {
 #pragma unroll
@@ -108,6 +120,13 @@ __device__ __forceinline__ ChunkLen make_chunk(uint32_t k, int kshift)
 }
 
 // relaxed gpu-scope accesses (cross-block words of the persistent frontier grid)
+__device__ __forceinline__ uint64_t ld_relaxed_u64(const uint64_t *p)
+{
+    uint64_t v;
+    asm volatile("ld.relaxed.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+    return v;
+}
+
 __device__ __forceinline__ uint32_t ld_relaxed_u32(const uint32_t *p)
 {
     uint32_t v;
@@ -120,6 +139,26 @@ __device__ __forceinline__ void st_relaxed_u64(uint64_t *p, uint64_t v)
     asm volatile("st.relaxed.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
 }
 
+// block-wide exclusive scan of a u64 (256 threads); returns the block total in `total`
+template <int NT>
+__device__ __forceinline__ uint64_t block_excl_u64(uint64_t x, uint64_t &total, uint64_t *s_warp)
+{
+    const uint32_t lane = lane_id(), wid = threadIdx.x >> 5;
+    uint64_t wt;
+    const uint64_t ex = warp_excl_u64(x, wt);
+    if (lane == 31) s_warp[wid] = wt;
+    __syncthreads();
+    uint64_t pre = 0, tot = 0;
+#pragma unroll
+    for (int w = 0; w < NT / 32; ++w) {
+        const uint64_t v = s_warp[w];
+        if (w < (int)wid) pre += v;
+        tot += v;
+    }
+    __syncthreads();
+    total = tot;
+    return pre + ex;
+}
 
 
 // --------------------------------------------------------------------------
@@ -484,9 +523,10 @@ __global__ void __launch_bounds__(kFrontierThreads, 2) frontier_kernel(FrontierA
                         rv[u] = __ldg(reinterpret_cast<const uint4 *>(a.rec + v));
                         if (vlow && __ldg(a.umax + v) < vlow) rv[u] = make_uint4(0, 0, 0, 0);  // skipped list
                     }
-                    // depth in input ids (relabelled graphs: one scattered store per vertex
-                    // into the L2-resident depth array, instead of a gather pass at the end)
-                    if (((bb >> lane) & 1) && depth) depth[a.old_of_new ? __ldg(a.old_of_new + v) : v] = (int32_t)level;
+                    if ((bb >> lane) & 1) {
+                        if (a.depth_stored) a.depth_stored[v] = (int32_t)level;  // stored-id order (coalesced)
+                        if (!a.depth_stored_only && depth) depth[v] = (int32_t)level;
+                    }
                 }
             }
             // per-list work nch*CW + d < 2^31.1 (deg < 2^26); the 32-lane sums fit
@@ -1215,6 +1255,12 @@ __global__ void gather64_kernel(const double *stored, const uint32_t *new_of_old
 
 // depth_out[old_of_new[i]] = depth_stored[i] as a gather over input ids:
 // depth_out[v] = depth_stored[new_of_old[v]] (coalesced stores).
+__global__ void map_depth_kernel(const int32_t *stored, const uint32_t *new_of_old, int32_t *out, uint64_t n)
+{
+    for (uint64_t v = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; v < n; v += (uint64_t)gridDim.x * blockDim.x)
+        out[v] = stored[new_of_old[v]];
+}
+
 __global__ void map_parent_kernel(const uint32_t *pin, const uint32_t *old_of_new, uint32_t *pout, uint64_t n)
 {
     for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x) {
@@ -1263,6 +1309,14 @@ cudaError_t launch_gather64(const double *stored, const uint32_t *new_of_old, do
                             cudaStream_t s)
 {
     gather64_kernel<<<grid_for(n), 256, 0, s>>>(stored, new_of_old, out, n);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_map_depth(const int32_t *stored, const uint32_t *new_of_old, int32_t *out, uint64_t n,
+                             cudaStream_t s)
+{
+    const unsigned blocks = (unsigned)std::max<uint64_t>(1, std::min<uint64_t>((n + 255) / 256, 148 * 16));
+    map_depth_kernel<<<blocks, 256, 0, s>>>(stored, new_of_old, out, n);
     return cudaGetLastError();
 }
 

@@ -58,7 +58,8 @@ struct XchgArgs {
 struct FrontierArgs {           // level end (a7) + next level plan (a1-a4), one launch
     uint32_t *vis, *prev;      // visited bitmap now / at the previous level end
     const uint32_t *iso;       // degree-0 vertices (never probed): count as visited for the visited prefix
-    const uint32_t *old_of_new;  // relabelled graphs: input id of each stored id (depth is written in input ids), else null
+    int32_t *depth_stored;     // depth by stored id (relabelled graphs)
+    int depth_stored_only;     // 1: depth_stored is the only depth output (relabelled graphs)
     int consume;               // 1: frontier = vis itself, vis reset (SSSP relaxed set)
     const uint32_t *deg32;     // degrees (pass 1)
     const uint32_t *umax;      // largest neighbour of each list
@@ -97,6 +98,8 @@ cudaError_t launch_gather32(const uint32_t *stored, const uint32_t *new_of_old, 
                             cudaStream_t s);
 cudaError_t launch_gather64(const double *stored, const uint32_t *new_of_old, double *out, uint64_t n,
                             cudaStream_t s);
+cudaError_t launch_map_depth(const int32_t *stored, const uint32_t *new_of_old, int32_t *out, uint64_t n,
+                             cudaStream_t s);
 cudaError_t launch_map_parent(const uint32_t *pin, const uint32_t *old_of_new, uint32_t *pout, uint64_t n,
                               cudaStream_t s);
 
