@@ -109,7 +109,12 @@ FrontierArgs frontier_args(DeviceGraph &d, cudaGraphConditionalHandle cond, bool
     a.depth_stored_only = d.old_of_new ? 1 : 0;
     a.deg32 = d.deg32;
     a.umax = d.umax;
+    a.skipw = d.skipw;
+#ifdef EFG_NO_LSKIP
+    a.lskip = 0;  // tuning experiment: record-level skip only
+#else
     a.lskip = (d.prefix_skip && !consume) ? 1u : 0u;
+#endif
     a.rec = d.rec;
     a.chunks = d.chunks;
     a.tiles = d.tiles;
@@ -196,6 +201,7 @@ void device_free(DeviceGraph &d)
     cudaFree(d.rec);
     cudaFree(d.deg32);
     cudaFree(d.umax);
+    cudaFree(d.skipw);
     cudaFree(d.iso);
     cudaFree(d.vlist);
     cudaFree(d.weights);
@@ -276,6 +282,7 @@ efg_status device_upload(efg_graph *g, const efg_build_opts &o)
     EFG_TRY(dev_alloc(d, &d.deg32, d.nwords * 32));
     CUDA_TRY(cudaMemcpyAsync(d.deg32, deg.data(), d.nwords * 32 * 4, cudaMemcpyHostToDevice, s));
     EFG_TRY(dev_alloc(d, &d.umax, d.nwords * 32));
+    EFG_TRY(dev_alloc(d, &d.skipw, d.nwords));
     CUDA_TRY(cudaMemsetAsync(d.umax, 0, d.nwords * 32 * 4, s));
     CUDA_TRY(cudaMemcpyAsync(d.umax, h.umax.data(), h.n * 4, cudaMemcpyHostToDevice, s));
     {

@@ -164,6 +164,7 @@ struct DeviceGraph {
     VRec *rec = nullptr;               // n records
     uint32_t *deg32 = nullptr;         // n degrees (padded to the bitmap size)
     uint32_t *umax = nullptr;          // n largest neighbour per list (padded to the bitmap size)
+    uint32_t *skipw = nullptr;         // frontier_kernel scratch: skipped lists per bitmap word
     uint32_t *iso = nullptr;           // bitmap of the degree-0 vertices and the padding (nwords)
     uint64_t *vlist = nullptr;         // n+1 (SSSP weight indexing / decode)
     float *weights = nullptr;          // m or null

@@ -384,14 +384,16 @@ __global__ void __launch_bounds__(kFrontierThreads, 2) frontier_kernel(FrontierA
         // word (one coalesced 128-byte load per word)
         uint32_t todo = __ballot_sync(FULL, nq != 0);
         while (todo) {
-            uint32_t dv[kB], uv[kB];
+            uint32_t dv[kB], uv[kB], jv[kB];
 #pragma unroll
             for (int u = 0; u < kB; ++u) {
                 dv[u] = 0;
-                uv[u] = 0;
+                uv[u] = FULL;
+                jv[u] = 32;
                 if (todo) {
                     const int j = __ffs(todo) - 1;
                     todo &= todo - 1;
+                    jv[u] = j;
                     const uint32_t bits = __shfl_sync(FULL, nq, j);
                     if ((bits >> lane) & 1) {
                         dv[u] = __ldg(a.deg32 + (w0 + j) * 32 + lane);
@@ -402,6 +404,10 @@ __global__ void __launch_bounds__(kFrontierThreads, 2) frontier_kernel(FrontierA
 #pragma unroll
             for (int u = 0; u < kB; ++u) {
                 const uint32_t d = dv[u];
+                if (vlow) {  // skipped lists of this word -> skipw (phase 2 drops them)
+                    const uint32_t sm = __ballot_sync(FULL, uv[u] < vlow);
+                    if (lane == 0 && jv[u] < 32) a.skipw[w0 + jv[u]] = sm;
+                }
                 if (uv[u] < vlow) {  // skipped list (vlow = 0: never)
                     sk += d;
                     continue;
@@ -489,8 +495,11 @@ __global__ void __launch_bounds__(kFrontierThreads, 2) frontier_kernel(FrontierA
     constexpr int kS = 2;                         // non-empty words planned together
     for (uint64_t w0 = 32ull * gw; w0 < a.nwords; w0 += WG) {
         const uint64_t w = w0 + lane;
-        uint32_t nb = 0;
+        uint32_t nb = 0, skw = 0;
         if (w < a.nwords) {
+            // lists skipped in phase 1 are not planned (a word's mask is valid
+            // wherever phase 1 saw owned new bits, i.e. wherever it is used)
+            if (vlow) skw = a.skipw[w];
             const uint32_t x = a.vis[w];
             if (a.consume) {  // SSSP: the relaxed set itself is the next frontier; reset it
                 nb = x;
@@ -502,7 +511,7 @@ __global__ void __launch_bounds__(kFrontierThreads, 2) frontier_kernel(FrontierA
             }
         }
         const bool own = w >= a.own_lo_w && w < a.own_hi_w;
-        const uint32_t nq = own ? nb : 0u;
+        const uint32_t nq = own ? nb & ~skw : 0u;
         uint32_t todo = __ballot_sync(FULL, nb != 0);
         while (todo) {
             uint32_t jw[kS], bq[kS], wl[kS], nc[kS];
@@ -519,10 +528,7 @@ __global__ void __launch_bounds__(kFrontierThreads, 2) frontier_kernel(FrontierA
                     bq[u] = __shfl_sync(FULL, nq, j);
                     const uint32_t bb = __shfl_sync(FULL, nb, j);
                     const uint32_t v = (uint32_t)((w0 + j) * 32 + lane);
-                    if ((bq[u] >> lane) & 1) {
-                        rv[u] = __ldg(reinterpret_cast<const uint4 *>(a.rec + v));
-                        if (vlow && __ldg(a.umax + v) < vlow) rv[u] = make_uint4(0, 0, 0, 0);  // skipped list
-                    }
+                    if ((bq[u] >> lane) & 1) rv[u] = __ldg(reinterpret_cast<const uint4 *>(a.rec + v));
                     if ((bb >> lane) & 1) {
                         if (a.depth_stored) a.depth_stored[v] = (int32_t)level;  // stored-id order (coalesced)
                         if (!a.depth_stored_only && depth) depth[v] = (int32_t)level;

@@ -64,6 +64,7 @@ struct FrontierArgs {           // level end (a7) + next level plan (a1-a4), one
     const uint32_t *deg32;     // degrees (pass 1)
     const uint32_t *umax;      // largest neighbour of each list
     uint32_t lskip;            // BFS: lists whose largest neighbour is below ctrl->vpre_used are not planned
+    uint32_t *skipw;           // scratch (nwords): per bitmap word, the skipped lists (phase 1 -> phase 2)
     const VRec *rec;           // vertex records (pass 2)
     ChunkDesc *chunks;         // out: chunk descriptors
     uint32_t *tiles;           // out: first chunk of each tile (+ sentinel)
