@@ -464,7 +464,7 @@ def main():
         rs = float(rank_d.sum().item())
         pr = {"iters": 50, "damping": 0.85, "ms": pms, "ms_per_iter": pms / 50,
               "gteps": 50 * int(info["m"]) / (pms * 1e-3) / 1e9, "unit": "GTEPS (edges pushed / s)",
-              "rank_sum": rs, "accumulate": "fp64 atomicAdd (push, P:185)"}
+              "rank_sum": rs, "accumulate": "fp64; symmetric graph: each vertex gathers r(u)/deg(u) over its own list (one atomicAdd per list run; push with an atomic per edge, P:185, for directed graphs)"}
 
     # ---- cpu baseline: the oracle on a bounded sample (rank 0, N=1 only) ----
     cpu = None

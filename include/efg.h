@@ -210,6 +210,11 @@ efg_status efg_pagerank(efg_graph *g, double damping, uint32_t iters, double *ra
                                * nor probed; their bytes are still staged.  0: every element
                                * is decoded and probed (the paper's expansion, Alg. 1).
                                * Results are identical either way. */
+#define EFG_OPT_PAGERANK_PULL 3 /* 1 (default): efg_pagerank on a symmetric whole-graph handle
+                                 * gathers r(u)/deg(u) over each vertex's own list (one fp64
+                                 * atomic per list run instead of one per edge); 0 (and every
+                                 * directed or row-range handle): push along every edge with
+                                 * fp64 atomicAdd.  Same sums, other order (C21). */
 
 /* Set a per-handle option.  Errors: EFG_EINVAL (unknown option / value),
  * EFG_ESTATE (host-only handle). */

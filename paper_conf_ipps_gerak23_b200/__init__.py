@@ -91,6 +91,10 @@ class Graph:
         all below the visited prefix; False = decode and probe every element."""
         check(lib.efg_set_option(self._h, _abi.EFG_OPT_PREFIX_SKIP, 1 if on else 0), "efg_set_option")
 
+    def set_pagerank_pull(self, on: bool) -> None:
+        """EFG_OPT_PAGERANK_PULL: True (default) = gather on symmetric graphs, False = push."""
+        check(lib.efg_set_option(self._h, _abi.EFG_OPT_PAGERANK_PULL, 1 if on else 0), "efg_set_option")
+
     def free(self) -> None:
         if self._h:
             lib.efg_free(self._h)

@@ -169,6 +169,10 @@ extern "C" efg_status efg_set_option(efg_graph *g, int option, int64_t value)
         if (value != 0 && value != 1) return set_error(EFG_EINVAL, "EFG_OPT_LEVEL_LOOP: 0 or 1");
         g->dev.level_loop = (int)value;
         return EFG_OK;
+    case EFG_OPT_PAGERANK_PULL:
+        if (value != 0 && value != 1) return set_error(EFG_EINVAL, "EFG_OPT_PAGERANK_PULL: 0 or 1");
+        g->dev.pr_pull = (int)value;
+        return EFG_OK;
     case EFG_OPT_PREFIX_SKIP:
         if (value != 0 && value != 1) return set_error(EFG_EINVAL, "EFG_OPT_PREFIX_SKIP: 0 or 1");
         if (g->dev.prefix_skip != (int)value) {

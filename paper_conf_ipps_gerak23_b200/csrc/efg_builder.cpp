@@ -211,6 +211,7 @@ efg_status build_host(uint64_t n, uint64_t m, const uint32_t *src, const uint32_
         out.m_input = m;
         out.k = k;
         out.row_lo = lo;
+        out.symmetric = sym;
         out.row_hi = hi;
 
         // ---- pass 1: a-priori sizes -> offsets ----

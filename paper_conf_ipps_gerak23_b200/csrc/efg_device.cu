@@ -91,6 +91,7 @@ ExpandArgs expand_args(DeviceGraph &d, uint32_t *out)
     a.dist = d.fbuf;
     a.rank = d.dbuf;
     a.next = d.dbuf ? d.dbuf + d.n : nullptr;
+    a.contrib = d.dbuf ? d.dbuf + 2 * d.n + 1 : nullptr;
     a.max_stats = kMaxLevelStats;
     a.hot_words = (uint32_t)std::min<uint64_t>(kHotWords, d.nwords) & ~3u;
     a.k = d.k;
@@ -734,8 +735,12 @@ efg_status device_pagerank(efg_graph *g, double damping, uint32_t iters, double 
     DeviceGraph &d = g->dev;
     CUDA_TRY(cudaSetDevice(d.device));
     cudaStream_t s = stream_of(d);
-    if (!d.dbuf) EFG_TRY(dev_alloc(d, &d.dbuf, 2 * d.n + 1));
-    double *r = d.dbuf, *next = d.dbuf + d.n, *dsum = d.dbuf + 2 * d.n;
+    if (!d.dbuf) EFG_TRY(dev_alloc(d, &d.dbuf, 3 * d.n + 1));
+    double *r = d.dbuf, *next = d.dbuf + d.n, *dsum = d.dbuf + 2 * d.n, *contrib = d.dbuf + 2 * d.n + 1;
+    // pull (no atomics per edge) where every list is also the vertex's in-list:
+    // symmetric graphs on a whole-graph handle; push otherwise
+    const bool pull = g->host.symmetric && g->host.row_lo == 0 && g->host.row_hi == g->host.n && d.pr_pull;
+    const int pmode = pull ? kModePrPull : kModePagerank;
     const bool rank_dev = is_device_ptr(rank);
     cudaEvent_t ev0, ev1;
     CUDA_TRY(cudaEventCreate(&ev0));
@@ -745,12 +750,13 @@ efg_status device_pagerank(efg_graph *g, double damping, uint32_t iters, double 
     CUDA_TRY(cudaMemsetAsync(next, 0, d.n * 8, s));
     uint32_t launches = 0;
     EFG_TRY(start_traversal(d, 0, d.n, d.depth, nullptr, launches));  // frontier = every vertex
-    const int blocks = d.num_sms * expand_occupancy(kModePagerank);
+    const int blocks = d.num_sms * expand_occupancy(pmode);
+    if (pull) CUDA_TRY(launch_pr_contrib(r, d.deg32, contrib, d.n, s));
     for (uint32_t it = 0; it < iters; ++it) {
         CUDA_TRY(cudaMemsetAsync(dsum, 0, 8, s));
         CUDA_TRY(launch_pr_dangling(r, d.deg32, d.n, dsum, s));
-        CUDA_TRY(launch_expand(kModePagerank, expand_args(d, nullptr), blocks, s));
-        CUDA_TRY(launch_pr_update(r, next, d.n, damping, dsum, s));
+        CUDA_TRY(launch_expand(pmode, expand_args(d, nullptr), blocks, s));
+        CUDA_TRY(launch_pr_update(r, next, d.n, damping, dsum, pull ? contrib : nullptr, d.deg32, s));
     }
     // ranks back to input ids (next[] is free scratch now)
     double *src = r;

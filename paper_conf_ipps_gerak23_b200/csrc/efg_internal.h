@@ -32,6 +32,7 @@ struct HostEFG {
     std::vector<uint32_t> umax;     // n: largest neighbour (list's last element, P:218 u), 0 if empty
     uint64_t fwd_bytes = 0, lower_bytes = 0, upper_bytes = 0, apriori_bits = 0;
     uint64_t row_lo = 0, row_hi = 0;
+    bool symmetric = false;         // built with EFG_SYMMETRIZE: out-lists = in-lists
     double build_seconds = 0.0;
 };
 
@@ -198,6 +199,7 @@ struct DeviceGraph {
     LevelStat *stats_host = nullptr;   // pinned mirror of stats
     int level_loop = 0;                // 0 = CUDA graph (device loop), 1 = host loop + events
     int prefix_skip = 1;               // EFG_OPT_PREFIX_SKIP
+    int pr_pull = 1;                   // EFG_OPT_PAGERANK_PULL
     cudaGraph_t loop_graph[2] = {nullptr, nullptr};      // per mode (visit, visit+parent)
     cudaGraphExec_t loop_exec[2] = {nullptr, nullptr};
     uint64_t own_lo_w = 0, own_hi_w = 0;   // bitmap words of the owned rows (frontier filter)

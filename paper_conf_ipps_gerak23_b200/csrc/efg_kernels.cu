@@ -1015,6 +1015,7 @@ __global__ void __launch_bounds__(kExpandThreads, 1) expand_kernel(ExpandArgs a)
                 sp.aux = a.vlist[cur.v] + r0;
                 sp.aux2 = a.dist[cur.v];
             }
+            if (MODE == kModePrPull) sp.aux = cur.v;  // the list's vertex gathers its neighbours' shares
             if (MODE == kModePagerank) {  // push r(u)/deg(u) along every edge
                 const double share = a.rank[cur.v] / (double)a.deg32[cur.v];
                 sp.aux = (uint64_t)__double_as_longlong(share);
@@ -1091,6 +1092,8 @@ __global__ void __launch_bounds__(kExpandThreads, 1) expand_kernel(ExpandArgs a)
                 if (j) r.x &= FULL >> select_in_word(__brev(r.x), j);  // drop j stop bits
                 uint32_t l = r.w & 63, lmask = (1u << l) - 1;
                 uint32_t e = Er0 + c;  // batch element index (modes without the skip keep every record)
+                uint32_t pr_slot = FULL;  // PageRank pull: slot being summed and its partial sum
+                double pr_acc = 0.0;
 
                 // one element: next stop bit -> select1(i) - i, lower field, value
                 auto decode = [&](uint32_t &x, uint32_t &slot_of) {
@@ -1137,6 +1140,23 @@ __global__ void __launch_bounds__(kExpandThreads, 1) expand_kernel(ExpandArgs a)
                             if (u < cntu && nd[u] < cd[u]) {  // non-negative floats order like their bits
                                 const int old = atomicMin(reinterpret_cast<int *>(a.dist) + xv[u], __float_as_int(nd[u]));
                                 if (__float_as_int(nd[u]) < old) atomicOr(a.vis + (xv[u] >> 5), 1u << (xv[u] & 31));
+                            }
+                        }
+                    } else if (MODE == kModePrPull) {
+                        // pull (symmetric graphs): the lane sums contrib[u] = r(u)/deg(u) of its
+                        // run's neighbours and adds the sum once per list it leaves
+                        double cv[kU];
+#pragma unroll
+                        for (int u = 0; u < kU; ++u) cv[u] = u < cntu ? __ldg(a.contrib + xv[u]) : 0.0;
+#pragma unroll
+                        for (int u = 0; u < kU; ++u) {
+                            if (u < cntu) {
+                                if (sv[u] != pr_slot) {
+                                    if (pr_slot != FULL) atomicAdd(a.next + ws.slot[pr_slot].aux, pr_acc);
+                                    pr_slot = sv[u];
+                                    pr_acc = 0.0;
+                                }
+                                pr_acc += cv[u];
                             }
                         }
                     } else if (MODE == kModePagerank) {
@@ -1203,6 +1223,7 @@ __global__ void __launch_bounds__(kExpandThreads, 1) expand_kernel(ExpandArgs a)
                     }
                     visit(xv, sv, ev, cntu);
                 }
+                if (MODE == kModePrPull && pr_slot != FULL) atomicAdd(a.next + ws.slot[pr_slot].aux, pr_acc);
             }
             __syncwarp();
             Er0 = Er1;
@@ -1225,13 +1246,22 @@ __global__ void pr_dangling_kernel(const double *rank, const uint32_t *deg32, ui
     if ((threadIdx.x & 31) == 0 && acc != 0.0) atomicAdd(dsum, acc);
 }
 
-__global__ void pr_update_kernel(double *rank, double *next, uint64_t n, double damping, const double *dsum)
+__global__ void pr_update_kernel(double *rank, double *next, uint64_t n, double damping, const double *dsum,
+                                 double *contrib, const uint32_t *deg32)
 {
     const double base = (1.0 - damping) / (double)n, dn = *dsum / (double)n;
     for (uint64_t v = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; v < n; v += (uint64_t)gridDim.x * blockDim.x) {
-        rank[v] = base + damping * (next[v] + dn);
+        const double r = base + damping * (next[v] + dn);
+        rank[v] = r;
         next[v] = 0.0;
+        if (contrib) contrib[v] = deg32[v] ? r / (double)deg32[v] : 0.0;  // pull: next iteration's shares
     }
+}
+
+__global__ void pr_contrib_kernel(const double *rank, const uint32_t *deg32, double *contrib, uint64_t n)
+{
+    for (uint64_t v = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; v < n; v += (uint64_t)gridDim.x * blockDim.x)
+        contrib[v] = deg32[v] ? rank[v] / (double)deg32[v] : 0.0;
 }
 
 __global__ void fill_kernel(uint32_t *p, uint32_t val, uint64_t n)
@@ -1286,9 +1316,15 @@ cudaError_t launch_pr_dangling(const double *rank, const uint32_t *deg32, uint64
 }
 
 cudaError_t launch_pr_update(double *rank, double *next, uint64_t n, double damping, const double *dsum,
-                             cudaStream_t s)
+                             double *contrib, const uint32_t *deg32, cudaStream_t s)
 {
-    pr_update_kernel<<<grid_for(n), 256, 0, s>>>(rank, next, n, damping, dsum);
+    pr_update_kernel<<<grid_for(n), 256, 0, s>>>(rank, next, n, damping, dsum, contrib, deg32);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_pr_contrib(const double *rank, const uint32_t *deg32, double *contrib, uint64_t n, cudaStream_t s)
+{
+    pr_contrib_kernel<<<grid_for(n), 256, 0, s>>>(rank, deg32, contrib, n);
     return cudaGetLastError();
 }
 
@@ -1350,6 +1386,8 @@ static cudaError_t expand_set_attrs()
         e = cudaFuncSetAttribute(expand_kernel<kModeSssp>, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes);
     if (e == cudaSuccess)
         e = cudaFuncSetAttribute(expand_kernel<kModePagerank>, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes);
+    if (e == cudaSuccess)
+        e = cudaFuncSetAttribute(expand_kernel<kModePrPull>, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes);
     if (e == cudaSuccess) done = true;
     return e;
 }
@@ -1377,6 +1415,9 @@ cudaError_t launch_expand(int mode, const ExpandArgs &a, int blocks, cudaStream_
         break;
     case kModePagerank:
         expand_kernel<kModePagerank><<<blocks, kExpandThreads, sm, s>>>(a);
+        break;
+    case kModePrPull:
+        expand_kernel<kModePrPull><<<blocks, kExpandThreads, sm, s>>>(a);
         break;
     default:
         expand_kernel<kModeDecode><<<blocks, kExpandThreads, sm, s>>>(a);

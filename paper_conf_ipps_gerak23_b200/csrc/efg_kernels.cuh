@@ -13,6 +13,7 @@ enum ExpandMode : int {
     kModeDecode = 2,       // efg_decode: store the decoded value in CSR order
     kModeSssp = 3,         // SSSP relax: atomicMin on fp32 dist, mark relaxed vertices
     kModePagerank = 4,     // PageRank push: next[v] += r(u)/deg(u)
+    kModePrPull = 5,       // PageRank pull (symmetric graphs): next[u] += sum of contrib[v] over u's list
 };
 
 struct ExpandArgs {
@@ -30,6 +31,7 @@ struct ExpandArgs {
     float *dist;               // SSSP: distances (stored ids)
     const double *rank;        // PageRank: current ranks (stored ids)
     double *next;              // PageRank: accumulated pushes
+    const double *contrib;     // PageRank pull: r(v)/deg(v) per vertex
     uint32_t max_stats;
     uint32_t hot_words;        // bitmap words with a shared-memory snapshot (multiple of 4)
     uint32_t k;                // forward-pointer quantum (chunk length); 0 = none
@@ -92,7 +94,8 @@ size_t expand_smem_bytes();
 // pout[old_of_new[i]] = pin[i] == ~0u ? ~0u : old_of_new[pin[i]]  (parents back to input ids)
 cudaError_t launch_pr_dangling(const double *rank, const uint32_t *deg32, uint64_t n, double *dsum, cudaStream_t s);
 cudaError_t launch_pr_update(double *rank, double *next, uint64_t n, double damping, const double *dsum,
-                             cudaStream_t s);
+                             double *contrib, const uint32_t *deg32, cudaStream_t s);
+cudaError_t launch_pr_contrib(const double *rank, const uint32_t *deg32, double *contrib, uint64_t n, cudaStream_t s);
 cudaError_t launch_fill(uint32_t *p, uint32_t val, uint64_t n, cudaStream_t s);
 cudaError_t launch_fill_f64(double *p, double val, uint64_t n, cudaStream_t s);
 cudaError_t launch_gather32(const uint32_t *stored, const uint32_t *new_of_old, uint32_t *out, uint64_t n,

@@ -378,9 +378,22 @@ def test_pagerank_vs_fp64_oracle(efg, reorder):
     flags = efg.EFG_DEFAULT_FLAGS | (efg.EFG_REORDER_DEGREE if reorder else 0)
     g = efg.Graph.build(n, src, dst, flags=flags)
     ov, oe = oracle.csr_build(n, src, dst)
+    ref = oracle.pagerank(ov, oe, 0.85, 50)
+    for pull in (True, False):  # gather over own lists / push along every edge
+        g.set_pagerank_pull(pull)
+        got = g.pagerank(0.85, 50)
+        rel = np.abs(got - ref).sum() / np.abs(ref).sum()
+        assert rel < 1e-6, (pull, rel)
+        assert abs(got.sum() - 1.0) < 1e-9
+    g.free()
+
+
+def test_pagerank_directed_uses_push(efg):
+    """A directed handle's lists are out-lists only: PageRank pushes (pull option ignored)."""
+    n, src, dst = synth.rmat(12, 8, seed=23)
+    g = efg.Graph.build(n, src, dst, flags=efg.EFG_DEDUP | efg.EFG_DROP_SELF_LOOPS)
+    ov, oe = oracle.csr_build(n, src, dst, symmetrize=False)
     got = g.pagerank(0.85, 50)
     ref = oracle.pagerank(ov, oe, 0.85, 50)
-    rel = np.abs(got - ref).sum() / np.abs(ref).sum()
-    assert rel < 1e-6, rel
-    assert abs(got.sum() - 1.0) < 1e-9
+    assert np.abs(got - ref).sum() / np.abs(ref).sum() < 1e-6
     g.free()
