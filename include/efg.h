@@ -161,8 +161,11 @@ typedef struct efg_stats {
     uint64_t *level_frontier;  /* in/out: |F_L| per level (level_cap entries)        */
     uint64_t *level_edges;     /* in/out: E_L = sum of frontier degrees per level    */
     float *level_expand_ms;    /* in/out: expand kernel time per level, or NULL      */
-    float *level_end_ms;       /* in/out: compact + plan time per level (host loop   *
-                                *         only, CUDA events), or NULL                */
+    float *level_end_ms;       /* in/out: level-end + plan kernel time per level     *
+                                *         (host loop only, CUDA events), or NULL     */
+    uint64_t d2h_bytes;        /* out: device->host bytes the call moved for host    *
+                                *       outputs (a host depth array travels as one   *
+                                *       byte per vertex when every depth < 127)      */
 } efg_stats;
 
 /*

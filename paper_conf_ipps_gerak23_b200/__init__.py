@@ -182,7 +182,7 @@ class Graph:
             sd = {"levels": L, "edges_traversed": st.edges_traversed,
                   "vertices_reached": st.vertices_reached, "device_ms": st.device_ms,
                   "expand_ms": st.expand_ms, "expand_launches": st.expand_launches,
-                  "kernel_launches": st.kernel_launches,
+                  "kernel_launches": st.kernel_launches, "d2h_bytes": st.d2h_bytes,
                   "level_frontier": arrs[0][:min(L, level_cap)].copy(),
                   "level_edges": arrs[1][:min(L, level_cap)].copy(),
                   "level_expand_ms": arrs[2][:min(L, level_cap)].copy(),

@@ -203,6 +203,8 @@ void device_free(DeviceGraph &d)
     cudaFree(d.deg32);
     cudaFree(d.umax);
     cudaFree(d.skipw);
+    cudaFree(d.depth8);
+    if (d.depth8_host) cudaFreeHost(d.depth8_host);
     cudaFree(d.iso);
     cudaFree(d.vlist);
     cudaFree(d.weights);
@@ -505,9 +507,34 @@ efg_status device_bfs(efg_graph *g, uint32_t source, int32_t *depth, uint32_t *p
         CUDA_TRY(cudaEventRecord(ev1, s));
     }
     if (parent && relabel) CUDA_TRY(launch_map_parent(pd, d.old_of_new, pout, d.n, s));
-    if (!depth_dev) CUDA_TRY(cudaMemcpyAsync(depth, dd, d.n * 4, cudaMemcpyDeviceToHost, s));
-    if (parent && !parent_dev) CUDA_TRY(cudaMemcpyAsync(parent, pout, d.n * 4, cudaMemcpyDeviceToHost, s));
+    uint64_t d2h = 0;
+    // a host depth array crosses PCIe as one byte per vertex when every depth
+    // fits (levels < 127: [-1, 126]); the host widens it (OpenMP)
+    bool narrow8 = false;
+    if (!depth_dev) {
+        narrow8 = levels < 127 && d.n >= 4096;  // levels is final here in both loop modes
+        if (narrow8) {
+            if (!d.depth8) EFG_TRY(dev_alloc(d, &d.depth8, d.n));
+            if (!d.depth8_host) CUDA_TRY(cudaMallocHost(reinterpret_cast<void **>(&d.depth8_host), d.n));
+            CUDA_TRY(launch_pack8(dd, d.depth8, d.n, s));
+            CUDA_TRY(cudaMemcpyAsync(d.depth8_host, d.depth8, d.n, cudaMemcpyDeviceToHost, s));
+            d2h += d.n;
+        } else {
+            CUDA_TRY(cudaMemcpyAsync(depth, dd, d.n * 4, cudaMemcpyDeviceToHost, s));
+            d2h += d.n * 4;
+        }
+    }
+    if (parent && !parent_dev) {
+        CUDA_TRY(cudaMemcpyAsync(parent, pout, d.n * 4, cudaMemcpyDeviceToHost, s));
+        d2h += d.n * 4;
+    }
     CUDA_TRY(cudaStreamSynchronize(s));
+    if (narrow8) {
+        const int8_t *src8 = d.depth8_host;
+        const int64_t nn = (int64_t)d.n;
+#pragma omp parallel for schedule(static)
+        for (int64_t i = 0; i < nn; ++i) depth[i] = src8[i];
+    }
 
     float total_ms = 0.f;
     cudaEventElapsedTime(&total_ms, ev0, ev1);
@@ -542,6 +569,7 @@ efg_status device_bfs(efg_graph *g, uint32_t source, int32_t *depth, uint32_t *p
         st->expand_launches = levels;
         st->kernel_launches = launches;
         st->expand_bytes = 0;
+        st->d2h_bytes = d2h;
         for (uint32_t i = 0; i < std::min<uint32_t>((uint32_t)lf.size(), st->level_cap); ++i) {
             if (st->level_frontier) st->level_frontier[i] = lf[i];
             if (st->level_edges) st->level_edges[i] = le[i];

@@ -166,6 +166,8 @@ struct DeviceGraph {
     uint32_t *deg32 = nullptr;         // n degrees (padded to the bitmap size)
     uint32_t *umax = nullptr;          // n largest neighbour per list (padded to the bitmap size)
     uint32_t *skipw = nullptr;         // frontier_kernel scratch: skipped lists per bitmap word
+    int8_t *depth8 = nullptr;          // host depth transfer: 1 byte per vertex (device) ...
+    int8_t *depth8_host = nullptr;     // ... and its pinned host staging buffer
     uint32_t *iso = nullptr;           // bitmap of the degree-0 vertices and the padding (nwords)
     uint64_t *vlist = nullptr;         // n+1 (SSSP weight indexing / decode)
     float *weights = nullptr;          // m or null

@@ -1297,6 +1297,21 @@ __global__ void map_depth_kernel(const int32_t *stored, const uint32_t *new_of_o
         out[v] = stored[new_of_old[v]];
 }
 
+// host depth transfer: one byte per vertex (every depth in [-1, 126])
+__global__ void pack8_kernel(const int32_t *in, int8_t *out, uint64_t n)
+{
+    for (uint64_t i = (blockIdx.x * (uint64_t)blockDim.x + threadIdx.x) * 4; i < n; i += (uint64_t)gridDim.x * blockDim.x * 4) {
+        if (i + 4 <= n) {
+            const int4 v = *reinterpret_cast<const int4 *>(in + i);
+            const uint32_t b = (uint32_t)(uint8_t)v.x | (uint32_t)(uint8_t)v.y << 8 | (uint32_t)(uint8_t)v.z << 16 |
+                               (uint32_t)(uint8_t)v.w << 24;
+            *reinterpret_cast<uint32_t *>(out + i) = b;
+        } else {
+            for (uint64_t j = i; j < n; ++j) out[j] = (int8_t)in[j];
+        }
+    }
+}
+
 __global__ void map_parent_kernel(const uint32_t *pin, const uint32_t *old_of_new, uint32_t *pout, uint64_t n)
 {
     for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x) {
@@ -1359,6 +1374,13 @@ cudaError_t launch_map_depth(const int32_t *stored, const uint32_t *new_of_old, 
 {
     const unsigned blocks = (unsigned)std::max<uint64_t>(1, std::min<uint64_t>((n + 255) / 256, 148 * 16));
     map_depth_kernel<<<blocks, 256, 0, s>>>(stored, new_of_old, out, n);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_pack8(const int32_t *in, int8_t *out, uint64_t n, cudaStream_t s)
+{
+    const unsigned blocks = (unsigned)std::max<uint64_t>(1, std::min<uint64_t>((n / 4 + 255) / 256, 148 * 8));
+    pack8_kernel<<<blocks, 256, 0, s>>>(in, out, n);
     return cudaGetLastError();
 }
 
