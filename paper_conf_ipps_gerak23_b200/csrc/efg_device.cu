@@ -205,6 +205,8 @@ void device_free(DeviceGraph &d)
     cudaFree(d.skipw);
     cudaFree(d.depth8);
     if (d.depth8_host) cudaFreeHost(d.depth8_host);
+    for (int c = 0; c < kD2HChunks; ++c)
+        if (d.d2h_ev[c]) cudaEventDestroy(d.d2h_ev[c]);
     cudaFree(d.iso);
     cudaFree(d.vlist);
     cudaFree(d.weights);
@@ -516,8 +518,15 @@ efg_status device_bfs(efg_graph *g, uint32_t source, int32_t *depth, uint32_t *p
         if (narrow8) {
             if (!d.depth8) EFG_TRY(dev_alloc(d, &d.depth8, d.n));
             if (!d.depth8_host) CUDA_TRY(cudaMallocHost(reinterpret_cast<void **>(&d.depth8_host), d.n));
+            if (!d.d2h_ev[0])
+                for (int c = 0; c < kD2HChunks; ++c) CUDA_TRY(cudaEventCreateWithFlags(&d.d2h_ev[c], cudaEventDisableTiming));
             CUDA_TRY(launch_pack8(dd, d.depth8, d.n, s));
-            CUDA_TRY(cudaMemcpyAsync(d.depth8_host, d.depth8, d.n, cudaMemcpyDeviceToHost, s));
+            // chunked copy: the host widens chunk c while chunks > c are in flight
+            for (int c = 0; c < kD2HChunks; ++c) {
+                const uint64_t c0 = d.n * c / kD2HChunks, c1 = d.n * (c + 1) / kD2HChunks;
+                CUDA_TRY(cudaMemcpyAsync(d.depth8_host + c0, d.depth8 + c0, c1 - c0, cudaMemcpyDeviceToHost, s));
+                CUDA_TRY(cudaEventRecord(d.d2h_ev[c], s));
+            }
             d2h += d.n;
         } else {
             CUDA_TRY(cudaMemcpyAsync(depth, dd, d.n * 4, cudaMemcpyDeviceToHost, s));
@@ -528,13 +537,16 @@ efg_status device_bfs(efg_graph *g, uint32_t source, int32_t *depth, uint32_t *p
         CUDA_TRY(cudaMemcpyAsync(parent, pout, d.n * 4, cudaMemcpyDeviceToHost, s));
         d2h += d.n * 4;
     }
-    CUDA_TRY(cudaStreamSynchronize(s));
     if (narrow8) {
         const int8_t *src8 = d.depth8_host;
-        const int64_t nn = (int64_t)d.n;
+        for (int c = 0; c < kD2HChunks; ++c) {
+            CUDA_TRY(cudaEventSynchronize(d.d2h_ev[c]));
+            const int64_t c0 = (int64_t)(d.n * c / kD2HChunks), c1 = (int64_t)(d.n * (c + 1) / kD2HChunks);
 #pragma omp parallel for schedule(static)
-        for (int64_t i = 0; i < nn; ++i) depth[i] = src8[i];
+            for (int64_t i = c0; i < c1; ++i) depth[i] = src8[i];
+        }
     }
+    CUDA_TRY(cudaStreamSynchronize(s));
 
     float total_ms = 0.f;
     cudaEventElapsedTime(&total_ms, ev0, ev1);

@@ -154,6 +154,7 @@ constexpr uint32_t kTileWork = EFG_TILE_WORK;         // work units per tile (a3
 constexpr uint32_t kChunkWork = 32;          // per-chunk overhead in work units
 
 constexpr unsigned kMaxGrid = 4096;
+constexpr int kD2HChunks = 8;               // host depth transfer pipeline depth
 
 struct DeviceGraph {
     int device = -1;
@@ -168,6 +169,7 @@ struct DeviceGraph {
     uint32_t *skipw = nullptr;         // frontier_kernel scratch: skipped lists per bitmap word
     int8_t *depth8 = nullptr;          // host depth transfer: 1 byte per vertex (device) ...
     int8_t *depth8_host = nullptr;     // ... and its pinned host staging buffer
+    cudaEvent_t d2h_ev[8] = {};        // chunked depth8 copy: one event per chunk
     uint32_t *iso = nullptr;           // bitmap of the degree-0 vertices and the padding (nwords)
     uint64_t *vlist = nullptr;         // n+1 (SSSP weight indexing / decode)
     float *weights = nullptr;          // m or null
