@@ -121,7 +121,7 @@ FrontierArgs frontier_args(DeviceGraph &d, cudaGraphConditionalHandle cond, bool
     a.tiles = d.tiles;
     a.ctrl = d.ctrl;
     a.status = d.status;
-    a.barrier = reinterpret_cast<unsigned long long *>(d.status + 4 * kMaxGrid);
+    a.barrier = reinterpret_cast<unsigned long long *>(d.status + 5 * kMaxGrid);
     a.big = d.big;
     a.trace = d.trace;
     a.stats = d.stats;
@@ -324,8 +324,8 @@ efg_status device_upload(efg_graph *g, const efg_build_opts &o)
     EFG_TRY(dev_alloc(d, &d.tiles, d.max_tiles + 1));
     EFG_TRY(dev_alloc(d, &d.chunks, d.max_chunks));
     EFG_TRY(dev_alloc(d, &d.depth, h.n));
-    EFG_TRY(dev_alloc(d, &d.status, 4 * kMaxGrid + 1));  // + the grid-barrier counter
-    CUDA_TRY(cudaMemsetAsync(d.status, 0, (4 * kMaxGrid + 1) * 8, s));
+    EFG_TRY(dev_alloc(d, &d.status, 5 * kMaxGrid + 1));  // + the grid-barrier counter
+    CUDA_TRY(cudaMemsetAsync(d.status, 0, (5 * kMaxGrid + 1) * 8, s));
     if (std::getenv("EFG_FRONTIER_TRACE")) EFG_TRY(dev_alloc(d, &d.trace, 8 * kMaxGrid));
     // lists planned grid-wide: more than one chunk (deg > k) or more than one
     // tile of work (deg > kTileWork - kChunkWork)

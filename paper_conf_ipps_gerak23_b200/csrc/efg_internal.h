@@ -96,7 +96,6 @@ struct LevelCtrl {
     uint64_t total_ne;  // sum of E_L (= edges traversed, reading C18)
     uint32_t vmin2[2];  // frontier_kernel of level L: smallest vertex neither visited nor isolated, in
                         // slot L & 1 (atomicMin); the expand of level L reads it as its visited prefix
-    uint32_t nbig2[2];  // frontier_kernel of level L: BigList entries appended (slot L & 1)
     uint32_t vpre_used; // visited prefix the last BFS expand used (0: none); lower bound for the next level end
 };
 
@@ -187,7 +186,7 @@ struct DeviceGraph {
     uint32_t *new_of_old = nullptr;    // its inverse (n) or null
     int32_t *depth_st = nullptr;       // depth by stored id (relabelled graphs)
     int32_t *step_depth = nullptr;     // stepwise traversal: caller's depth buffer
-    uint64_t *status = nullptr;        // frontier_kernel: 4 x [kMaxGrid] per-block aggregates + barrier counter
+    uint64_t *status = nullptr;        // frontier_kernel: 5 x [kMaxGrid] per-block aggregates + barrier counter
     BigList *big = nullptr;
     unsigned long long *trace = nullptr;  // debug: frontier_kernel phase timestamps            // frontier_kernel: multi-chunk / multi-tile lists of a level
     uint64_t max_big = 0;

@@ -179,8 +179,6 @@ __global__ void init_kernel(InitArgs a)
         a.ctrl->total_ne = 0;
         a.ctrl->vmin2[0] = FULL;
         a.ctrl->vmin2[1] = FULL;
-        a.ctrl->nbig2[0] = 0;
-        a.ctrl->nbig2[1] = 0;
         a.ctrl->vpre_used = 0;
         if (a.parent) a.parent[a.v0] = (uint32_t)a.v0;
     }
@@ -330,8 +328,8 @@ __device__ __forceinline__ void warp_excl_u32_n(uint32_t (&x)[N], uint32_t (&tot
 __global__ void __launch_bounds__(kFrontierThreads, 2) frontier_kernel(FrontierArgs a)
 {
     constexpr int NT = kFrontierThreads, NW = NT / 32;
-    __shared__ uint64_t s_q[NW], s_wk[NW], s_ch[NW], s_sk[NW], s_all[NW];
-    __shared__ uint64_t s_pre[4], s_tot[4];
+    __shared__ uint64_t s_q[NW], s_wk[NW], s_ch[NW], s_sk[NW], s_bg[NW], s_all[NW];
+    __shared__ uint64_t s_pre[5], s_tot[5];
 
     const uint32_t tid = threadIdx.x, lane = tid & 31, wid = tid >> 5, b = blockIdx.x;
 #define FTRACE(p)                                                      \
@@ -344,7 +342,6 @@ __global__ void __launch_bounds__(kFrontierThreads, 2) frontier_kernel(FrontierA
     int32_t *depth = ctrl->depth;
     if (b == 0 && tid == 0) {  // slots of the next level end
         ctrl->vmin2[(level & 1) ^ 1] = FULL;
-        ctrl->nbig2[(level & 1) ^ 1] = 0;
     }
     const ChunkLen cl = make_chunk(a.k, a.kshift);
     const uint64_t CH = cl.ch, CW = kChunkWork;
@@ -355,7 +352,10 @@ __global__ void __launch_bounds__(kFrontierThreads, 2) frontier_kernel(FrontierA
     const uint32_t gw = b * NW + wid;
     const uint64_t WG = 32ull * G;  // words between a warp's groups
     const uint32_t lt = (1u << lane) - 1;
-    constexpr int kB = 8;  // pass 1: non-empty words whose degree loads are in flight together
+#ifndef EFG_KB
+#define EFG_KB 8
+#endif
+    constexpr int kB = EFG_KB;  // pass 1: non-empty words whose degree loads are in flight together
 
     // ---- 1: count, work and chunks of the warp's new (owned) vertices ----
     // BFS list skip: a list whose largest neighbour is below the visited
@@ -365,6 +365,7 @@ __global__ void __launch_bounds__(kFrontierThreads, 2) frontier_kernel(FrontierA
     const uint32_t vlow = a.lskip ? ctrl->vpre_used : 0u;
     uint32_t cq = 0, all = 0, ch = 0;  // lane partials
     uint64_t wk = 0, sk = 0;
+    uint32_t bg = 0;  // lists planned grid-wide (phase 3)
     uint32_t vmin = FULL;  // smallest vertex of this warp's range that is neither visited nor isolated
     for (uint64_t w0 = 32ull * gw; w0 < a.nwords; w0 += WG) {
         const uint64_t w = w0 + lane;
@@ -415,12 +416,14 @@ __global__ void __launch_bounds__(kFrontierThreads, 2) frontier_kernel(FrontierA
                 const uint32_t nch = d ? (uint32_t)cl.div((uint64_t)d + CH - 1) : 0u;
                 wk += (uint64_t)nch * CW + d;
                 ch += nch;
+                bg += (nch > 1 || (uint64_t)nch * CW + d > kTileWork) ? 1u : 0u;
             }
         }
     }
     const uint64_t cqw = warp_sum_u64(cq), allw = warp_sum_u64(all), chw = warp_sum_u64(ch);
     wk = warp_sum_u64(wk);
     sk = warp_sum_u64(sk);
+    const uint64_t bgw = warp_sum_u64(bg);
 #pragma unroll
     for (int d = 16; d; d >>= 1) vmin = min(vmin, __shfl_xor_sync(FULL, vmin, d));
     if (lane == 0) {
@@ -429,6 +432,7 @@ __global__ void __launch_bounds__(kFrontierThreads, 2) frontier_kernel(FrontierA
         s_wk[wid] = wk;
         s_ch[wid] = chw;
         s_sk[wid] = sk;
+        s_bg[wid] = bgw;
         if (vmin != FULL) atomicMin(&ctrl->vmin2[level & 1], vmin);
     }
     __syncthreads();
@@ -436,16 +440,16 @@ __global__ void __launch_bounds__(kFrontierThreads, 2) frontier_kernel(FrontierA
     // publish the block's aggregates (frontier vertices, work units, chunks,
     // skipped-list edges), barrier, then every block sums its predecessors'
     // (region r by warp r)
-    if (wid < 4) {
-        const uint64_t *src = wid == 0 ? s_q : (wid == 1 ? s_wk : (wid == 2 ? s_ch : s_sk));
+    if (wid < 5) {
+        const uint64_t *src = wid == 0 ? s_q : (wid == 1 ? s_wk : (wid == 2 ? s_ch : (wid == 3 ? s_sk : s_bg)));
         const uint64_t agg = warp_sum_u64(lane < NW ? src[lane] : 0);
         if (lane == 0) st_relaxed_u64(a.status + wid * kMaxGrid + b, agg);
-    } else if (wid == 4) {
+    } else if (wid == 5) {
         const uint64_t blk_all = warp_sum_u64(lane < NW ? s_all[lane] : 0);
         if (lane == 0 && blk_all) atomicAdd(reinterpret_cast<unsigned long long *>(&ctrl->nnew), blk_all);
     }
     grid_barrier(a.barrier);
-    if (wid < 4) {
+    if (wid < 5) {
         uint64_t pre, tot;
         sum_published(a.status + wid * kMaxGrid, b, pre, tot);
         if (lane == 0) {
@@ -482,7 +486,10 @@ __global__ void __launch_bounds__(kFrontierThreads, 2) frontier_kernel(FrontierA
     FTRACE(2);
     uint64_t run = s_pre[1];
     uint32_t crun = (uint32_t)s_pre[2];  // chunks of a level < 2^32 (n + m/k)
+    uint32_t brun = (uint32_t)s_pre[4];  // this warp's first BigList entry (no atomics)
+    const uint32_t nbig = (uint32_t)s_tot[4];
     for (uint32_t w = 0; w < wid; ++w) {
+        brun += (uint32_t)s_bg[w];
         run += s_wk[w];
         crun += (uint32_t)s_ch[w];
     }
@@ -588,9 +595,8 @@ __global__ void __launch_bounds__(kFrontierThreads, 2) frontier_kernel(FrontierA
                 }
                 const uint32_t bm = __ballot_sync(FULL, big);
                 if (bm) {
-                    uint32_t base = 0;
-                    if (lane == 0) base = atomicAdd(&ctrl->nbig2[level & 1], (uint32_t)__popc(bm));
-                    base = __shfl_sync(FULL, base, 0);
+                    const uint32_t base = brun;
+                    brun += __popc(bm);
                     if (big) {
                         BigList bl;
                         bl.W = W;
@@ -609,13 +615,13 @@ __global__ void __launch_bounds__(kFrontierThreads, 2) frontier_kernel(FrontierA
         }
     }
     FTRACE(5);
+    if (nbig == 0) return;  // grid-uniform: no long list this level
     grid_barrier(a.barrier);
     FTRACE(6);
 
     // ---- 3: the long lists, one per lane (lists of > 8 chunks or tiles: one
     // per warp, lanes over chunks / tiles): descriptors and the tile
     // boundaries of the list's window (Fig. 4 rule) ----
-    const uint32_t nbig = ld_relaxed_u32(&ctrl->nbig2[level & 1]);
     const bool udiv = a.k && CW + CH < (1ull << 31);  // 32-bit chunk division (rel < 2^31.1 - CW - CH)
     const uint32_t CWH = (uint32_t)(CW + CH);
     auto tile_chunk = [&](uint32_t rel, uint32_t nch) -> uint32_t {
@@ -624,8 +630,11 @@ __global__ void __launch_bounds__(kFrontierThreads, 2) frontier_kernel(FrontierA
         if (udiv && nch > 1) c = min((rel + CWH - 1) / CWH, nch);
         return c;
     };
-    for (uint64_t e0 = (uint64_t)gw * 32; e0 < nbig; e0 += 32ull * G) {
-        const uint64_t e = e0 + lane;
+    // entry e = gw + G*(lane + 32*i): consecutive entries (neighbouring ids,
+    // i.e. similar degrees: the relabelled hubs come together) go to
+    // different warps
+    for (uint64_t e0 = gw; e0 < nbig; e0 += 32ull * G) {
+        const uint64_t e = e0 + (uint64_t)lane * G;
         uint64_t W = 0, cs = 0, off_l = 0;
         uint32_t d = 0, ub = 0, v = 0, nch = 0;
         if (e < nbig) {

@@ -71,7 +71,7 @@ struct FrontierArgs {           // level end (a7) + next level plan (a1-a4), one
     ChunkDesc *chunks;         // out: chunk descriptors
     uint32_t *tiles;           // out: first chunk of each tile (+ sentinel)
     LevelCtrl *ctrl;           // in: level, seq, depth ptr; out: nf, ne, nwork, nchunks, ntiles, xlevel, vmin2
-    uint64_t *status;          // four per-block aggregate regions of kMaxGrid words
+    uint64_t *status;          // five per-block aggregate regions of kMaxGrid words
     unsigned long long *barrier;  // grid-barrier arrival counter (grows by gridDim.x per barrier)
     BigList *big;              // scratch: lists planned by the whole grid
     unsigned long long *trace; // debug (EFG_FRONTIER_TRACE): per block, 8 phase timestamps, or null
