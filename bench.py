@@ -58,6 +58,8 @@ def parse():
     p.add_argument("--reorder", default="degree", choices=["none", "degree"],
                    help="EFG_REORDER_DEGREE relabelling at build time (results stay in input ids)")
     p.add_argument("--profile-levels", action="store_true", help="print per-level stats to stderr")
+    p.add_argument("--sssp", action="store_true",
+                   help="also time SSSP (NEXT-1) over the same graph built with synthetic weights")
     p.add_argument("--no-pagerank", action="store_true",
                    help="skip the PageRank measurement (BASELINE configs[1]: BFS and PageRank)")
     return p.parse_args()
@@ -511,6 +513,39 @@ def main():
               "gteps": 50 * int(info["m"]) / (pms * 1e-3) / 1e9, "unit": "GTEPS (edges pushed / s)",
               "rank_sum": rs, "accumulate": "fp64; symmetric graph: each vertex gathers r(u)/deg(u) over its own list (one atomicAdd per list run; push with an atomic per edge, P:185, for directed graphs)"}
 
+    # ---- SSSP (NEXT-1; BASELINE configs[3] "BFS and SSSP with synthetic
+    # weights"): frontier Bellman-Ford over the EFG, fp32 weights (reading C20) ----
+    sssp = None
+    if world == 1 and args.sssp:
+        n3, s3, d3, _ = make_graph_edges(args.config, args.scale)
+        w3 = synth.weights(s3, d3, 2000 + args.config)
+        g3 = efg.Graph.build(n3, s3, d3, device=local, stream=stream.cuda_stream, flags=flags, weights=w3)
+        del s3, d3, w3
+        dist_d = torch.empty(n, dtype=torch.float32, device=dev)
+        with torch.cuda.stream(stream):
+            g3.sssp(int(my[0]), dist=dist_d)  # warm-up
+        torch.cuda.synchronize()
+        q0 = torch.cuda.Event(enable_timing=True)
+        q1 = torch.cuda.Event(enable_timing=True)
+        relaxed, iters, nsrc = 0, 0, min(3, len(stats))
+        q0.record(stream)
+        with torch.cuda.stream(stream):
+            for s, _ in stats[:nsrc]:
+                _, sst = g3.sssp(s, dist=dist_d, stats=True)
+                relaxed += sst["edges_relaxed"]
+                iters += sst["iterations"]
+        q1.record(stream)
+        torch.cuda.synchronize()
+        qms = q0.elapsed_time(q1)
+        sssp = {"sources": nsrc, "ms_per_source": qms / nsrc, "iterations_per_source": iters / nsrc,
+                "edges_relaxed_per_source": relaxed / nsrc,
+                "gteps_reached_edges": nsrc * float(np.mean([st["edges_traversed"] for _, st in stats[:nsrc]]))
+                / (qms * 1e-3) / 1e9,
+                "relax_gteps": relaxed / (qms * 1e-3) / 1e9,
+                "note": "frontier Bellman-Ford, fp32 __fadd_rn + int-punned atomicMin; bit-exact vs fp32 "
+                        "Dijkstra in tests"}
+        g3.free()
+
     # ---- cpu baseline: the oracle on a bounded sample (rank 0, N=1 only) ----
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
@@ -570,6 +605,7 @@ def main():
             "alt_no_reorder": alt,
             "alt_no_prefix_skip": alt_ns,
             "pagerank": pr,
+            "sssp": sssp,
         }
         print(json.dumps(line), flush=True)
     g.free()

@@ -235,7 +235,10 @@ class Graph:
             dist = np.empty(n, np.float32)
         st = _abi.Stats() if stats else None
         check(lib.efg_sssp(self._h, source, _ptr(dist), C.byref(st) if st else None), "efg_sssp")
-        return dist
+        if not stats:
+            return dist
+        return dist, {"iterations": st.levels, "edges_relaxed": st.edges_traversed,
+                      "device_ms": st.device_ms}
 
     def pagerank(self, damping: float = 0.85, iters: int = 50, rank=None):
         n = self.info["n"]

@@ -242,15 +242,23 @@ def test_stats_levels(efg):
 @pytest.mark.slow
 def test_c2_rmat24_full_size(efg):
     # BASELINE.json configs[1] at full size, bench launch configuration
+    # (degree relabelling + prefix/list skip, as bench.py times it; then the
+    # input order and the full decode)
     n, src, dst = synth.config_edges(2)
-    g = efg.Graph.build(n, src, dst)
     ov, oe = oracle.csr_build(n, src, dst)
-    del src, dst
     deg = np.diff(ov)
     srcs = synth.sources(n, 2, seed=1002, nonisolated_mask=deg > 0)
-    for s in np.concatenate([[0], srcs]):
-        d = g.bfs(int(s))
-        assert np.array_equal(d, oracle.bfs(ov, oe, int(s)))
+    refs = {int(s): oracle.bfs(ov, oe, int(s)) for s in np.concatenate([[0], srcs])}
+    g = efg.Graph.build(n, src, dst, flags=efg.EFG_DEFAULT_FLAGS | efg.EFG_REORDER_DEGREE)
+    for s, ref in refs.items():
+        assert np.array_equal(g.bfs(s), ref)
+    g.set_prefix_skip(False)
+    assert np.array_equal(g.bfs(int(srcs[0])), refs[int(srcs[0])])
+    g.free()
+    g = efg.Graph.build(n, src, dst)
+    del src, dst
+    for s, ref in refs.items():
+        assert np.array_equal(g.bfs(s), ref)
     # decode of sampled vertex ranges (hubs and tail)
     for a, b in [(0, 64), (n // 2, n // 2 + 4096), (n - 5000, n)]:
         assert np.array_equal(g.decode(a, b), oe[ov[a]:ov[b]])
