@@ -177,6 +177,11 @@ typedef struct efg_stats {
  * 0xFFFFFFFF.  depth / parent: host or device, n entries, caller-allocated.
  * With a partitioned handle the call is collective over the communicator:
  * every rank calls it with the same source and receives the full depth array.
+ * Completion: with device outputs (depth and parent, if any) and st == NULL
+ * the call only enqueues the BFS on the handle's stream (efg_build_opts
+ * stream) and returns; the outputs are valid once that stream is
+ * synchronised (stream order, as cudaMemcpyAsync).  Otherwise it returns with
+ * the outputs written.
  * Errors: EFG_ERANGE (source >= n), EFG_ESTATE, EFG_ECUDA, EFG_ENCCL.
  */
 efg_status efg_bfs(efg_graph *g, uint32_t source, int32_t *depth, uint32_t *parent,

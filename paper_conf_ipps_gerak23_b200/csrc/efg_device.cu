@@ -427,6 +427,23 @@ efg_status device_bfs(efg_graph *g, uint32_t source, int32_t *depth, uint32_t *p
     const bool graph_mode = d.level_loop == 0;
     if (graph_mode) EFG_TRY(build_loop_graph(d, mode));
 
+    // device outputs and no statistics: enqueue the whole BFS on the handle's
+    // stream and return (stream-ordered, like cudaMemcpyAsync); back-to-back
+    // calls then run without a host round trip in between
+    if (graph_mode && !st && depth_dev && (!parent || parent_dev)) {
+        uint32_t launches = 0;
+        if (relabel)
+            CUDA_TRY(cudaMemsetAsync(d.depth_st, 0xFF, d.n * 4, s));
+        else
+            CUDA_TRY(cudaMemsetAsync(dd, 0xFF, d.n * 4, s));
+        if (pd) CUDA_TRY(cudaMemsetAsync(pd, 0xFF, d.n * 4, s));
+        EFG_TRY(start_traversal(d, source, (uint64_t)source + 1, dd, pd, launches));
+        CUDA_TRY(cudaGraphLaunch(d.loop_exec[mode], s));
+        if (relabel) CUDA_TRY(launch_map_depth(d.depth_st, d.new_of_old, dd, d.n, s));
+        if (parent && relabel) CUDA_TRY(launch_map_parent(pd, d.old_of_new, pout, d.n, s));
+        return EFG_OK;
+    }
+
     cudaEvent_t ev0, ev1;
     CUDA_TRY(cudaEventCreate(&ev0));
     CUDA_TRY(cudaEventCreate(&ev1));
