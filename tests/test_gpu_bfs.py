@@ -294,6 +294,21 @@ def test_long_path_many_levels(efg):
     g.free()
 
 
+@pytest.mark.parametrize("plen", [125, 126, 127, 128, 300])
+def test_host_depth_transfer_levels_boundary(efg, plen):
+    """Host depth arrays cross PCIe as 1 byte per vertex only while every depth
+    fits [-1, 126]: paths around the boundary, plus unreached vertices (-1)."""
+    n = 5000
+    src = np.arange(plen - 1, dtype=np.uint32)
+    g = efg.Graph.build(n, src, src + 1)
+    d, _, st = g.bfs(0, stats=True)
+    ref = np.full(n, -1, np.int32)
+    ref[:plen] = np.arange(plen)
+    assert np.array_equal(d, ref)
+    assert st["d2h_bytes"] == (n if plen < 127 else 4 * n)
+    g.free()
+
+
 def test_reorder_degree_bfs_in_input_ids(efg):
     n, src, dst = synth.rmat(14, 16, seed=11)
     g = efg.Graph.build(n, src, dst, flags=efg.EFG_DEFAULT_FLAGS | efg.EFG_REORDER_DEGREE)
