@@ -257,23 +257,6 @@ __global__ void xchg_kernel(XchgArgs a)
 // reduced into ctrl->vmin2[level & 1], which the next expand reads; the
 // other slot is reset for the following level end.
 // --------------------------------------------------------------------------
-// cp.async (LDGSTS) 16 B global -> shared, zero-filled beyond src_size (0 or 16)
-__device__ __forceinline__ void cp_async16_zfill(void *dst, const void *src, uint32_t src_size)
-{
-    asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(
-                     static_cast<uint32_t>(__cvta_generic_to_shared(dst))),
-                 "l"(src), "r"(src_size)
-                 : "memory");
-}
-
-__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
-
-template <int N>
-__device__ __forceinline__ void cp_async_wait()
-{
-    asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory");
-}
-
 // Grid-wide barrier of a persistent grid (every block resident): a 64-bit
 // arrival counter that only grows (each barrier adds gridDim.x), release on
 // arrival, acquire while polling with a short back-off.
@@ -347,7 +330,6 @@ __global__ void __launch_bounds__(kFrontierThreads, 2) frontier_kernel(FrontierA
     constexpr int NT = kFrontierThreads, NW = NT / 32;
     __shared__ uint64_t s_q[NW], s_wk[NW], s_ch[NW], s_sk[NW], s_bg[NW], s_all[NW];
     __shared__ uint64_t s_pre[5], s_tot[5];
-    __shared__ __align__(16) uint4 s_rec[NW][2][2][32];  // phase 2: record staging, 2 stages x 2 words per warp
 
     const uint32_t tid = threadIdx.x, lane = tid & 31, wid = tid >> 5, b = blockIdx.x;
 #define FTRACE(p)                                                      \
@@ -518,7 +500,6 @@ __global__ void __launch_bounds__(kFrontierThreads, 2) frontier_kernel(FrontierA
     // lists go to the BigList table (phase 3) ----
     const bool narrow = a.k == 0 || a.k >= 32;  // per-lane work < 2^27: 32-bit scans
     constexpr int kS = 2;                         // non-empty words planned together
-    static_assert(kS == 2, "s_rec is sized for 2 words per pipeline stage");
     for (uint64_t w0 = 32ull * gw; w0 < a.nwords; w0 += WG) {
         const uint64_t w = w0 + lane;
         uint32_t nb = 0, skw = 0;
@@ -539,64 +520,28 @@ __global__ void __launch_bounds__(kFrontierThreads, 2) frontier_kernel(FrontierA
         const bool own = w >= a.own_lo_w && w < a.own_hi_w;
         const uint32_t nq = own ? nb & ~skw : 0u;
         uint32_t todo = __ballot_sync(FULL, nb != 0);
-        // software pipeline over pairs of non-empty words: the records of the
-        // next pair travel global -> shared (cp.async, zero-filled where a
-        // bit is clear; no registers held) while the current pair is planned
-        auto take = [&](uint32_t (&jj)[kS]) {
-#pragma unroll
-            for (int u = 0; u < kS; ++u) {
-                jj[u] = 32;
-                if (todo) {
-                    jj[u] = __ffs(todo) - 1;
-                    todo &= todo - 1;
-                }
-            }
-        };
-        auto issue = [&](const uint32_t (&jj)[kS], uint32_t stg) {
-#pragma unroll
-            for (int u = 0; u < kS; ++u)
-                if (jj[u] < 32) {
-                    const uint32_t bits = __shfl_sync(FULL, nq, jj[u]);
-                    const bool on = (bits >> lane) & 1;
-                    const VRec *src = on ? a.rec + (w0 + jj[u]) * 32 + lane : a.rec;
-                    cp_async16_zfill(&s_rec[wid][stg][u][lane], src, on ? 16u : 0u);
-                }
-            cp_async_commit();
-        };
-        uint32_t jn[kS], stg = 0;
-        take(jn);
-        if (jn[0] < 32) issue(jn, 0);
-        while (jn[0] < 32) {
+        while (todo) {
             uint32_t jw[kS], bq[kS], wl[kS], nc[kS];
             uint4 rv[kS];
 #pragma unroll
-            for (int u = 0; u < kS; ++u) jw[u] = jn[u];
-            take(jn);
-            if (jn[0] < 32) {
-                issue(jn, stg ^ 1);
-                cp_async_wait<1>();
-            } else {
-                cp_async_wait<0>();
-            }
-            __syncwarp();
-#pragma unroll
             for (int u = 0; u < kS; ++u) {
+                jw[u] = 32;
                 bq[u] = 0;
                 rv[u] = make_uint4(0, 0, 0, 0);
-                if (jw[u] < 32) {
-                    const uint32_t j = jw[u];
+                if (todo) {
+                    const int j = __ffs(todo) - 1;
+                    todo &= todo - 1;
+                    jw[u] = j;
                     bq[u] = __shfl_sync(FULL, nq, j);
                     const uint32_t bb = __shfl_sync(FULL, nb, j);
                     const uint32_t v = (uint32_t)((w0 + j) * 32 + lane);
-                    rv[u] = s_rec[wid][stg][u][lane];
+                    if ((bq[u] >> lane) & 1) rv[u] = __ldg(reinterpret_cast<const uint4 *>(a.rec + v));
                     if ((bb >> lane) & 1) {
                         if (a.depth_stored) a.depth_stored[v] = (int32_t)level;  // stored-id order (coalesced)
                         if (!a.depth_stored_only && depth) depth[v] = (int32_t)level;
                     }
                 }
             }
-            __syncwarp();  // stage stg is refilled two pairs later
-            stg ^= 1;
             // per-list work nch*CW + d < 2^31.1 (deg < 2^26); the 32-lane sums fit
             // 32 bits when k >= 32 (< 2^27 per list), else the work is scanned
             // as (w >> 5, w & 31)
