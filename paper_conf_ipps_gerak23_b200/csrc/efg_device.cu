@@ -340,7 +340,7 @@ efg_status device_upload(efg_graph *g, const efg_build_opts &o)
     CUDA_TRY(cudaMallocHost(reinterpret_cast<void **>(&d.ctrl_host), sizeof(LevelCtrl)));
     CUDA_TRY(cudaMallocHost(reinterpret_cast<void **>(&d.stats_host), kMaxLevelStats * sizeof(LevelStat)));
     // persistent grids of the frontier kernels: 2 blocks per SM, whole bitmap words
-    d.frontier_blocks = (unsigned)std::min<uint64_t>(2 * (uint64_t)d.num_sms, kMaxGrid);
+    d.frontier_blocks = (unsigned)std::min<uint64_t>((1024 / kFrontierThreads) * (uint64_t)d.num_sms, kMaxGrid);
     if (const char *e = std::getenv("EFG_FRONTIER_BLOCKS"))  // tuning knob (blocks of compact / plan)
         d.frontier_blocks = (unsigned)std::max(1, std::min(atoi(e), (int)kMaxGrid));
     const uint64_t per = (d.nwords + d.frontier_blocks - 1) / d.frontier_blocks;

@@ -141,7 +141,10 @@ constexpr uint32_t kRoundWords = EFG_ROUND_WORDS;        // upper-bit words deco
 #define EFG_HOT_WORDS 4
 #endif
 constexpr uint32_t kHotWords = EFG_HOT_WORDS;     // > 4: shared-memory visited snapshot of the first 32*kHotWords ids (off: vpre covers the visited prefix)
-constexpr int kFrontierThreads = 512;        // frontier_kernel (16 warps)
+#ifndef EFG_FRONTIER_THREADS
+#define EFG_FRONTIER_THREADS 256
+#endif
+constexpr int kFrontierThreads = EFG_FRONTIER_THREADS;  // frontier_kernel (8 warps; 1024 threads per SM)
 constexpr int kBitmapAlign = 1024;           // bitmap words are padded to a multiple of this
 // Step a3 partitions "work units" rather than bare edges: a chunk costs
 // kChunkWork units (descriptor, staging, set-up) plus one per element, so a

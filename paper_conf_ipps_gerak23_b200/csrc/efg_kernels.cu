@@ -325,7 +325,7 @@ __device__ __forceinline__ void warp_excl_u32_n(uint32_t (&x)[N], uint32_t (&tot
     }
 }
 
-__global__ void __launch_bounds__(kFrontierThreads, 2) frontier_kernel(FrontierArgs a)
+__global__ void __launch_bounds__(kFrontierThreads, 1024 / kFrontierThreads) frontier_kernel(FrontierArgs a)
 {
     constexpr int NT = kFrontierThreads, NW = NT / 32;
     __shared__ uint64_t s_q[NW], s_wk[NW], s_ch[NW], s_sk[NW], s_bg[NW], s_all[NW];
@@ -499,7 +499,10 @@ __global__ void __launch_bounds__(kFrontierThreads, 2) frontier_kernel(FrontierA
     // descriptors (a4) and tile boundaries (a3) of single-chunk lists; longer
     // lists go to the BigList table (phase 3) ----
     const bool narrow = a.k == 0 || a.k >= 32;  // per-lane work < 2^27: 32-bit scans
-    constexpr int kS = 2;                         // non-empty words planned together
+#ifndef EFG_KS
+#define EFG_KS 3
+#endif
+    constexpr int kS = EFG_KS;                    // non-empty words planned together
     for (uint64_t w0 = 32ull * gw; w0 < a.nwords; w0 += WG) {
         const uint64_t w = w0 + lane;
         uint32_t nb = 0, skw = 0;
