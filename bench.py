@@ -20,8 +20,12 @@ rows a1-a7) from one seeded source over the BASELINE.json configs[1] graph
 
 ``--impl reference`` runs the reference arm: the oracle, as it stands, on the
 host cores, same config/metric (each step = one oracle BFS).
-With N > 1 (torchrun) ranks run disjoint seeded sources (independent BFS
-problems, no data-path collective): "scaling": "weak".
+With N > 1 (torchrun) the default is the north_star's 1-D row partition: each
+rank holds a byte-balanced row range of the EFG, every BFS level exchanges the
+new-vertex bitmap (all_to_all + OR + all_gather over NCCL), "scaling":
+"strong"; ``--mode replicas`` runs independent BFS problems per rank on
+disjoint sources (no data-path collective, "scaling": "weak").
+Also reported on one GPU: PageRank (50 iterations) and SSSP over the same graph.
 """
 from __future__ import annotations
 
@@ -58,8 +62,8 @@ def parse():
     p.add_argument("--reorder", default="degree", choices=["none", "degree"],
                    help="EFG_REORDER_DEGREE relabelling at build time (results stay in input ids)")
     p.add_argument("--profile-levels", action="store_true", help="print per-level stats to stderr")
-    p.add_argument("--sssp", action="store_true",
-                   help="also time SSSP (NEXT-1) over the same graph built with synthetic weights")
+    p.add_argument("--no-sssp", action="store_true",
+                   help="skip the SSSP (NEXT-1) timing over the same graph built with synthetic weights")
     p.add_argument("--no-pagerank", action="store_true",
                    help="skip the PageRank measurement (BASELINE configs[1]: BFS and PageRank)")
     return p.parse_args()
@@ -521,7 +525,7 @@ def main():
     # ---- SSSP (NEXT-1; BASELINE configs[3] "BFS and SSSP with synthetic
     # weights"): frontier Bellman-Ford over the EFG, fp32 weights (reading C20) ----
     sssp = None
-    if world == 1 and args.sssp:
+    if world == 1 and not args.no_sssp:
         n3, s3, d3, _ = make_graph_edges(args.config, args.scale)
         w3 = synth.weights(s3, d3, 2000 + args.config)
         g3 = efg.Graph.build(n3, s3, d3, device=local, stream=stream.cuda_stream, flags=flags, weights=w3)
