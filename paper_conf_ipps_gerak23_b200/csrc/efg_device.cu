@@ -468,6 +468,8 @@ efg_status device_bfs(efg_graph *g, uint32_t source, int32_t *depth, uint32_t *p
         CUDA_TRY(cudaMemcpyAsync(d.ctrl_host, d.ctrl, sizeof(LevelCtrl), cudaMemcpyDeviceToHost, s));
         CUDA_TRY(cudaStreamSynchronize(s));
         levels = d.ctrl_host->nlevels;
+        if (d.ctrl_host->fault)
+            return set_error(EFG_ECUDA, "frontier_kernel: grid barrier timed out (grid not co-resident)");
         const uint32_t ns = std::min(levels, kMaxLevelStats);
         if (ns) {
             CUDA_TRY(cudaMemcpyAsync(d.stats_host, d.stats, ns * sizeof(LevelStat), cudaMemcpyDeviceToHost, s));
@@ -486,6 +488,7 @@ efg_status device_bfs(efg_graph *g, uint32_t source, int32_t *depth, uint32_t *p
             CUDA_TRY(cudaMemcpyAsync(d.ctrl_host, d.ctrl, sizeof(LevelCtrl), cudaMemcpyDeviceToHost, s));
             CUDA_TRY(cudaStreamSynchronize(s));
             const LevelCtrl c = *d.ctrl_host;
+            if (c.fault) return set_error(EFG_ECUDA, "frontier_kernel: grid barrier timed out (grid not co-resident)");
             if (c.nf == 0) break;
             lf.push_back(c.nf);
             le.push_back(c.ne);

@@ -97,6 +97,7 @@ struct LevelCtrl {
     uint32_t vmin2[2];  // frontier_kernel of level L: smallest vertex neither visited nor isolated, in
                         // slot L & 1 (atomicMin); the expand of level L reads it as its visited prefix
     uint32_t vpre_used; // visited prefix the last BFS expand used (0: none); lower bound for the next level end
+    uint32_t fault;     // a frontier_kernel grid barrier timed out (sticky; reported by the host)
 };
 
 // A frontier list whose chunk descriptors and tile boundaries are written by

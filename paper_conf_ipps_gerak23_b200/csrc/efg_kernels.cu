@@ -260,7 +260,10 @@ __global__ void xchg_kernel(XchgArgs a)
 // Grid-wide barrier of a persistent grid (every block resident): a 64-bit
 // arrival counter that only grows (each barrier adds gridDim.x), release on
 // arrival, acquire while polling with a short back-off.
-__device__ __forceinline__ void grid_barrier(unsigned long long *count)
+// A barrier that has waited 4 s (a grid that is not co-resident, e.g. another
+// kernel holding SMs forever) gives up and raises ctrl->fault, which the host
+// reports as an error, instead of hanging the device.
+__device__ __forceinline__ void grid_barrier(unsigned long long *count, uint32_t *fault)
 {
     __syncthreads();
     if (threadIdx.x == 0) {
@@ -268,11 +271,16 @@ __device__ __forceinline__ void grid_barrier(unsigned long long *count)
         unsigned long long old;
         asm volatile("atom.add.release.gpu.global.u64 %0, [%1], 1;" : "=l"(old) : "l"(count) : "memory");
         const unsigned long long target = (old / gridDim.x + 1) * gridDim.x;
-        for (;;) {
+        const unsigned long long t0 = globaltimer();
+        for (uint32_t it = 0;; ++it) {
             unsigned long long cur;
             asm volatile("ld.acquire.gpu.global.u64 %0, [%1];" : "=l"(cur) : "l"(count) : "memory");
             if (cur >= target) break;
             __nanosleep(32);
+            if ((it & 1023) == 1023 && globaltimer() - t0 > 4000000000ull) {
+                atomicExch(fault, 1u);
+                break;
+            }
         }
         __threadfence();
     }
@@ -448,7 +456,7 @@ __global__ void __launch_bounds__(kFrontierThreads, 1024 / kFrontierThreads) fro
         const uint64_t blk_all = warp_sum_u64(lane < NW ? s_all[lane] : 0);
         if (lane == 0 && blk_all) atomicAdd(reinterpret_cast<unsigned long long *>(&ctrl->nnew), blk_all);
     }
-    grid_barrier(a.barrier);
+    grid_barrier(a.barrier, &ctrl->fault);
     if (wid < 5) {
         uint64_t pre, tot;
         sum_published(a.status + wid * kMaxGrid, b, pre, tot);
@@ -619,7 +627,7 @@ __global__ void __launch_bounds__(kFrontierThreads, 1024 / kFrontierThreads) fro
     }
     FTRACE(5);
     if (nbig == 0) return;  // grid-uniform: no long list this level
-    grid_barrier(a.barrier);
+    grid_barrier(a.barrier, &ctrl->fault);
     FTRACE(6);
 
     // ---- 3: the long lists, one per lane (lists of > 8 chunks or tiles: one
