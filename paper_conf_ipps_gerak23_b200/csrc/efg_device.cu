@@ -79,6 +79,7 @@ ExpandArgs expand_args(DeviceGraph &d, uint32_t *out)
     ExpandArgs a;
     a.data = d.data;
     a.chunks = d.chunks;
+    a.cvtx = d.cvtx;
     a.tiles = d.tiles;
     a.deg32 = d.deg32;
     a.ctrl = d.ctrl;
@@ -118,6 +119,7 @@ FrontierArgs frontier_args(DeviceGraph &d, cudaGraphConditionalHandle cond, bool
 #endif
     a.rec = d.rec;
     a.chunks = d.chunks;
+    a.cvtx = d.cvtx;
     a.tiles = d.tiles;
     a.ctrl = d.ctrl;
     a.status = d.status;
@@ -214,6 +216,7 @@ void device_free(DeviceGraph &d)
     cudaFree(d.prev);
     cudaFree(d.tiles);
     cudaFree(d.chunks);
+    cudaFree(d.cvtx);
     cudaFree(d.depth);
     cudaFree(d.parent);
     cudaFree(d.parent2);
@@ -254,6 +257,8 @@ efg_status device_upload(efg_graph *g, const efg_build_opts &o)
 
     // EF data, padded so 32-bit word reads past the last list stay in bounds
     d.data_bytes = h.data.size();
+    if (d.data_bytes >= (1ull << kOffBits))
+        return set_error(EFG_ENOTSUP, "efg_build: EF data of 1 TiB or more is not supported on the device");
     const uint64_t padded = ((d.data_bytes + 64) + 15) & ~15ull;
     EFG_TRY(dev_alloc(d, &d.data, padded));
     CUDA_TRY(cudaMemsetAsync(d.data, 0, padded, s));
@@ -323,6 +328,7 @@ efg_status device_upload(efg_graph *g, const efg_build_opts &o)
     d.max_tiles = (h.m + (uint64_t)kChunkWork * d.max_chunks) / kTileWork + 2;
     EFG_TRY(dev_alloc(d, &d.tiles, d.max_tiles + 1));
     EFG_TRY(dev_alloc(d, &d.chunks, d.max_chunks));
+    EFG_TRY(dev_alloc(d, &d.cvtx, d.max_chunks));
     EFG_TRY(dev_alloc(d, &d.depth, h.n));
     EFG_TRY(dev_alloc(d, &d.status, 5 * kMaxGrid + 1));  // + the grid-barrier counter
     CUDA_TRY(cudaMemsetAsync(d.status, 0, (5 * kMaxGrid + 1) * 8, s));

@@ -56,27 +56,28 @@ efg_status build_host(uint64_t n, uint64_t m, const uint32_t *src, const uint32_
 // Packed 16-byte vertex record: one aligned 128-bit load gives everything the
 // frontier step a1 needs (degree, data offset, l, upper-section length).
 struct alignas(16) VRec {
-    uint64_t off_l;   // bits 0..57: offsets[v] (byte offset in data); bits 58..63: l
+    uint64_t off_l;   // bits 0..39: offsets[v] (byte offset in data); bits 40..45: l; 46..63: 0
     uint32_t deg;     // vlist[v+1]-vlist[v]
     uint32_t ubytes;  // upper-bits section length in bytes
 };
 static_assert(sizeof(VRec) == 16, "VRec must be 16 bytes");
 
-constexpr int kOffBits = 58;
+constexpr int kOffBits = 40;                            // data byte offsets < 2^40 (1 TiB)
 constexpr uint64_t kOffMask = (1ull << kOffBits) - 1;
+constexpr int kCcShift = 46;                            // ChunkDesc: chunk index above l
 
 // Chunk descriptor (step a1, written by frontier_kernel, read by expand_kernel):
 // one k-aligned piece of a frontier vertex's list.  The expand
 // kernel derives the chunk's bit ranges from it and the forward pointers (a4).
 struct alignas(16) ChunkDesc {
-    uint64_t off_l;  // the list's VRec.off_l: byte offset in data (58 bits) | l << 58
-    uint32_t deg;    // list length
-    uint32_t ubytes; // upper-bits section bytes of the list
-    uint32_t v;      // source vertex (stored id)
-    uint32_t cc;     // chunk index within the list (rank of its first element r0 = cc*k)
-    uint32_t pad[2];
+    uint64_t off_l_cc;  // the list's VRec.off_l (offset: 40 bits, l: bits 40-45) | chunk index cc << 46
+                        // (rank of the chunk's first element r0 = cc*k; cc < 2^17 for deg < 2^26)
+    uint32_t deg;       // list length
+    uint32_t ubytes;    // upper-bits section bytes of the list
 };
-static_assert(sizeof(ChunkDesc) == 32, "ChunkDesc must be 32 bytes");
+static_assert(sizeof(ChunkDesc) == 16, "ChunkDesc must be 16 bytes");
+// The chunk's source vertex lives in a parallel array (cvtx), read only by the
+// modes that need it (parents, decode, SSSP, PageRank): a BFS moves 16 B per chunk.
 
 // Level control block (device), written by the advance kernel.
 struct LevelCtrl {
@@ -182,6 +183,7 @@ struct DeviceGraph {
     uint32_t *tiles = nullptr;         // tile table: first chunk of each tile (max_tiles + 1)
     uint64_t max_tiles = 0;
     ChunkDesc *chunks = nullptr;       // chunk descriptors of the level (max_chunks)
+    uint32_t *cvtx = nullptr;          // source vertex of each chunk (max_chunks)
     uint64_t max_chunks = 0;
     int32_t *depth = nullptr;          // internal depth (n)
     uint32_t *parent = nullptr;        // internal parent (n), lazily allocated

@@ -595,10 +595,9 @@ __global__ void __launch_bounds__(kFrontierThreads, 1024 / kFrontierThreads) fro
                 const uint64_t wlen = (uint64_t)nch * CW + d;
                 const bool big = mine && (nch > 1 || wlen > kTileWork);
                 if (mine && !big) {
-                    if (nch == 1) {  // a4: the list's only chunk
-                        uint4 *dp = reinterpret_cast<uint4 *>(a.chunks + C);
-                        dp[0] = make_uint4(rv[u].x, rv[u].y, d, ub);
-                        dp[1] = make_uint4((uint32_t)((w0 + jw[u]) * 32 + lane), 0u, 0u, 0u);
+                    if (nch == 1) {  // a4: the list's only chunk (cc = 0)
+                        *reinterpret_cast<uint4 *>(a.chunks + C) = make_uint4(rv[u].x, rv[u].y, d, ub);
+                        a.cvtx[C] = (uint32_t)((w0 + jw[u]) * 32 + lane);
                     }
                     // a3: a tile boundary t*T inside [W, W + wlen) starts at this chunk or the next
                     const uint64_t t = (W + kTileWork - 1) / kTileWork;
@@ -663,9 +662,9 @@ __global__ void __launch_bounds__(kFrontierThreads, 1024 / kFrontierThreads) fro
         const bool huge = nch > 8 || t_hi - t_lo > 8;
         if (!huge) {
             for (uint32_t j = 0; j < nch; ++j) {
-                uint4 *dp = reinterpret_cast<uint4 *>(a.chunks + cs + j);
-                dp[0] = make_uint4((uint32_t)off_l, (uint32_t)(off_l >> 32), d, ub);
-                dp[1] = make_uint4(v, j, 0u, 0u);
+                const uint64_t oc = off_l | ((uint64_t)j << kCcShift);
+                *reinterpret_cast<uint4 *>(a.chunks + cs + j) = make_uint4((uint32_t)oc, (uint32_t)(oc >> 32), d, ub);
+                a.cvtx[cs + j] = v;
             }
             for (uint64_t t = t_lo; t < t_hi; ++t)
                 a.tiles[t] = (uint32_t)(cs + tile_chunk((uint32_t)(t * kTileWork - W), nch));
@@ -679,9 +678,9 @@ __global__ void __launch_bounds__(kFrontierThreads, 1024 / kFrontierThreads) fro
             const uint32_t od = __shfl_sync(FULL, d, o), oub = __shfl_sync(FULL, ub, o);
             const uint32_t ov = __shfl_sync(FULL, v, o), onch = __shfl_sync(FULL, nch, o);
             for (uint32_t j = lane; j < onch; j += 32) {
-                uint4 *dp = reinterpret_cast<uint4 *>(a.chunks + ocs + j);
-                dp[0] = make_uint4((uint32_t)ooff, (uint32_t)(ooff >> 32), od, oub);
-                dp[1] = make_uint4(ov, j, 0u, 0u);
+                const uint64_t oc = ooff | ((uint64_t)j << kCcShift);
+                *reinterpret_cast<uint4 *>(a.chunks + ocs + j) = make_uint4((uint32_t)oc, (uint32_t)(oc >> 32), od, oub);
+                a.cvtx[ocs + j] = ov;
             }
             const uint64_t owl = (uint64_t)onch * CW + od;
             const uint64_t ot_lo = (oW + kTileWork - 1) / kTileWork, ot_hi = (oW + owl + kTileWork - 1) / kTileWork;
@@ -923,14 +922,13 @@ __global__ void __launch_bounds__(kExpandThreads, 1) expand_kernel(ExpandArgs a)
         uint64_t lb = 0, A0 = 0, A1 = 0;
         uint32_t l = 0, nel = 0, hib = 0, v = 0, cc = 0;
         if (valid) {
-            const uint4 *dp = reinterpret_cast<const uint4 *>(a.chunks + c);
-            const uint4 d0 = dp[0], d1 = dp[1];
+            const uint4 d0 = *reinterpret_cast<const uint4 *>(a.chunks + c);
             const uint64_t offl = ((uint64_t)d0.y << 32) | d0.x;
             const uint64_t off = offl & kOffMask;
             const uint32_t deg = d0.z, ubytes = d0.w;
-            l = (uint32_t)(offl >> kOffBits);
-            v = d1.x;
-            cc = d1.y;
+            l = (uint32_t)(offl >> kOffBits) & 63;
+            cc = (uint32_t)(offl >> kCcShift);
+            if (MODE != kModeVisit) v = a.cvtx[c];
             const uint64_t F = a.k ? (kpow2 ? (uint64_t)(deg >> kshift) : (uint64_t)deg / a.k) : 0;  // forward pointers (C8)
             const uint64_t Lb = ((uint64_t)deg * l + 7) >> 3;            // lower section bytes
             const uint64_t lbase = (off + 4 * F) * 8;

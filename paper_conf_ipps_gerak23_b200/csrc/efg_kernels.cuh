@@ -19,6 +19,7 @@ enum ExpandMode : int {
 struct ExpandArgs {
     const uint8_t *data;       // EF data (device, 4-byte aligned, padded)
     const ChunkDesc *chunks;   // chunk descriptors of the level (frontier_kernel)
+    const uint32_t *cvtx;      // source vertex of each chunk (modes other than plain BFS)
     const uint32_t *tiles;     // tile table: first chunk of tile t (ntiles + 1 entries)
     const uint32_t *deg32;     // degrees (PageRank share)
     LevelCtrl *ctrl;           // nf, ne, ntiles of this level; parent pointer; level
@@ -69,6 +70,7 @@ struct FrontierArgs {           // level end (a7) + next level plan (a1-a4), one
     uint32_t *skipw;           // scratch (nwords): per bitmap word, the skipped lists (phase 1 -> phase 2)
     const VRec *rec;           // vertex records (pass 2)
     ChunkDesc *chunks;         // out: chunk descriptors
+    uint32_t *cvtx;            // out: source vertex of each chunk
     uint32_t *tiles;           // out: first chunk of each tile (+ sentinel)
     LevelCtrl *ctrl;           // in: level, seq, depth ptr; out: nf, ne, nwork, nchunks, ntiles, xlevel, vmin2
     uint64_t *status;          // five per-block aggregate regions of kMaxGrid words
