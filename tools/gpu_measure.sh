@@ -11,7 +11,7 @@ if [ "$2" != "skip-tests" ]; then
   timeout 600 python -c "import __graft_entry__ as g; g.smoke()" > $O/smoke_$TAG.log 2>&1; echo "smoke rc=$?"
 fi
 timeout 900 python bench.py > $O/bench_$TAG.json 2> $O/bench_$TAG.err; echo "bench rc=$?"; tail -1 $O/bench_$TAG.json
-NB="--steps 2 --warmup 1 --no-cpu-baseline --no-alt --no-pagerank"
+NB="--steps 2 --warmup 1 --no-cpu-baseline --no-alt --no-pagerank --no-sssp"
 timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file $O/launches_$TAG.csv \
   python bench.py $NB > /dev/null 2>&1; echo "ncu list rc=$?"
 python tools/launches.py $O/launches_$TAG.csv > $O/launches_${TAG}_summary.txt 2>&1; cat $O/launches_${TAG}_summary.txt
