@@ -2,7 +2,7 @@
 default GPU test run): the CUDA path (bench.py's build: degree relabelling,
 prefix/list skip) against the oracle on the same seeded graph.
 
-  python tools/verify_full.py --config 3 --sources 3 > profiles/r1_verify_c3.json
+  python tests/verify_full.py --config 3 --sources 3 > profiles/r1_verify_c3.json
 
 For every sampled source: depth bit-exact vs the oracle's FIFO BFS over its
 own CSR (oracle.csr_build, no product code).  Prints one JSON line.
