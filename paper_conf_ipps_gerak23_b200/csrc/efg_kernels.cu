@@ -972,8 +972,18 @@ __global__ void __launch_bounds__(kExpandThreads, 1) expand_kernel(ExpandArgs a)
         B.buf = buf;
         nbuf ^= 1;
         uint32_t tot_e, tot_w;
-        B.eb = warp_excl_u32(fits ? nel : 0u, tot_e);
-        B.wb = warp_excl_u32(fits ? nwd : 0u, tot_w);
+        if (kpow2 && a.k <= 1024) {
+            // one scan for both: a batch holds < 2^15 elements and < 2^16 words
+            uint32_t t;
+            const uint32_t ex = warp_excl_u32(fits ? (nel | nwd << 16) : 0u, t);
+            B.eb = ex & 0xffffu;
+            B.wb = ex >> 16;
+            tot_e = t & 0xffffu;
+            tot_w = t >> 16;
+        } else {
+            B.eb = warp_excl_u32(fits ? nel : 0u, tot_e);
+            B.wb = warp_excl_u32(fits ? nwd : 0u, tot_w);
+        }
         const uint32_t tot_b = __shfl_sync(FULL, sb + bytes, B.cnt - 1);  // bytes of the fitting prefix
         B.ne = tot_e;
         B.nw = tot_w;
