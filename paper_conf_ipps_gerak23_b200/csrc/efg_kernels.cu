@@ -1088,9 +1088,16 @@ __global__ void __launch_bounds__(kExpandThreads, 1) expand_kernel(ExpandArgs a)
                 const uint32_t hb = 32 * g + sp.HB - (run + ex);
                 bool keep = wd != 0;
                 uint32_t kex = ex, ktot = tot;  // kept-element prefix (= all without the skip)
+                const uint32_t nzm = __ballot_sync(FULL, wd != 0);
                 if (pskip) {
                     keep = keep && hb + (31 - __clz(wd)) - (pc - 1) >= (vpre >> l);
-                    kex = warp_excl_u32(keep ? pc : 0u, ktot);
+                    const uint32_t km0 = __ballot_sync(FULL, keep);
+                    if (km0 == 0) {  // every word of these 32 skipped
+                        kex = 0;
+                        ktot = 0;
+                    } else if (km0 != nzm) {  // some skipped: scan the kept popcounts
+                        kex = warp_excl_u32(keep ? pc : 0u, ktot);
+                    }
                 }
                 const uint32_t km = __ballot_sync(FULL, keep);
                 if (keep) {
