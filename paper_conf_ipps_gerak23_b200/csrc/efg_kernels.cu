@@ -708,21 +708,22 @@ __global__ void __launch_bounds__(kFrontierThreads, 1024 / kFrontierThreads) fro
 //   (rounds)    lays the batch's upper-bit words end to end (kRoundWords per
 //               round), masks each chunk's first/last word and keeps the
 //               non-zero words as 16-byte records {word, hi base, lower-field
-//               base, l} with the popcount prefix of each (the rank of its
-//               first stop bit: the segmented scan of P:171-177, segments =
-//               chunks);
-//   (decode)    a5: splits the round's elements evenly over the lanes; a lane
-//               finds select1 of its first element once (maxle over the record
-//               prefix, Fig. 4 rule, then an in-word select) and walks its run
-//               serially: the next set bit (ffs) gives select1(i) - i, the lower
-//               field is a funnel shift of two shared-memory words, x = hi << l
-//               | lo; an exhausted word is refilled from the next record without
-//               a branch (every record has a set bit);
-//   (visit)     a6: kU elements per lane in flight: hot ids answer from a
-//               per-CTA shared-memory copy of their visited bits (a snapshot of
-//               the level start, updated by this CTA's discoveries), the others
-//               probe the global bitmap, and atomicOr decides (stale reads are
-//               benign, C16).
+//               base, l | slot} (bases relative to the record's first stop bit)
+//               with the kept-element prefix of each (the segmented scan of
+//               P:171-177, segments = chunks); BFS prefix skip: a word whose
+//               ids are all below the visited prefix vpre gets no record;
+//   (decode)    a5: splits the round's kept elements evenly over the lanes; a
+//               lane finds select1 of its first element once (maxle over the
+//               record prefix, Fig. 4 rule, then an in-word select) and walks
+//               its run serially: the next set bit (bfind on the reversed word)
+//               gives select1(i) - i, the lower field is a funnel shift of two
+//               shared-memory words, x = hi << l | lo; an exhausted word is
+//               refilled from the next record without a branch (every record
+//               has a set bit);
+//   (visit)     a6: kU elements per lane in flight: ids below vpre are known
+//               visited (register compare), the others probe the global bitmap
+//               and atomicOr decides (stale reads are benign, C16); SSSP relax,
+//               PageRank push / pull and decode use the same walk.
 // --------------------------------------------------------------------------
 struct SlotP {        // one chunk of the batch being decoded (shared memory)
     uint32_t lsmb;    // shared-window bit address of element e's lower field = lsmb + e*l (mod 2^32)
