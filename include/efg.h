@@ -266,6 +266,41 @@ efg_status efg_xchg_unpack(efg_graph *g, int world, const uint64_t *bounds, uint
 efg_status efg_bfs_finish_level(efg_graph *g, uint64_t *global_new);
 efg_status efg_bfs_end(efg_graph *g, efg_stats *st);
 
+/* ---- multi-GPU exchange over peer memory (NVLink / NVSwitch), no NCCL ----
+ *
+ * The same per-level exchange as pack / all-to-all / reduce / all-gather /
+ * unpack (owners OR the P ranks' new bits of their rows, every
+ * rank receives the OR of every owner), done by the library's kernels reading
+ * and writing the other ranks' HBM directly.  Level loop:
+ *   efg_bfs_expand; efg_xchg_peer; efg_bfs_finish_level
+ * Setup, once per handle and partition (collective: every rank, same world):
+ *   efg_peer_alloc   allocates this rank's exchange region (cudaMalloc, 4 *
+ *                    (64 + 2 * ceil32(ceil(n/32))) bytes, owned by the handle,
+ *                    zeroed) and returns its device address and its 64-byte
+ *                    CUDA IPC handle; either may be NULL.
+ *   (caller)         all-gathers the handles (e.g. torch.distributed) — or, for
+ *                    several handles on one device in one process, the addresses.
+ *   efg_peer_open    maps the other ranks' regions: ipc_handles = world * 64
+ *                    bytes (rank order; cudaIpcOpenMemHandle with lazy peer
+ *                    access), or regions = world device addresses (same
+ *                    process); exactly one of the two is non-NULL.  bounds as in
+ *                    efg_xchg_geometry (bounds[0] = 0, bounds[world] = n).
+ *   efg_xchg_peer    enqueues the exchange on the handle's stream (three
+ *                    kernels; two cross-rank barriers over flags in the regions)
+ *                    and returns.  Every rank must call it once per level.
+ * Ranks that share one device must use distinct non-blocking streams (the
+ * barrier kernels of one rank wait for the others' kernels).  A barrier that
+ * waits more than 4 s gives up; the next efg_bfs_finish_level then returns
+ * EFG_ECUDA.  efg_free unmaps and frees everything.
+ * Errors: EFG_EINVAL (bad world / rank / bounds / pointers), EFG_ESTATE (open
+ * before alloc, exchange before open, host-only handle), EFG_ECUDA.
+ */
+#define EFG_IPC_HANDLE_BYTES 64
+efg_status efg_peer_alloc(efg_graph *g, int world, void **region, uint8_t *ipc_handle);
+efg_status efg_peer_open(efg_graph *g, int world, int rank, const uint64_t *bounds, const uint8_t *ipc_handles,
+                         void *const *regions);
+efg_status efg_xchg_peer(efg_graph *g);
+
 /*
  * efg_partition — the 1-D row partition (efg_build_opts.row_lo / row_hi):
  * rank r owns vertices [bounds[r], bounds[r+1]).  Boundaries balance

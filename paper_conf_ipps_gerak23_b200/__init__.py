@@ -213,6 +213,32 @@ class Graph:
         b = np.ascontiguousarray(bounds, np.uint64)
         check(lib.efg_xchg_unpack(self._h, b.size - 1, _ptr(b), S, _ptr(gathered)), "efg_xchg_unpack")
 
+    # -- the same exchange over peer memory (efg_peer_alloc / _open / efg_xchg_peer) --
+    def peer_alloc(self, world: int) -> tuple[int, bytes]:
+        """Allocate this rank's exchange region; returns (device address, 64-byte IPC handle)."""
+        reg = C.c_void_p()
+        h = (C.c_uint8 * 64)()
+        check(lib.efg_peer_alloc(self._h, world, C.byref(reg), h), "efg_peer_alloc")
+        return int(reg.value or 0), bytes(h)
+
+    def peer_open(self, rank: int, bounds: np.ndarray, *, handles: list[bytes] | None = None,
+                  regions: list[int] | None = None) -> None:
+        """Map every rank's region: IPC handles (one process per GPU) or, for
+        handles sharing one process, their device addresses."""
+        b = np.ascontiguousarray(bounds, np.uint64)
+        world = b.size - 1
+        if (handles is None) == (regions is None):
+            raise ValueError("peer_open: pass exactly one of handles / regions")
+        if handles is not None:
+            hb = np.frombuffer(b"".join(handles), np.uint8).copy()
+            check(lib.efg_peer_open(self._h, world, rank, _ptr(b), _ptr(hb), None), "efg_peer_open")
+        else:
+            rg = (C.c_void_p * world)(*regions)
+            check(lib.efg_peer_open(self._h, world, rank, _ptr(b), None, rg), "efg_peer_open")
+
+    def xchg_peer(self) -> None:
+        check(lib.efg_xchg_peer(self._h), "efg_xchg_peer")
+
     def bfs_finish_level(self) -> int:
         n = C.c_uint64()
         check(lib.efg_bfs_finish_level(self._h, C.byref(n)), "efg_bfs_finish_level")

@@ -69,6 +69,9 @@ SIGNATURES = [
     ("efg_xchg_pack", C.c_int, [C.c_void_p, C.c_int, C.c_void_p, C.c_uint64, C.c_void_p]),
     ("efg_xchg_reduce", C.c_int, [C.c_void_p, C.c_int, C.c_uint64, C.c_void_p, C.c_void_p]),
     ("efg_xchg_unpack", C.c_int, [C.c_void_p, C.c_int, C.c_void_p, C.c_uint64, C.c_void_p]),
+    ("efg_peer_alloc", C.c_int, [C.c_void_p, C.c_int, C.POINTER(C.c_void_p), C.c_void_p]),
+    ("efg_peer_open", C.c_int, [C.c_void_p, C.c_int, C.c_int, C.c_void_p, C.c_void_p, C.c_void_p]),
+    ("efg_xchg_peer", C.c_int, [C.c_void_p]),
     ("efg_bfs_finish_level", C.c_int, [C.c_void_p, C.POINTER(C.c_uint64)]),
     ("efg_bfs_end", C.c_int, [C.c_void_p, C.POINTER(Stats)]),
     ("efg_partition", C.c_int, [C.c_uint64, C.c_void_p, C.c_void_p, C.c_int, C.c_void_p]),

@@ -263,6 +263,32 @@ extern "C" efg_status efg_xchg_unpack(efg_graph *g, int world, const uint64_t *b
     return device_xchg(g, 2, world, bounds, slice_words, nullptr, gathered);
 }
 
+extern "C" efg_status efg_peer_alloc(efg_graph *g, int world, void **region, uint8_t *ipc_handle)
+{
+    clear_error();
+    EFG_TRY(check_handle(g));
+    if (world < 1 || world > kPeerMaxWorld) return set_error(EFG_EINVAL, "efg_peer_alloc: world outside [1, 64]");
+    return device_peer_alloc(g, world, region, ipc_handle);
+}
+
+extern "C" efg_status efg_peer_open(efg_graph *g, int world, int rank, const uint64_t *bounds,
+                                    const uint8_t *ipc_handles, void *const *regions)
+{
+    clear_error();
+    EFG_TRY(check_handle(g));
+    if (world < 1 || world > kPeerMaxWorld || rank < 0 || rank >= world || !bounds ||
+        (ipc_handles == nullptr) == (regions == nullptr))
+        return set_error(EFG_EINVAL, "efg_peer_open: bad args");
+    return device_peer_open(g, world, rank, bounds, ipc_handles, regions);
+}
+
+extern "C" efg_status efg_xchg_peer(efg_graph *g)
+{
+    clear_error();
+    EFG_TRY(check_handle(g));
+    return device_xchg_peer(g);
+}
+
 extern "C" efg_status efg_bfs_finish_level(efg_graph *g, uint64_t *global_new)
 {
     clear_error();

@@ -200,6 +200,7 @@ void device_drop_graphs(DeviceGraph &d)
 void device_free(DeviceGraph &d)
 {
     device_drop_graphs(d);
+    device_peer_close(d);
     cudaFree(d.data);
     cudaFree(d.rec);
     cudaFree(d.deg32);
@@ -229,6 +230,7 @@ void device_free(DeviceGraph &d)
     cudaFree(d.stats);
     cudaFree(d.xchg_bounds);
     cudaFree(d.ctrl);
+    cudaFree(d.peer_region);
     cudaFree(d.fbuf);
     cudaFree(d.dbuf);
     if (d.ctrl_host) cudaFreeHost(d.ctrl_host);
@@ -664,6 +666,7 @@ efg_status device_step_finish(efg_graph *g, uint64_t *global_new)
     CUDA_TRY(cudaMemcpyAsync(d.ctrl_host, d.ctrl, sizeof(LevelCtrl), cudaMemcpyDeviceToHost, s));
     CUDA_TRY(cudaStreamSynchronize(s));
     const LevelCtrl c = *d.ctrl_host;
+    if (c.fault) return set_error(EFG_ECUDA, "partitioned level: a grid or peer barrier timed out");
     if (c.nnew == 0 && d.old_of_new) {  // traversal over: depth back to input ids
         CUDA_TRY(launch_map_depth(d.depth_st, d.new_of_old, d.step_depth, d.n, s));
         CUDA_TRY(cudaStreamSynchronize(s));
@@ -694,6 +697,121 @@ efg_status device_step_end(efg_graph *g, efg_stats *st)
         if (st->level_frontier) st->level_frontier[i] = d.step_lf[i];
         if (st->level_edges) st->level_edges[i] = d.step_le[i];
     }
+    return EFG_OK;
+}
+
+// ---------------------------------------------------------------------------
+// Peer-memory exchange (efg.h "multi-GPU", peer_kernel in efg_kernels.cu).
+// ---------------------------------------------------------------------------
+void device_peer_close(DeviceGraph &d)
+{
+    for (int p = 0; p < kPeerMaxWorld; ++p)
+        if (d.peer_ipc[p]) {
+            cudaIpcCloseMemHandle(d.peer_ipc[p]);
+            d.peer_ipc[p] = nullptr;
+        }
+    cudaFree(d.peer_ptrs);
+    d.peer_ptrs = nullptr;
+    d.peer_world = 0;
+    d.peer_rank = -1;
+}
+
+efg_status device_peer_alloc(efg_graph *g, int world, void **region, uint8_t *ipc_handle)
+{
+    DeviceGraph &d = g->dev;
+    CUDA_TRY(cudaSetDevice(d.device));
+    cudaStream_t s = stream_of(d);
+    CUDA_TRY(cudaStreamSynchronize(s));
+    device_peer_close(d);
+    if (!d.peer_region) {
+        // its own allocation: an IPC handle maps exactly this region
+        EFG_TRY(dev_alloc(d, &d.peer_region, peer_region_words(d.nwords)));
+    }
+    CUDA_TRY(cudaMemset(d.peer_region, 0, peer_region_words(d.nwords) * 4));  // flags = epoch 0
+    d.peer_epoch = 0;
+    d.peer_alloc_world = world;
+    if (region) *region = d.peer_region;
+    if (ipc_handle) {
+        cudaIpcMemHandle_t h;
+        CUDA_TRY(cudaIpcGetMemHandle(&h, d.peer_region));
+        static_assert(sizeof(h) == EFG_IPC_HANDLE_BYTES, "cudaIpcMemHandle_t size");
+        std::memcpy(ipc_handle, &h, sizeof(h));
+    }
+    return EFG_OK;
+}
+
+efg_status device_peer_open(efg_graph *g, int world, int rank, const uint64_t *bounds, const uint8_t *ipc_handles,
+                            void *const *regions)
+{
+    DeviceGraph &d = g->dev;
+    CUDA_TRY(cudaSetDevice(d.device));
+    cudaStream_t s = stream_of(d);
+    if (!d.peer_region || d.peer_alloc_world != world)
+        return set_error(EFG_ESTATE, "efg_peer_open: call efg_peer_alloc with the same world first");
+    if (bounds[0] != 0 || bounds[world] != d.n)
+        return set_error(EFG_EINVAL, "efg_peer_open: bounds must span [0, n)");
+    for (int r = 0; r < world; ++r)
+        if (bounds[r + 1] < bounds[r] || bounds[r] % 64)
+            return set_error(EFG_EINVAL, "efg_peer_open: bounds must be non-decreasing multiples of 64");
+    device_peer_close(d);
+    std::vector<uint32_t *> ptrs(world);
+    for (int p = 0; p < world; ++p) {
+        if (p == rank) {
+            ptrs[p] = d.peer_region;
+        } else if (regions) {
+            ptrs[p] = static_cast<uint32_t *>(regions[p]);
+        } else {
+            cudaIpcMemHandle_t h;
+            std::memcpy(&h, ipc_handles + (size_t)p * EFG_IPC_HANDLE_BYTES, sizeof(h));
+            void *ptr = nullptr;
+            const cudaError_t e = cudaIpcOpenMemHandle(&ptr, h, cudaIpcMemLazyEnablePeerAccess);
+            if (e != cudaSuccess) {
+                cudaGetLastError();
+                device_peer_close(d);
+                return set_error(EFG_ECUDA, std::string("efg_peer_open: cudaIpcOpenMemHandle(rank ") +
+                                                std::to_string(p) + "): " + cudaGetErrorString(e));
+            }
+            d.peer_ipc[p] = ptr;
+            ptrs[p] = static_cast<uint32_t *>(ptr);
+        }
+    }
+    EFG_TRY(dev_alloc(d, &d.peer_ptrs, (uint64_t)world));
+    CUDA_TRY(cudaMemcpyAsync(d.peer_ptrs, ptrs.data(), world * sizeof(uint32_t *), cudaMemcpyHostToDevice, s));
+    if ((uint64_t)world + 1 > d.xchg_bounds_cap) {
+        cudaFree(d.xchg_bounds);
+        d.xchg_bounds = nullptr;
+        EFG_TRY(dev_alloc(d, &d.xchg_bounds, (uint64_t)world + 1));
+        d.xchg_bounds_cap = (uint64_t)world + 1;
+    }
+    CUDA_TRY(cudaMemcpyAsync(d.xchg_bounds, bounds, (world + 1) * 8, cudaMemcpyHostToDevice, s));
+    CUDA_TRY(cudaStreamSynchronize(s));
+    d.peer_world = world;
+    d.peer_rank = rank;
+    return EFG_OK;
+}
+
+efg_status device_xchg_peer(efg_graph *g)
+{
+    DeviceGraph &d = g->dev;
+    if (!d.peer_ptrs) return set_error(EFG_ESTATE, "efg_xchg_peer: call efg_peer_open first");
+    CUDA_TRY(cudaSetDevice(d.device));
+    cudaStream_t s = stream_of(d);
+    PeerArgs a;
+    a.peers = d.peer_ptrs;
+    a.local = d.peer_region;
+    a.bounds = d.xchg_bounds;
+    a.vis = d.vis;
+    a.prev = d.prev;
+    a.fault = &d.ctrl->fault;
+    a.nwords = d.nwords;
+    a.world = d.peer_world;
+    a.rank = d.peer_rank;
+    a.epoch = d.peer_epoch + 1;
+    for (int op = 0; op < 3; ++op) {
+        a.op = op;
+        CUDA_TRY(launch_peer(a, d.num_sms, s));
+    }
+    d.peer_epoch += 2;
     return EFG_OK;
 }
 

@@ -214,6 +214,13 @@ struct DeviceGraph {
     uint64_t own_lo_w = 0, own_hi_w = 0;   // bitmap words of the owned rows (frontier filter)
     uint64_t *xchg_bounds = nullptr;       // device copy of the partition bounds
     uint64_t xchg_bounds_cap = 0;
+    // peer-memory exchange (efg_peer_alloc / efg_peer_open / efg_xchg_peer)
+    uint32_t *peer_region = nullptr;       // this rank's region (own cudaMalloc: IPC-exportable)
+    uint32_t **peer_ptrs = nullptr;        // device array [peer_world] of region bases
+    void *peer_ipc[64] = {};               // IPC-opened peer bases (closed on free)
+    int peer_world = 0, peer_rank = -1;
+    int peer_alloc_world = 0;
+    uint32_t peer_epoch = 0;               // last barrier epoch used
     // stepwise (partitioned) traversal state
     uint32_t step_levels = 0;
     uint64_t step_reached = 0, step_edges = 0;
@@ -242,6 +249,11 @@ efg_status device_step_expand(efg_graph *g);
 efg_status device_step_finish(efg_graph *g, uint64_t *global_new);
 efg_status device_step_end(efg_graph *g, efg_stats *st);
 // op 0 = pack (out = send), 1 = reduce (in = recv, out = mine), 2 = unpack (in = gathered)
+efg_status device_peer_alloc(efg_graph *g, int world, void **region, uint8_t *ipc_handle);
+efg_status device_peer_open(efg_graph *g, int world, int rank, const uint64_t *bounds, const uint8_t *ipc_handles,
+                            void *const *regions);
+efg_status device_xchg_peer(efg_graph *g);
+void device_peer_close(DeviceGraph &d);
 efg_status device_xchg(efg_graph *g, int op, int world, const uint64_t *bounds, uint64_t slice_words,
                        uint32_t *out, const uint32_t *in);
 }  // namespace efg

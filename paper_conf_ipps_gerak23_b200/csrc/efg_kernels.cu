@@ -222,6 +222,80 @@ __global__ void xchg_kernel(XchgArgs a)
 }
 
 // --------------------------------------------------------------------------
+// Peer-memory exchange (SURVEY §8(e) "B200-native upgrade"): the same OR-reduce
+// to owners + all-gather as pack / all-to-all / reduce / all-gather / unpack,
+// with no collective library and no intermediate slices: owners read every
+// rank's published new bits straight from its HBM over NVLink and store the
+// OR into every rank's result buffer.  Three launches per level, in stream
+// order on each rank:
+//   op 0  publish:  pub[w] = vis[w] & ~prev[w]                 (local)
+//   op 1  barrier e; for owned words w: m = OR_p pub_p[w]; res_p[w] = m for all p
+//   op 2  barrier e+1; vis[w] |= res[w]                       (local)
+// Barrier e: block 0 stores e into flags[rank] of every rank (release, system
+// scope), every block waits until all of its own flags reach e (acquire).
+// Reuse is safe without more barriers: a rank republishes (op 0 of the next
+// level) only after its barrier e+1, which every rank passes only after all
+// ops 1 (the readers of pub) completed; owners write res (op 1 of the next
+// level) only after barrier e+2, i.e. after every rank's op 2 read it.
+// A wait longer than 4 s (a rank that never arrives) raises *fault and gives
+// up instead of holding the device.
+// --------------------------------------------------------------------------
+__device__ __forceinline__ bool peer_barrier(const PeerArgs &a, uint32_t e)
+{
+    if (blockIdx.x == 0 && threadIdx.x < (unsigned)a.world) {
+        __threadfence_system();
+        uint32_t *f = a.peers[threadIdx.x] + a.rank;
+        asm volatile("st.release.sys.global.u32 [%0], %1;" ::"l"(f), "r"(e) : "memory");
+    }
+    __shared__ int ok;
+    if (threadIdx.x == 0) ok = 1;
+    __syncthreads();
+    if (threadIdx.x < (unsigned)a.world) {
+        const uint32_t *f = a.local + threadIdx.x;
+        const unsigned long long t0 = globaltimer();
+        for (uint32_t it = 0;; ++it) {
+            uint32_t cur;
+            asm volatile("ld.acquire.sys.global.u32 %0, [%1];" : "=r"(cur) : "l"(f) : "memory");
+            if ((int32_t)(cur - e) >= 0) break;
+            __nanosleep(64);
+            if ((it & 255) == 255 && globaltimer() - t0 > 4000000000ull) {
+                atomicExch(a.fault, 1u);
+                ok = 0;
+                break;
+            }
+        }
+    }
+    __syncthreads();
+    return ok != 0;
+}
+
+__global__ void peer_kernel(PeerArgs a)
+{
+    const uint64_t pub = kPeerFlagWords, res = kPeerFlagWords + peer_pad(a.nwords);
+    const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+    const uint64_t t0 = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
+    if (a.op == 0) {
+        for (uint64_t w = t0; w < a.nwords; w += stride) a.local[pub + w] = a.vis[w] & ~a.prev[w];
+        return;
+    }
+    if (!peer_barrier(a, a.op == 1 ? a.epoch : a.epoch + 1)) return;
+    if (a.op == 1) {
+        const uint64_t w0 = a.bounds[a.rank] / 32, w1 = (a.bounds[a.rank + 1] + 31) / 32;
+        for (uint64_t w = w0 + t0; w < w1; w += stride) {
+            uint32_t m = 0;
+            for (int p = 0; p < a.world; ++p) m |= __ldcv(a.peers[p] + pub + w);
+            for (int p = 0; p < a.world; ++p) __stcg(a.peers[p] + res + w, m);
+        }
+        __threadfence_system();
+        return;
+    }
+    for (uint64_t w = t0; w < a.nwords; w += stride) {
+        const uint32_t m = __ldcv(a.local + res + w);
+        if (m) a.vis[w] |= m;
+    }
+}
+
+// --------------------------------------------------------------------------
 // frontier_kernel: the level end (a7) fused with the next level's plan
 // (a1 + a2 + a3 + a4), one launch per level.
 //
@@ -1513,6 +1587,16 @@ cudaError_t launch_xchg(const XchgArgs &a, cudaStream_t s)
     const uint64_t total = (uint64_t)(a.op == 1 ? 1 : a.world) * a.S;
     const unsigned blocks = (unsigned)std::max<uint64_t>(1, std::min<uint64_t>((total + 255) / 256, 148 * 8));
     xchg_kernel<<<blocks, 256, 0, s>>>(a);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_peer(const PeerArgs &a, int max_blocks, cudaStream_t s)
+{
+    // a small grid: the spinning blocks of one rank must leave room for the
+    // other ranks' kernels when several ranks share a device (tests)
+    const unsigned blocks = (unsigned)std::max<uint64_t>(1, std::min<uint64_t>((a.nwords + 255) / 256,
+                                                                               (uint64_t)max_blocks));
+    peer_kernel<<<blocks, 256, 0, s>>>(a);
     return cudaGetLastError();
 }
 

@@ -58,6 +58,28 @@ struct XchgArgs {
     const uint32_t *in;
 };
 
+// Peer-memory exchange (efg_xchg_peer): every rank's region, mapped into every
+// rank (CUDA IPC over NVLink / NVSwitch, or plain pointers on one device), is
+//   [flags: kPeerFlagWords u32 | pub: peer_pad(nwords) u32 | res: nwords u32]
+// flags[p] = the last barrier epoch rank p signalled to this rank.
+constexpr int kPeerMaxWorld = 64;
+constexpr uint64_t kPeerFlagWords = 64;
+__host__ __device__ inline uint64_t peer_pad(uint64_t nwords) { return (nwords + 31) & ~31ull; }
+__host__ __device__ inline uint64_t peer_region_words(uint64_t nwords) { return kPeerFlagWords + 2 * peer_pad(nwords); }
+
+struct PeerArgs {
+    uint32_t *const *peers;        // device array [world]: region base of every rank (own included)
+    uint32_t *local;               // this rank's region
+    const uint64_t *bounds;        // device copy of the vertex bounds (world+1)
+    uint32_t *vis;
+    const uint32_t *prev;
+    uint32_t *fault;               // LevelCtrl.fault: a barrier wait timed out
+    uint64_t nwords;
+    uint32_t epoch;                // barrier epoch of ops 1 and 2
+    int world, rank;
+    int op;                        // 0 publish, 1 owner OR + broadcast, 2 unpack
+};
+
 struct FrontierArgs {           // level end (a7) + next level plan (a1-a4), one launch
     uint32_t *vis, *prev;      // visited bitmap now / at the previous level end
     const uint32_t *iso;       // degree-0 vertices (never probed): count as visited for the visited prefix
@@ -91,6 +113,7 @@ cudaError_t launch_init(const InitArgs &a, cudaStream_t s);
 cudaError_t launch_frontier(const FrontierArgs &a, unsigned blocks, cudaStream_t s);
 int frontier_occupancy();  // resident frontier_kernel blocks per SM (its grid must fit: blocks spin on predecessors)
 cudaError_t launch_xchg(const XchgArgs &a, cudaStream_t s);
+cudaError_t launch_peer(const PeerArgs &a, int max_blocks, cudaStream_t s);
 int expand_occupancy(int mode);
 size_t expand_smem_bytes();
 // pout[old_of_new[i]] = pin[i] == ~0u ? ~0u : old_of_new[pin[i]]  (parents back to input ids)

@@ -128,3 +128,61 @@ def simulated_partitioned_bfs(graphs, source: int, depths, bounds: np.ndarray, m
             break
         counts.append(news[0])
     return counts
+
+
+# ---------------------------------------------------------------------------
+# The same exchange over peer memory (efg.h "exchange over peer memory"): the
+# library's kernels read and write the other ranks' HBM over NVLink; this
+# module only all-gathers the 64-byte CUDA IPC handles once per partition.
+# ---------------------------------------------------------------------------
+def peer_setup(g, rank: int, bounds: np.ndarray, group=None) -> None:
+    """Collective: allocate this rank's region, all-gather the IPC handles,
+    map the other ranks' regions."""
+    import torch.distributed as dist
+    world = bounds.size - 1
+    _, handle = g.peer_alloc(world)
+    handles = [None] * world
+    dist.all_gather_object(handles, handle, group=group)
+    g.peer_open(rank, bounds, handles=handles)
+
+
+def partitioned_bfs_peer(g, source: int, depth):
+    """One partitioned BFS after peer_setup: per level expand, peer exchange,
+    level end.  Returns the list of global new-vertex counts per level."""
+    g.bfs_begin(source, depth)
+    counts = [1]
+    while True:
+        g.bfs_expand()
+        g.xchg_peer()
+        new = g.bfs_finish_level()
+        if new == 0:
+            break
+        counts.append(new)
+    return counts
+
+
+def simulated_peer_setup(graphs, bounds: np.ndarray) -> None:
+    """All `world` rank handles in one process on one device (tests): the
+    regions are mapped by address instead of IPC.  Each handle must have been
+    built on its own non-blocking stream."""
+    world = bounds.size - 1
+    regions = [g.peer_alloc(world)[0] for g in graphs]
+    for r, g in enumerate(graphs):
+        g.peer_open(r, bounds, regions=regions)
+
+
+def simulated_partitioned_bfs_peer(graphs, source: int, depths):
+    for g, d in zip(graphs, depths):
+        g.bfs_begin(source, d)
+    counts = [1]
+    while True:
+        for g in graphs:
+            g.bfs_expand()
+        for g in graphs:      # every rank's barrier kernels are enqueued before any wait
+            g.xchg_peer()
+        news = [g.bfs_finish_level() for g in graphs]
+        assert len(set(news)) == 1, news
+        if news[0] == 0:
+            break
+        counts.append(news[0])
+    return counts

@@ -369,6 +369,54 @@ def test_partitioned_bfs_simulated_ranks(efg, world):
             g.free()
 
 
+@pytest.mark.parametrize("world", [1, 2, 3, 4])
+def test_partitioned_bfs_peer_exchange_simulated_ranks(efg, world):
+    """SURVEY §8(e) over peer memory (efg_peer_* / efg_xchg_peer): the owner
+    OR-reduce + broadcast and the cross-rank barriers run in the library's
+    kernels; here the ranks share one device (regions mapped by address, one
+    non-blocking stream per rank).  Every rank's depth must equal the oracle's,
+    over several BFS on the same mapping (barrier epochs keep counting)."""
+    import torch
+    from paper_conf_ipps_gerak23_b200.dist import simulated_peer_setup, simulated_partitioned_bfs_peer
+    n, src, dst = synth.rmat(14, 16, seed=13)
+    ov, oe = oracle.csr_build(n, src, dst)
+    for flags in (efg.EFG_DEFAULT_FLAGS, efg.EFG_DEFAULT_FLAGS | efg.EFG_REORDER_DEGREE):
+        whole = efg.Graph.build(n, src, dst, flags=flags, device=-1)
+        vlist, _, offsets, _ = whole.export()
+        bounds = efg.partition(vlist, offsets, world)
+        whole.free()
+        streams = [torch.cuda.Stream() for _ in range(world)]
+        graphs = [efg.Graph.build(n, src, dst, flags=flags, stream=streams[r].cuda_stream,
+                                  rows=(int(bounds[r]), int(bounds[r + 1]))) for r in range(world)]
+        simulated_peer_setup(graphs, bounds)
+        for s in (0, 3, 9999, n - 1):
+            depths = [torch.empty(n, dtype=torch.int32, device="cuda") for _ in range(world)]
+            torch.cuda.synchronize()
+            simulated_partitioned_bfs_peer(graphs, s, depths)
+            torch.cuda.synchronize()
+            ref = oracle.bfs(ov, oe, s)
+            for d in depths:
+                assert np.array_equal(d.cpu().numpy(), ref)
+        for g in graphs:
+            g.free()
+
+
+def test_peer_exchange_errors(efg):
+    n, src, dst = synth.rmat(10, 8, seed=3)
+    g = efg.Graph.build(n, src, dst)
+    bounds = np.array([0, n], np.uint64)
+    with pytest.raises(efg.EFGError):
+        g.xchg_peer()                       # before efg_peer_open
+    with pytest.raises(efg.EFGError):
+        g.peer_open(0, bounds, regions=[0])  # before efg_peer_alloc
+    reg, h = g.peer_alloc(1)
+    assert reg != 0 and len(h) == 64
+    with pytest.raises(efg.EFGError):
+        g.peer_open(0, np.array([0, n - 1], np.uint64), regions=[reg])  # bounds do not span [0, n)
+    g.peer_open(0, bounds, regions=[reg])
+    g.free()
+
+
 @pytest.mark.parametrize("reorder", [False, True])
 def test_sssp_bit_exact_vs_dijkstra(efg, reorder):
     """NEXT-1: fp32 frontier Bellman-Ford == fp32 Dijkstra bit for bit (C20)."""
