@@ -22,8 +22,11 @@ rows a1-a7) from one seeded source over the BASELINE.json configs[1] graph
 host cores, same config/metric (each step = one oracle BFS).
 With N > 1 (torchrun) the default is the north_star's 1-D row partition: each
 rank holds a byte-balanced row range of the EFG, every BFS level exchanges the
-new-vertex bitmap (all_to_all + OR + all_gather over NCCL), "scaling":
-"strong"; ``--mode replicas`` runs independent BFS problems per rank on
+new-vertex bitmap ("scaling": "strong"): by default the library's kernels
+read every rank's new bits over NVLink peer memory and broadcast the owners'
+OR (``--xchg peer``; CUDA IPC handles all-gathered once), or all_to_all + OR +
+all_gather with torch.distributed over NCCL (``--xchg nccl``).
+``--mode replicas`` runs independent BFS problems per rank on
 disjoint sources (no data-path collective, "scaling": "weak").
 Also reported on one GPU: PageRank (50 iterations) and SSSP over the same graph.
 """
@@ -59,6 +62,10 @@ def parse():
     p.add_argument("--mode", default="partition", choices=["partition", "replicas"],
                    help="N > 1: 1-D partitioned BFS with a per-level NCCL exchange (SURVEY 8(e)), "
                         "or independent replicas on disjoint sources")
+    p.add_argument("--xchg", default="peer", choices=["peer", "nccl"],
+                   help="N > 1 partition mode: per-level exchange by the library's kernels over "
+                        "NVLink peer memory (CUDA IPC, efg_xchg_peer) or all_to_all + all_gather "
+                        "with torch.distributed (efg_xchg_pack/reduce/unpack)")
     p.add_argument("--reorder", default="degree", choices=["none", "degree"],
                    help="EFG_REORDER_DEGREE relabelling at build time (results stay in input ids)")
     p.add_argument("--profile-levels", action="store_true", help="print per-level stats to stderr")
@@ -243,7 +250,8 @@ def run_partitioned(args, rank, world, local):
     import torch.distributed as dist
     import synth
     import paper_conf_ipps_gerak23_b200 as efg
-    from paper_conf_ipps_gerak23_b200.dist import TorchTransport, partitioned_bfs
+    from paper_conf_ipps_gerak23_b200.dist import (TorchTransport, partitioned_bfs, partitioned_bfs_peer,
+                                                   peer_setup)
 
     dev = torch.device("cuda", local)
     stream = torch.cuda.Stream(device=dev)
@@ -274,9 +282,14 @@ def run_partitioned(args, rank, world, local):
     depth = torch.empty(n, dtype=torch.int32, device=dev)
     tr = TorchTransport(stage_on_host=dist.get_backend() != "nccl")
     mk = lambda k: torch.zeros(k, dtype=torch.int32, device=dev)  # noqa: E731
+    if args.xchg == "peer":
+        peer_setup(g, rank, b)  # IPC handles all-gathered once; no collective per level
+        one_bfs = lambda s: partitioned_bfs_peer(g, s, depth)  # noqa: E731
+    else:
+        one_bfs = lambda s: partitioned_bfs(g, s, depth, b, tr, mk)  # noqa: E731
     with torch.cuda.stream(stream):
         for s in srcs[:args.warmup]:
-            partitioned_bfs(g, int(s), depth, b, tr, mk)
+            one_bfs(int(s))
     torch.cuda.synchronize()
     dist.barrier()
     torch.cuda.synchronize()
@@ -288,7 +301,7 @@ def run_partitioned(args, rank, world, local):
     e0.record(stream)
     with torch.cuda.stream(stream):
         for s in srcs[args.warmup:]:
-            partitioned_bfs(g, int(s), depth, b, tr, mk)
+            one_bfs(int(s))
             st = g.bfs_end()
             edges += st["edges_traversed"]  # this rank's rows
     e1.record(stream)
@@ -309,7 +322,11 @@ def run_partitioned(args, rank, world, local):
             "data": "synthetic",
             "config": {"workload": cfgname, "n": int(n), "reorder": args.reorder,
                        "parallelism": f"1-D row partition over {world} GPUs, per-level bitmap "
-                                      "exchange (all_to_all + OR + all_gather, NCCL)",
+                                      + ("exchange by the library's kernels over peer memory "
+                                         "(owner OR + broadcast, CUDA IPC over NVLink)"
+                                         if args.xchg == "peer" else
+                                         "exchange (all_to_all + OR + all_gather, NCCL)"),
+                       "xchg": args.xchg,
                        "bounds": [int(x) for x in b],
                        "l2_policy": "inputs larger than L2"},
             "clocks": clocks, "gpu_launches": None,
