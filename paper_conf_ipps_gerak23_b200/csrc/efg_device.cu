@@ -570,8 +570,7 @@ efg_status device_bfs(efg_graph *g, uint32_t source, int32_t *depth, uint32_t *p
         for (int c = 0; c < kD2HChunks; ++c) {
             CUDA_TRY(cudaEventSynchronize(d.d2h_ev[c]));
             const int64_t c0 = (int64_t)(d.n * c / kD2HChunks), c1 = (int64_t)(d.n * (c + 1) / kD2HChunks);
-#pragma omp parallel for schedule(static)
-            for (int64_t i = c0; i < c1; ++i) depth[i] = src8[i];
+            host_widen_i8_i32(src8 + c0, depth + c0, c1 - c0);
         }
     }
     CUDA_TRY(cudaStreamSynchronize(s));

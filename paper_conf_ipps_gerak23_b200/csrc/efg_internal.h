@@ -258,6 +258,11 @@ efg_status device_xchg(efg_graph *g, int op, int world, const uint64_t *bounds, 
                        uint32_t *out, const uint32_t *in);
 }  // namespace efg
 
+// host widening of the compact depth transfer (efg_host_widen.cpp): dst[i] = src[i], OpenMP
+namespace efg {
+void host_widen_i8_i32(const int8_t *src, int32_t *dst, int64_t n);
+}  // namespace efg
+
 // error handling (efg_error.cpp)
 namespace efg {
 efg_status set_error(efg_status s, const std::string &msg);

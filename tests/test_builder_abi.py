@@ -165,3 +165,22 @@ def test_row_range_build_keeps_only_owned_lists():
     assert part.info["row_lo"] == 1024 and part.info["row_hi"] == 2048
     with pytest.raises(efg.EFGError):
         efg.Graph.build(n, src, dst, device=-1, rows=(100, 2048))
+
+
+def test_host_widen_i8_i32():
+    """Host side of the compact depth transfer (efg_host_widen.cpp): the
+    streaming-store widening equals a plain int8 -> int32 copy at every length
+    and alignment, and writes nothing outside [0, n)."""
+    import ctypes as C
+    from paper_conf_ipps_gerak23_b200 import _abi
+    f = getattr(C.CDLL(_abi.LIB_PATH), "_ZN3efg17host_widen_i8_i32EPKaPil")
+    f.restype = None
+    f.argtypes = [C.c_void_p, C.c_void_p, C.c_int64]
+    rng = np.random.default_rng(5)
+    for n in (0, 1, 7, 8, 63, 64, 65, 1000, 4097, 100003):
+        for off in (0, 1, 3, 8):
+            s = rng.integers(-1, 127, size=n + 16).astype(np.int8)
+            d = np.full(n + 16, 777, np.int32)
+            f(s.ctypes.data + off, d.ctypes.data + 4 * off, n)
+            assert np.array_equal(d[off:off + n], s[off:off + n].astype(np.int32)), (n, off)
+            assert np.all(d[:off] == 777) and np.all(d[off + n:] == 777)
