@@ -298,12 +298,14 @@ def run_partitioned(args, rank, world, local):
     e0 = torch.cuda.Event(enable_timing=True)
     e1 = torch.cuda.Event(enable_timing=True)
     edges = 0
+    launches = 0
     e0.record(stream)
     with torch.cuda.stream(stream):
         for s in srcs[args.warmup:]:
             one_bfs(int(s))
             st = g.bfs_end()
             edges += st["edges_traversed"]  # this rank's rows
+            launches += st["kernel_launches"]
     e1.record(stream)
     torch.cuda.synchronize()
     clocks = clk.stop()
@@ -329,7 +331,8 @@ def run_partitioned(args, rank, world, local):
                        "xchg": args.xchg,
                        "bounds": [int(x) for x in b],
                        "l2_policy": "inputs larger than L2"},
-            "clocks": clocks, "gpu_launches": None,
+            "clocks": clocks, "gpu_launches": launches,
+            "gpu_launches_note": "rank 0's kernels (every rank launches the same number per level)",
             "e2e": None, "cpu_baseline": None,
         }
         print(json.dumps(line), flush=True)

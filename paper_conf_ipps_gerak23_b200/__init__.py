@@ -252,8 +252,8 @@ class Graph:
         check(lib.efg_bfs_end(self._h, C.byref(st)), "efg_bfs_end")
         L = min(st.levels + 1, level_cap)
         return {"levels": st.levels, "edges_traversed": st.edges_traversed,
-                "vertices_reached": st.vertices_reached, "level_frontier": lf[:L].copy(),
-                "level_edges": le[:L].copy()}
+                "vertices_reached": st.vertices_reached, "kernel_launches": st.kernel_launches,
+                "level_frontier": lf[:L].copy(), "level_edges": le[:L].copy()}
 
     def sssp(self, source: int, dist=None, stats: bool = False):
         n = self.info["n"]

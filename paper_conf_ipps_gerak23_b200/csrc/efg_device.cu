@@ -639,6 +639,7 @@ efg_status device_step_begin(efg_graph *g, uint32_t source, int32_t *depth)
         CUDA_TRY(cudaMemsetAsync(depth, 0xFF, d.n * 4, s));
     uint32_t launches = 0;
     EFG_TRY(start_traversal(d, source, (uint64_t)source + 1, depth, nullptr, launches));
+    d.step_launches = launches;
     CUDA_TRY(cudaMemcpyAsync(d.ctrl_host, d.ctrl, sizeof(LevelCtrl), cudaMemcpyDeviceToHost, s));
     CUDA_TRY(cudaStreamSynchronize(s));
     d.step_lf.push_back(d.ctrl_host->nf);
@@ -653,6 +654,7 @@ efg_status device_step_expand(efg_graph *g)
     const int blocks = d.num_sms * expand_occupancy(kModeVisit);
     CUDA_TRY(launch_expand(kModeVisit, expand_args(d, nullptr), blocks, stream_of(d)));
     ++d.step_levels;
+    ++d.step_launches;
     return EFG_OK;
 }
 
@@ -662,12 +664,14 @@ efg_status device_step_finish(efg_graph *g, uint64_t *global_new)
     CUDA_TRY(cudaSetDevice(d.device));
     cudaStream_t s = stream_of(d);
     EFG_TRY(launch_level_end(d, 0, s));
+    ++d.step_launches;
     CUDA_TRY(cudaMemcpyAsync(d.ctrl_host, d.ctrl, sizeof(LevelCtrl), cudaMemcpyDeviceToHost, s));
     CUDA_TRY(cudaStreamSynchronize(s));
     const LevelCtrl c = *d.ctrl_host;
     if (c.fault) return set_error(EFG_ECUDA, "partitioned level: a grid or peer barrier timed out");
     if (c.nnew == 0 && d.old_of_new) {  // traversal over: depth back to input ids
         CUDA_TRY(launch_map_depth(d.depth_st, d.new_of_old, d.step_depth, d.n, s));
+        ++d.step_launches;
         CUDA_TRY(cudaStreamSynchronize(s));
     }
     if (c.nnew) {
@@ -692,6 +696,7 @@ efg_status device_step_end(efg_graph *g, efg_stats *st)
     st->edges_traversed = edges;      // this rank's rows
     st->vertices_reached = reached;   // this rank's rows
     st->expand_launches = d.step_levels;
+    st->kernel_launches = d.step_launches;
     for (uint32_t i = 0; i < std::min<uint32_t>((uint32_t)d.step_lf.size(), st->level_cap); ++i) {
         if (st->level_frontier) st->level_frontier[i] = d.step_lf[i];
         if (st->level_edges) st->level_edges[i] = d.step_le[i];
@@ -809,6 +814,7 @@ efg_status device_xchg_peer(efg_graph *g)
     for (int op = 0; op < 3; ++op) {
         a.op = op;
         CUDA_TRY(launch_peer(a, d.num_sms, s));
+        ++d.step_launches;
     }
     d.peer_epoch += 2;
     return EFG_OK;
@@ -839,6 +845,7 @@ efg_status device_xchg(efg_graph *g, int op, int world, const uint64_t *bounds, 
     a.out = out;
     a.in = in;
     CUDA_TRY(launch_xchg(a, s));
+    ++d.step_launches;
     return EFG_OK;
 }
 

@@ -223,6 +223,7 @@ struct DeviceGraph {
     uint32_t peer_epoch = 0;               // last barrier epoch used
     // stepwise (partitioned) traversal state
     uint32_t step_levels = 0;
+    uint32_t step_launches = 0;            // kernels this stepwise BFS launched (efg_stats.kernel_launches)
     uint64_t step_reached = 0, step_edges = 0;
     std::vector<uint64_t> step_lf, step_le;
 };

@@ -6,7 +6,7 @@ ROOT=$(cd "$(dirname "$0")/.." && pwd)
 OUT=$ROOT/build/var_$NAME; mkdir -p $OUT
 CS=$ROOT/paper_conf_ipps_gerak23_b200/csrc
 F="-gencode arch=compute_100a,code=sm_100a -O3 -std=c++17 -I $ROOT/include -I $CS -Xcompiler -fPIC,-fopenmp -lineinfo $DEFS"
-for s in efg_api.cu efg_builder.cpp efg_device.cu efg_error.cpp efg_kernels.cu; do
+for s in $(cd $CS && ls *.cu *.cpp); do
   nvcc $F -c $CS/$s -o $OUT/$s.o &
 done
 wait
