@@ -627,9 +627,9 @@ def main():
                                    "loop, same sources, on the library stream)"},
             "e2e": {"value": e2e_val, "unit": UNIT, "h2d_bytes_per_step": 4,
                     "d2h_bytes_per_step": int(np.mean(d2h_bytes)) if d2h_bytes else None,
-                    "d2h_note": "depth array into a pinned host buffer; one byte per vertex "
-                                "over PCIe when every depth < 127, widened to int32 on the host "
-                                "inside the call"},
+                    "d2h_note": "depth array into a pinned host buffer; 4 bits per vertex "
+                                "over PCIe when the BFS has < 15 levels (1 byte when every "
+                                "depth < 127), widened to int32 on the host inside the call"},
             "cpu_baseline": cpu,
             "alt_no_reorder": alt,
             "alt_no_prefix_skip": alt_ns,

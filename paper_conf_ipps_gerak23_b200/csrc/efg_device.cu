@@ -538,39 +538,52 @@ efg_status device_bfs(efg_graph *g, uint32_t source, int32_t *depth, uint32_t *p
     }
     if (parent && relabel) CUDA_TRY(launch_map_parent(pd, d.old_of_new, pout, d.n, s));
     uint64_t d2h = 0;
-    // a host depth array crosses PCIe as one byte per vertex when every depth
-    // fits (levels < 127: [-1, 126]); the host widens it (OpenMP)
-    bool narrow8 = false;
-    if (!depth_dev) {
-        narrow8 = levels < 127 && d.n >= 4096;  // levels is final here in both loop modes
-        if (narrow8) {
-            if (!d.depth8) EFG_TRY(dev_alloc(d, &d.depth8, d.n));
-            if (!d.depth8_host) CUDA_TRY(cudaMallocHost(reinterpret_cast<void **>(&d.depth8_host), d.n));
-            if (!d.d2h_ev[0])
-                for (int c = 0; c < kD2HChunks; ++c) CUDA_TRY(cudaEventCreateWithFlags(&d.d2h_ev[c], cudaEventDisableTiming));
+    // a host depth array crosses PCIe as 4 bits per vertex when every depth
+    // is < 15 (code = depth + 1, 0 = unreached), else as one byte per vertex
+    // when every depth is < 127 ([-1, 126]); the host widens it
+    // (efg_host_widen.cpp) chunk by chunk as the chunks land
+    int narrow = 0;  // 4 or 8 bits per vertex, 0 = int32 copy
+    if (!depth_dev && d.n >= 4096) narrow = levels < 15 ? 4 : levels < 127 ? 8 : 0;  // depth <= levels; levels is final here
+    // chunk c: vertices [cv(c), cv(c+1)), multiples of 8 (one 4-bit word = 8 vertices)
+    auto cv = [&](int c) -> uint64_t {
+        return c == kD2HChunks ? d.n : (((d.n + 7) / 8) * c / kD2HChunks) * 8;
+    };
+    if (narrow) {
+        if (!d.depth8) EFG_TRY(dev_alloc(d, &d.depth8, d.n + 8));
+        if (!d.depth8_host) CUDA_TRY(cudaMallocHost(reinterpret_cast<void **>(&d.depth8_host), d.n + 8));
+        if (!d.d2h_ev[0])
+            for (int c = 0; c < kD2HChunks; ++c) CUDA_TRY(cudaEventCreateWithFlags(&d.d2h_ev[c], cudaEventDisableTiming));
+        if (narrow == 4)
+            CUDA_TRY(launch_pack4(dd, reinterpret_cast<uint32_t *>(d.depth8), d.n, s));
+        else
             CUDA_TRY(launch_pack8(dd, d.depth8, d.n, s));
-            // chunked copy: the host widens chunk c while chunks > c are in flight
-            for (int c = 0; c < kD2HChunks; ++c) {
-                const uint64_t c0 = d.n * c / kD2HChunks, c1 = d.n * (c + 1) / kD2HChunks;
-                CUDA_TRY(cudaMemcpyAsync(d.depth8_host + c0, d.depth8 + c0, c1 - c0, cudaMemcpyDeviceToHost, s));
-                CUDA_TRY(cudaEventRecord(d.d2h_ev[c], s));
-            }
-            d2h += d.n;
-        } else {
-            CUDA_TRY(cudaMemcpyAsync(depth, dd, d.n * 4, cudaMemcpyDeviceToHost, s));
-            d2h += d.n * 4;
+        // chunked copy: the host widens chunk c while chunks > c are in flight
+        for (int c = 0; c < kD2HChunks; ++c) {
+            const uint64_t b0 = narrow == 4 ? cv(c) / 2 : cv(c);
+            const uint64_t b1 = narrow == 4 ? (cv(c + 1) + 7) / 8 * 4 : cv(c + 1);
+            if (b1 > b0)
+                CUDA_TRY(cudaMemcpyAsync(d.depth8_host + b0, d.depth8 + b0, b1 - b0, cudaMemcpyDeviceToHost, s));
+            CUDA_TRY(cudaEventRecord(d.d2h_ev[c], s));
+            d2h += b1 - b0;
         }
+    } else if (!depth_dev) {
+        CUDA_TRY(cudaMemcpyAsync(depth, dd, d.n * 4, cudaMemcpyDeviceToHost, s));
+        d2h += d.n * 4;
     }
     if (parent && !parent_dev) {
         CUDA_TRY(cudaMemcpyAsync(parent, pout, d.n * 4, cudaMemcpyDeviceToHost, s));
         d2h += d.n * 4;
     }
-    if (narrow8) {
-        const int8_t *src8 = d.depth8_host;
+    if (narrow) {
         for (int c = 0; c < kD2HChunks; ++c) {
             CUDA_TRY(cudaEventSynchronize(d.d2h_ev[c]));
-            const int64_t c0 = (int64_t)(d.n * c / kD2HChunks), c1 = (int64_t)(d.n * (c + 1) / kD2HChunks);
-            host_widen_i8_i32(src8 + c0, depth + c0, c1 - c0);
+            const uint64_t v0 = cv(c), v1 = cv(c + 1);
+            if (v1 <= v0) continue;
+            if (narrow == 4)
+                host_widen_u4_i32(reinterpret_cast<const uint32_t *>(d.depth8_host) + v0 / 8, depth + v0,
+                                  (int64_t)(v1 - v0));
+            else
+                host_widen_i8_i32(d.depth8_host + v0, depth + v0, (int64_t)(v1 - v0));
         }
     }
     CUDA_TRY(cudaStreamSynchronize(s));

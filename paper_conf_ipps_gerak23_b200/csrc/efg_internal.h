@@ -262,6 +262,8 @@ efg_status device_xchg(efg_graph *g, int op, int world, const uint64_t *bounds, 
 // host widening of the compact depth transfer (efg_host_widen.cpp): dst[i] = src[i], OpenMP
 namespace efg {
 void host_widen_i8_i32(const int8_t *src, int32_t *dst, int64_t n);
+// dst[i] = nibble i of src (8 per word, low nibble first) - 1; n vertices from a word boundary
+void host_widen_u4_i32(const uint32_t *src, int32_t *dst, int64_t n);
 }  // namespace efg
 
 // error handling (efg_error.cpp)

@@ -1487,6 +1487,34 @@ cudaError_t launch_map_depth(const int32_t *stored, const uint32_t *new_of_old, 
     return cudaGetLastError();
 }
 
+// host depth transfer in 4-bit codes (every depth < 15): out word g holds
+// depth + 1 of vertices 8g .. 8g+7 (low nibble first; 0 = unreached)
+__global__ void pack4_kernel(const int32_t *in, uint32_t *out, uint64_t n)
+{
+    const uint64_t G = (n + 7) / 8;
+    for (uint64_t g = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; g < G; g += (uint64_t)gridDim.x * blockDim.x) {
+        const uint64_t i = 8 * g;
+        uint32_t w = 0;
+        if (i + 8 <= n) {
+            const int4 a = *reinterpret_cast<const int4 *>(in + i);
+            const int4 b = *reinterpret_cast<const int4 *>(in + i + 4);
+            w = ((uint32_t)(a.x + 1) & 15u) | ((uint32_t)(a.y + 1) & 15u) << 4 | ((uint32_t)(a.z + 1) & 15u) << 8 |
+                ((uint32_t)(a.w + 1) & 15u) << 12 | ((uint32_t)(b.x + 1) & 15u) << 16 |
+                ((uint32_t)(b.y + 1) & 15u) << 20 | ((uint32_t)(b.z + 1) & 15u) << 24 | ((uint32_t)(b.w + 1) & 15u) << 28;
+        } else {
+            for (uint64_t j = i; j < n; ++j) w |= ((uint32_t)(in[j] + 1) & 15u) << (4 * (j - i));
+        }
+        out[g] = w;
+    }
+}
+
+cudaError_t launch_pack4(const int32_t *in, uint32_t *out, uint64_t n, cudaStream_t s)
+{
+    const unsigned blocks = (unsigned)std::max<uint64_t>(1, std::min<uint64_t>((n / 8 + 255) / 256, 148 * 8));
+    pack4_kernel<<<blocks, 256, 0, s>>>(in, out, n);
+    return cudaGetLastError();
+}
+
 cudaError_t launch_pack8(const int32_t *in, int8_t *out, uint64_t n, cudaStream_t s)
 {
     const unsigned blocks = (unsigned)std::max<uint64_t>(1, std::min<uint64_t>((n / 4 + 255) / 256, 148 * 8));

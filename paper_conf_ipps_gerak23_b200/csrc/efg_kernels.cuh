@@ -130,6 +130,7 @@ cudaError_t launch_gather64(const double *stored, const uint32_t *new_of_old, do
 cudaError_t launch_map_depth(const int32_t *stored, const uint32_t *new_of_old, int32_t *out, uint64_t n,
                              cudaStream_t s);
 cudaError_t launch_pack8(const int32_t *in, int8_t *out, uint64_t n, cudaStream_t s);  // n % 4 handled
+cudaError_t launch_pack4(const int32_t *in, uint32_t *out, uint64_t n, cudaStream_t s);  // n % 8 handled
 cudaError_t launch_map_parent(const uint32_t *pin, const uint32_t *old_of_new, uint32_t *pout, uint64_t n,
                               cudaStream_t s);
 

@@ -184,3 +184,25 @@ def test_host_widen_i8_i32():
             f(s.ctypes.data + off, d.ctypes.data + 4 * off, n)
             assert np.array_equal(d[off:off + n], s[off:off + n].astype(np.int32)), (n, off)
             assert np.all(d[:off] == 777) and np.all(d[off + n:] == 777)
+
+
+def test_host_widen_u4_i32():
+    """4-bit codes of the compact depth transfer: vertex i is nibble i & 7 of
+    word i >> 3 (low nibble first), depth = code - 1 (code 0 = unreached)."""
+    import ctypes as C
+    from paper_conf_ipps_gerak23_b200 import _abi
+    f = getattr(C.CDLL(_abi.LIB_PATH), "_ZN3efg17host_widen_u4_i32EPKjPil")
+    f.restype = None
+    f.argtypes = [C.c_void_p, C.c_void_p, C.c_int64]
+    rng = np.random.default_rng(6)
+    for n in (0, 1, 7, 8, 9, 63, 64, 65, 1000, 4097, 100003):
+        for off in (0, 1, 8):
+            depth = rng.integers(-1, 15, size=n).astype(np.int32)
+            codes = (depth + 1).astype(np.uint32)
+            words = np.zeros((n + 7) // 8 + 1, np.uint32)
+            for j in range(8):
+                np.bitwise_or.at(words, np.arange(j, n, 8) // 8, codes[j::8] << np.uint32(4 * j))
+            d = np.full(n + 16, 777, np.int32)
+            f(words.ctypes.data, d.ctypes.data + 4 * off, n)
+            assert np.array_equal(d[off:off + n], depth), (n, off)
+            assert np.all(d[:off] == 777) and np.all(d[off + n:] == 777)

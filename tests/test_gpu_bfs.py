@@ -294,10 +294,11 @@ def test_long_path_many_levels(efg):
     g.free()
 
 
-@pytest.mark.parametrize("plen", [125, 126, 127, 128, 300])
+@pytest.mark.parametrize("plen", [1, 2, 13, 14, 15, 16, 125, 126, 127, 128, 300])
 def test_host_depth_transfer_levels_boundary(efg, plen):
-    """Host depth arrays cross PCIe as 1 byte per vertex only while every depth
-    fits [-1, 126]: paths around the boundary, plus unreached vertices (-1)."""
+    """Host depth arrays cross PCIe as 4 bits per vertex while the BFS has
+    fewer than 15 levels, as 1 byte while every depth fits [-1, 126], else as
+    int32: paths around both boundaries, plus unreached vertices (-1)."""
     n = 5000
     src = np.arange(plen - 1, dtype=np.uint32)
     g = efg.Graph.build(n, src, src + 1)
@@ -305,7 +306,7 @@ def test_host_depth_transfer_levels_boundary(efg, plen):
     ref = np.full(n, -1, np.int32)
     ref[:plen] = np.arange(plen)
     assert np.array_equal(d, ref)
-    assert st["d2h_bytes"] == (n if plen < 127 else 4 * n)
+    assert st["d2h_bytes"] == ((n + 7) // 8 * 4 if plen < 15 else n if plen < 127 else 4 * n)
     g.free()
 
 
