@@ -778,7 +778,9 @@ __global__ void __launch_bounds__(kFrontierThreads, 1024 / kFrontierThreads) fro
 //               no select is needed) and stages the lower fields and upper
 //               words into shared memory with TMA bulk copies (cp.async.bulk,
 //               completion on a per-buffer mbarrier), one batch ahead of the
-//               decoder (double buffering);
+//               decoder (double buffering); BFS chunk skip: a chunk whose
+//               last element (high part = its forward pointer) is below
+//               the visited prefix becomes an empty slot, nothing staged;
 //   (rounds)    lays the batch's upper-bit words end to end (kRoundWords per
 //               round), masks each chunk's first/last word and keeps the
 //               non-zero words as 16-byte records {word, hi base, lower-field
@@ -925,6 +927,10 @@ constexpr bool kUseHot = kHotWords > 4;  // shared-memory visited snapshot compi
 #define EFG_KU 4
 #endif
 constexpr int kU = EFG_KU;  // elements per lane whose probes are in flight together
+#ifndef EFG_CHUNK_SKIP
+#define EFG_CHUNK_SKIP 1
+#endif
+constexpr bool kChunkSkip = EFG_CHUNK_SKIP;  // BFS: k-chunks wholly below the visited prefix are not staged
 
 template <int MODE>
 __global__ void __launch_bounds__(kExpandThreads, 1) expand_kernel(ExpandArgs a)
@@ -996,6 +1002,7 @@ __global__ void __launch_bounds__(kExpandThreads, 1) expand_kernel(ExpandArgs a)
         const bool valid = c < cend;
         uint64_t lb = 0, A0 = 0, A1 = 0;
         uint32_t l = 0, nel = 0, hib = 0, v = 0, cc = 0;
+        bool skipc = false;  // an empty slot: no elements, no words, no bytes
         if (valid) {
             const uint4 d0 = *reinterpret_cast<const uint4 *>(a.chunks + c);
             const uint64_t offl = ((uint64_t)d0.y << 32) | d0.x;
@@ -1013,9 +1020,13 @@ __global__ void __launch_bounds__(kExpandThreads, 1) expand_kernel(ExpandArgs a)
             // chunk cc starts right after element r0-1, whose stop bit is
             // fwd[cc-1] + r0 - 1; it ends after element r1-1 (C14)
             hib = cc ? ld_u32_unaligned(data32, off + 4 * (uint64_t)(cc - 1)) : 0u;
-            const uint64_t b1 = r1 < deg ? (uint64_t)ld_u32_unaligned(data32, off + 4 * (uint64_t)cc) + r1
-                                         : 8ull * ubytes;
-            nel = (uint32_t)(r1 - r0);
+            const uint32_t fwdc = r1 < deg ? ld_u32_unaligned(data32, off + 4 * (uint64_t)cc) : 0u;
+            const uint64_t b1 = r1 < deg ? (uint64_t)fwdc + r1 : 8ull * ubytes;
+            // BFS chunk skip: fwd[cc] is the high part of the chunk's last
+            // element, so fwd[cc] < vpre >> l puts every element of the chunk
+            // below the visited prefix: nothing to stage, decode or probe
+            skipc = kChunkSkip && pskip && r1 < deg && fwdc < (vpre >> l);
+            nel = skipc ? 0u : (uint32_t)(r1 - r0);
             lb = lbase + r0 * l;
             A0 = U0 + (cc ? (uint64_t)hib + r0 : 0);
             A1 = U0 + b1;
@@ -1026,7 +1037,7 @@ __global__ void __launch_bounds__(kExpandThreads, 1) expand_kernel(ExpandArgs a)
         uint32_t bytes = 0, lsz = 0;
         bool ustage = false, merged = false;
         uint32_t nwd = 0;
-        if (valid) {
+        if (valid && !skipc) {
             if (l) {
                 lg0 = (lb >> 3) & ~15ull;
                 lg1 = ((((lb + (uint64_t)nel * l - 1) >> 5) * 4 + 8) + 15) & ~15ull;
