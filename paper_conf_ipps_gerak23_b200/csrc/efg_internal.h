@@ -152,7 +152,7 @@ constexpr int kBitmapAlign = 1024;           // bitmap words are padded to a mul
 // kChunkWork units (descriptor, staging, set-up) plus one per element, so a
 // tile of kTileWork units holds at most kTileWork/kChunkWork chunks.
 #ifndef EFG_TILE_WORK
-#define EFG_TILE_WORK 1024
+#define EFG_TILE_WORK 2048
 #endif
 constexpr uint32_t kTileWork = EFG_TILE_WORK;         // work units per tile (a3)
 constexpr uint32_t kChunkWork = 32;          // per-chunk overhead in work units
