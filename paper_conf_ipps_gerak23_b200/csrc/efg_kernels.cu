@@ -435,7 +435,7 @@ __global__ void __launch_bounds__(kFrontierThreads, 1024 / kFrontierThreads) fro
     const uint64_t WG = 32ull * G;  // words between a warp's groups
     const uint32_t lt = (1u << lane) - 1;
 #ifndef EFG_KB
-#define EFG_KB 8
+#define EFG_KB 4
 #endif
     constexpr int kB = EFG_KB;  // pass 1: non-empty words whose degree loads are in flight together
 
