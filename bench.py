@@ -4,8 +4,9 @@
 Contract (driver): ``python bench.py --gpus N --steps K --warmup W`` prints ONE
 JSON line on rank 0.  A "step" is one full BFS (all levels: frontier
 materialisation, scan, partition, decode, visit, compaction — SURVEY §8(a)
-rows a1-a7) from one seeded source over the BASELINE.json configs[1] graph
-(RMAT scale 24, edgefactor 16) resident in HBM.
+rows a1-a7) from one seeded source over the BASELINE.json configs[2] graph
+(Twitter-shaped power-law graph, the config the 1/2/4/8-GPU metric is quoted
+on; ``--config 2`` = RMAT-24/ef16, ``--config 4`` = web-shaped) resident in HBM.
 
   value      whole-job GTEPS = sum over ranks of traversed edges / max-over-ranks
              device time (traversed edges = sum of degrees of reached vertices,
@@ -16,10 +17,14 @@ rows a1-a7) from one seeded source over the BASELINE.json configs[1] graph
              frontier + 21 B per frontier vertex) / its
              CUDA-event time, against MEASURED_PEAKS.json hbm_gbs
   cpu_baseline  the oracle (plain single-threaded FIFO BFS over CSR) timed on
-             this host on a bounded sample (one BFS of the same graph)
+             this host on a bounded sample (one BFS of the same graph, pinned to
+             one core, in a spawned process that overlaps the GPU work), with a
+             bit-exact depth check against the GPU BFS from that source
 
-``--impl reference`` runs the reference arm: the oracle, as it stands, on the
-host cores, same config/metric (each step = one oracle BFS).
+``--impl reference`` runs the reference arm: the oracle, as it stands, on one
+host core, same config/metric; each step is a bounded sample of one BFS (the
+oracle's FIFO BFS from that step's source, stopped after 2^28 scanned edges:
+or_bfs_bounded), so that the whole run stays within minutes on C3/C4.
 With N > 1 (torchrun) the default is the north_star's 1-D row partition: each
 rank holds a byte-balanced row range of the EFG, every BFS level exchanges the
 new-vertex bitmap ("scaling": "strong"): by default the library's kernels
@@ -55,10 +60,13 @@ def parse():
     p.add_argument("--steps", type=int, default=10)
     p.add_argument("--warmup", type=int, default=3)
     p.add_argument("--impl", default="efg", choices=["efg", "reference"])
-    p.add_argument("--config", type=int, default=2, help="BASELINE.json config index (1-based)")
+    p.add_argument("--config", type=int, default=3, help="BASELINE.json config index (1-based); "
+                   "3 = twitter_like, the config of the 1/2/4/8-GPU metric")
     p.add_argument("--scale", type=int, default=None, help="override RMAT scale (debug only)")
     p.add_argument("--no-cpu-baseline", action="store_true")
-    p.add_argument("--no-alt", action="store_true", help="skip the reorder=none comparison run")
+    p.add_argument("--no-alt", action="store_true", help="skip the reorder=none comparison run "
+                   "(run by default on the configs that name it: C2 and C4 'with and without reordering')")
+    p.add_argument("--alt", action="store_true", help="force the reorder=none comparison run")
     p.add_argument("--mode", default="partition", choices=["partition", "replicas"],
                    help="N > 1: 1-D partitioned BFS with a per-level NCCL exchange (SURVEY 8(e)), "
                         "or independent replicas on disjoint sources")
@@ -70,10 +78,18 @@ def parse():
                    help="EFG_REORDER_DEGREE relabelling at build time (results stay in input ids)")
     p.add_argument("--profile-levels", action="store_true", help="print per-level stats to stderr")
     p.add_argument("--no-sssp", action="store_true",
-                   help="skip the SSSP (NEXT-1) timing over the same graph built with synthetic weights")
+                   help="skip the SSSP (NEXT-1) timing over the same graph built with synthetic weights "
+                        "(on by default on C4, BASELINE configs[3] 'BFS and SSSP')")
+    p.add_argument("--sssp", action="store_true", help="force the SSSP timing on other configs")
     p.add_argument("--no-pagerank", action="store_true",
-                   help="skip the PageRank measurement (BASELINE configs[1]: BFS and PageRank)")
-    return p.parse_args()
+                   help="skip the PageRank measurement (on by default on C2, BASELINE configs[1]: "
+                        "BFS and PageRank)")
+    p.add_argument("--pagerank", action="store_true", help="force the PageRank timing on other configs")
+    a = p.parse_args()
+    a.do_alt = (a.alt or a.config in (2, 4)) and not a.no_alt
+    a.do_sssp = (a.sssp or a.config == 4) and not a.no_sssp
+    a.do_pagerank = (a.pagerank or a.config == 2) and not a.no_pagerank
+    return a
 
 
 def dist_env():
@@ -176,16 +192,17 @@ class ClockSampler:
 
 
 def load_traffic(workload: str, reorder: str):
-    """dram bytes per expand launch from the committed ncu capture of this
-    workload (profiles/r1_expand_traffic.json), or None."""
-    path = os.path.join(ROOT, "profiles", "r1_expand_traffic.json")
-    if not os.path.exists(path):
-        return None
-    with open(path) as f:
-        t = json.load(f)
-    if t.get("workload") != workload or t.get("reorder") != reorder:
-        return None
-    return t
+    """dram bytes per expand launch from the newest committed ncu capture of
+    this workload (profiles/r<NN>_expand_traffic*.json, written by
+    tools/expand_traffic.py), or None."""
+    import glob
+    for path in sorted(glob.glob(os.path.join(ROOT, "profiles", "r*_expand_traffic*.json")), reverse=True):
+        with open(path) as f:
+            t = json.load(f)
+        if t.get("workload") == workload and t.get("reorder") == reorder:
+            t["file"] = os.path.relpath(path, ROOT)
+            return t
+    return None
 
 
 def load_peak():
@@ -204,17 +221,89 @@ def make_graph_edges(cfg: int, scale: int | None):
     return n, src, dst, time.time() - t0
 
 
-def cpu_count_used() -> int:
-    return 1  # the oracle is single-threaded by construction
+def cpu_model() -> str:
+    try:
+        with open("/proc/cpuinfo") as f:
+            for line in f:
+                if line.startswith("model name"):
+                    return line.split(":", 1)[1].strip()
+    except OSError:
+        pass
+    return "unknown"
+
+
+REF_STEP_EDGES = 1 << 28  # reference-arm step: FIFO BFS stopped after this many scanned edges
+
+
+def _cpu_baseline_child(cfg: int, scale, index: int, count: int, out_dir: str, core: int):
+    """Spawned process (bench.py cpu_baseline leg): the oracle's CSR of the
+    same seeded graph, then ONE plain single-threaded FIFO BFS from the first
+    timed source, pinned to `core` (the parent keeps off that core).  Writes
+    depth.npy and meta.json to out_dir."""
+    import oracle
+    import synth
+    n, src, dst = synth.config_edges(cfg, scale_override=scale)
+    os.sched_setaffinity(0, {core})
+    t0 = time.time()
+    ov, oe = oracle.csr_build(n, src, dst)
+    csr_s = time.time() - t0
+    del src, dst
+    deg = np.diff(ov)
+    s0 = int(synth.sources(n, count, seed=1000 + cfg, nonisolated_mask=deg > 0)[index])
+    t = time.perf_counter()
+    d = oracle.bfs(ov, oe, s0)
+    cs = time.perf_counter() - t
+    np.save(os.path.join(out_dir, "depth.npy"), d)
+    with open(os.path.join(out_dir, "meta.json"), "w") as f:
+        json.dump({"source": s0, "bfs_s": cs, "csr_s": csr_s, "edges": int(deg[d >= 0].sum()),
+                   "core": core, "affinity": sorted(os.sched_getaffinity(0))}, f)
+
+
+def start_cpu_baseline(args, count: int, index: int):
+    """Start the cpu_baseline child on the last host core and move this
+    process (and every thread it creates from now on) off that core."""
+    import multiprocessing as mp
+    import tempfile
+    cores = sorted(os.sched_getaffinity(0))
+    core = cores[-1]
+    out_dir = tempfile.mkdtemp(prefix="efg_cpu_baseline_")
+    proc = mp.get_context("spawn").Process(target=_cpu_baseline_child,
+                                            args=(args.config, args.scale, index, count, out_dir, core))
+    proc.start()
+    if len(cores) > 1:
+        os.sched_setaffinity(0, set(cores[:-1]))
+    return proc, out_dir
+
+
+def finish_cpu_baseline(proc, out_dir: str, g, n: int):
+    proc.join()
+    if proc.exitcode != 0:
+        return {"unavailable": f"cpu_baseline process exited with {proc.exitcode}"}
+    with open(os.path.join(out_dir, "meta.json")) as f:
+        meta = json.load(f)
+    dref = np.load(os.path.join(out_dir, "depth.npy"))
+    ok = bool(np.array_equal(dref, g.bfs(meta["source"])))
+    return {"value": meta["edges"] / meta["bfs_s"] / 1e9, "unit": UNIT, "cores": 1, "kind": "oracle",
+            "sample": f"one single-threaded FIFO BFS (source {meta['source']}, {meta['edges']} edges) over "
+                      f"the oracle CSR of the same graph ({meta['bfs_s']:.1f} s; CSR build "
+                      f"{meta['csr_s']:.1f} s untimed), pinned to host core {meta['core']} "
+                      f"(sched_setaffinity = taskset -c {meta['core']}; bench's own threads kept off it)",
+            "cpu_model": cpu_model(), "host_cores": os.cpu_count(),
+            "parity_bit_exact": ok, "parity_source": meta["source"]}
 
 
 def run_reference(args, rank, world):
-    """Reference arm: the oracle (plain CPU BFS) on the host, rank 0 only."""
+    """Reference arm: the oracle (plain CPU BFS) on one host core, rank 0 only.
+    Each step (warm-up and timed) is a bounded sample of one BFS: the oracle's
+    FIFO BFS from that step's source, stopped once REF_STEP_EDGES adjacency
+    entries were scanned (or_bfs_bounded); GTEPS = scanned edges / time."""
     if rank != 0:
         return
     import oracle
     import synth
     n, src, dst, gen_s = make_graph_edges(args.config, args.scale)
+    core = sorted(os.sched_getaffinity(0))[-1]
+    os.sched_setaffinity(0, {core})
     t0 = time.time()
     vlist, elist = oracle.csr_build(n, src, dst)
     csr_s = time.time() - t0
@@ -223,23 +312,27 @@ def run_reference(args, rank, world):
     srcs = synth.sources(n, args.warmup + args.steps, seed=1000 + args.config,
                          nonisolated_mask=deg > 0)
     for s in srcs[:args.warmup]:
-        oracle.bfs(vlist, elist, int(s))
-    edges, secs = 0, 0.0
+        oracle.bfs_bounded(vlist, elist, int(s), REF_STEP_EDGES)
+    edges, secs, full = 0, 0.0, 0
     for s in srcs[args.warmup:]:
         t = time.perf_counter()
-        d = oracle.bfs(vlist, elist, int(s))
+        d, nv, scanned = oracle.bfs_bounded(vlist, elist, int(s), REF_STEP_EDGES)
         secs += time.perf_counter() - t
-        edges += int(deg[d >= 0].sum())
+        edges += scanned
+        full += int(scanned < REF_STEP_EDGES)
     v = edges / secs / 1e9
     cfgname = synth.CONFIGS[args.config]["name"] + (f"_scale{args.scale}" if args.scale else "")
+    sample = (f"{args.steps} single-threaded FIFO BFS over the oracle CSR, each stopped after "
+              f"{REF_STEP_EDGES} scanned edges ({full} ran to completion); pinned to host core {core}")
     line = {"impl": "reference", "metric": METRIC, "value": v, "unit": UNIT, "n_gpus": args.gpus,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": secs / args.steps * 1e3,
             "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u32",
             "data": "synthetic",
             "config": {"workload": cfgname, "n": int(n), "m_directed": int(vlist[-1]),
-                       "sources": args.steps, "csr_build_s": round(csr_s, 2)},
-            "cpu_baseline": {"value": v, "unit": UNIT, "cores": 1, "kind": "oracle",
-                             "sample": f"{args.steps} single-threaded FIFO BFS over the oracle CSR"},
+                       "sources": args.steps, "csr_build_s": round(csr_s, 2),
+                       "step_edges_cap": REF_STEP_EDGES},
+            "cpu_baseline": {"value": v, "unit": UNIT, "cores": 1, "kind": "oracle", "sample": sample,
+                             "cpu_model": cpu_model()},
             "e2e": {"value": v, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
 
@@ -346,6 +439,11 @@ def main():
     if args.impl == "reference":
         run_reference(args, rank, world)
         return
+    # the oracle baseline runs in a spawned process on its own core while this
+    # process builds and measures (started before any thread pool exists here)
+    cpu_job = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        cpu_job = start_cpu_baseline(args, args.warmup + args.steps, args.warmup)
 
     import torch
     import synth
@@ -479,7 +577,7 @@ def main():
 
     # ---- the same measurement without the degree relabelling (transparency) ----
     alt = None
-    if world == 1 and args.reorder == "degree" and not args.no_alt:
+    if world == 1 and args.reorder == "degree" and args.do_alt:
         n2, s2, d2, _ = make_graph_edges(args.config, args.scale)
         g2 = efg.Graph.build(n2, s2, d2, device=local, stream=stream.cuda_stream)
         del s2, d2
@@ -524,7 +622,7 @@ def main():
     # ---- PageRank over the same EFG (BASELINE configs[1] "BFS and PageRank"):
     # 50 push iterations, fp64 accumulation (reading C21) ----
     pr = None
-    if world == 1 and not args.no_pagerank:
+    if world == 1 and args.do_pagerank:
         rank_d = torch.empty(n, dtype=torch.float64, device=dev)
         with torch.cuda.stream(stream):
             g.pagerank(0.85, 50, rank=rank_d)  # warm-up (builds the all-vertex plan once)
@@ -545,7 +643,7 @@ def main():
     # ---- SSSP (NEXT-1; BASELINE configs[3] "BFS and SSSP with synthetic
     # weights"): frontier Bellman-Ford over the EFG, fp32 weights (reading C20) ----
     sssp = None
-    if world == 1 and not args.no_sssp:
+    if world == 1 and args.do_sssp:
         n3, s3, d3, _ = make_graph_edges(args.config, args.scale)
         w3 = synth.weights(s3, d3, 2000 + args.config)
         g3 = efg.Graph.build(n3, s3, d3, device=local, stream=stream.cuda_stream, flags=flags, weights=w3)
@@ -577,22 +675,10 @@ def main():
 
     # ---- cpu baseline: the oracle on a bounded sample (rank 0, N=1 only) ----
     cpu = None
-    if rank == 0 and world == 1 and not args.no_cpu_baseline:
-        import oracle
-        t0 = time.time()
-        ov, oe = oracle.csr_build(n, *synth.config_edges(args.config, scale_override=args.scale)[1:])
-        csr_s = time.time() - t0
-        s0 = stats[0][0]
-        t = time.perf_counter()
-        dref = oracle.bfs(ov, oe, s0)
-        cs = time.perf_counter() - t
-        ce = int(np.diff(ov)[dref >= 0].sum())
-        ok = bool(np.array_equal(dref, g.bfs(s0)))
-        cpu = {"value": ce / cs / 1e9, "unit": UNIT, "cores": 1, "kind": "oracle",
-               "sample": f"one single-threaded FIFO BFS (source {s0}) over the oracle CSR of the "
-                         f"same graph ({cs:.1f} s; CSR build {csr_s:.1f} s untimed)",
-               "parity_bit_exact": ok}
-        del ov, oe
+    if cpu_job is not None:
+        cpu = finish_cpu_baseline(*cpu_job, g, n)
+        if "parity_source" in cpu and cpu["parity_source"] != stats[0][0]:
+            cpu["parity_note"] = "source differs from the first timed source"
 
     if rank == 0:
         cfgname = synth.CONFIGS[args.config]["name"] + (f"_scale{args.scale}" if args.scale else "")
@@ -617,7 +703,13 @@ def main():
                          "achieved": achieved, "peak": peak, "unit": "GB/s",
                          "frac": achieved / peak,
                          "traffic": (trf or {}).get("dram_bytes_per_launch"),
-                         "traffic_source": (trf or {}).get("source"),
+                         "traffic_source": ((trf or {}).get("source") or "") + (
+                             f" ({trf['file']})" if trf else ""),
+                         # ncu-measured DRAM bandwidth of the heaviest expand launch
+                         # (dram__bytes_read+write / gpu__time_duration, cold cache)
+                         "dram_heavy_launch": (trf or {}).get("heavy"),
+                         "frac_dram_heavy_launch": ((trf or {}).get("heavy") or {}).get("gbps", 0) / peak
+                         if trf and trf.get("heavy") else None,
                          "alg_bytes_per_launch": alg_bytes / max(exp_launch, 1),
                          "peak_source": peak_src,
                          "expand_launches": exp_launch, "expand_ms_total": exp_ms,

@@ -17,7 +17,12 @@
  *   - A handle is not safe for concurrent calls from several threads; distinct
  *     handles are independent.  All GPU work of a handle is issued on the
  *     stream given at build time, and every call synchronises that stream
- *     before returning (results are complete on return).
+ *     before returning (results are complete on return) — except the
+ *     enqueue-only form of efg_bfs (device outputs, st == NULL) and the
+ *     partitioned step calls, which are stream-ordered (see each call).
+ *   - A device-side barrier that times out (efg_bfs, the peer exchange) sets a
+ *     sticky fault in the handle; every later synchronous call on it returns
+ *     EFG_ECUDA.
  */
 #ifndef EFG_H
 #define EFG_H
@@ -56,8 +61,11 @@ typedef struct efg_graph efg_graph; /* opaque: host EFG arrays + device copy */
 
 typedef struct efg_build_opts {
     /* Forward-pointer quantum k (§VI-C; k = 512 in the paper's
-     * experiments).  0 disables forward pointers (lists are then never
-     * split across warps).  Default 512. */
+     * experiments).  0 disables forward pointers.  Default 512.  Any k
+     * is accepted: the host arrays (efg_export) use k; the device copy splits
+     * lists into k-element chunks when 1 <= k <= 512 and every list has fewer
+     * than 2^18 chunks, else it re-samples the pointers every 512 elements
+     * (efg_info_t.device_quantum).  Results do not depend on k. */
     uint32_t fwd_quantum;
     /* EFG_* flags above.  Default EFG_DEFAULT_FLAGS. */
     uint32_t flags;
@@ -122,6 +130,11 @@ typedef struct efg_info_t {
     uint64_t device_bytes;   /* device memory held by the handle                   */
     uint64_t row_lo, row_hi; /* owned row range (whole graph: 0, n)                */
     double build_seconds;    /* host builder wall time                             */
+    uint32_t device_quantum; /* chunk length of the device copy: fwd_quantum when  *
+                              * 1 <= k <= 512 and ceil(deg/k) < 2^18 for every    *
+                              * list, else 512 (the device copy's forward         *
+                              * pointers are re-sampled; the host arrays keep k)  */
+    uint32_t reserved_;
 } efg_info_t;
 
 efg_status efg_info(const efg_graph *g, efg_info_t *info);
@@ -175,14 +188,22 @@ typedef struct efg_stats {
  * (reading C15).  parent (nullable): some neighbour u with depth[u] ==
  * depth[v]-1 (any valid one, reading C28); parent[source] = source; unreached
  * 0xFFFFFFFF.  depth / parent: host or device, n entries, caller-allocated.
- * With a partitioned handle the call is collective over the communicator:
- * every rank calls it with the same source and receives the full depth array.
+ * Partitioned handle (row_lo/row_hi): the call is COLLECTIVE
+ * over the peer exchange opened with efg_peer_alloc / efg_peer_open — every
+ * rank calls it with the same source; each level expands the rank's own rows,
+ * ORs the new bits over peer memory (efg_xchg_peer) and ends the level over
+ * the now-global bitmap, so every rank receives the full depth array.  The
+ * loop ends on the device when the global new count is 0 (identical on every
+ * rank).  Without an open peer exchange it returns EFG_ESTATE (drive the
+ * levels with efg_bfs_begin / expand / xchg_* / finish_level instead);
+ * parent != NULL returns EFG_ENOTSUP.  st then counts this rank's rows.
  * Completion: with device outputs (depth and parent, if any) and st == NULL
  * the call only enqueues the BFS on the handle's stream (efg_build_opts
  * stream) and returns; the outputs are valid once that stream is
- * synchronised (stream order, as cudaMemcpyAsync).  Otherwise it returns with
- * the outputs written.
- * Errors: EFG_ERANGE (source >= n), EFG_ESTATE, EFG_ECUDA, EFG_ENCCL.
+ * synchronised (stream order, as cudaMemcpyAsync).  A barrier time-out in
+ * that form is reported by the next synchronous call.  Otherwise it returns
+ * with the outputs written.
+ * Errors: EFG_ERANGE (source >= n), EFG_ESTATE, EFG_ENOTSUP, EFG_ECUDA.
  */
 efg_status efg_bfs(efg_graph *g, uint32_t source, int32_t *depth, uint32_t *parent,
                    efg_stats *st);
@@ -192,7 +213,8 @@ efg_status efg_bfs(efg_graph *g, uint32_t source, int32_t *depth, uint32_t *pare
  * §VI-F): frontier Bellman-Ford, relaxed vertices marked in a bitmap, fp32
  * distances with single-rounding adds (dist[u] + w, no contraction; reading
  * C20).  dist: host or device, n entries; unreached = +inf.
- * Errors: EFG_EINVAL (graph built without weights), EFG_ERANGE, EFG_ESTATE.
+ * Errors: EFG_EINVAL (graph built without weights), EFG_ERANGE, EFG_ESTATE,
+ * EFG_ENOTSUP (partitioned handle).
  */
 efg_status efg_sssp(efg_graph *g, uint32_t source, float *dist, efg_stats *st);
 
@@ -202,6 +224,7 @@ efg_status efg_sssp(efg_graph *g, uint32_t source, float *dist, efg_stats *st);
  * r' = (1-d)/N + d*(sum_{u in N(v)} r(u)/deg(u) + D/N), D = rank mass on
  * degree-0 vertices, exactly `iters` iterations, fp64 accumulation.
  * rank: host or device, n doubles.
+ * Errors: EFG_EINVAL, EFG_ESTATE, EFG_ENOTSUP (partitioned handle).
  */
 efg_status efg_pagerank(efg_graph *g, double damping, uint32_t iters, double *rank,
                         efg_stats *st);

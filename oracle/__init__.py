@@ -57,6 +57,8 @@ def lib():
         L.or_csr_free.argtypes = [C.c_void_p]
         L.or_bfs.restype = C.c_uint64
         L.or_bfs.argtypes = [C.c_uint64, u64p, u32p, C.c_uint32, i32p]
+        L.or_bfs_bounded.restype = C.c_uint64
+        L.or_bfs_bounded.argtypes = [C.c_uint64, u64p, u32p, C.c_uint32, i32p, C.c_uint64, u64p]
         L.or_ef_lower_bits.restype = C.c_uint32
         L.or_ef_lower_bits.argtypes = [C.c_uint64, C.c_uint64]
         L.or_ef_sections.restype = None
@@ -120,6 +122,18 @@ def bfs(vlist: np.ndarray, elist: np.ndarray, source: int) -> np.ndarray:
     el = elist if elist.size else np.zeros(1, np.uint32)
     lib().or_bfs(n, _ptr(vlist, u64p), _ptr(el, u32p), source, _ptr(depth, i32p))
     return depth
+
+
+def bfs_bounded(vlist: np.ndarray, elist: np.ndarray, source: int, max_edges: int):
+    """FIFO BFS stopped once `max_edges` adjacency entries were scanned:
+    (depth, dequeued vertices, edges scanned).  Assigned depths are final."""
+    n = vlist.size - 1
+    depth = np.empty(n, np.int32)
+    el = elist if elist.size else np.zeros(1, np.uint32)
+    scanned = np.zeros(1, np.uint64)
+    nv = lib().or_bfs_bounded(n, _ptr(vlist, u64p), _ptr(el, u32p), source, _ptr(depth, i32p),
+                              max_edges, _ptr(scanned, u64p))
+    return depth, int(nv), int(scanned[0])
 
 
 # --------------------------------------------------------------------------

@@ -14,6 +14,8 @@
  *                   C11 (drop duplicates and self-loops) and C12 (symmetrise).
  *   or_bfs          BFS depth by its plain definition: FIFO queue BFS
  *                   (Alg. 1 semantics, §III-B).  depth = hop distance.
+ *   or_bfs_bounded  the same BFS stopped after a budget of scanned edges
+ *                   (bench.py reference arm: a bounded sample per step).
  *   or_ef_*         Elias-Fano list encoding / naive decoding (§IV,
  *                   Fig. 2, forward pointers P:157 §VI-C, EFG layout
  *                   P:111-117 §V), step by step in the order of SURVEY §8(c).
@@ -149,6 +151,41 @@ uint64_t or_bfs(uint64_t n, const uint64_t *vlist, const uint32_t *elist, uint32
     }
     free(q);
     return tail;
+}
+
+/* Bounded sample of the same FIFO BFS (bench.py reference arm only: a timed
+ * step must stay within seconds on the largest configs).  Identical to or_bfs
+ * except that it stops dequeuing once the adjacency entries scanned reach
+ * max_edges (the current vertex's list is always finished).  Every depth it
+ * assigns is final (a FIFO BFS assigns a vertex's depth once, at discovery),
+ * so depth[] is or_bfs's depth on the discovered vertices and -1 elsewhere.
+ * *edges_scanned = adjacency entries scanned (= sum of the degrees of the
+ * dequeued vertices).  Returns the number of dequeued vertices. */
+uint64_t or_bfs_bounded(uint64_t n, const uint64_t *vlist, const uint32_t *elist, uint32_t source,
+                        int32_t *depth, uint64_t max_edges, uint64_t *edges_scanned)
+{
+    for (uint64_t v = 0; v < n; ++v) depth[v] = -1;
+    *edges_scanned = 0;
+    if (source >= n) return 0;
+    uint32_t *q = (uint32_t *)malloc((n ? n : 1) * sizeof(uint32_t));
+    if (!q) return 0;
+    uint64_t head = 0, tail = 0, scanned = 0;
+    depth[source] = 0;
+    q[tail++] = source;
+    while (head < tail && scanned < max_edges) {
+        uint32_t u = q[head++];
+        for (uint64_t e = vlist[u]; e < vlist[u + 1]; ++e) {
+            uint32_t v = elist[e];
+            if (depth[v] < 0) {
+                depth[v] = depth[u] + 1;
+                q[tail++] = v;
+            }
+        }
+        scanned += vlist[u + 1] - vlist[u];
+    }
+    free(q);
+    *edges_scanned = scanned;
+    return head;
 }
 
 /* ------------------------------------------------------------------------- */

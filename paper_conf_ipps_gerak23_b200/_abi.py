@@ -36,7 +36,8 @@ class Info(C.Structure):
                 ("fwd_bytes", C.c_uint64), ("lower_bytes", C.c_uint64), ("upper_bytes", C.c_uint64),
                 ("apriori_bits", C.c_uint64), ("vertex_bytes", C.c_uint64),
                 ("device_bytes", C.c_uint64), ("row_lo", C.c_uint64), ("row_hi", C.c_uint64),
-                ("build_seconds", C.c_double)]
+                ("build_seconds", C.c_double), ("device_quantum", C.c_uint32),
+                ("reserved_", C.c_uint32)]
 
 
 class Stats(C.Structure):

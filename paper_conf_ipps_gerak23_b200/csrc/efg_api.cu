@@ -29,6 +29,9 @@ using namespace efg;
 
 namespace {
 
+// a handle of a 1-D row partition (efg_build_opts.row_lo / row_hi)
+bool partitioned(const efg_graph *g) { return !(g->host.row_lo == 0 && g->host.row_hi == g->host.n); }
+
 efg_status check_handle(efg_graph *g)
 {
     if (!g) return set_error(EFG_EINVAL, "null handle");
@@ -110,6 +113,7 @@ extern "C" efg_status efg_info(const efg_graph *g, efg_info_t *info)
     info->row_lo = h.row_lo;
     info->row_hi = h.row_hi;
     info->build_seconds = h.build_seconds;
+    info->device_quantum = g->on_device ? g->dev.k : 0;
     return EFG_OK;
 }
 
@@ -192,6 +196,7 @@ extern "C" efg_status efg_sssp(efg_graph *g, uint32_t source, float *dist, efg_s
     if (source >= g->dev.n) return set_error(EFG_ERANGE, "efg_sssp: source >= n");
     if (!dist) return set_error(EFG_EINVAL, "efg_sssp: dist is NULL");
     if (!g->dev.weights && g->host.m) return set_error(EFG_EINVAL, "efg_sssp: graph built without weights");
+    if (partitioned(g)) return set_error(EFG_ENOTSUP, "efg_sssp: not available on a partitioned (row-range) handle");
     const uint32_t s = g->host.new_of_old.empty() ? source : g->host.new_of_old[source];
     return device_sssp(g, s, dist, st);
 }
@@ -202,6 +207,7 @@ extern "C" efg_status efg_pagerank(efg_graph *g, double damping, uint32_t iters,
     EFG_TRY(check_handle(g));
     if (!rank) return set_error(EFG_EINVAL, "efg_pagerank: rank is NULL");
     if (!(damping >= 0.0 && damping <= 1.0)) return set_error(EFG_EINVAL, "efg_pagerank: damping outside [0,1]");
+    if (partitioned(g)) return set_error(EFG_ENOTSUP, "efg_pagerank: not available on a partitioned (row-range) handle");
     return device_pagerank(g, damping, iters, rank, st);
 }
 

@@ -74,6 +74,60 @@ int kshift_of(uint32_t k)
 
 cudaStream_t stream_of(const DeviceGraph &d) { return static_cast<cudaStream_t>(d.stream); }
 
+// The chunk length of the device copy.  The expand kernel stages one chunk's
+// lower fields in a kStageBytes buffer (<= 512 elements of <= 31 bits fit) and
+// stores the chunk index in kCcBits of the descriptor; a format quantum k
+// (any k >= 0 is a valid EFG) outside those limits — k = 0 (no
+// pointers), k > 512, or ceil(deg/k) >= 2^kCcBits — is served by re-sampling
+// the forward pointers at kMaxDeviceQuantum for the device (reading R3).
+uint32_t device_quantum(uint32_t k, uint64_t maxdeg)
+{
+    if (k >= 1 && k <= kMaxDeviceQuantum && (maxdeg + k - 1) / k < (1ull << kCcBits)) return k;
+    return kMaxDeviceQuantum;
+}
+
+// Device EF data with forward pointers every kd elements (fwd[j] =
+// select1((j+1)kd - 1) - ((j+1)kd - 1), the high part of that element): the
+// lower and upper sections are copied unchanged, the pointers are recomputed by
+// a select1 scan over the upper bits of each list.
+void resample_forward_pointers(const HostEFG &h, uint32_t kd, std::vector<uint8_t> &data,
+                               std::vector<uint64_t> &offsets)
+{
+    const uint64_t n = h.n;
+    offsets.assign(n + 1, 0);
+    for (uint64_t v = 0; v < n; ++v) {
+        const uint64_t dv = h.vlist[v + 1] - h.vlist[v];
+        const uint64_t hf = h.k ? 4 * (dv / h.k) : 0;
+        offsets[v + 1] = offsets[v] + (h.offsets[v + 1] - h.offsets[v]) - hf + 4 * (dv / kd);
+    }
+    data.assign(offsets[n], 0);
+#pragma omp parallel for schedule(dynamic, 1024)
+    for (int64_t v = 0; v < (int64_t)n; ++v) {
+        const uint64_t dv = h.vlist[v + 1] - h.vlist[v];
+        if (!dv) continue;
+        const uint64_t hf = h.k ? 4 * (dv / h.k) : 0;
+        const uint64_t body = h.offsets[v + 1] - h.offsets[v] - hf;  // lower + upper bytes
+        const uint64_t F = dv / kd, lower = (dv * h.nlb[v] + 7) / 8;
+        uint8_t *out = data.data() + offsets[v];
+        std::memcpy(out + 4 * F, h.data.data() + h.offsets[v] + hf, body);
+        const uint8_t *up = out + 4 * F + lower;
+        const uint64_t U = body - lower;
+        uint64_t ones = 0, target = kd - 1, j = 0;
+        for (uint64_t b = 0; b < U && j < F; ++b) {
+            const uint32_t byte = up[b], pc = (uint32_t)__builtin_popcount(byte);
+            while (j < F && ones + pc > target) {  // element `target` has its stop bit in this byte
+                uint32_t t = byte;
+                for (uint64_t r = target - ones; r; --r) t &= t - 1;
+                const uint32_t f = (uint32_t)(b * 8 + (uint64_t)__builtin_ctz(t) - target);
+                std::memcpy(out + 4 * j, &f, 4);
+                ++j;
+                target += kd;
+            }
+            ones += pc;
+        }
+    }
+}
+
 ExpandArgs expand_args(DeviceGraph &d, uint32_t *out)
 {
     ExpandArgs a;
@@ -103,6 +157,7 @@ ExpandArgs expand_args(DeviceGraph &d, uint32_t *out)
 FrontierArgs frontier_args(DeviceGraph &d, cudaGraphConditionalHandle cond, bool consume = false)
 {
     FrontierArgs a;
+    a.cond_global = 0;
     a.consume = consume ? 1 : 0;
     a.vis = d.vis;
     a.prev = d.prev;
@@ -140,17 +195,50 @@ FrontierArgs frontier_args(DeviceGraph &d, cudaGraphConditionalHandle cond, bool
 
 // level end + next plan: one launch (every block resident, see frontier_kernel)
 efg_status launch_level_end(DeviceGraph &d, cudaGraphConditionalHandle cond, cudaStream_t s,
-                            bool consume = false)
+                            bool consume = false, bool cond_global = false)
 {
-    CUDA_TRY(launch_frontier(frontier_args(d, cond, consume),
-                             (unsigned)((d.nwords + d.words_per_block - 1) / d.words_per_block), s));
+    FrontierArgs fa = frontier_args(d, cond, consume);
+    fa.cond_global = cond_global ? 1 : 0;
+    CUDA_TRY(launch_frontier(fa, (unsigned)((d.nwords + d.words_per_block - 1) / d.words_per_block), s));
     return EFG_OK;
 }
 
-// Build (once per handle and mode) the graph: while (frontier) { expand; frontier }
+PeerArgs peer_args(DeviceGraph &d, int op)
+{
+    PeerArgs a;
+    a.peers = d.peer_ptrs;
+    a.local = d.peer_region;
+    a.bounds = d.xchg_bounds;
+    a.vis = d.vis;
+    a.prev = d.prev;
+    a.fault = &d.ctrl->fault;
+    a.epoch = &d.ctrl->peer_epoch;
+    a.nwords = d.nwords;
+    a.world = d.peer_world;
+    a.rank = d.peer_rank;
+    a.op = op;
+    return a;
+}
+
+// the three peer-exchange launches of one level (publish, owner OR + broadcast, unpack)
+efg_status launch_peer_exchange(DeviceGraph &d, cudaStream_t s)
+{
+    for (int op = 0; op < 3; ++op) CUDA_TRY(launch_peer(peer_args(d, op), d.num_sms, s));
+    return EFG_OK;
+}
+
+// a handle of a 1-D row partition (efg_build_opts.row_lo / row_hi)
+bool partitioned(const efg_graph *g) { return !(g->host.row_lo == 0 && g->host.row_hi == g->host.n); }
+
+// Build (once per handle and mode) the graph:
+//   while (frontier) { expand; frontier }                          (modes 0, 1)
+//   while (global new) { expand; peer exchange; frontier }         (mode 2: partitioned)
+constexpr int kLoopPartitioned = 2;
 efg_status build_loop_graph(DeviceGraph &d, int mode)
 {
     if (d.loop_exec[mode]) return EFG_OK;
+    const bool part = mode == kLoopPartitioned;
+    const int emode = part ? (int)kModeVisit : mode;
     cudaGraph_t g;
     CUDA_TRY(cudaGraphCreate(&g, 0));
     cudaGraphConditionalHandle cond;
@@ -166,9 +254,11 @@ efg_status build_loop_graph(DeviceGraph &d, int mode)
     cudaStream_t cs;
     CUDA_TRY(cudaStreamCreateWithFlags(&cs, cudaStreamNonBlocking));
     CUDA_TRY(cudaStreamBeginCaptureToGraph(cs, body, nullptr, nullptr, 0, cudaStreamCaptureModeRelaxed));
-    const int blocks = d.num_sms * expand_occupancy(mode);
-    cudaError_t e1 = launch_expand(mode, expand_args(d, nullptr), blocks, cs);
-    efg_status st = e1 == cudaSuccess ? launch_level_end(d, cond, cs) : EFG_ECUDA;
+    const int blocks = d.num_sms * expand_occupancy(emode);
+    cudaError_t e1 = launch_expand(emode, expand_args(d, nullptr), blocks, cs);
+    efg_status st = e1 == cudaSuccess ? EFG_OK : EFG_ECUDA;
+    if (st == EFG_OK && part) st = launch_peer_exchange(d, cs);
+    if (st == EFG_OK) st = launch_level_end(d, cond, cs, false, part);
     cudaGraph_t captured;
     cudaError_t e2 = cudaStreamEndCapture(cs, &captured);
     cudaStreamDestroy(cs);
@@ -189,7 +279,7 @@ efg_status build_loop_graph(DeviceGraph &d, int mode)
 void device_drop_graphs(DeviceGraph &d)
 {
     if (d.device >= 0) cudaSetDevice(d.device);
-    for (int m = 0; m < 2; ++m) {
+    for (int m = 0; m < DeviceGraph::kLoopGraphs; ++m) {
         if (d.loop_exec[m]) cudaGraphExecDestroy(d.loop_exec[m]);
         if (d.loop_graph[m]) cudaGraphDestroy(d.loop_graph[m]);
         d.loop_exec[m] = nullptr;
@@ -253,18 +343,30 @@ efg_status device_upload(efg_graph *g, const efg_build_opts &o)
     d.num_sms = prop.multiProcessorCount;
 
     // the expand kernel stages select1(i) - i (< 2 * degree) in 27 bits
-    for (uint64_t v = 0; v < h.n; ++v)
-        if (h.vlist[v + 1] - h.vlist[v] >= (1ull << 26))
-            return set_error(EFG_ENOTSUP, "efg_build: a vertex degree >= 2^26 is not supported on the device");
+    uint64_t maxdeg = 0;
+    for (uint64_t v = 0; v < h.n; ++v) maxdeg = std::max<uint64_t>(maxdeg, h.vlist[v + 1] - h.vlist[v]);
+    if (maxdeg >= (1ull << 26))
+        return set_error(EFG_ENOTSUP, "efg_build: a vertex degree >= 2^26 is not supported on the device");
+
+    // device chunk quantum (reading R3): the format's k when every
+    // chunk fits the kernel's staging buffer and chunk-index field, else the
+    // forward pointers are re-sampled at kMaxDeviceQuantum for the device copy
+    d.k = device_quantum(h.k, maxdeg);
+    std::vector<uint8_t> rdata;       // re-sampled EF data (k != d.k), else empty
+    std::vector<uint64_t> roffsets;   // its per-vertex offsets
+    if (d.k != h.k) resample_forward_pointers(h, d.k, rdata, roffsets);
+    const std::vector<uint8_t> &ddata = d.k != h.k ? rdata : h.data;
+    const std::vector<uint64_t> &doffsets = d.k != h.k ? roffsets : h.offsets;
 
     // EF data, padded so 32-bit word reads past the last list stay in bounds
-    d.data_bytes = h.data.size();
+    d.data_bytes = ddata.size();
     if (d.data_bytes >= (1ull << kOffBits))
         return set_error(EFG_ENOTSUP, "efg_build: EF data of 1 TiB or more is not supported on the device");
     const uint64_t padded = ((d.data_bytes + 64) + 15) & ~15ull;
     EFG_TRY(dev_alloc(d, &d.data, padded));
     CUDA_TRY(cudaMemsetAsync(d.data, 0, padded, s));
-    if (d.data_bytes) CUDA_TRY(cudaMemcpyAsync(d.data, h.data.data(), d.data_bytes, cudaMemcpyHostToDevice, s));
+    if (d.data_bytes) CUDA_TRY(cudaMemcpyAsync(d.data, ddata.data(), d.data_bytes, cudaMemcpyHostToDevice, s));
+    CUDA_TRY(cudaStreamSynchronize(s));  // ddata may be a temporary
 
     // bitmap geometry
     const uint64_t words = (h.n + 31) / 32;
@@ -279,11 +381,11 @@ efg_status device_upload(efg_graph *g, const efg_build_opts &o)
     for (int64_t v = 0; v < (int64_t)h.n; ++v) {
         const uint64_t dv = h.vlist[v + 1] - h.vlist[v];
         const uint32_t l = h.nlb[v];
-        const uint64_t size = h.offsets[v + 1] - h.offsets[v];
-        const uint64_t fwd = h.k ? 4 * (dv / h.k) : 0;
+        const uint64_t size = doffsets[v + 1] - doffsets[v];
+        const uint64_t fwd = d.k ? 4 * (dv / d.k) : 0;
         const uint64_t lower = (dv * l + 7) / 8;
         VRec r;
-        r.off_l = (h.offsets[v] & kOffMask) | ((uint64_t)l << kOffBits);
+        r.off_l = (doffsets[v] & kOffMask) | ((uint64_t)l << kOffBits);
         r.deg = (uint32_t)dv;
         r.ubytes = (uint32_t)(dv ? size - fwd - lower : 0);
         rec[v] = r;
@@ -326,7 +428,7 @@ efg_status device_upload(efg_graph *g, const efg_build_opts &o)
     EFG_TRY(dev_alloc(d, &d.prev, d.nwords));
     // a level has at most one chunk per frontier vertex plus one per k elements
     const uint64_t rows = (h.row_hi > h.row_lo) ? h.row_hi - h.row_lo : h.n;
-    d.max_chunks = rows + (h.k ? h.m / h.k : 0) + 1;
+    d.max_chunks = rows + h.m / d.k + 1;
     d.max_tiles = (h.m + (uint64_t)kChunkWork * d.max_chunks) / kTileWork + 2;
     EFG_TRY(dev_alloc(d, &d.tiles, d.max_tiles + 1));
     EFG_TRY(dev_alloc(d, &d.chunks, d.max_chunks));
@@ -338,7 +440,7 @@ efg_status device_upload(efg_graph *g, const efg_build_opts &o)
     // lists planned grid-wide: more than one chunk (deg > k) or more than one
     // tile of work (deg > kTileWork - kChunkWork)
     {
-        const uint64_t q = h.k ? std::min<uint64_t>(h.k, kTileWork - kChunkWork) : kTileWork - kChunkWork;
+        const uint64_t q = std::min<uint64_t>(d.k, kTileWork - kChunkWork);
         d.max_big = std::min<uint64_t>(rows, h.m / q + 1);
         EFG_TRY(dev_alloc(d, &d.big, d.max_big));
     }
@@ -431,7 +533,18 @@ efg_status device_bfs(efg_graph *g, uint32_t source, int32_t *depth, uint32_t *p
         pd = (parent_dev && !relabel) ? parent : d.parent;
         pout = parent_dev ? parent : (relabel ? d.parent2 : d.parent);
     }
-    const int mode = parent ? kModeVisitParent : kModeVisit;
+    // partitioned handle: the BFS is collective over the peer exchange (every
+    // rank calls efg_bfs with the same source; each level = expand own rows,
+    // exchange the new bits, level end over the global bitmap)
+    const bool part = partitioned(g);
+    if (part && !d.peer_ptrs)
+        return set_error(EFG_ESTATE, "efg_bfs: a partitioned handle runs a collective BFS over the peer exchange: "
+                                     "call efg_peer_alloc / efg_peer_open first (or drive the levels with "
+                                     "efg_bfs_begin / efg_bfs_expand / efg_xchg_* / efg_bfs_finish_level)");
+    if (part && parent)
+        return set_error(EFG_ENOTSUP, "efg_bfs: parents are not available on a partitioned handle");
+    const int emode = parent ? kModeVisitParent : kModeVisit;  // expand mode
+    const int mode = part ? kLoopPartitioned : emode;            // loop graph
     const bool graph_mode = d.level_loop == 0;
     if (graph_mode) EFG_TRY(build_loop_graph(d, mode));
 
@@ -477,7 +590,8 @@ efg_status device_bfs(efg_graph *g, uint32_t source, int32_t *depth, uint32_t *p
         CUDA_TRY(cudaStreamSynchronize(s));
         levels = d.ctrl_host->nlevels;
         if (d.ctrl_host->fault)
-            return set_error(EFG_ECUDA, "frontier_kernel: grid barrier timed out (grid not co-resident)");
+            return set_error(EFG_ECUDA, "a grid or peer barrier timed out (grid not co-resident, or a rank "
+                                        "missing from the collective); sticky until efg_free");
         const uint32_t ns = std::min(levels, kMaxLevelStats);
         if (ns) {
             CUDA_TRY(cudaMemcpyAsync(d.stats_host, d.stats, ns * sizeof(LevelStat), cudaMemcpyDeviceToHost, s));
@@ -489,15 +603,17 @@ efg_status device_bfs(efg_graph *g, uint32_t source, int32_t *depth, uint32_t *p
             const LevelStat &x = d.stats_host[i];
             lms.push_back(x.t1 > x.t0 ? (float)((double)(x.t1 - x.t0) * 1e-6) : 0.f);
         }
-        launches += 2 * levels + (relabel ? 1 : 0);
+        launches += (part ? 5 : 2) * levels + (relabel ? 1 : 0);
     } else {
-        const int blocks = d.num_sms * expand_occupancy(mode);
+        const int blocks = d.num_sms * expand_occupancy(emode);
         for (;;) {
             CUDA_TRY(cudaMemcpyAsync(d.ctrl_host, d.ctrl, sizeof(LevelCtrl), cudaMemcpyDeviceToHost, s));
             CUDA_TRY(cudaStreamSynchronize(s));
             const LevelCtrl c = *d.ctrl_host;
-            if (c.fault) return set_error(EFG_ECUDA, "frontier_kernel: grid barrier timed out (grid not co-resident)");
-            if (c.nf == 0) break;
+            if (c.fault)
+                return set_error(EFG_ECUDA, "a grid or peer barrier timed out (grid not co-resident, or a rank "
+                                            "missing from the collective); sticky until efg_free");
+            if ((part ? c.nnew : c.nf) == 0) break;  // partitioned: the global new count
             lf.push_back(c.nf);
             le.push_back(c.ne);
             cudaEvent_t a, b;
@@ -509,11 +625,12 @@ efg_status device_bfs(efg_graph *g, uint32_t source, int32_t *depth, uint32_t *p
             CUDA_TRY(cudaEventCreate(&ec));
             lev.push_back(ec);
             CUDA_TRY(cudaEventRecord(a, s));
-            CUDA_TRY(launch_expand(mode, expand_args(d, nullptr), blocks, s));
+            CUDA_TRY(launch_expand(emode, expand_args(d, nullptr), blocks, s));
             CUDA_TRY(cudaEventRecord(b, s));
+            if (part) EFG_TRY(launch_peer_exchange(d, s));
             EFG_TRY(launch_level_end(d, 0, s));
             CUDA_TRY(cudaEventRecord(ec, s));
-            launches += 2;
+            launches += part ? 5 : 2;
             if (d.trace) {  // debug: phase end times of frontier_kernel, max over blocks (us after the first start)
                 const unsigned nb = (unsigned)((d.nwords + d.words_per_block - 1) / d.words_per_block);
                 std::vector<unsigned long long> t(8 * nb);
@@ -722,6 +839,7 @@ efg_status device_step_end(efg_graph *g, efg_stats *st)
 // ---------------------------------------------------------------------------
 void device_peer_close(DeviceGraph &d)
 {
+    device_drop_graphs(d);  // a captured partitioned loop refers to the peer table
     for (int p = 0; p < kPeerMaxWorld; ++p)
         if (d.peer_ipc[p]) {
             cudaIpcCloseMemHandle(d.peer_ipc[p]);
@@ -745,7 +863,7 @@ efg_status device_peer_alloc(efg_graph *g, int world, void **region, uint8_t *ip
         EFG_TRY(dev_alloc(d, &d.peer_region, peer_region_words(d.nwords)));
     }
     CUDA_TRY(cudaMemset(d.peer_region, 0, peer_region_words(d.nwords) * 4));  // flags = epoch 0
-    d.peer_epoch = 0;
+    CUDA_TRY(cudaMemset(&d.ctrl->peer_epoch, 0, sizeof(uint32_t)));           // exchange counter
     d.peer_alloc_world = world;
     if (region) *region = d.peer_region;
     if (ipc_handle) {
@@ -812,24 +930,8 @@ efg_status device_xchg_peer(efg_graph *g)
     DeviceGraph &d = g->dev;
     if (!d.peer_ptrs) return set_error(EFG_ESTATE, "efg_xchg_peer: call efg_peer_open first");
     CUDA_TRY(cudaSetDevice(d.device));
-    cudaStream_t s = stream_of(d);
-    PeerArgs a;
-    a.peers = d.peer_ptrs;
-    a.local = d.peer_region;
-    a.bounds = d.xchg_bounds;
-    a.vis = d.vis;
-    a.prev = d.prev;
-    a.fault = &d.ctrl->fault;
-    a.nwords = d.nwords;
-    a.world = d.peer_world;
-    a.rank = d.peer_rank;
-    a.epoch = d.peer_epoch + 1;
-    for (int op = 0; op < 3; ++op) {
-        a.op = op;
-        CUDA_TRY(launch_peer(a, d.num_sms, s));
-        ++d.step_launches;
-    }
-    d.peer_epoch += 2;
+    EFG_TRY(launch_peer_exchange(d, stream_of(d)));
+    d.step_launches += 3;
     return EFG_OK;
 }
 

@@ -65,13 +65,16 @@ static_assert(sizeof(VRec) == 16, "VRec must be 16 bytes");
 constexpr int kOffBits = 40;                            // data byte offsets < 2^40 (1 TiB)
 constexpr uint64_t kOffMask = (1ull << kOffBits) - 1;
 constexpr int kCcShift = 46;                            // ChunkDesc: chunk index above l
+constexpr int kCcBits = 64 - kCcShift;                  // chunk index field: cc < 2^18
+constexpr uint32_t kMaxDeviceQuantum = 512;             // largest device chunk (its lower fields fit a staging buffer)
 
 // Chunk descriptor (step a1, written by frontier_kernel, read by expand_kernel):
 // one k-aligned piece of a frontier vertex's list.  The expand
 // kernel derives the chunk's bit ranges from it and the forward pointers (a4).
 struct alignas(16) ChunkDesc {
     uint64_t off_l_cc;  // the list's VRec.off_l (offset: 40 bits, l: bits 40-45) | chunk index cc << 46
-                        // (rank of the chunk's first element r0 = cc*k; cc < 2^17 for deg < 2^26)
+                        // (rank of the chunk's first element r0 = cc*k; device_upload picks the
+                        // device quantum k so that ceil(deg/k) < 2^kCcBits for every list)
     uint32_t deg;       // list length
     uint32_t ubytes;    // upper-bits section bytes of the list
 };
@@ -99,6 +102,7 @@ struct LevelCtrl {
                         // slot L & 1 (atomicMin); the expand of level L reads it as its visited prefix
     uint32_t vpre_used; // visited prefix the last BFS expand used (0: none); lower bound for the next level end
     uint32_t fault;     // a frontier_kernel grid barrier timed out (sticky; reported by the host)
+    uint32_t peer_epoch;  // peer exchange counter (efg_xchg_peer / partitioned efg_bfs): +2 per exchange
 };
 
 // A frontier list whose chunk descriptors and tile boundaries are written by
@@ -209,8 +213,9 @@ struct DeviceGraph {
     int level_loop = 0;                // 0 = CUDA graph (device loop), 1 = host loop + events
     int prefix_skip = 1;               // EFG_OPT_PREFIX_SKIP
     int pr_pull = 1;                   // EFG_OPT_PAGERANK_PULL
-    cudaGraph_t loop_graph[2] = {nullptr, nullptr};      // per mode (visit, visit+parent)
-    cudaGraphExec_t loop_exec[2] = {nullptr, nullptr};
+    static constexpr int kLoopGraphs = 3;                 // visit, visit+parent, partitioned visit
+    cudaGraph_t loop_graph[kLoopGraphs] = {};
+    cudaGraphExec_t loop_exec[kLoopGraphs] = {};
     uint64_t own_lo_w = 0, own_hi_w = 0;   // bitmap words of the owned rows (frontier filter)
     uint64_t *xchg_bounds = nullptr;       // device copy of the partition bounds
     uint64_t xchg_bounds_cap = 0;
@@ -220,7 +225,6 @@ struct DeviceGraph {
     void *peer_ipc[64] = {};               // IPC-opened peer bases (closed on free)
     int peer_world = 0, peer_rank = -1;
     int peer_alloc_world = 0;
-    uint32_t peer_epoch = 0;               // last barrier epoch used
     // stepwise (partitioned) traversal state
     uint32_t step_levels = 0;
     uint32_t step_launches = 0;            // kernels this stepwise BFS launched (efg_stats.kernel_launches)

@@ -276,9 +276,15 @@ __global__ void peer_kernel(PeerArgs a)
     const uint64_t t0 = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
     if (a.op == 0) {
         for (uint64_t w = t0; w < a.nwords; w += stride) a.local[pub + w] = a.vis[w] & ~a.prev[w];
+        // barrier epochs of this exchange: E - 1 (op 1) and E (op 2), E = the
+        // counter after this increment (a device counter, so a captured level
+        // loop advances it every iteration; every rank runs the same number of
+        // exchanges, so the counters agree)
+        if (blockIdx.x == 0 && threadIdx.x == 0) *a.epoch += 2;
         return;
     }
-    if (!peer_barrier(a, a.op == 1 ? a.epoch : a.epoch + 1)) return;
+    const uint32_t E = *a.epoch;
+    if (!peer_barrier(a, a.op == 1 ? E - 1 : E)) return;
     if (a.op == 1) {
         const uint64_t w0 = a.bounds[a.rank] / 32, w1 = (a.bounds[a.rank + 1] + 31) / 32;
         for (uint64_t w = w0 + t0; w < w1; w += stride) {
@@ -563,7 +569,14 @@ __global__ void __launch_bounds__(kFrontierThreads, 1024 / kFrontierThreads) fro
                 a.stats[level].t1 = 0;
             }
         }
-        if (a.cond) cudaGraphSetConditional(a.cond, nf ? 1u : 0u);
+        if (a.cond) {
+            // loop while the next frontier is non-empty: this rank's owned part
+            // (whole graph), or the global new set (partitioned: identical on
+            // every rank after the exchange, so all ranks stop together); a
+            // timed-out grid or peer barrier ends the loop (sticky fault)
+            const uint64_t more = a.cond_global ? __ldcg(&ctrl->nnew) : nf;
+            cudaGraphSetConditional(a.cond, (more && !__ldcg(&ctrl->fault)) ? 1u : 0u);
+        }
     }
     FTRACE(2);
     uint64_t run = s_pre[1];
@@ -1058,8 +1071,9 @@ __global__ void __launch_bounds__(kExpandThreads, 1) expand_kernel(ExpandArgs a)
         B.buf = buf;
         nbuf ^= 1;
         uint32_t tot_e, tot_w;
-        if (kpow2 && a.k <= 1024) {
-            // one scan for both: a batch holds < 2^15 elements and < 2^16 words
+        if (kpow2 && a.k <= 1024 && __all_sync(FULL, !fits || nwd < 2048)) {
+            // one scan for both: a batch holds < 2^15 elements (32 chunks of <= 512)
+            // and, with every chunk under 2048 words, < 2^16 words
             uint32_t t;
             const uint32_t ex = warp_excl_u32(fits ? (nel | nwd << 16) : 0u, t);
             B.eb = ex & 0xffffu;

@@ -75,7 +75,8 @@ struct PeerArgs {
     const uint32_t *prev;
     uint32_t *fault;               // LevelCtrl.fault: a barrier wait timed out
     uint64_t nwords;
-    uint32_t epoch;                // barrier epoch of ops 1 and 2
+    uint32_t *epoch;               // device exchange counter (LevelCtrl.peer_epoch): op 0 adds 2,
+                                   // ops 1 and 2 wait on barrier epochs counter-1 and counter
     int world, rank;
     int op;                        // 0 publish, 1 owner OR + broadcast, 2 unpack
 };
@@ -104,6 +105,8 @@ struct FrontierArgs {           // level end (a7) + next level plan (a1-a4), one
     uint32_t k;
     int32_t kshift;
     cudaGraphConditionalHandle cond;  // graph-mode loop condition, 0 = host loop
+    int cond_global;                  // 1: loop while the global new count (ctrl->nnew) is non-zero
+                                      // (partitioned traversal), 0: while this rank's frontier is
     uint64_t nwords, words_per_block;
     uint64_t own_lo_w, own_hi_w;  // owned bitmap words: only these enter the frontier
 };

@@ -24,3 +24,44 @@ def test_reference_arm_json_line():
     assert d["config"]["workload"] == "rmat16_ef16"
     assert d["cpu_baseline"]["kind"] == "oracle" and d["cpu_baseline"]["cores"] == 1
     assert d["e2e"]["h2d_bytes_per_step"] == 0 and d["e2e"]["value"] == d["value"]
+
+
+def test_cpu_baseline_child_pinned_and_checked():
+    """bench.py's cpu_baseline leg: a spawned process builds the oracle CSR of
+    the same seeded graph, times one FIFO BFS pinned to one core, and the
+    parent compares that depth with the traversal it is handed (here a stub
+    returning the oracle's own answer, and one returning a wrong answer)."""
+    import numpy as np
+    import bench
+    import oracle
+    import synth
+
+    class Args:
+        config, scale = 1, None
+
+    n, src, dst = synth.config_edges(1)
+    ov, oe = oracle.csr_build(n, src, dst)
+
+    class Stub:
+        def __init__(self, wrong):
+            self.wrong = wrong
+
+        def bfs(self, s):
+            d = oracle.bfs(ov, oe, s)
+            if self.wrong:
+                d[np.flatnonzero(d > 0)[0]] += 1
+            return d
+
+    before = os.sched_getaffinity(0)
+    try:
+        for wrong in (False, True):
+            job = bench.start_cpu_baseline(Args, 4, 1)
+            cpu = bench.finish_cpu_baseline(*job, Stub(wrong), n)
+            os.sched_setaffinity(0, before)
+            assert cpu["kind"] == "oracle" and cpu["cores"] == 1 and cpu["value"] > 0
+            assert cpu["parity_bit_exact"] is (not wrong)
+            srcs = synth.sources(n, 4, seed=1001, nonisolated_mask=np.diff(ov) > 0)
+            assert cpu["parity_source"] == int(srcs[1])
+            assert "taskset -c" in cpu["sample"] and cpu["cpu_model"]
+    finally:
+        os.sched_setaffinity(0, before)

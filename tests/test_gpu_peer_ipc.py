@@ -47,11 +47,24 @@ def _worker(rank: int, port: int, q):
         ov, oe = oracle.csr_build(n, src, dst)
         bad = []
         for s in SOURCES:
+            ref = oracle.bfs(ov, oe, s)
             depth = torch.empty(n, dtype=torch.int32, device="cuda")
-            partitioned_bfs_peer(g, s, depth)
+            partitioned_bfs_peer(g, s, depth)  # stepwise calls
             torch.cuda.synchronize()
-            if not np.array_equal(depth.cpu().numpy(), oracle.bfs(ov, oe, s)):
-                bad.append(s)
+            if not np.array_equal(depth.cpu().numpy(), ref):
+                bad.append(("stepwise", s))
+            # collective efg_bfs: enqueue-only (device depth) and synchronous (host depth),
+            # graph loop and host loop
+            for host_loop in (False, True):
+                g.set_level_loop(host_loop)
+                depth.fill_(-7)
+                g.bfs(s, depth=depth)
+                torch.cuda.synchronize()
+                if not np.array_equal(depth.cpu().numpy(), ref):
+                    bad.append(("collective-device", host_loop, s))
+                if not np.array_equal(g.bfs(s), ref):
+                    bad.append(("collective-host", host_loop, s))
+            g.set_level_loop(False)
         dist.barrier()
         g.free()
         dist.destroy_process_group()

@@ -147,3 +147,40 @@ def test_bfs_rmat_invariants():
     vlist, elist = oracle.csr_build(n, src, dst)
     for s in (0, 1, 100):
         graph500_validate(vlist, elist, s, oracle.bfs(vlist, elist, s))
+
+
+def test_bfs_bounded_sample():
+    """or_bfs_bounded (bench.py reference-arm sample): every depth it assigns is
+    the Floyd-Warshall hop distance, it scans at least the budget (or finishes
+    the BFS), the scanned count is the degree sum of the dequeued vertices, and
+    an unlimited budget is the full BFS."""
+    rng = np.random.default_rng(12)
+    for t in range(40):
+        n = int(rng.integers(2, 65))
+        m = int(rng.integers(0, 4 * n))
+        src = rng.integers(0, n, m).astype(np.uint32)
+        dst = rng.integers(0, n, m).astype(np.uint32)
+        vlist, elist = oracle.csr_build(n, src, dst)
+        deg = np.diff(vlist)
+        d = _fw_dist(n, list(zip(src.tolist(), dst.tolist())))
+        for s in rng.integers(0, n, 3):
+            s = int(s)
+            full = d[s]
+            for budget in (0, 1, 5, int(rng.integers(0, 2 * m + 2)), 2**63):
+                got, nv, scanned = oracle.bfs_bounded(vlist, elist, s, budget)
+                assigned = got >= 0
+                assert np.array_equal(got[assigned], full[assigned])
+                assert got[s] == 0
+                # the dequeued vertices are the nv closest (FIFO order: by depth)
+                reached = int((full >= 0).sum())
+                assert nv <= reached
+                assert scanned >= min(budget, int(deg[full >= 0].sum())) or nv == reached
+                if budget == 2**63:
+                    assert np.array_equal(got, full) and nv == reached
+                    assert scanned == int(deg[full >= 0].sum())
+                # every vertex at depth < the last dequeued depth was dequeued, hence
+                # all of its neighbours have depths assigned
+                if nv:
+                    dq_depths = np.sort(full[full >= 0])[:nv]
+                    for u in np.flatnonzero((full >= 0) & (full < dq_depths[-1])):
+                        assert np.all(got[elist[vlist[u]:vlist[u + 1]]] >= 0)
