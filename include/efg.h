@@ -247,6 +247,13 @@ efg_status efg_pagerank(efg_graph *g, double damping, uint32_t iters, double *ra
                                  * directed or row-range handle): push along every edge with
                                  * fp64 atomicAdd.  Same sums, other order (C21). */
 
+#define EFG_OPT_EXPAND_VARIANT 4 /* tuning / A-B switch of the expand kernel, bit mask (default 3):
+                                  * bit 0: batches of balanced chunks are decoded lane-per-chunk
+                                  * (each lane walks its own chunk) instead of by word records
+                                  * split evenly over the lanes; bit 1: a batch of adjacent chunks
+                                  * is staged by one bulk copy of its byte span.  Results are
+                                  * identical for every value. */
+
 /* Set a per-handle option.  Errors: EFG_EINVAL (unknown option / value),
  * EFG_ESTATE (host-only handle). */
 efg_status efg_set_option(efg_graph *g, int option, int64_t value);

@@ -95,6 +95,10 @@ class Graph:
         """EFG_OPT_PAGERANK_PULL: True (default) = gather on symmetric graphs, False = push."""
         check(lib.efg_set_option(self._h, _abi.EFG_OPT_PAGERANK_PULL, 1 if on else 0), "efg_set_option")
 
+    def set_expand_variant(self, mask: int) -> None:
+        """EFG_OPT_EXPAND_VARIANT (A/B switch): bit 0 lane-per-chunk decode, bit 1 span staging."""
+        check(lib.efg_set_option(self._h, _abi.EFG_OPT_EXPAND_VARIANT, int(mask)), "efg_set_option")
+
     def free(self) -> None:
         if self._h:
             lib.efg_free(self._h)

@@ -22,6 +22,7 @@ EFG_REORDER_DEGREE = 0x8
 EFG_OPT_LEVEL_LOOP = 1
 EFG_OPT_PREFIX_SKIP = 2
 EFG_OPT_PAGERANK_PULL = 3
+EFG_OPT_EXPAND_VARIANT = 4
 
 
 class BuildOpts(C.Structure):

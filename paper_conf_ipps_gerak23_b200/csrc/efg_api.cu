@@ -184,6 +184,13 @@ extern "C" efg_status efg_set_option(efg_graph *g, int option, int64_t value)
             efg::device_drop_graphs(g->dev);  // the captured level loops carry the old value
         }
         return EFG_OK;
+    case EFG_OPT_EXPAND_VARIANT:
+        if (value < 0 || value > 3) return set_error(EFG_EINVAL, "EFG_OPT_EXPAND_VARIANT: 0..3");
+        if (g->dev.expand_variant != (int)value) {
+            g->dev.expand_variant = (int)value;
+            efg::device_drop_graphs(g->dev);
+        }
+        return EFG_OK;
     default:
         return set_error(EFG_EINVAL, "efg_set_option: unknown option");
     }

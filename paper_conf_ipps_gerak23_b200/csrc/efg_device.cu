@@ -151,6 +151,7 @@ ExpandArgs expand_args(DeviceGraph &d, uint32_t *out)
     a.hot_words = (uint32_t)std::min<uint64_t>(kHotWords, d.nwords) & ~3u;
     a.k = d.k;
     a.pskip = d.prefix_skip ? 1u : 0u;
+    a.variant = (uint32_t)d.expand_variant;
     return a;
 }
 

@@ -928,6 +928,8 @@ __device__ __forceinline__ void fence_proxy_async()
 struct Batch {
     uint32_t cnt, ne, nw, buf;   // chunks, elements, upper words, staging buffer
     uint32_t lsmb, lflags, HB, eb, wb, nwd, v, cc;
+    uint32_t nel;                // elements of this lane's chunk
+    bool lpc;                    // warp-uniform: decode lane-per-chunk (see expand_kernel)
     uint64_t usrc;
 };
 
@@ -944,6 +946,14 @@ constexpr int kU = EFG_KU;  // elements per lane whose probes are in flight toge
 #define EFG_CHUNK_SKIP 1
 #endif
 constexpr bool kChunkSkip = EFG_CHUNK_SKIP;  // BFS: k-chunks wholly below the visited prefix are not staged
+#ifndef EFG_LPC
+#define EFG_LPC 1
+#endif
+constexpr bool kLpc = EFG_LPC;  // lane-per-chunk decode of balanced batches (no word records)
+#ifndef EFG_SPAN_STAGE
+#define EFG_SPAN_STAGE 1
+#endif
+constexpr bool kSpanStage = EFG_SPAN_STAGE;  // one bulk copy per batch when the chunks' bytes are adjacent
 
 template <int MODE>
 __global__ void __launch_bounds__(kExpandThreads, 1) expand_kernel(ExpandArgs a)
@@ -1063,10 +1073,34 @@ __global__ void __launch_bounds__(kExpandThreads, 1) expand_kernel(ExpandArgs a)
             lsz = (uint32_t)(lg1 - lg0);
             bytes = merged ? (uint32_t)(max(lg1, ug1) - lg0) : lsz + (ustage ? (uint32_t)(ug1 - ug0) : 0u);
         }
+        // Two staging layouts; the one that fits more chunks wins:
+        //   sum:  each chunk's ranges packed one after the other (one or two
+        //         bulk copies per chunk; a lane issues its own);
+        //   span: ONE bulk copy of [S, E), the byte span of consecutive chunks
+        //         whose staged bytes are single ranges — frontier lists in id
+        //         order are laid out in increasing offset order, so on
+        //         dense levels the span is the chunks' bytes plus small gaps,
+        //         without per-chunk 16-byte rounding
         uint32_t tb;
         const uint32_t sb = warp_excl_u32(bytes, tb);
-        const bool fits = valid && sb + bytes <= kStageBytes;
-        B.cnt = __popc(__ballot_sync(FULL, fits));  // a prefix of the lanes; >= 1 (one chunk always fits)
+        const bool fits_sum = valid && sb + bytes <= kStageBytes;
+        const uint64_t rs = l ? lg0 : ug0;  // this lane's single range [rs, rs + bytes)
+        const uint32_t hm = __ballot_sync(FULL, valid && bytes);
+        const uint64_t S = hm ? __shfl_sync(FULL, rs, __ffs(hm) - 1) : 0ull;
+        uint32_t E = 0;  // span end relative to S, inclusive max over lanes <= this one
+        if (valid && bytes) E = (rs >= S && rs + bytes - S < (1ull << 30)) ? (uint32_t)(rs + bytes - S) : (1u << 30);
+#pragma unroll
+        for (int d = 1; d < 32; d <<= 1) {
+            const uint32_t t = __shfl_up_sync(FULL, E, d);
+            if ((int)lane >= d) E = max(E, t);
+        }
+        const bool fits_span = valid && E <= kStageBytes;
+        const bool one = __all_sync(FULL, !(valid && l && ustage && !merged));
+        const uint32_t cnt_sum = __popc(__ballot_sync(FULL, fits_sum));
+        const uint32_t cnt_span = __popc(__ballot_sync(FULL, fits_span));
+        const bool span = kSpanStage && (a.variant & 2) && one && cnt_span >= cnt_sum;  // warp-uniform
+        const bool fits = span ? fits_span : fits_sum;
+        B.cnt = span ? cnt_span : cnt_sum;  // a prefix of the lanes; >= 1 (one chunk always fits)
         const uint32_t buf = nbuf;
         B.buf = buf;
         nbuf ^= 1;
@@ -1084,13 +1118,19 @@ __global__ void __launch_bounds__(kExpandThreads, 1) expand_kernel(ExpandArgs a)
             B.eb = warp_excl_u32(fits ? nel : 0u, tot_e);
             B.wb = warp_excl_u32(fits ? nwd : 0u, tot_w);
         }
-        const uint32_t tot_b = __shfl_sync(FULL, sb + bytes, B.cnt - 1);  // bytes of the fitting prefix
+        const uint32_t tot_b = __shfl_sync(FULL, span ? E : sb + bytes, B.cnt - 1);  // bytes of the fitting prefix
         B.ne = tot_e;
         B.nw = tot_w;
         B.nwd = nwd;
         B.v = v;
         B.cc = cc;
-        const uint32_t base = buf * kStageBytes + sb;  // stage-area byte offset of this chunk
+        B.nel = fits ? nel : 0u;
+        // lane-per-chunk decode when the lanes' chunks are balanced enough:
+        // >= 50 % of the warp's element slots busy (the degree relabelling puts
+        // lists of similar length next to each other in the frontier)
+        B.lpc = kLpc && (a.variant & 1) && 2 * tot_e >= 32 * __reduce_max_sync(FULL, B.nel);
+        // stage-area byte offset of this chunk's first staged byte
+        const uint32_t base = buf * kStageBytes + (span ? (bytes ? (uint32_t)(rs - S) : 0u) : sb);
         const uint32_t lsm = sbits + (l ? base * 8 + (uint32_t)(lb - lg0 * 8) : buf * kStageBytes * 8);
         B.lsmb = lsm - B.eb * l;
         B.lflags = l | ((uint32_t)(A0 & 31) << 8) | ((uint32_t)((A1 - 1) & 31) << 16) | (ustage ? 1u << 24 : 0u);
@@ -1106,7 +1146,13 @@ __global__ void __launch_bounds__(kExpandThreads, 1) expand_kernel(ExpandArgs a)
         __syncwarp();
         if (lane == 0) mbar_arrive_expect_tx(&ws.mbar[buf], tot_b);
         __syncwarp();
-        if (fits) {
+        if (span) {
+            if (lane == 0 && tot_b) {
+                fence_proxy_async();
+                bulk_g2s(reinterpret_cast<uint8_t *>(&ws.stage[0][0]) + buf * kStageBytes, data + S, tot_b,
+                         &ws.mbar[buf]);
+            }
+        } else if (fits) {
             fence_proxy_async();
             uint8_t *dst = reinterpret_cast<uint8_t *>(&ws.stage[0][0]) + base;
             if (merged) {
@@ -1118,6 +1164,91 @@ __global__ void __launch_bounds__(kExpandThreads, 1) expand_kernel(ExpandArgs a)
         }
         return true;
     };
+
+    // ---- a6 (and the other modes' visit functors) for kU decoded elements ----
+        auto visit = [&](const uint32_t (&xv)[kU], const uint32_t (&sv)[kU], const uint32_t (&ev)[kU],
+                         int cntu, uint32_t &pr_slot, double &pr_acc) {
+            if (MODE == kModeDecode) {
+#pragma unroll
+                for (int u = 0; u < kU; ++u)
+                    if (u < cntu) a.out[ws.slot[sv[u]].aux + (ev[u] - ws.slot[sv[u]].eb)] = xv[u];
+            } else if (MODE == kModeSssp) {
+                // relax: d' = fl32(dist(u) + w), single rounding (reading C20)
+                float nd[kU], cd[kU];
+#pragma unroll
+                for (int u = 0; u < kU; ++u) {
+                    nd[u] = INFINITY;
+                    cd[u] = 0.f;
+                    if (u < cntu) {
+                        const SlotP &sp = ws.slot[sv[u]];
+                        nd[u] = __fadd_rn(sp.aux2, __ldg(a.weights + sp.aux + (ev[u] - sp.eb)));
+                        cd[u] = a.dist[xv[u]];
+                    }
+                }
+#pragma unroll
+                for (int u = 0; u < kU; ++u) {
+                    if (u < cntu && nd[u] < cd[u]) {  // non-negative floats order like their bits
+                        const int old = atomicMin(reinterpret_cast<int *>(a.dist) + xv[u], __float_as_int(nd[u]));
+                        if (__float_as_int(nd[u]) < old) atomicOr(a.vis + (xv[u] >> 5), 1u << (xv[u] & 31));
+                    }
+                }
+            } else if (MODE == kModePrPull) {
+                // pull (symmetric graphs): the lane sums contrib[u] = r(u)/deg(u) of its
+                // run's neighbours and adds the sum once per list it leaves
+                double cv[kU];
+#pragma unroll
+                for (int u = 0; u < kU; ++u) cv[u] = u < cntu ? __ldg(a.contrib + xv[u]) : 0.0;
+#pragma unroll
+                for (int u = 0; u < kU; ++u) {
+                    if (u < cntu) {
+                        if (sv[u] != pr_slot) {
+                            if (pr_slot != FULL) atomicAdd(a.next + ws.slot[pr_slot].aux, pr_acc);
+                            pr_slot = sv[u];
+                            pr_acc = 0.0;
+                        }
+                        pr_acc += cv[u];
+                    }
+                }
+            } else if (MODE == kModePagerank) {
+#pragma unroll
+                for (int u = 0; u < kU; ++u)
+                    if (u < cntu)
+                        atomicAdd(a.next + xv[u], __longlong_as_double((long long)ws.slot[sv[u]].aux));
+            } else {
+                // Alg. 1 line 3: hot ids answer from shared memory
+                // ids below vpre are known visited without a memory access
+                bool need[kU];
+#pragma unroll
+                for (int u = 0; u < kU; ++u) {
+                    need[u] = u < cntu && xv[u] >= vpre;
+                    if (kUseHot) {
+                        const uint32_t hw = (need[u] && xv[u] < hot_limit) ? s_hot[xv[u] >> 5] : 0u;
+                        need[u] = need[u] && !((hw >> (xv[u] & 31)) & 1);
+                    }
+                }
+                uint32_t gv[kU];
+#pragma unroll
+                for (int u = 0; u < kU; ++u) gv[u] = need[u] ? a.vis[xv[u] >> 5] : FULL;
+                uint32_t hit = 1;
+#pragma unroll
+                for (int u = 0; u < kU; ++u) hit &= shf_r_wrap(gv[u], gv[u], xv[u]);
+                const bool miss = !(hit & 1);
+                if (!__any_sync(__activemask(), miss)) return;  // most probes of a heavy level end here
+#pragma unroll
+                for (int u = 0; u < kU; ++u) {
+                    const uint32_t bit = 1u << (xv[u] & 31);
+                    if (!(gv[u] & bit)) {  // line 4 (the atomic decides)
+                        if (MODE == kModeVisit) {
+                            atomicOr(a.vis + (xv[u] >> 5), bit);
+                        } else {
+                            const uint32_t old = atomicOr(a.vis + (xv[u] >> 5), bit);
+                            if (!(old & bit)) parent[xv[u]] = (uint32_t)ws.slot[sv[u]].aux;
+                        }
+                        if (kUseHot && xv[u] < hot_limit) atomicOr(s_hot + (xv[u] >> 5), bit);
+                    }
+                }
+            }
+        };
 
     Batch cur, nxt;
     bool have = produce(cur);
@@ -1156,6 +1287,92 @@ __global__ void __launch_bounds__(kExpandThreads, 1) expand_kernel(ExpandArgs a)
         __syncwarp();
         mbar_wait(&ws.mbar[buf], (phase >> buf) & 1);
         phase ^= 1u << buf;
+
+        if (cur.lpc) {
+            // ---- lane-per-chunk: lane i walks chunk i of the batch serially
+            // from the staged bytes (a5): the next stop bit of its upper words
+            // gives select1(j) - j, its lower field the low bits; no word
+            // records, no lane-start search.  With the prefix skip the lane
+            // first steps over whole words whose last stop bit is below
+            // vpre >> l (their elements are visited; P:157's pointers already
+            // dropped whole chunks) ----
+            if (lane < cnt && cur.nel) {
+                const uint32_t nel = cur.nel, l = cur.lflags & 63, lmask = (1u << l) - 1;
+                const uint32_t a0s = (cur.lflags >> 8) & 31, a1s = (cur.lflags >> 16) & 31;
+                const bool staged = (cur.lflags >> 24) & 1;
+                const uint32_t nwd = cur.nwd, ebase = cur.eb;
+                const uint64_t usrc = cur.usrc;
+                uint32_t la = cur.lsmb + ebase * l;          // lower field of element j
+                uint32_t hcur = cur.HB + 32u * cur.wb - ebase;  // hi = hcur + p - j for a stop bit at p of word gl
+                uint32_t gl = 0, j = 0;
+                auto word = [&](uint32_t g) -> uint32_t {
+                    uint32_t w = staged ? st32[usrc + g] : ldg_u32(data32 + usrc + g);
+                    if (g == 0) w &= FULL << a0s;
+                    if (g == nwd - 1) w &= FULL >> (31 - a1s);
+                    return w;
+                };
+                uint32_t w = word(0);
+                if (pskip) {
+                    const uint32_t h0 = vpre >> l;
+                    // whole words whose last stop bit has a high part below h0
+                    while (gl + 1 < nwd) {
+                        const uint32_t pc = __popc(w);
+                        if (pc && hcur + (31 - __clz(w)) - (j + pc - 1) >= h0) break;
+                        j += pc;
+                        la += pc * l;
+                        ++gl;
+                        hcur += 32;
+                        w = word(gl);
+                    }
+                }
+                uint32_t uw = __brev(w);  // reversed: the next stop bit is the leading one
+                uint32_t e = ebase + j;
+                auto decode1 = [&](uint32_t &x) {
+                    while (uw == 0) {
+                        ++gl;
+                        hcur += 32;
+                        uw = __brev(word(gl));
+                    }
+                    const uint32_t p = clz_nz(uw);
+                    uw ^= 0x80000000u >> p;
+                    const uint32_t hi = hcur + p - j;  // select1(j) - j
+                    const uint32_t ad = (la >> 3) & ~3u;
+                    const uint32_t lo = shf_r_wrap(lds_u32(ad), lds_u32(ad + 4), la) & lmask;
+                    x = (hi << l) | lo;
+                    la += l;
+                    ++j;
+                    ++e;
+                };
+                uint32_t pr_slot = FULL;  // PageRank pull partial sum (one list per lane)
+                double pr_acc = 0.0;
+                for (; j + kU <= nel;) {
+                    uint32_t xv[kU], sv[kU], ev[kU];
+#pragma unroll
+                    for (int u = 0; u < kU; ++u) {
+                        ev[u] = e;
+                        sv[u] = lane;
+                        decode1(xv[u]);
+                    }
+                    visit(xv, sv, ev, kU, pr_slot, pr_acc);
+                }
+                if (j < nel) {
+                    uint32_t xv[kU], sv[kU], ev[kU];
+                    const int cntu = (int)(nel - j);
+#pragma unroll
+                    for (int u = 0; u < kU; ++u) {
+                        xv[u] = 0;
+                        sv[u] = lane;
+                        ev[u] = e;
+                        if (u < cntu) decode1(xv[u]);
+                    }
+                    visit(xv, sv, ev, cntu, pr_slot, pr_acc);
+                }
+                if (MODE == kModePrPull && pr_slot != FULL) atomicAdd(a.next + ws.slot[pr_slot].aux, pr_acc);
+            }
+            __syncwarp();
+            cur = nxt;
+            continue;
+        }
 
         uint32_t Er0 = 0;  // batch element index at the round start
         for (uint32_t ga = 0; ga < NW; ga += kRoundWords) {
@@ -1251,90 +1468,6 @@ __global__ void __launch_bounds__(kExpandThreads, 1) expand_kernel(ExpandArgs a)
                     ++e;
                 };
 
-                auto visit = [&](const uint32_t (&xv)[kU], const uint32_t (&sv)[kU], const uint32_t (&ev)[kU],
-                                 int cntu) {
-                    if (MODE == kModeDecode) {
-#pragma unroll
-                        for (int u = 0; u < kU; ++u)
-                            if (u < cntu) a.out[ws.slot[sv[u]].aux + (ev[u] - ws.slot[sv[u]].eb)] = xv[u];
-                    } else if (MODE == kModeSssp) {
-                        // relax: d' = fl32(dist(u) + w), single rounding (reading C20)
-                        float nd[kU], cd[kU];
-#pragma unroll
-                        for (int u = 0; u < kU; ++u) {
-                            nd[u] = INFINITY;
-                            cd[u] = 0.f;
-                            if (u < cntu) {
-                                const SlotP &sp = ws.slot[sv[u]];
-                                nd[u] = __fadd_rn(sp.aux2, __ldg(a.weights + sp.aux + (ev[u] - sp.eb)));
-                                cd[u] = a.dist[xv[u]];
-                            }
-                        }
-#pragma unroll
-                        for (int u = 0; u < kU; ++u) {
-                            if (u < cntu && nd[u] < cd[u]) {  // non-negative floats order like their bits
-                                const int old = atomicMin(reinterpret_cast<int *>(a.dist) + xv[u], __float_as_int(nd[u]));
-                                if (__float_as_int(nd[u]) < old) atomicOr(a.vis + (xv[u] >> 5), 1u << (xv[u] & 31));
-                            }
-                        }
-                    } else if (MODE == kModePrPull) {
-                        // pull (symmetric graphs): the lane sums contrib[u] = r(u)/deg(u) of its
-                        // run's neighbours and adds the sum once per list it leaves
-                        double cv[kU];
-#pragma unroll
-                        for (int u = 0; u < kU; ++u) cv[u] = u < cntu ? __ldg(a.contrib + xv[u]) : 0.0;
-#pragma unroll
-                        for (int u = 0; u < kU; ++u) {
-                            if (u < cntu) {
-                                if (sv[u] != pr_slot) {
-                                    if (pr_slot != FULL) atomicAdd(a.next + ws.slot[pr_slot].aux, pr_acc);
-                                    pr_slot = sv[u];
-                                    pr_acc = 0.0;
-                                }
-                                pr_acc += cv[u];
-                            }
-                        }
-                    } else if (MODE == kModePagerank) {
-#pragma unroll
-                        for (int u = 0; u < kU; ++u)
-                            if (u < cntu)
-                                atomicAdd(a.next + xv[u], __longlong_as_double((long long)ws.slot[sv[u]].aux));
-                    } else {
-                        // Alg. 1 line 3: hot ids answer from shared memory
-                        // ids below vpre are known visited without a memory access
-                        bool need[kU];
-#pragma unroll
-                        for (int u = 0; u < kU; ++u) {
-                            need[u] = u < cntu && xv[u] >= vpre;
-                            if (kUseHot) {
-                                const uint32_t hw = (need[u] && xv[u] < hot_limit) ? s_hot[xv[u] >> 5] : 0u;
-                                need[u] = need[u] && !((hw >> (xv[u] & 31)) & 1);
-                            }
-                        }
-                        uint32_t gv[kU];
-#pragma unroll
-                        for (int u = 0; u < kU; ++u) gv[u] = need[u] ? a.vis[xv[u] >> 5] : FULL;
-                        uint32_t hit = 1;
-#pragma unroll
-                        for (int u = 0; u < kU; ++u) hit &= shf_r_wrap(gv[u], gv[u], xv[u]);
-                        const bool miss = !(hit & 1);
-                        if (!__any_sync(__activemask(), miss)) return;  // most probes of a heavy level end here
-#pragma unroll
-                        for (int u = 0; u < kU; ++u) {
-                            const uint32_t bit = 1u << (xv[u] & 31);
-                            if (!(gv[u] & bit)) {  // line 4 (the atomic decides)
-                                if (MODE == kModeVisit) {
-                                    atomicOr(a.vis + (xv[u] >> 5), bit);
-                                } else {
-                                    const uint32_t old = atomicOr(a.vis + (xv[u] >> 5), bit);
-                                    if (!(old & bit)) parent[xv[u]] = (uint32_t)ws.slot[sv[u]].aux;
-                                }
-                                if (kUseHot && xv[u] < hot_limit) atomicOr(s_hot + (xv[u] >> 5), bit);
-                            }
-                        }
-                    }
-                };
-
                 // main loop: kU elements per step, no per-element guards
                 for (; c + kU <= c1; c += kU) {
                     uint32_t xv[kU], sv[kU], ev[kU];
@@ -1343,7 +1476,7 @@ __global__ void __launch_bounds__(kExpandThreads, 1) expand_kernel(ExpandArgs a)
                         ev[u] = e;
                         decode(xv[u], sv[u]);
                     }
-                    visit(xv, sv, ev, kU);
+                    visit(xv, sv, ev, kU, pr_slot, pr_acc);
                 }
                 // tail: < kU elements
                 if (c < c1) {
@@ -1356,7 +1489,7 @@ __global__ void __launch_bounds__(kExpandThreads, 1) expand_kernel(ExpandArgs a)
                         ev[u] = e;
                         if (u < cntu) decode(xv[u], sv[u]);
                     }
-                    visit(xv, sv, ev, cntu);
+                    visit(xv, sv, ev, cntu, pr_slot, pr_acc);
                 }
                 if (MODE == kModePrPull && pr_slot != FULL) atomicAdd(a.next + ws.slot[pr_slot].aux, pr_acc);
             }
