@@ -160,6 +160,10 @@ constexpr int kBitmapAlign = 1024;           // bitmap words are padded to a mul
 #endif
 constexpr uint32_t kTileWork = EFG_TILE_WORK;         // work units per tile (a3)
 constexpr uint32_t kChunkWork = 32;          // per-chunk overhead in work units
+#ifndef EFG_TILE_BIG_MIN_WORK
+#define EFG_TILE_BIG_MIN_WORK (1ull << 27)
+#endif
+constexpr uint64_t kTileBigMinWork = EFG_TILE_BIG_MIN_WORK;  // levels with this much work use 2 x kTileWork tiles
 
 constexpr unsigned kMaxGrid = 4096;
 constexpr int kD2HChunks = 8;               // host depth transfer pipeline depth

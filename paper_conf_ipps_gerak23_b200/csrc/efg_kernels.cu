@@ -547,10 +547,15 @@ __global__ void __launch_bounds__(kFrontierThreads, 1024 / kFrontierThreads) fro
     }
     __syncthreads();
     const uint64_t nf = s_tot[0];
+    // tile size of this level (a3): 2 x kTileWork on levels with plenty of work
+    // (longer batches of short lists per warp), kTileWork otherwise (enough
+    // tiles for every expand warp on small levels).  Lists of <= kTileWork
+    // units cross at most one tile boundary either way (phase 2).
+    const uint64_t TW = s_tot[1] >= kTileBigMinWork ? 2ull * kTileWork : (uint64_t)kTileWork;
     if (b == gridDim.x - 1 && tid == 0) {  // level totals
         const uint64_t nwork = s_tot[1], nchunks = s_tot[2];
         const uint64_t ne = nwork - CW * nchunks + s_tot[3];  // every frontier list's edges
-        const uint64_t ntiles = (nwork + kTileWork - 1) / kTileWork;
+        const uint64_t ntiles = (nwork + TW - 1) / TW;
         ctrl->nf = nf;
         ctrl->nwork = nwork;
         ctrl->nchunks = nchunks;
@@ -687,8 +692,8 @@ __global__ void __launch_bounds__(kFrontierThreads, 1024 / kFrontierThreads) fro
                         a.cvtx[C] = (uint32_t)((w0 + jw[u]) * 32 + lane);
                     }
                     // a3: a tile boundary t*T inside [W, W + wlen) starts at this chunk or the next
-                    const uint64_t t = (W + kTileWork - 1) / kTileWork;
-                    if (t * kTileWork < W + wlen) a.tiles[t] = C + (t * kTileWork > W ? 1u : 0u);
+                    const uint64_t t = (W + TW - 1) / TW;
+                    if (t * TW < W + wlen) a.tiles[t] = C + (t * TW > W ? 1u : 0u);
                 }
                 const uint32_t bm = __ballot_sync(FULL, big);
                 if (bm) {
@@ -745,7 +750,7 @@ __global__ void __launch_bounds__(kFrontierThreads, 1024 / kFrontierThreads) fro
             nch = __ldcg(&bp->nch);
         }
         const uint64_t wl = (uint64_t)nch * CW + d;
-        const uint64_t t_lo = (W + kTileWork - 1) / kTileWork, t_hi = (W + wl + kTileWork - 1) / kTileWork;
+        const uint64_t t_lo = (W + TW - 1) / TW, t_hi = (W + wl + TW - 1) / TW;
         const bool huge = nch > 8 || t_hi - t_lo > 8;
         if (!huge) {
             for (uint32_t j = 0; j < nch; ++j) {
@@ -754,7 +759,7 @@ __global__ void __launch_bounds__(kFrontierThreads, 1024 / kFrontierThreads) fro
                 a.cvtx[cs + j] = v;
             }
             for (uint64_t t = t_lo; t < t_hi; ++t)
-                a.tiles[t] = (uint32_t)(cs + tile_chunk((uint32_t)(t * kTileWork - W), nch));
+                a.tiles[t] = (uint32_t)(cs + tile_chunk((uint32_t)(t * TW - W), nch));
         }
         uint32_t hm = __ballot_sync(FULL, huge);
         while (hm) {
@@ -770,9 +775,9 @@ __global__ void __launch_bounds__(kFrontierThreads, 1024 / kFrontierThreads) fro
                 a.cvtx[ocs + j] = ov;
             }
             const uint64_t owl = (uint64_t)onch * CW + od;
-            const uint64_t ot_lo = (oW + kTileWork - 1) / kTileWork, ot_hi = (oW + owl + kTileWork - 1) / kTileWork;
+            const uint64_t ot_lo = (oW + TW - 1) / TW, ot_hi = (oW + owl + TW - 1) / TW;
             for (uint64_t t = ot_lo + lane; t < ot_hi; t += 32)
-                a.tiles[t] = (uint32_t)(ocs + tile_chunk((uint32_t)(t * kTileWork - oW), onch));
+                a.tiles[t] = (uint32_t)(ocs + tile_chunk((uint32_t)(t * TW - oW), onch));
         }
     }
     FTRACE(7);
@@ -954,6 +959,10 @@ constexpr bool kLpc = EFG_LPC;  // lane-per-chunk decode of balanced batches (no
 #define EFG_SPAN_STAGE 1
 #endif
 constexpr bool kSpanStage = EFG_SPAN_STAGE;  // one bulk copy per batch when the chunks' bytes are adjacent
+#ifndef EFG_FAST_SINGLE
+#define EFG_FAST_SINGLE 1
+#endif
+constexpr bool kFastSingle = EFG_FAST_SINGLE;  // producer fast path for batches of whole short lists
 
 template <int MODE>
 __global__ void __launch_bounds__(kExpandThreads, 1) expand_kernel(ExpandArgs a)
@@ -1023,11 +1032,76 @@ __global__ void __launch_bounds__(kExpandThreads, 1) expand_kernel(ExpandArgs a)
         }
         const uint64_t c = cnext + lane;
         const bool valid = c < cend;
+        uint4 d0 = make_uint4(0, 0, 0, 0);
+        if (valid) d0 = *reinterpret_cast<const uint4 *>(a.chunks + c);
+        // fast path: every chunk of the batch is a whole short list (deg < k:
+        // no forward pointers, cc = 0, bytes [lower][upper] contiguous)
+        // with a stageable upper section — the common case on the levels that
+        // expand millions of small lists.  One span copy stages them all.
+        // (a list whose bytes + alignment slack exceed a buffer takes the general path)
+        const uint32_t lsec = ((d0.z * ((d0.y >> (kOffBits - 32)) & 63)) + 7) >> 3;
+        if (kFastSingle && (a.variant & 2) &&
+            __all_sync(FULL, !valid || ((uint64_t)d0.z < CH && d0.w <= kUpperStageMax &&
+                                        lsec + d0.w + 40 <= kStageBytes))) {
+            const uint64_t off = (((uint64_t)d0.y << 32) | d0.x) & kOffMask;
+            const uint32_t l = (d0.y >> (kOffBits - 32)) & 63, deg = d0.z, ub = d0.w;
+            const uint64_t U0b = off + ((deg * l + 7) >> 3);  // byte address of the upper section
+            const uint64_t rs = off & ~15ull;                  // staged range: the whole list + 8 B
+            const uint64_t re = (U0b + ub + 8 + 15) & ~15ull;  // (two-word lower windows), 16-B aligned
+            const uint64_t S = __shfl_sync(FULL, rs, 0);       // lane 0 is valid (cnext < cend)
+            uint32_t E = valid ? ((rs >= S && re - S < (1ull << 30)) ? (uint32_t)(re - S) : (1u << 30)) : 0u;
+#pragma unroll
+            for (int d = 1; d < 32; d <<= 1) {
+                const uint32_t t = __shfl_up_sync(FULL, E, d);
+                if ((int)lane >= d) E = max(E, t);
+            }
+            const bool fits = valid && E <= kStageBytes;
+            const uint32_t cnt = __popc(__ballot_sync(FULL, fits));
+            // sparse frontiers leave gaps between the lists: when packing the
+            // lists one after the other would fit more of them, take the
+            // general path (which then stages them per chunk)
+            uint32_t tsum;
+            const uint32_t ssum = warp_excl_u32(valid ? (uint32_t)(re - rs) : 0u, tsum);
+            const uint32_t cnt_sum = __popc(__ballot_sync(FULL, valid && ssum + (uint32_t)(re - rs) <= kStageBytes));
+            if (cnt >= cnt_sum) {
+                B.cnt = cnt;
+                const uint32_t buf = nbuf;
+                B.buf = buf;
+                nbuf ^= 1;
+                const uint64_t A0 = U0b * 8, A1 = A0 + 8ull * ub;
+                const uint32_t nel = fits ? deg : 0u;
+                const uint32_t nwd = fits ? (uint32_t)(((A1 - 1) >> 5) - (A0 >> 5) + 1) : 0u;
+                uint32_t t;  // < 2^15 elements (32 lists of < 512), < 2^16 words (32 x <= 241)
+                const uint32_t ex = warp_excl_u32(nel | nwd << 16, t);
+                B.eb = ex & 0xffffu;
+                B.wb = ex >> 16;
+                B.ne = t & 0xffffu;
+                B.nw = t >> 16;
+                B.nwd = nwd;
+                B.nel = nel;
+                B.cc = 0;
+                B.v = (MODE != kModeVisit && valid) ? a.cvtx[c] : 0u;
+                B.lpc = kLpc && (a.variant & 1) && 2 * B.ne >= 32 * __reduce_max_sync(FULL, nel);
+                const uint32_t sbase = buf * kStageBytes;
+                B.lsmb = sbits + 8 * (sbase + (uint32_t)(off - S)) - B.eb * l;
+                B.lflags = l | ((uint32_t)(A0 & 31) << 8) | ((uint32_t)((A1 - 1) & 31) << 16) | (1u << 24);
+                B.HB = 0u - 32u * B.wb - (uint32_t)(A0 & 31) + B.eb;
+                B.usrc = (sbase + (uint32_t)((A0 >> 5) * 4 - S)) >> 2;
+                cnext += B.cnt;
+                const uint32_t tot_b = __shfl_sync(FULL, E, B.cnt - 1);
+                __syncwarp();
+                if (lane == 0) {
+                    mbar_arrive_expect_tx(&ws.mbar[buf], tot_b);
+                    fence_proxy_async();
+                    bulk_g2s(reinterpret_cast<uint8_t *>(&ws.stage[0][0]) + sbase, data + S, tot_b, &ws.mbar[buf]);
+                }
+                return true;
+            }
+        }
         uint64_t lb = 0, A0 = 0, A1 = 0;
         uint32_t l = 0, nel = 0, hib = 0, v = 0, cc = 0;
         bool skipc = false;  // an empty slot: no elements, no words, no bytes
         if (valid) {
-            const uint4 d0 = *reinterpret_cast<const uint4 *>(a.chunks + c);
             const uint64_t offl = ((uint64_t)d0.y << 32) | d0.x;
             const uint64_t off = offl & kOffMask;
             const uint32_t deg = d0.z, ubytes = d0.w;

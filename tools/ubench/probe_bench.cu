@@ -3,6 +3,7 @@
 // red.global.or, and shared-memory random loads, with 8 independent probes per
 // thread in flight.  Used to size the visit step (a6) of the expand kernel.
 #include <cstdio>
+#include <cstdlib>
 #include <cstdint>
 #include <cuda_runtime.h>
 
@@ -37,8 +38,9 @@ __global__ void probe(const uint32_t* __restrict__ a, uint32_t* b, uint32_t nwor
     if (acc == 0x12345678) out[0] = acc;
 }
 
-int main() {
-    const uint32_t nwords = (1u << 24) / 32;  // 16.7M bits = 2 MiB (RMAT-24 visited bitmap)
+int main(int argc, char **argv) {
+    // default 16.7M bits = 2 MiB (RMAT-24 visited bitmap); argv[1] = bits (C3: 41652230)
+    const uint32_t nwords = (argc > 1 ? (uint32_t)atoll(argv[1]) : (1u << 24)) / 32;
     uint32_t *a, *b, *out;
     cudaMalloc(&a, nwords * 4); cudaMalloc(&b, nwords * 4); cudaMalloc(&out, 4);
     cudaMemset(a, 0x55, nwords * 4); cudaMemset(b, 0, nwords * 4);
