@@ -112,6 +112,31 @@ void efg_default_opts(efg_build_opts *o);
 efg_status efg_build(uint64_t n, uint64_t m, const uint32_t *src, const uint32_t *dst,
                      const efg_build_opts *opts, efg_graph **out);
 
+/*
+ * efg_build_stream — efg_build over edges produced on demand instead of held in
+ * caller arrays (a rank builds only its rows of a graph larger
+ * than host memory allows as an edge list, e.g. RMAT-29/ef32, BASELINE
+ * configs[4]).
+ *   gen(user, first, count, src, dst, w) must write samples [first, first +
+ *   count) of the edge list into src[0..count), dst[0..count) and, when
+ *   `weighted` != 0, w[0..count) (else w is NULL).  It is called from one
+ *   thread at a time, chunk by chunk in increasing `first`, TWICE over [0, m)
+ *   (a counting pass, then a scatter pass), and must return the same samples
+ *   both times (e.g. a counter-based generator).  Its buffers belong to the
+ *   library and are only valid during the call.
+ *   n, opts, out: as efg_build (opts->weights is ignored; weights come from gen).
+ * Memory: the builder holds the adjacency of the materialised rows only — the
+ * owned rows of a row-range handle (row_lo/row_hi) without EFG_REORDER_DEGREE;
+ * every row otherwise (the relabelling needs every degree) — never the edge
+ * list: 4 bytes per directed entry (8 when weighted) plus the EFG.
+ * The result equals efg_build on the concatenated samples.
+ * Errors: as efg_build.
+ */
+typedef void (*efg_edge_gen_fn)(void *user, uint64_t first, uint64_t count, uint32_t *src, uint32_t *dst,
+                                float *w);
+efg_status efg_build_stream(uint64_t n, uint64_t m, efg_edge_gen_fn gen, void *user, int weighted,
+                            const efg_build_opts *opts, efg_graph **out);
+
 /* Release everything the handle owns (host and device).  NULL-safe. */
 void efg_free(efg_graph *g);
 

@@ -81,6 +81,27 @@ class Graph:
         check(lib.efg_build(n, src.size, _ptr(src), _ptr(dst), C.byref(o), C.byref(h)), "efg_build")
         return cls(h.value, stream)
 
+    @classmethod
+    def build_stream(cls, n: int, m: int, gen_fn: int, gen_user: int, *, weighted: bool = False,
+                     k: int = 512, flags: int = EFG_DEFAULT_FLAGS, device: int = 0,
+                     stream: int | None = None, n_threads: int = 0, rows: tuple[int, int] | None = None):
+        """efg_build_stream: edges produced on demand by a C callback (efg_edge_gen_fn
+        address `gen_fn`, its context address `gen_user`), read twice in chunks; the
+        edge list is never materialised."""
+        o = _abi.BuildOpts()
+        lib.efg_default_opts(C.byref(o))
+        o.fwd_quantum = k
+        o.flags = flags
+        o.device = device
+        o.n_threads = n_threads
+        o.stream = stream
+        if rows is not None:
+            o.row_lo, o.row_hi = int(rows[0]), int(rows[1])
+        h = C.c_void_p()
+        check(lib.efg_build_stream(n, m, gen_fn, gen_user, 1 if weighted else 0, C.byref(o), C.byref(h)),
+              "efg_build_stream")
+        return cls(h.value, stream)
+
     def set_level_loop(self, host: bool) -> None:
         """EFG_OPT_LEVEL_LOOP: False = device-side CUDA-graph loop (default),
         True = host loop with per-level CUDA-event timing of the expand kernel."""

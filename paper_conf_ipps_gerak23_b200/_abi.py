@@ -56,6 +56,8 @@ SIGNATURES = [
     ("efg_default_opts", None, [C.POINTER(BuildOpts)]),
     ("efg_build", C.c_int, [C.c_uint64, C.c_uint64, C.c_void_p, C.c_void_p, C.POINTER(BuildOpts),
                             C.POINTER(C.c_void_p)]),
+    ("efg_build_stream", C.c_int, [C.c_uint64, C.c_uint64, C.c_void_p, C.c_void_p, C.c_int,
+                                   C.POINTER(BuildOpts), C.POINTER(C.c_void_p)]),
     ("efg_free", None, [C.c_void_p]),
     ("efg_info", C.c_int, [C.c_void_p, C.POINTER(Info)]),
     ("efg_export", C.c_int, [C.c_void_p, C.c_void_p, C.c_void_p, C.c_void_p, C.c_void_p]),

@@ -50,10 +50,12 @@ extern "C" void efg_default_opts(efg_build_opts *o)
     o->device = 0;
 }
 
-extern "C" efg_status efg_build(uint64_t n, uint64_t m, const uint32_t *src, const uint32_t *dst,
-                                const efg_build_opts *opts, efg_graph **out)
+namespace {
+
+// common part of efg_build / efg_build_stream: options, host build, upload
+template <class HostBuild>
+efg_status build_common(uint64_t n, const efg_build_opts *opts, efg_graph **out, HostBuild &&host_build)
 {
-    clear_error();
     if (!out) return set_error(EFG_EINVAL, "efg_build: out is NULL");
     *out = nullptr;
     efg_build_opts o;
@@ -62,12 +64,11 @@ extern "C" efg_status efg_build(uint64_t n, uint64_t m, const uint32_t *src, con
     else
         efg_default_opts(&o);
     if (n == 0 || n > 0xFFFFFFFFull) return set_error(EFG_EINVAL, "efg_build: need 1 <= n <= 2^32-1");
-    if (m && (!src || !dst)) return set_error(EFG_EINVAL, "efg_build: src/dst is NULL");
     if (o.row_hi > o.row_lo && (o.row_lo % 64 || (o.row_hi % 64 && o.row_hi < n)))
         return set_error(EFG_EINVAL, "efg_build: row range bounds must be multiples of 64 (or n)");
     efg_graph *g = new (std::nothrow) efg_graph();
     if (!g) return set_error(EFG_ENOMEM, "efg_build: handle allocation failed");
-    efg_status st = build_host(n, m, src, dst, o, g->host);
+    efg_status st = host_build(o, g->host);
     if (st != EFG_OK) {
         delete g;
         return st;
@@ -83,6 +84,36 @@ extern "C" efg_status efg_build(uint64_t n, uint64_t m, const uint32_t *src, con
     }
     *out = g;
     return EFG_OK;
+}
+
+}  // namespace
+
+extern "C" efg_status efg_build(uint64_t n, uint64_t m, const uint32_t *src, const uint32_t *dst,
+                                const efg_build_opts *opts, efg_graph **out)
+{
+    clear_error();
+    if (m && (!src || !dst)) {
+        if (out) *out = nullptr;
+        return set_error(EFG_EINVAL, "efg_build: src/dst is NULL");
+    }
+    return build_common(n, opts, out, [&](const efg_build_opts &o, HostEFG &h) {
+        return build_host(n, m, src, dst, o, h);
+    });
+}
+
+extern "C" efg_status efg_build_stream(uint64_t n, uint64_t m, efg_edge_gen_fn gen, void *user, int weighted,
+                                       const efg_build_opts *opts, efg_graph **out)
+{
+    clear_error();
+    if (m && !gen) {
+        if (out) *out = nullptr;
+        return set_error(EFG_EINVAL, "efg_build_stream: gen is NULL");
+    }
+    return build_common(n, opts, out, [&](const efg_build_opts &o, HostEFG &h) {
+        efg_build_opts o2 = o;
+        o2.weights = nullptr;
+        return build_host_stream(n, m, gen, user, weighted, o2, h);
+    });
 }
 
 extern "C" void efg_free(efg_graph *g)

@@ -49,6 +49,8 @@ ListGeom list_geom(uint64_t n, uint64_t u, uint32_t k);
 // Builder (efg_builder.cpp).  Returns EFG_OK or an error with set_error().
 efg_status build_host(uint64_t n, uint64_t m, const uint32_t *src, const uint32_t *dst,
                       const efg_build_opts &o, HostEFG &out);
+efg_status build_host_stream(uint64_t n, uint64_t m, efg_edge_gen_fn gen, void *user, int weighted,
+                             const efg_build_opts &o, HostEFG &out);
 
 // ---------------------------------------------------------------------------
 // Device layout

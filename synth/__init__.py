@@ -57,6 +57,8 @@ def lib():
         L.synth_web_hosts.restype = C.c_uint64
         L.synth_web_hosts.argtypes = [C.c_uint64, C.c_double, C.c_uint64, C.c_uint64, u64p,
                                       C.c_uint64]
+        L.synth_gen_range.restype = None
+        L.synth_gen_range.argtypes = [C.c_void_p, C.c_uint64, C.c_uint64, u32p, u32p, f32p]
         L.synth_web_host_of.restype = None
         L.synth_web_host_of.argtypes = [C.c_uint64, u64p, u32p]
         L.synth_web.restype = None
@@ -177,3 +179,73 @@ def config_edges(c: int, scale_override: int | None = None, permute: bool | None
     if perm_flag:
         apply_permutation(permutation(n, 100 + c), src, dst)
     return n, src, dst
+
+
+# ---------------------------------------------------------------------------
+# Streamed generation (efg_build_stream): samples produced on demand by range
+# ---------------------------------------------------------------------------
+class _GenCtx(C.Structure):
+    _fields_ = [("kind", C.c_int), ("scale", C.c_int), ("n", C.c_uint64), ("seed", C.c_uint64),
+                ("a", C.c_double), ("b", C.c_double), ("c", C.c_double),
+                ("alpha_src", C.c_double), ("alpha_dst", C.c_double), ("rho", C.c_double),
+                ("host_start", C.c_void_p), ("n_hosts", C.c_uint64), ("host_of", C.c_void_p),
+                ("p_intra", C.c_double), ("p_near", C.c_double), ("zipf_alpha", C.c_double),
+                ("perm", C.c_void_p), ("wseed", C.c_uint64)]
+
+
+class StreamGen:
+    """A config's edge generator as a C callback (synth_gen_range, the
+    efg_edge_gen_fn signature): `fn` and `user` are raw addresses to hand to
+    efg_build_stream; samples [first, first+count) equal the same indices of
+    config_edges(c).  Keeps its arrays alive."""
+
+    def __init__(self, n: int, m: int, ctx: _GenCtx, keep: list):
+        self.n, self.m, self._ctx, self._keep = n, m, ctx, keep
+        self.fn = C.cast(lib().synth_gen_range, C.c_void_p).value
+        self.user = C.addressof(ctx)
+
+    def range(self, first: int, count: int, weighted: bool = False):
+        src = np.empty(count, np.uint32)
+        dst = np.empty(count, np.uint32)
+        w = np.empty(count, np.float32) if weighted else None
+        lib().synth_gen_range(C.byref(self._ctx), first, count, _ptr(src, u32p), _ptr(dst, u32p),
+                              _ptr(w, f32p) if weighted else None)
+        return (src, dst, w) if weighted else (src, dst)
+
+
+def config_stream(c: int, scale_override: int | None = None, permute: bool | None = None,
+                  weight_seed: int | None = None) -> StreamGen:
+    """StreamGen of BASELINE.json config c (same samples as config_edges)."""
+    cfg = CONFIGS[c]
+    perm_flag = cfg["permute"] if permute is None else permute
+    ctx = _GenCtx()
+    keep = []
+    ctx.seed = c
+    ctx.wseed = 2000 + c if weight_seed is None else weight_seed
+    if cfg["kind"] == "rmat":
+        scale = scale_override if scale_override is not None else cfg["scale"]
+        n, m = 1 << scale, cfg["ef"] << scale
+        ctx.kind, ctx.scale, ctx.n = 0, scale, n
+        ctx.a, ctx.b, ctx.c = RMAT_ABC
+    elif cfg["kind"] == "chunglu":
+        n, m = cfg["n"], cfg["m"]
+        ctx.kind, ctx.n = 1, n
+        ctx.alpha_src, ctx.alpha_dst, ctx.rho = cfg["alpha_src"], cfg["alpha_dst"], cfg["rho"]
+    elif cfg["kind"] == "web":
+        n, m = cfg["n"], cfg["m"]
+        hs = np.zeros(n + 1, np.uint64)
+        nh = lib().synth_web_hosts(n, 1.5, 20000, c, _ptr(hs, u64p), n)
+        hs = np.ascontiguousarray(hs[:nh + 1])
+        host_of = np.empty(n, np.uint32)
+        lib().synth_web_host_of(nh, _ptr(hs, u64p), _ptr(host_of, u32p))
+        keep += [hs, host_of]
+        ctx.kind, ctx.n = 2, n
+        ctx.host_start, ctx.n_hosts, ctx.host_of = hs.ctypes.data, nh, host_of.ctypes.data
+        ctx.p_intra, ctx.p_near, ctx.zipf_alpha = 0.85, 0.10, 1.4
+    else:
+        raise ValueError(cfg)
+    if perm_flag:
+        p = permutation(n, 100 + c)
+        keep.append(p)
+        ctx.perm = p.ctypes.data
+    return StreamGen(n, m, ctx, keep)

@@ -44,12 +44,13 @@ uint64_t synth_draw(uint64_t seed, uint64_t i, uint64_t j) { return draw(seed, i
 
 /* R-MAT / Kronecker edge sampler: for each of `scale` bit levels (MSB first)
  * pick a quadrant with probabilities a, b, c, 1-a-b-c.  `m` undirected samples. */
-void synth_rmat(int scale, uint64_t m, double a, double b, double c, uint64_t seed,
-                uint32_t *src, uint32_t *dst)
+static void rmat_range(int scale, uint64_t first, uint64_t m, double a, double b, double c, uint64_t seed,
+                       uint32_t *src, uint32_t *dst)
 {
     const double ab = a + b, abc = a + b + c;
 #pragma omp parallel for schedule(static)
-    for (int64_t e = 0; e < (int64_t)m; ++e) {
+    for (int64_t i = 0; i < (int64_t)m; ++i) {
+        const uint64_t e = first + (uint64_t)i;
         uint32_t u = 0, v = 0;
         for (int lvl = 0; lvl < scale; ++lvl) {
             double r = unif(draw(seed, (uint64_t)e, (uint64_t)lvl));
@@ -61,9 +62,15 @@ void synth_rmat(int scale, uint64_t m, double a, double b, double c, uint64_t se
             u = (u << 1) | ub;
             v = (v << 1) | vb;
         }
-        src[e] = u;
-        dst[e] = v;
+        src[i] = u;
+        dst[i] = v;
     }
+}
+
+void synth_rmat(int scale, uint64_t m, double a, double b, double c, uint64_t seed,
+                uint32_t *src, uint32_t *dst)
+{
+    rmat_range(scale, 0, m, a, b, c, seed, src, dst);
 }
 
 /* uniform random endpoints in [0,n) */
@@ -112,23 +119,30 @@ static inline uint32_t zipf_draw(uint64_t n, double alpha, double r)
     return (uint32_t)xi;
 }
 
+static void chunglu_range(uint64_t n, uint64_t first, uint64_t m, double alpha_src, double alpha_dst,
+                          double rho, uint64_t seed, uint32_t *src, uint32_t *dst)
+{
+#pragma omp parallel for schedule(static)
+    for (int64_t i = 0; i < (int64_t)m; ++i) {
+        const uint64_t e = first + (uint64_t)i;
+        uint64_t r0 = draw(seed, e, 0);
+        if (e > 0 && unif(r0) < rho) {
+            /* reciprocal copy of an earlier sample (index drawn from [0,e)) */
+            uint64_t j = (uint64_t)((__uint128_t)draw(seed, e, 1) * e >> 64);
+            uint32_t u = zipf_draw(n, alpha_src, unif(draw(seed, j, 2)));
+            uint32_t v = zipf_draw(n, alpha_dst, unif(draw(seed, j, 3)));
+            src[i] = v; dst[i] = u;
+        } else {
+            src[i] = zipf_draw(n, alpha_src, unif(draw(seed, e, 2)));
+            dst[i] = zipf_draw(n, alpha_dst, unif(draw(seed, e, 3)));
+        }
+    }
+}
+
 void synth_chunglu(uint64_t n, uint64_t m, double alpha_src, double alpha_dst, double rho,
                    uint64_t seed, uint32_t *src, uint32_t *dst)
 {
-#pragma omp parallel for schedule(static)
-    for (int64_t e = 0; e < (int64_t)m; ++e) {
-        uint64_t r0 = draw(seed, (uint64_t)e, 0);
-        if (e > 0 && unif(r0) < rho) {
-            /* reciprocal copy of an earlier sample (index drawn from [0,e)) */
-            uint64_t j = (uint64_t)((__uint128_t)draw(seed, (uint64_t)e, 1) * (uint64_t)e >> 64);
-            uint32_t u = zipf_draw(n, alpha_src, unif(draw(seed, j, 2)));
-            uint32_t v = zipf_draw(n, alpha_dst, unif(draw(seed, j, 3)));
-            src[e] = v; dst[e] = u;
-        } else {
-            src[e] = zipf_draw(n, alpha_src, unif(draw(seed, (uint64_t)e, 2)));
-            dst[e] = zipf_draw(n, alpha_dst, unif(draw(seed, (uint64_t)e, 3)));
-        }
-    }
+    chunglu_range(n, 0, m, alpha_src, alpha_dst, rho, seed, src, dst);
 }
 
 /* Web-shaped locality graph.  Vertices are grouped into contiguous "hosts" of
@@ -163,12 +177,13 @@ static inline int64_t geom_off(double p, double r)
     return 1 + (int64_t)floor(log(1.0 - r) / log(1.0 - p));
 }
 
-void synth_web(uint64_t n, uint64_t m, const uint64_t *host_start, uint64_t n_hosts,
-               const uint32_t *host_of, double p_intra, double p_near, double zipf_alpha,
-               uint64_t seed, uint32_t *src, uint32_t *dst)
+static void web_range(uint64_t n, uint64_t first, uint64_t m, const uint64_t *host_start, uint64_t n_hosts,
+                      const uint32_t *host_of, double p_intra, double p_near, double zipf_alpha,
+                      uint64_t seed, uint32_t *src, uint32_t *dst)
 {
 #pragma omp parallel for schedule(static)
-    for (int64_t e = 0; e < (int64_t)m; ++e) {
+    for (int64_t i = 0; i < (int64_t)m; ++i) {
+        const int64_t e = (int64_t)(first + (uint64_t)i);
         uint64_t u = (uint64_t)((__uint128_t)draw(seed, (uint64_t)e, 0) * n >> 64);
         uint64_t h = host_of[u];
         double kind = unif(draw(seed, (uint64_t)e, 1));
@@ -196,9 +211,16 @@ void synth_web(uint64_t n, uint64_t m, const uint64_t *host_start, uint64_t n_ho
             if (draw(seed, (uint64_t)e, 5) & 1) v = lo;
             else v = lo + (uint64_t)((__uint128_t)draw(seed, (uint64_t)e, 4) * (hi - lo) >> 64);
         }
-        src[e] = (uint32_t)u;
-        dst[e] = (uint32_t)v;
+        src[i] = (uint32_t)u;
+        dst[i] = (uint32_t)v;
     }
+}
+
+void synth_web(uint64_t n, uint64_t m, const uint64_t *host_start, uint64_t n_hosts,
+               const uint32_t *host_of, double p_intra, double p_near, double zipf_alpha,
+               uint64_t seed, uint32_t *src, uint32_t *dst)
+{
+    web_range(n, 0, m, host_start, n_hosts, host_of, p_intra, p_near, zipf_alpha, seed, src, dst);
 }
 
 /* host_of[v] for v in [0,n) given host_start */
@@ -225,3 +247,43 @@ void synth_weights(uint64_t m, const uint32_t *src, const uint32_t *dst, uint64_
 }
 
 float synth_weight_pair(uint64_t seed, uint32_t u, uint32_t v) { return weight_of(seed, u, v); }
+
+/* ------------------------------------------------------------------------- */
+/* Range generation for streamed builds (efg_build_stream): a context names a */
+/* config's generator; synth_gen_range writes samples [first, first+count),   */
+/* identical to the same indices of the whole-array generator, then the       */
+/* optional relabelling and the optional weights.  Matches efg_edge_gen_fn.   */
+/* ------------------------------------------------------------------------- */
+typedef struct synth_gen_ctx {
+    int kind;                 /* 0 rmat, 1 chunglu, 2 web, 3 uniform */
+    int scale;
+    uint64_t n, seed;
+    double a, b, c;           /* rmat */
+    double alpha_src, alpha_dst, rho;  /* chunglu */
+    const uint64_t *host_start;        /* web */
+    uint64_t n_hosts;
+    const uint32_t *host_of;
+    double p_intra, p_near, zipf_alpha;
+    const uint32_t *perm;     /* relabelling x -> perm[x], or NULL */
+    uint64_t wseed;           /* weight seed (weights written when w != NULL) */
+} synth_gen_ctx;
+
+void synth_gen_range(void *vctx, uint64_t first, uint64_t count, uint32_t *src, uint32_t *dst, float *w)
+{
+    const synth_gen_ctx *g = (const synth_gen_ctx *)vctx;
+    switch (g->kind) {
+    case 0: rmat_range(g->scale, first, count, g->a, g->b, g->c, g->seed, src, dst); break;
+    case 1: chunglu_range(g->n, first, count, g->alpha_src, g->alpha_dst, g->rho, g->seed, src, dst); break;
+    case 2: web_range(g->n, first, count, g->host_start, g->n_hosts, g->host_of, g->p_intra, g->p_near,
+                      g->zipf_alpha, g->seed, src, dst); break;
+    default:
+#pragma omp parallel for schedule(static)
+        for (int64_t i = 0; i < (int64_t)count; ++i) {
+            const uint64_t e = first + (uint64_t)i;
+            src[i] = (uint32_t)((__uint128_t)draw(g->seed, e, 0) * g->n >> 64);
+            dst[i] = (uint32_t)((__uint128_t)draw(g->seed, e, 1) * g->n >> 64);
+        }
+    }
+    if (g->perm) synth_apply_permutation(count, g->perm, src, dst);
+    if (w) synth_weights(count, src, dst, g->wseed, w);
+}
