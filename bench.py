@@ -74,6 +74,8 @@ def parse():
                    help="N > 1 partition mode: per-level exchange by the library's kernels over "
                         "NVLink peer memory (CUDA IPC, efg_xchg_peer) or all_to_all + all_gather "
                         "with torch.distributed (efg_xchg_pack/reduce/unpack)")
+    p.add_argument("--permute", action="store_true",
+                   help="random relabelling of the generator's ids (P:248-258 'random ordering' arm)")
     p.add_argument("--reorder", default="degree", choices=["none", "degree"],
                    help="EFG_REORDER_DEGREE relabelling at build time (results stay in input ids)")
     p.add_argument("--profile-levels", action="store_true", help="print per-level stats to stderr")
@@ -221,6 +223,19 @@ def make_graph_edges(cfg: int, scale: int | None):
     return n, src, dst, time.time() - t0
 
 
+def build_graph(efg, args, *, permute=None, weighted=False, **kw):
+    """The config's EFG built from its generator (efg_build_stream: the edge list
+    is never materialised in this process, which keeps C4/C5 within host RAM).
+    Returns (graph, generator-setup seconds)."""
+    import synth
+    t0 = time.time()
+    sg = synth.config_stream(args.config, scale_override=args.scale, permute=permute)
+    gen_s = time.time() - t0
+    g = efg.Graph.build_stream(sg.n, sg.m, sg.fn, sg.user, weighted=weighted,
+                               n_threads=os.cpu_count() or 1, **kw)
+    return g, gen_s
+
+
 def cpu_model() -> str:
     try:
         with open("/proc/cpuinfo") as f:
@@ -235,14 +250,14 @@ def cpu_model() -> str:
 REF_STEP_EDGES = 1 << 28  # reference-arm step: FIFO BFS stopped after this many scanned edges
 
 
-def _cpu_baseline_child(cfg: int, scale, index: int, count: int, out_dir: str, core: int):
+def _cpu_baseline_child(cfg: int, scale, index: int, count: int, out_dir: str, core: int, permute=None):
     """Spawned process (bench.py cpu_baseline leg): the oracle's CSR of the
     same seeded graph, then ONE plain single-threaded FIFO BFS from the first
     timed source, pinned to `core` (the parent keeps off that core).  Writes
     depth.npy and meta.json to out_dir."""
     import oracle
     import synth
-    n, src, dst = synth.config_edges(cfg, scale_override=scale)
+    n, src, dst = synth.config_edges(cfg, scale_override=scale, permute=permute)
     os.sched_setaffinity(0, {core})
     t0 = time.time()
     ov, oe = oracle.csr_build(n, src, dst)
@@ -268,7 +283,8 @@ def start_cpu_baseline(args, count: int, index: int):
     core = cores[-1]
     out_dir = tempfile.mkdtemp(prefix="efg_cpu_baseline_")
     proc = mp.get_context("spawn").Process(target=_cpu_baseline_child,
-                                            args=(args.config, args.scale, index, count, out_dir, core))
+                                            args=(args.config, args.scale, index, count, out_dir, core,
+                                                  args.permute or None))
     proc.start()
     if len(cores) > 1:
         os.sched_setaffinity(0, set(cores[:-1]))
@@ -338,46 +354,63 @@ def run_reference(args, rank, world):
 
 
 def run_partitioned(args, rank, world, local):
-    """N ranks, one BFS at a time over the 1-D row partition (strong scaling)."""
+    """N ranks, one collective BFS at a time over the 1-D row partition (strong
+    scaling).  Each rank builds only its rows from the generator
+    (efg_build_stream); per level the library expands the rank's rows, ORs the
+    new bits over peer memory and ends the level on the device (efg_bfs on a
+    partitioned handle: no host round trip per level).  --xchg nccl drives the
+    same levels step by step with torch.distributed collectives instead."""
     import torch
     import torch.distributed as dist
     import synth
     import paper_conf_ipps_gerak23_b200 as efg
-    from paper_conf_ipps_gerak23_b200.dist import (TorchTransport, partitioned_bfs, partitioned_bfs_peer,
-                                                   peer_setup)
+    from paper_conf_ipps_gerak23_b200.dist import TorchTransport, partitioned_bfs, peer_setup
 
     dev = torch.device("cuda", local)
     stream = torch.cuda.Stream(device=dev)
-    n, src, dst, gen_s = make_graph_edges(args.config, args.scale)
     flags = efg.EFG_DEFAULT_FLAGS | (efg.EFG_REORDER_DEGREE if args.reorder == "degree" else 0)
     cdev = dev if dist.get_backend() == "nccl" else torch.device("cpu")
+    sg = synth.config_stream(args.config, scale_override=args.scale, permute=args.permute or None)
+    n = sg.n
     bounds = torch.zeros(world + 1, dtype=torch.int64, device=cdev)
-    deg_in = torch.zeros(n, dtype=torch.int64, device=cdev)
-    if rank == 0:  # byte-balanced partition of the whole graph (host-only handle)
-        whole = efg.Graph.build(n, src, dst, device=-1, flags=flags, n_threads=os.cpu_count() or 1)
-        vl, _, of, _ = whole.export()
-        pm = whole.perm()
-        b = efg.partition(vl, of, world)
-        bounds.copy_(torch.from_numpy(b.astype(np.int64)))
-        d = np.empty(n, np.int64)
-        d[pm] = np.diff(vl).astype(np.int64)
-        deg_in.copy_(torch.from_numpy(d))
-        whole.free()
-    dist.broadcast(bounds, 0)
-    dist.broadcast(deg_in, 0)
-    b = bounds.cpu().numpy().astype(np.uint64)
-    deg = deg_in.cpu().numpy()
+    srcs_t = torch.zeros(args.warmup + args.steps, dtype=torch.int64, device=cdev)
     nthr = max(1, (os.cpu_count() or 1) // world)
-    g = efg.Graph.build(n, src, dst, device=local, stream=stream.cuda_stream, flags=flags,
-                        rows=(int(b[rank]), int(b[rank + 1])), n_threads=nthr)
-    del src, dst
-    srcs = synth.sources(n, args.warmup + args.steps, seed=1000 + args.config, nonisolated_mask=deg > 0)
+    if rank == 0:
+        if args.reorder == "degree":
+            # byte-balanced bounds need the relabelled sizes: one host-only
+            # whole-graph build on rank 0 (efg_partition, SURVEY 8(e))
+            whole = efg.Graph.build_stream(n, sg.m, sg.fn, sg.user, device=-1, flags=flags,
+                                           n_threads=os.cpu_count() or 1)
+            vl, _, of, _ = whole.export()
+            b = efg.partition(vl, of, world)
+            pm = whole.perm()
+            deg = np.empty(n, np.int64)
+            deg[pm] = np.diff(vl).astype(np.int64)
+            whole.free()
+        else:
+            # generator order (e.g. permuted RMAT, C5): equal vertex ranges, 64-aligned
+            b = np.array([min(n, (n * r // world + 63) // 64 * 64) for r in range(world)] + [n], np.uint64)
+            deg = None
+        if deg is not None:
+            s = synth.sources(n, args.warmup + args.steps, seed=1000 + args.config, nonisolated_mask=deg > 0)
+        else:
+            s = synth.sources(n, args.warmup + args.steps, seed=1000 + args.config)
+        bounds.copy_(torch.from_numpy(b.astype(np.int64)))
+        srcs_t.copy_(torch.from_numpy(s.astype(np.int64)))
+    dist.broadcast(bounds, 0)
+    dist.broadcast(srcs_t, 0)
+    b = bounds.cpu().numpy().astype(np.uint64)
+    srcs = srcs_t.cpu().numpy()
+    t0 = time.time()
+    g = efg.Graph.build_stream(n, sg.m, sg.fn, sg.user, device=local, stream=stream.cuda_stream, flags=flags,
+                               rows=(int(b[rank]), int(b[rank + 1])), n_threads=nthr)
+    build_s = time.time() - t0
     depth = torch.empty(n, dtype=torch.int32, device=dev)
     tr = TorchTransport(stage_on_host=dist.get_backend() != "nccl")
     mk = lambda k: torch.zeros(k, dtype=torch.int32, device=dev)  # noqa: E731
     if args.xchg == "peer":
         peer_setup(g, rank, b)  # IPC handles all-gathered once; no collective per level
-        one_bfs = lambda s: partitioned_bfs_peer(g, s, depth)  # noqa: E731
+        one_bfs = lambda s: g.bfs(s, depth=depth)  # noqa: E731  collective, enqueue-only
     else:
         one_bfs = lambda s: partitioned_bfs(g, s, depth, b, tr, mk)  # noqa: E731
     with torch.cuda.stream(stream):
@@ -390,43 +423,64 @@ def run_partitioned(args, rank, world, local):
     clk.start()
     e0 = torch.cuda.Event(enable_timing=True)
     e1 = torch.cuda.Event(enable_timing=True)
-    edges = 0
-    launches = 0
     e0.record(stream)
     with torch.cuda.stream(stream):
         for s in srcs[args.warmup:]:
             one_bfs(int(s))
-            st = g.bfs_end()
-            edges += st["edges_traversed"]  # this rank's rows
-            launches += st["kernel_launches"]
     e1.record(stream)
     torch.cuda.synchronize()
     clocks = clk.stop()
     ms = e0.elapsed_time(e1)
-    t = torch.tensor([ms], dtype=torch.float64, device=cdev)
+    # traversed edges of this rank's rows (untimed statistics pass; the
+    # collective call with statistics synchronises)
+    edges, launches = 0, 0
+    for s in srcs[args.warmup:]:
+        if args.xchg == "peer":
+            _, _, st = g.bfs(int(s), depth=depth, stats=True)
+        else:
+            partitioned_bfs(g, int(s), depth, b, tr, mk)
+            st = g.bfs_end()
+        edges += st["edges_traversed"]
+        launches += st["kernel_launches"]
+    # e2e: the same collective calls with a pinned host depth array
+    hdepth = torch.empty(n, dtype=torch.int32, pin_memory=True)
+    dist.barrier()
+    t1 = time.perf_counter()
+    if args.xchg == "peer":
+        for s in srcs[args.warmup:]:
+            g.bfs(int(s), depth=hdepth)
+    e2e_s = time.perf_counter() - t1
+    t = torch.tensor([ms, e2e_s], dtype=torch.float64, device=cdev)
     e = torch.tensor([edges], dtype=torch.float64, device=cdev)
     dist.all_reduce(t, op=dist.ReduceOp.MAX)
     dist.all_reduce(e, op=dist.ReduceOp.SUM)
-    value = float(e.item()) / (float(t.item()) * 1e-3) / 1e9
+    value = float(e.item()) / (float(t[0].item()) * 1e-3) / 1e9
     if rank == 0:
         cfgname = synth.CONFIGS[args.config]["name"] + (f"_scale{args.scale}" if args.scale else "")
+        gpus = torch.cuda.device_count()
         line = {
             "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
-            "warmup": args.warmup, "ms_per_step": float(t.item()) / args.steps,
+            "warmup": args.warmup, "ms_per_step": float(t[0].item()) / args.steps,
             "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "u32",
             "data": "synthetic",
-            "config": {"workload": cfgname, "n": int(n), "reorder": args.reorder,
-                       "parallelism": f"1-D row partition over {world} GPUs, per-level bitmap "
-                                      + ("exchange by the library's kernels over peer memory "
-                                         "(owner OR + broadcast, CUDA IPC over NVLink)"
-                                         if args.xchg == "peer" else
-                                         "exchange (all_to_all + OR + all_gather, NCCL)"),
-                       "xchg": args.xchg,
-                       "bounds": [int(x) for x in b],
+            "config": {"workload": cfgname, "n": int(n), "reorder": args.reorder, "permute": bool(args.permute),
+                       "parallelism": f"1-D row partition over {world} ranks on {min(world, gpus)} GPU(s), "
+                                      "per-level bitmap "
+                                      + ("exchange by the library's kernels over peer memory (owner OR + "
+                                         "broadcast, CUDA IPC), collective efg_bfs with the level loop on "
+                                         "the device" if args.xchg == "peer" else
+                                         "exchange (all_to_all + OR + all_gather, torch.distributed)"),
+                       "ranks_per_gpu": world / max(1, min(world, gpus)),
+                       "xchg": args.xchg, "bounds": [int(x) for x in b],
+                       "build_s_rank0": round(build_s, 2),
                        "l2_policy": "inputs larger than L2"},
             "clocks": clocks, "gpu_launches": launches,
             "gpu_launches_note": "rank 0's kernels (every rank launches the same number per level)",
-            "e2e": None, "cpu_baseline": None,
+            "e2e": ({"value": float(e.item()) / float(t[1].item()) / 1e9, "unit": UNIT, "h2d_bytes_per_step": 4,
+                     "d2h_bytes_per_step": None,
+                     "d2h_note": "every rank receives the full depth array in a pinned host buffer"}
+                    if args.xchg == "peer" else None),
+            "cpu_baseline": None,
         }
         print(json.dumps(line), flush=True)
     g.free()
@@ -442,7 +496,9 @@ def main():
     # the oracle baseline runs in a spawned process on its own core while this
     # process builds and measures (started before any thread pool exists here)
     cpu_job = None
-    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+    # (C4's oracle CSR alone needs ~130 GB of host memory next to this process's
+    # build: its parity runs in tests/verify_full.py instead)
+    if rank == 0 and world == 1 and not args.no_cpu_baseline and args.config != 4:
         cpu_job = start_cpu_baseline(args, args.warmup + args.steps, args.warmup)
 
     import torch
@@ -464,10 +520,10 @@ def main():
     dev = torch.device("cuda", local)
     stream = torch.cuda.Stream(device=dev)
 
-    n, src, dst, gen_s = make_graph_edges(args.config, args.scale)
     flags = efg.EFG_DEFAULT_FLAGS | (efg.EFG_REORDER_DEGREE if args.reorder == "degree" else 0)
-    g = efg.Graph.build(n, src, dst, device=local, stream=stream.cuda_stream, flags=flags)
-    del src, dst
+    g, gen_s = build_graph(efg, args, device=local, stream=stream.cuda_stream, flags=flags,
+                           permute=args.permute or None)
+    n = g.n
     info = g.info
     vlist, nlb, offsets, _ = g.export()
     perm = g.perm()  # stored id -> input id
@@ -578,9 +634,7 @@ def main():
     # ---- the same measurement without the degree relabelling (transparency) ----
     alt = None
     if world == 1 and args.reorder == "degree" and args.do_alt:
-        n2, s2, d2, _ = make_graph_edges(args.config, args.scale)
-        g2 = efg.Graph.build(n2, s2, d2, device=local, stream=stream.cuda_stream)
-        del s2, d2
+        g2, _ = build_graph(efg, args, device=local, stream=stream.cuda_stream, permute=args.permute or None)
         with torch.cuda.stream(stream):
             for s in my[:args.warmup]:
                 g2.bfs(int(s), depth=depth)
@@ -644,10 +698,11 @@ def main():
     # weights"): frontier Bellman-Ford over the EFG, fp32 weights (reading C20) ----
     sssp = None
     if world == 1 and args.do_sssp:
-        n3, s3, d3, _ = make_graph_edges(args.config, args.scale)
-        w3 = synth.weights(s3, d3, 2000 + args.config)
-        g3 = efg.Graph.build(n3, s3, d3, device=local, stream=stream.cuda_stream, flags=flags, weights=w3)
-        del s3, d3, w3
+        # weighted build in the generator's order (no relabelling: the weighted
+        # builder keeps 8-byte adjacency entries; C4's generator order is its
+        # locality order, the paper's "with reordering" arm)
+        g3, _ = build_graph(efg, args, device=local, stream=stream.cuda_stream, weighted=True,
+                            permute=args.permute or None)
         dist_d = torch.empty(n, dtype=torch.float32, device=dev)
         with torch.cuda.stream(stream):
             g3.sssp(int(my[0]), dist=dist_d)  # warm-up

@@ -157,7 +157,7 @@ CONFIGS = {
     2: dict(name="rmat24_ef16", kind="rmat", scale=24, ef=16, permute=False),
     3: dict(name="twitter_like", kind="chunglu", n=41_652_230, m=1_468_365_182,
             alpha_src=0.85, alpha_dst=0.8, rho=0.18, permute=False),
-    4: dict(name="web_like", kind="web", n=100_000_000, m=3_500_000_000, permute=False),
+    4: dict(name="web_like", kind="web", n=100_000_000, m=6_300_000_000, permute=False),
     5: dict(name="rmat29_ef32", kind="rmat", scale=29, ef=32, permute=True),
 }
 
