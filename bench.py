@@ -74,6 +74,9 @@ def parse():
                    help="N > 1 partition mode: per-level exchange by the library's kernels over "
                         "NVLink peer memory (CUDA IPC, efg_xchg_peer) or all_to_all + all_gather "
                         "with torch.distributed (efg_xchg_pack/reduce/unpack)")
+    p.add_argument("--host-resident", action="store_true",
+                   help="out-of-core EFG (EFG_HOST_RESIDENT, P:34/P:222): EF data in pinned host memory, "
+                        "read by the kernels over the host link")
     p.add_argument("--permute", action="store_true",
                    help="random relabelling of the generator's ids (P:248-258 'random ordering' arm)")
     p.add_argument("--reorder", default="degree", choices=["none", "degree"],
@@ -521,6 +524,8 @@ def main():
     stream = torch.cuda.Stream(device=dev)
 
     flags = efg.EFG_DEFAULT_FLAGS | (efg.EFG_REORDER_DEGREE if args.reorder == "degree" else 0)
+    if args.host_resident:
+        flags |= efg.EFG_HOST_RESIDENT
     g, gen_s = build_graph(efg, args, device=local, stream=stream.cuda_stream, flags=flags,
                            permute=args.permute or None)
     n = g.n
@@ -751,6 +756,7 @@ def main():
                        "csr32_over_efg": (4 * info["m"] + 4 * (n + 1)) / (info["data_bytes"] + 17 * n),
                        "l2_policy": "inputs larger than L2 (EF data %.2f GB > 126 MB)" % (info["data_bytes"] / 1e9),
                        "parallelism": f"{world} independent BFS replicas" if world > 1 else "1 GPU",
+                       "data_location": "host (pinned, mapped: out-of-core)" if info["data_location"] else "HBM",
                        "build_s": round(info["build_seconds"], 2), "gen_s": round(gen_s, 2)},
             "clocks": clocks,
             "gpu_launches": launches,

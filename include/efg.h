@@ -55,6 +55,13 @@ typedef enum efg_status {
                                    * parent, dist, rank) stay in INPUT ids; efg_export and
                                    * efg_decode describe the relabelled graph, whose relabelling
                                    * efg_export_perm returns. */
+#define EFG_HOST_RESIDENT 0x10u   /* out-of-core EFG (§I, §VIII-B): the EF
+                                   * `data` array stays in pinned host memory mapped into
+                                   * the device's address space; the traversal kernels stage it
+                                   * over the host link (zero-copy) while the vertex records,
+                                   * bitmaps and work plan stay in HBM.  Without this flag the
+                                   * same happens automatically when `data` does not fit the
+                                   * device's free memory (efg_info_t.data_location). */
 #define EFG_DEFAULT_FLAGS (EFG_SYMMETRIZE | EFG_DEDUP | EFG_DROP_SELF_LOOPS)
 
 typedef struct efg_graph efg_graph; /* opaque: host EFG arrays + device copy */
@@ -159,7 +166,8 @@ typedef struct efg_info_t {
                               * 1 <= k <= 512 and ceil(deg/k) < 2^18 for every    *
                               * list, else 512 (the device copy's forward         *
                               * pointers are re-sampled; the host arrays keep k)  */
-    uint32_t reserved_;
+    uint32_t data_location;  /* 0: EF data in device memory (HBM); 1: pinned host  *
+                              * memory mapped into the device (out-of-core)       */
 } efg_info_t;
 
 efg_status efg_info(const efg_graph *g, efg_info_t *info);

@@ -16,11 +16,11 @@ import ctypes as C
 import numpy as np
 
 from . import _abi
-from ._abi import (EFG_DEDUP, EFG_DEFAULT_FLAGS, EFG_DROP_SELF_LOOPS, EFG_REORDER_DEGREE,  # noqa: F401
-                   EFG_SYMMETRIZE, EFGError, check, lib)
+from ._abi import (EFG_DEDUP, EFG_DEFAULT_FLAGS, EFG_DROP_SELF_LOOPS, EFG_HOST_RESIDENT,  # noqa: F401
+                   EFG_REORDER_DEGREE, EFG_SYMMETRIZE, EFGError, check, lib)
 
 __all__ = ["Graph", "EFGError", "EFG_DEFAULT_FLAGS", "EFG_SYMMETRIZE", "EFG_DEDUP",
-           "EFG_DROP_SELF_LOOPS", "EFG_REORDER_DEGREE", "version", "partition"]
+           "EFG_DROP_SELF_LOOPS", "EFG_REORDER_DEGREE", "EFG_HOST_RESIDENT", "version", "partition"]
 
 
 def version() -> str:

@@ -19,6 +19,7 @@ STATUS_NAMES = {0: "EFG_OK", 1: "EFG_EINVAL", 2: "EFG_ERANGE", 3: "EFG_ENOMEM", 
 EFG_SYMMETRIZE, EFG_DEDUP, EFG_DROP_SELF_LOOPS = 0x1, 0x2, 0x4
 EFG_DEFAULT_FLAGS = 0x7
 EFG_REORDER_DEGREE = 0x8
+EFG_HOST_RESIDENT = 0x10
 EFG_OPT_LEVEL_LOOP = 1
 EFG_OPT_PREFIX_SKIP = 2
 EFG_OPT_PAGERANK_PULL = 3
@@ -38,7 +39,7 @@ class Info(C.Structure):
                 ("apriori_bits", C.c_uint64), ("vertex_bytes", C.c_uint64),
                 ("device_bytes", C.c_uint64), ("row_lo", C.c_uint64), ("row_hi", C.c_uint64),
                 ("build_seconds", C.c_double), ("device_quantum", C.c_uint32),
-                ("reserved_", C.c_uint32)]
+                ("data_location", C.c_uint32)]
 
 
 class Stats(C.Structure):

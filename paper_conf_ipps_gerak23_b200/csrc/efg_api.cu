@@ -145,6 +145,7 @@ extern "C" efg_status efg_info(const efg_graph *g, efg_info_t *info)
     info->row_hi = h.row_hi;
     info->build_seconds = h.build_seconds;
     info->device_quantum = g->on_device ? g->dev.k : 0;
+    info->data_location = (g->on_device && g->dev.data_host) ? 1u : 0u;
     return EFG_OK;
 }
 

@@ -292,7 +292,10 @@ void device_free(DeviceGraph &d)
 {
     device_drop_graphs(d);
     device_peer_close(d);
-    cudaFree(d.data);
+    if (d.data_host)
+        cudaFreeHost(d.data_host);  // out-of-core: d.data is its device mapping
+    else
+        cudaFree(d.data);
     cudaFree(d.rec);
     cudaFree(d.deg32);
     cudaFree(d.umax);
@@ -364,10 +367,29 @@ efg_status device_upload(efg_graph *g, const efg_build_opts &o)
     if (d.data_bytes >= (1ull << kOffBits))
         return set_error(EFG_ENOTSUP, "efg_build: EF data of 1 TiB or more is not supported on the device");
     const uint64_t padded = ((d.data_bytes + 64) + 15) & ~15ull;
-    EFG_TRY(dev_alloc(d, &d.data, padded));
-    CUDA_TRY(cudaMemsetAsync(d.data, 0, padded, s));
-    if (d.data_bytes) CUDA_TRY(cudaMemcpyAsync(d.data, ddata.data(), d.data_bytes, cudaMemcpyHostToDevice, s));
-    CUDA_TRY(cudaStreamSynchronize(s));  // ddata may be a temporary
+    // out-of-core: keep `data` in pinned, mapped host memory when
+    // asked to, or when it does not fit the device's free memory next to the
+    // per-vertex arrays and the traversal workspace (~ 64 B per vertex + 20 B
+    // per chunk descriptor, estimated)
+    bool host_resident = (o.flags & EFG_HOST_RESIDENT) != 0;
+    if (!host_resident) {
+        size_t fr = 0, tot = 0;
+        CUDA_TRY(cudaMemGetInfo(&fr, &tot));
+        const uint64_t rest = 64 * h.n + 20 * (h.n + h.m / d.k + 1) + (256ull << 20);
+        host_resident = padded + rest > fr;
+    }
+    if (host_resident) {
+        CUDA_TRY(cudaHostAlloc(reinterpret_cast<void **>(&d.data_host), padded,
+                               cudaHostAllocMapped | cudaHostAllocPortable));
+        std::memset(d.data_host + d.data_bytes, 0, padded - d.data_bytes);
+        if (d.data_bytes) std::memcpy(d.data_host, ddata.data(), d.data_bytes);
+        CUDA_TRY(cudaHostGetDevicePointer(reinterpret_cast<void **>(&d.data), d.data_host, 0));
+    } else {
+        EFG_TRY(dev_alloc(d, &d.data, padded));
+        CUDA_TRY(cudaMemsetAsync(d.data, 0, padded, s));
+        if (d.data_bytes) CUDA_TRY(cudaMemcpyAsync(d.data, ddata.data(), d.data_bytes, cudaMemcpyHostToDevice, s));
+        CUDA_TRY(cudaStreamSynchronize(s));  // ddata may be a temporary
+    }
 
     // bitmap geometry
     const uint64_t words = (h.n + 31) / 32;

@@ -175,7 +175,8 @@ struct DeviceGraph {
     void *stream = nullptr;            // cudaStream_t
     uint64_t n = 0, nwords = 0;        // nwords = ceil(n/32) rounded up
     uint32_t k = 512;
-    uint8_t *data = nullptr;           // EF data + padding
+    uint8_t *data = nullptr;           // EF data + padding (device address; mapped host memory when out-of-core)
+    uint8_t *data_host = nullptr;      // out-of-core (EFG_HOST_RESIDENT): the pinned host allocation behind `data`
     uint64_t data_bytes = 0;
     VRec *rec = nullptr;               // n records
     uint32_t *deg32 = nullptr;         // n degrees (padded to the bitmap size)

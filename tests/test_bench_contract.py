@@ -37,7 +37,7 @@ def test_cpu_baseline_child_pinned_and_checked():
     import synth
 
     class Args:
-        config, scale = 1, None
+        config, scale, permute = 1, None, False
 
     n, src, dst = synth.config_edges(1)
     ov, oe = oracle.csr_build(n, src, dst)

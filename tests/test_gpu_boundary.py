@@ -164,3 +164,32 @@ def test_collective_bfs_on_partitioned_handles(efg, world):
             assert np.array_equal(d.cpu().numpy(), oracle.bfs(ov, oe, 5))
         for g in graphs:
             g.free()
+
+
+@pytest.mark.parametrize("reorder", [False, True])
+def test_host_resident_out_of_core(efg, reorder):
+    """EFG_HOST_RESIDENT (out-of-core, P:34 / P:222): the EF data stays in
+    pinned host memory mapped into the device; every traversal reads it over
+    the host link and gives the oracle's results."""
+    n, src, dst = synth.rmat(15, 16, seed=31)
+    w = synth.weights(src, dst, 2031)
+    flags = efg.EFG_DEFAULT_FLAGS | efg.EFG_HOST_RESIDENT | (efg.EFG_REORDER_DEGREE if reorder else 0)
+    g = efg.Graph.build(n, src, dst, flags=flags, weights=w)
+    assert g.info["data_location"] == 1
+    ov, oe = oracle.csr_build(n, src, dst)
+    if not reorder:
+        assert np.array_equal(g.decode(0, n), oe)
+    deg = np.diff(ov)
+    for s in np.concatenate([[0], synth.sources(n, 3, 1031, deg > 0)]):
+        assert np.array_equal(g.bfs(int(s)), oracle.bfs(ov, oe, int(s)))
+    u = np.repeat(np.arange(n, dtype=np.uint32), deg.astype(np.int64))
+    w_csr = synth.weights(u, oe, seed=2031)
+    got = g.sssp(3)
+    assert np.array_equal(got.view(np.uint32), oracle.sssp(ov, oe, w_csr, 3).view(np.uint32))
+    pr = g.pagerank(0.85, 50)
+    ref = oracle.pagerank(ov, oe, 0.85, 50)
+    assert np.abs(pr - ref).sum() / np.abs(ref).sum() < 1e-6
+    g.free()
+    g = efg.Graph.build(n, src, dst)
+    assert g.info["data_location"] == 0
+    g.free()
