@@ -239,6 +239,12 @@ def build_graph(efg, args, *, permute=None, weighted=False, **kw):
     return g, gen_s
 
 
+def peak_rss_gb() -> float:
+    """Peak resident set of this process (ru_maxrss, KiB on Linux) in GB."""
+    import resource
+    return resource.getrusage(resource.RUSAGE_SELF).ru_maxrss * 1024 / 1e9
+
+
 def cpu_model() -> str:
     try:
         with open("/proc/cpuinfo") as f:
@@ -757,7 +763,8 @@ def main():
                        "l2_policy": "inputs larger than L2 (EF data %.2f GB > 126 MB)" % (info["data_bytes"] / 1e9),
                        "parallelism": f"{world} independent BFS replicas" if world > 1 else "1 GPU",
                        "data_location": "host (pinned, mapped: out-of-core)" if info["data_location"] else "HBM",
-                       "build_s": round(info["build_seconds"], 2), "gen_s": round(gen_s, 2)},
+                       "build_s": round(info["build_seconds"], 2), "gen_s": round(gen_s, 2),
+                       "host_peak_rss_gb": round(peak_rss_gb(), 2)},
             "clocks": clocks,
             "gpu_launches": launches,
             "roofline": {"bound": "hbm", "kernel": "expand_kernel (a4+a5+a6)",

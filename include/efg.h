@@ -284,8 +284,10 @@ efg_status efg_pagerank(efg_graph *g, double damping, uint32_t iters, double *ra
                                   * bit 0: batches of balanced chunks are decoded lane-per-chunk
                                   * (each lane walks its own chunk) instead of by word records
                                   * split evenly over the lanes; bit 1: a batch of adjacent chunks
-                                  * is staged by one bulk copy of its byte span.  Results are
-                                  * identical for every value. */
+                                  * is staged by one bulk copy of its byte span; bit 2: frontier-
+                                  * order study — BFS expands each level's chunks in
+                                  * a pseudo-random ("arbitrary") order instead of the bitmap's
+                                  * id order.  Results are identical for every value. */
 
 /* Set a per-handle option.  Errors: EFG_EINVAL (unknown option / value),
  * EFG_ESTATE (host-only handle). */

@@ -204,6 +204,21 @@ efg_status launch_level_end(DeviceGraph &d, cudaGraphConditionalHandle cond, cud
     return EFG_OK;
 }
 
+// expand launch of one level (BFS modes); with the frontier-order study variant
+// the level's descriptors are first permuted into chunks_shuf
+cudaError_t launch_level_expand(DeviceGraph &d, int mode, cudaStream_t s)
+{
+    ExpandArgs a = expand_args(d, nullptr);
+    if ((d.expand_variant & 4) && d.chunks_shuf) {
+        const cudaError_t e = launch_shuffle_chunks(d.chunks, mode == kModeVisit ? nullptr : d.cvtx, d.chunks_shuf,
+                                                    d.cvtx_shuf, d.ctrl, d.num_sms * 8, s);
+        if (e != cudaSuccess) return e;
+        a.chunks = d.chunks_shuf;
+        a.cvtx = d.cvtx_shuf;
+    }
+    return launch_expand(mode, a, d.num_sms * expand_occupancy(mode), s);
+}
+
 PeerArgs peer_args(DeviceGraph &d, int op)
 {
     PeerArgs a;
@@ -255,8 +270,7 @@ efg_status build_loop_graph(DeviceGraph &d, int mode)
     cudaStream_t cs;
     CUDA_TRY(cudaStreamCreateWithFlags(&cs, cudaStreamNonBlocking));
     CUDA_TRY(cudaStreamBeginCaptureToGraph(cs, body, nullptr, nullptr, 0, cudaStreamCaptureModeRelaxed));
-    const int blocks = d.num_sms * expand_occupancy(emode);
-    cudaError_t e1 = launch_expand(emode, expand_args(d, nullptr), blocks, cs);
+    cudaError_t e1 = launch_level_expand(d, emode, cs);
     efg_status st = e1 == cudaSuccess ? EFG_OK : EFG_ECUDA;
     if (st == EFG_OK && part) st = launch_peer_exchange(d, cs);
     if (st == EFG_OK) st = launch_level_end(d, cond, cs, false, part);
@@ -312,6 +326,8 @@ void device_free(DeviceGraph &d)
     cudaFree(d.tiles);
     cudaFree(d.chunks);
     cudaFree(d.cvtx);
+    cudaFree(d.chunks_shuf);
+    cudaFree(d.cvtx_shuf);
     cudaFree(d.depth);
     cudaFree(d.parent);
     cudaFree(d.parent2);
@@ -566,6 +582,10 @@ efg_status device_bfs(efg_graph *g, uint32_t source, int32_t *depth, uint32_t *p
                                      "efg_bfs_begin / efg_bfs_expand / efg_xchg_* / efg_bfs_finish_level)");
     if (part && parent)
         return set_error(EFG_ENOTSUP, "efg_bfs: parents are not available on a partitioned handle");
+    if ((d.expand_variant & 4) && !d.chunks_shuf) {  // frontier-order study buffers
+        EFG_TRY(dev_alloc(d, &d.chunks_shuf, d.max_chunks));
+        EFG_TRY(dev_alloc(d, &d.cvtx_shuf, d.max_chunks));
+    }
     const int emode = parent ? kModeVisitParent : kModeVisit;  // expand mode
     const int mode = part ? kLoopPartitioned : emode;            // loop graph
     const bool graph_mode = d.level_loop == 0;
@@ -628,7 +648,6 @@ efg_status device_bfs(efg_graph *g, uint32_t source, int32_t *depth, uint32_t *p
         }
         launches += (part ? 5 : 2) * levels + (relabel ? 1 : 0);
     } else {
-        const int blocks = d.num_sms * expand_occupancy(emode);
         for (;;) {
             CUDA_TRY(cudaMemcpyAsync(d.ctrl_host, d.ctrl, sizeof(LevelCtrl), cudaMemcpyDeviceToHost, s));
             CUDA_TRY(cudaStreamSynchronize(s));
@@ -652,7 +671,7 @@ efg_status device_bfs(efg_graph *g, uint32_t source, int32_t *depth, uint32_t *p
             CUDA_TRY(cudaEventCreate(&ec));
             lev.push_back(ec);
             CUDA_TRY(cudaEventRecord(a, s));
-            CUDA_TRY(launch_expand(emode, expand_args(d, nullptr), blocks, s));
+            CUDA_TRY(launch_level_expand(d, emode, s));
             CUDA_TRY(cudaEventRecord(b, s));
             if (part) EFG_TRY(launch_peer_exchange(d, s));
             EFG_TRY(launch_level_end(d, 0, s));

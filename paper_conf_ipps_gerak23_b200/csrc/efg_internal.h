@@ -196,6 +196,8 @@ struct DeviceGraph {
     ChunkDesc *chunks = nullptr;       // chunk descriptors of the level (max_chunks)
     uint32_t *cvtx = nullptr;          // source vertex of each chunk (max_chunks)
     uint64_t max_chunks = 0;
+    ChunkDesc *chunks_shuf = nullptr;  // frontier-order study (EFG_OPT_EXPAND_VARIANT bit 2): permuted
+    uint32_t *cvtx_shuf = nullptr;     // copies of chunks / cvtx, lazily allocated
     int32_t *depth = nullptr;          // internal depth (n)
     uint32_t *parent = nullptr;        // internal parent (n), lazily allocated
     uint32_t *parent2 = nullptr;       // parent in input ids (reordered graphs), lazily

@@ -1662,7 +1662,27 @@ __global__ void map_parent_kernel(const uint32_t *pin, const uint32_t *old_of_ne
     }
 }
 
+// frontier-order study: the level's chunks in a pseudo-random order (an
+// "arbitrary order" frontier), same tiles (index ranges)
+__global__ void shuffle_chunks_kernel(const ChunkDesc *in, const uint32_t *cvin, ChunkDesc *out, uint32_t *cvout,
+                                      const LevelCtrl *ctrl)
+{
+    const uint64_t N = ctrl->nchunks;
+    for (uint64_t c = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; c < N; c += (uint64_t)gridDim.x * blockDim.x) {
+        const uint64_t d = (c * 2654435761ull + 12345ull) % N;
+        out[d] = in[c];
+        if (cvin) cvout[d] = cvin[c];
+    }
+}
+
 }  // namespace
+
+cudaError_t launch_shuffle_chunks(const ChunkDesc *in, const uint32_t *cvin, ChunkDesc *out, uint32_t *cvout,
+                                  const LevelCtrl *ctrl, int blocks, cudaStream_t s)
+{
+    shuffle_chunks_kernel<<<blocks, 256, 0, s>>>(in, cvin, out, cvout, ctrl);
+    return cudaGetLastError();
+}
 
 static unsigned grid_for(uint64_t n) { return (unsigned)std::max<uint64_t>(1, std::min<uint64_t>((n + 255) / 256, 148 * 16)); }
 

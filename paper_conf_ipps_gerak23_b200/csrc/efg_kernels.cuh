@@ -135,6 +135,11 @@ cudaError_t launch_map_depth(const int32_t *stored, const uint32_t *new_of_old, 
                              cudaStream_t s);
 cudaError_t launch_pack8(const int32_t *in, int8_t *out, uint64_t n, cudaStream_t s);  // n % 4 handled
 cudaError_t launch_pack4(const int32_t *in, uint32_t *out, uint64_t n, cudaStream_t s);  // n % 8 handled
+// frontier-order study: out[pi(c)] = in[c] for the
+// level's chunk descriptors, pi(c) = (c * 2654435761 + 12345) mod nchunks (a
+// bijection: the multiplier is prime and larger than any chunk count it meets)
+cudaError_t launch_shuffle_chunks(const ChunkDesc *in, const uint32_t *cvin, ChunkDesc *out, uint32_t *cvout,
+                                  const LevelCtrl *ctrl, int blocks, cudaStream_t s);
 cudaError_t launch_map_parent(const uint32_t *pin, const uint32_t *old_of_new, uint32_t *pout, uint64_t n,
                               cudaStream_t s);
 

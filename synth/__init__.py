@@ -55,7 +55,7 @@ def lib():
         L.synth_chunglu.argtypes = [C.c_uint64, C.c_uint64, C.c_double, C.c_double, C.c_double,
                                     C.c_uint64, u32p, u32p]
         L.synth_web_hosts.restype = C.c_uint64
-        L.synth_web_hosts.argtypes = [C.c_uint64, C.c_double, C.c_uint64, C.c_uint64, u64p,
+        L.synth_web_hosts.argtypes = [C.c_uint64, C.c_double, C.c_double, C.c_uint64, C.c_uint64, u64p,
                                       C.c_uint64]
         L.synth_gen_range.restype = None
         L.synth_gen_range.argtypes = [C.c_void_p, C.c_uint64, C.c_uint64, u32p, u32p, f32p]
@@ -106,11 +106,14 @@ def chunglu(n: int, m: int, alpha_src: float, alpha_dst: float, rho: float, seed
     return n, src, dst
 
 
+WEB_HOST_XM = 100.0 / 3.0  # Pareto(1.5) host sizes with mean ~100 pages
+
+
 def web(n: int, m: int, seed: int, pareto_alpha=1.5, host_cap=20000, p_intra=0.85,
-        p_near=0.10, zipf_alpha=1.4):
+        p_near=0.10, zipf_alpha=1.4, host_xm=WEB_HOST_XM):
     max_hosts = n
     hs = np.zeros(max_hosts + 1, np.uint64)
-    nh = lib().synth_web_hosts(n, pareto_alpha, host_cap, seed, _ptr(hs, u64p), max_hosts)
+    nh = lib().synth_web_hosts(n, pareto_alpha, host_xm, host_cap, seed, _ptr(hs, u64p), max_hosts)
     hs = np.ascontiguousarray(hs[:nh + 1])
     host_of = np.empty(n, np.uint32)
     lib().synth_web_host_of(nh, _ptr(hs, u64p), _ptr(host_of, u32p))
@@ -157,7 +160,7 @@ CONFIGS = {
     2: dict(name="rmat24_ef16", kind="rmat", scale=24, ef=16, permute=False),
     3: dict(name="twitter_like", kind="chunglu", n=41_652_230, m=1_468_365_182,
             alpha_src=0.85, alpha_dst=0.8, rho=0.18, permute=False),
-    4: dict(name="web_like", kind="web", n=100_000_000, m=6_300_000_000, permute=False),
+    4: dict(name="web_like", kind="web", n=100_000_000, m=5_200_000_000, permute=False),
     5: dict(name="rmat29_ef32", kind="rmat", scale=29, ef=32, permute=True),
 }
 
@@ -234,7 +237,7 @@ def config_stream(c: int, scale_override: int | None = None, permute: bool | Non
     elif cfg["kind"] == "web":
         n, m = cfg["n"], cfg["m"]
         hs = np.zeros(n + 1, np.uint64)
-        nh = lib().synth_web_hosts(n, 1.5, 20000, c, _ptr(hs, u64p), n)
+        nh = lib().synth_web_hosts(n, 1.5, WEB_HOST_XM, 20000, c, _ptr(hs, u64p), n)
         hs = np.ascontiguousarray(hs[:nh + 1])
         host_of = np.empty(n, np.uint32)
         lib().synth_web_host_of(nh, _ptr(hs, u64p), _ptr(host_of, u32p))

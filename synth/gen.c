@@ -152,14 +152,15 @@ void synth_chunglu(uint64_t n, uint64_t m, double alpha_src, double alpha_dst, d
  * first page of a Zipf-popular host.  host_start[] (n_hosts+1) is provided by
  * the caller from synth_web_hosts.  Ids are locality-ordered; callers permute
  * for the "random ordering" variant. */
-uint64_t synth_web_hosts(uint64_t n, double pareto_alpha, uint64_t cap, uint64_t seed,
+uint64_t synth_web_hosts(uint64_t n, double pareto_alpha, double xm, uint64_t cap, uint64_t seed,
                          uint64_t *host_start, uint64_t max_hosts)
 {
     uint64_t h = 0, pos = 0;
     while (pos < n && h < max_hosts) {
         double r = unif(draw(seed, h, 11));
-        /* Pareto(xm=1, alpha) size */
-        double s = pow(1.0 - r, -1.0 / pareto_alpha);
+        /* Pareto(xm, alpha) size: mean xm * alpha / (alpha - 1) (~100 pages for
+         * xm = 33.3, alpha = 1.5: SURVEY §8(d) C4) */
+        double s = xm * pow(1.0 - r, -1.0 / pareto_alpha);
         uint64_t sz = (uint64_t)s;
         if (sz < 1) sz = 1;
         if (sz > cap) sz = cap;

@@ -100,5 +100,7 @@ line = {"config": synth.CONFIGS[a.config]["name"], "order": a.order, "n": int(n)
                  + ("; SSSP fp32 distances bit-exact vs oracle fp32 Dijkstra" if a.sssp else ""),
         "efg_build_s": round(t_build, 1), "gen_s": round(t_gen, 1), "oracle_csr_s": round(t_csr, 1),
         "sources": res, "sssp": sres or None,
+        "host_peak_rss_gb": round(__import__("resource").getrusage(__import__("resource").RUSAGE_SELF).ru_maxrss
+                                  * 1024 / 1e9, 1),
         "all_exact": all(r["bit_exact"] for r in res + sres) and m_dir == int(ov[-1])}
 print(json.dumps(line))
