@@ -30,11 +30,12 @@ ap.add_argument("--levels", action="store_true")
 a = ap.parse_args()
 masks = [int(x) for x in a.masks.split(",")]
 
-n, src, dst = synth.config_edges(a.config, scale_override=a.scale)
+sg = synth.config_stream(a.config, scale_override=a.scale)
+n = sg.n
 flags = efg.EFG_DEFAULT_FLAGS | (efg.EFG_REORDER_DEGREE if a.reorder == "degree" else 0)
 stream = torch.cuda.Stream()
-g = efg.Graph.build(n, src, dst, stream=stream.cuda_stream, flags=flags, n_threads=os.cpu_count() or 1)
-del src, dst
+g = efg.Graph.build_stream(n, sg.m, sg.fn, sg.user, stream=stream.cuda_stream, flags=flags,
+                           n_threads=os.cpu_count() or 1)
 vl = g.export()[0]
 perm = g.perm()
 deg = np.empty(n, np.int64)
