@@ -350,9 +350,11 @@ efg_status efg_bfs_end(efg_graph *g, efg_stats *st);
  *                    access), or regions = world device addresses (same
  *                    process); exactly one of the two is non-NULL.  bounds as in
  *                    efg_xchg_geometry (bounds[0] = 0, bounds[world] = n).
- *   efg_xchg_peer    enqueues the exchange on the handle's stream (three
- *                    kernels; two cross-rank barriers over flags in the regions)
- *                    and returns.  Every rank must call it once per level.
+ *   efg_xchg_peer    enqueues the exchange on the handle's stream (five
+ *                    kernels: publish, barrier, owner OR + broadcast, barrier,
+ *                    unpack; the cross-rank barriers over flags in the regions
+ *                    spin in one block each) and returns.  Every rank must call
+ *                    it once per level.
  * Ranks that share one device must use distinct non-blocking streams (the
  * barrier kernels of one rank wait for the others' kernels).  A barrier that
  * waits more than 4 s gives up; the next efg_bfs_finish_level then returns

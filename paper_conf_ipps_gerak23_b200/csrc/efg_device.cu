@@ -239,7 +239,7 @@ PeerArgs peer_args(DeviceGraph &d, int op)
 // the three peer-exchange launches of one level (publish, owner OR + broadcast, unpack)
 efg_status launch_peer_exchange(DeviceGraph &d, cudaStream_t s)
 {
-    for (int op = 0; op < 3; ++op) CUDA_TRY(launch_peer(peer_args(d, op), d.num_sms, s));
+    for (int op : {0, 3, 1, 4, 2}) CUDA_TRY(launch_peer(peer_args(d, op), d.num_sms, s));
     return EFG_OK;
 }
 
@@ -646,7 +646,7 @@ efg_status device_bfs(efg_graph *g, uint32_t source, int32_t *depth, uint32_t *p
             const LevelStat &x = d.stats_host[i];
             lms.push_back(x.t1 > x.t0 ? (float)((double)(x.t1 - x.t0) * 1e-6) : 0.f);
         }
-        launches += (part ? 5 : 2) * levels + (relabel ? 1 : 0);
+        launches += (part ? 7 : 2) * levels + (relabel ? 1 : 0);
     } else {
         for (;;) {
             CUDA_TRY(cudaMemcpyAsync(d.ctrl_host, d.ctrl, sizeof(LevelCtrl), cudaMemcpyDeviceToHost, s));
@@ -676,7 +676,7 @@ efg_status device_bfs(efg_graph *g, uint32_t source, int32_t *depth, uint32_t *p
             if (part) EFG_TRY(launch_peer_exchange(d, s));
             EFG_TRY(launch_level_end(d, 0, s));
             CUDA_TRY(cudaEventRecord(ec, s));
-            launches += part ? 5 : 2;
+            launches += part ? 7 : 2;
             if (d.trace) {  // debug: phase end times of frontier_kernel, max over blocks (us after the first start)
                 const unsigned nb = (unsigned)((d.nwords + d.words_per_block - 1) / d.words_per_block);
                 std::vector<unsigned long long> t(8 * nb);
@@ -977,7 +977,7 @@ efg_status device_xchg_peer(efg_graph *g)
     if (!d.peer_ptrs) return set_error(EFG_ESTATE, "efg_xchg_peer: call efg_peer_open first");
     CUDA_TRY(cudaSetDevice(d.device));
     EFG_TRY(launch_peer_exchange(d, stream_of(d)));
-    d.step_launches += 3;
+    d.step_launches += 5;
     return EFG_OK;
 }
 

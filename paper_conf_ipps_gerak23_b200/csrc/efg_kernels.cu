@@ -226,11 +226,14 @@ __global__ void xchg_kernel(XchgArgs a)
 // to owners + all-gather as pack / all-to-all / reduce / all-gather / unpack,
 // with no collective library and no intermediate slices: owners read every
 // rank's published new bits straight from its HBM over NVLink and store the
-// OR into every rank's result buffer.  Three launches per level, in stream
-// order on each rank:
+// OR into every rank's result buffer.  Five launches per level, in stream
+// order on each rank (the barriers are one-block kernels, the data ops never
+// spin):
 //   op 0  publish:  pub[w] = vis[w] & ~prev[w]                 (local)
-//   op 1  barrier e; for owned words w: m = OR_p pub_p[w]; res_p[w] = m for all p
-//   op 2  barrier e+1; vis[w] |= res[w]                       (local)
+//   op 3  barrier e
+//   op 1  for owned words w: m = OR_p pub_p[w]; res_p[w] = m for all p
+//   op 4  barrier e+1
+//   op 2  vis[w] |= res[w]                                     (local)
 // Barrier e: block 0 stores e into flags[rank] of every rank (release, system
 // scope), every block waits until all of its own flags reach e (acquire).
 // Reuse is safe without more barriers: a rank republishes (op 0 of the next
@@ -276,15 +279,18 @@ __global__ void peer_kernel(PeerArgs a)
     const uint64_t t0 = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
     if (a.op == 0) {
         for (uint64_t w = t0; w < a.nwords; w += stride) a.local[pub + w] = a.vis[w] & ~a.prev[w];
-        // barrier epochs of this exchange: E - 1 (op 1) and E (op 2), E = the
-        // counter after this increment (a device counter, so a captured level
-        // loop advances it every iteration; every rank runs the same number of
-        // exchanges, so the counters agree)
+        // barrier epochs of this exchange: E - 1 (before op 1) and E (before
+        // op 2), E = the counter after this increment (a device counter, so a
+        // captured level loop advances it every iteration; every rank runs the
+        // same number of exchanges, so the counters agree)
         if (blockIdx.x == 0 && threadIdx.x == 0) *a.epoch += 2;
         return;
     }
-    const uint32_t E = *a.epoch;
-    if (!peer_barrier(a, a.op == 1 ? E - 1 : E)) return;
+    if (a.op == 3 || a.op == 4) {  // the barrier alone, one block (op 3: epoch E - 1, op 4: E)
+        const uint32_t E = *a.epoch;
+        peer_barrier(a, a.op == 3 ? E - 1 : E);
+        return;
+    }
     if (a.op == 1) {
         const uint64_t w0 = a.bounds[a.rank] / 32, w1 = (a.bounds[a.rank + 1] + 31) / 32;
         for (uint64_t w = w0 + t0; w < w1; w += stride) {
@@ -1872,10 +1878,13 @@ cudaError_t launch_xchg(const XchgArgs &a, cudaStream_t s)
 
 cudaError_t launch_peer(const PeerArgs &a, int max_blocks, cudaStream_t s)
 {
-    // a small grid: the spinning blocks of one rank must leave room for the
-    // other ranks' kernels when several ranks share a device (tests)
-    const unsigned blocks = (unsigned)std::max<uint64_t>(1, std::min<uint64_t>((a.nwords + 255) / 256,
-                                                                               (uint64_t)max_blocks));
+    // the barrier ops spin in ONE block (a rank waiting for the others holds
+    // one block's worth of an SM, which matters when ranks share a device);
+    // the data ops never wait
+    const unsigned blocks = (a.op == 3 || a.op == 4)
+                                ? 1u
+                                : (unsigned)std::max<uint64_t>(1, std::min<uint64_t>((a.nwords + 255) / 256,
+                                                                                     (uint64_t)max_blocks));
     peer_kernel<<<blocks, 256, 0, s>>>(a);
     return cudaGetLastError();
 }

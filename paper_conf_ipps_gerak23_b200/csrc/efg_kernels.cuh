@@ -79,7 +79,7 @@ struct PeerArgs {
     uint32_t *epoch;               // device exchange counter (LevelCtrl.peer_epoch): op 0 adds 2,
                                    // ops 1 and 2 wait on barrier epochs counter-1 and counter
     int world, rank;
-    int op;                        // 0 publish, 1 owner OR + broadcast, 2 unpack
+    int op;                        // 0 publish, 1 owner OR + broadcast, 2 unpack, 3 / 4 barrier (one block)
 };
 
 struct FrontierArgs {           // level end (a7) + next level plan (a1-a4), one launch
