@@ -52,8 +52,10 @@ static void rmat_range(int scale, uint64_t first, uint64_t m, double a, double b
     for (int64_t i = 0; i < (int64_t)m; ++i) {
         const uint64_t e = first + (uint64_t)i;
         uint32_t u = 0, v = 0;
+        /* draw(seed, e, lvl) with the per-sample part hoisted (same values) */
+        const uint64_t h = sm64(seed * 0xD1B54A32D192ED03ull + e);
         for (int lvl = 0; lvl < scale; ++lvl) {
-            double r = unif(draw(seed, (uint64_t)e, (uint64_t)lvl));
+            double r = unif(sm64(h ^ ((uint64_t)lvl * 0x9E3779B97F4A7C15ull + 0x632BE59BD9B4E019ull)));
             uint32_t ub, vb;
             if (r < a)        { ub = 0; vb = 0; }
             else if (r < ab)  { ub = 0; vb = 1; }
