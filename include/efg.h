@@ -280,14 +280,17 @@ efg_status efg_pagerank(efg_graph *g, double damping, uint32_t iters, double *ra
                                  * directed or row-range handle): push along every edge with
                                  * fp64 atomicAdd.  Same sums, other order (C21). */
 
-#define EFG_OPT_EXPAND_VARIANT 4 /* tuning / A-B switch of the expand kernel, bit mask (default 3):
+#define EFG_OPT_EXPAND_VARIANT 4 /* tuning / A-B switch of the expand kernel, bit mask (default 11):
                                   * bit 0: batches of balanced chunks are decoded lane-per-chunk
                                   * (each lane walks its own chunk) instead of by word records
                                   * split evenly over the lanes; bit 1: a batch of adjacent chunks
                                   * is staged by one bulk copy of its byte span; bit 2: frontier-
                                   * order study — BFS expands each level's chunks in
                                   * a pseudo-random ("arbitrary") order instead of the bitmap's
-                                  * id order.  Results are identical for every value. */
+                                  * id order; bit 3: a lane-per-chunk lane steps over the stop
+                                  * bits below the visited prefix inside its first kept word
+                                  * (select0) instead of decoding them.  Results are identical
+                                  * for every value. */
 
 /* Set a per-handle option.  Errors: EFG_EINVAL (unknown option / value),
  * EFG_ESTATE (host-only handle). */

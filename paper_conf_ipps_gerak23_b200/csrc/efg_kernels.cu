@@ -969,6 +969,10 @@ constexpr bool kSpanStage = EFG_SPAN_STAGE;  // one bulk copy per batch when the
 #define EFG_FAST_SINGLE 1
 #endif
 constexpr bool kFastSingle = EFG_FAST_SINGLE;  // producer fast path for batches of whole short lists
+#ifndef EFG_LPC_BITSKIP
+#define EFG_LPC_BITSKIP 1
+#endif
+constexpr bool kLpcBitSkip = EFG_LPC_BITSKIP;  // lane-per-chunk: skip the below-vpre stop bits of the first kept word
 
 template <int MODE>
 __global__ void __launch_bounds__(kExpandThreads, 1) expand_kernel(ExpandArgs a)
@@ -1403,6 +1407,19 @@ __global__ void __launch_bounds__(kExpandThreads, 1) expand_kernel(ExpandArgs a)
                         ++gl;
                         hcur += 32;
                         w = word(gl);
+                    }
+                    // inside the first kept word: the stop bit of element j + k at
+                    // position p has high part hcur + p - (j + k) = hcur - j + (zeros
+                    // of w below p), so the elements below h0 are the set bits
+                    // below zero number D - 1 of w, D = h0 + j - hcur (select0)
+                    const int32_t D = (int32_t)(h0 + j - hcur);
+                    if (kLpcBitSkip && (a.variant & 8) && D > 0 && D <= 32 - __popc(w)) {
+                        const uint32_t zpos = select_in_word(~w, (uint32_t)D - 1);
+                        const uint32_t below = w & ((1u << zpos) - 1);  // zpos < 32: w has a zero there
+                        const uint32_t cnt = __popc(below);
+                        w ^= below;
+                        j += cnt;
+                        la += cnt * l;
                     }
                 }
                 uint32_t uw = __brev(w);  // reversed: the next stop bit is the leading one
