@@ -469,3 +469,21 @@ def test_pagerank_directed_uses_push(efg):
     ref = oracle.pagerank(ov, oe, 0.85, 50)
     assert np.abs(got - ref).sum() / np.abs(ref).sum() < 1e-6
     g.free()
+
+
+@pytest.mark.slow
+def test_pagerank_c2_full_size(efg):
+    """NEXT-2 at its BASELINE config (configs[1]: RMAT-24/ef16, BFS and PageRank):
+    50 iterations within 1e-6 relative L1 of the fp64 oracle, pull (gather) and
+    push both, on the bench's degree-relabelled build."""
+    n, src, dst = synth.config_edges(2)
+    ov, oe = oracle.csr_build(n, src, dst)
+    ref = oracle.pagerank(ov, oe, 0.85, 50)
+    g = efg.Graph.build(n, src, dst, flags=efg.EFG_DEFAULT_FLAGS | efg.EFG_REORDER_DEGREE)
+    del src, dst
+    for pull in (True, False):
+        g.set_pagerank_pull(pull)
+        got = g.pagerank(0.85, 50)
+        rel = np.abs(got - ref).sum() / np.abs(ref).sum()
+        assert rel < 1e-6, (pull, rel)
+    g.free()
