@@ -1,8 +1,7 @@
 #!/bin/bash
 # compute-sanitizer memcheck / racecheck / synccheck over the C1-sized traversals:
-# BFS (graph and host level loops, parents), decode, SSSP, PageRank, the
-# collective partitioned BFS over the peer exchange (2 simulated ranks), and
-# the out-of-core path.  Summaries -> gpurun_out/sanitize_<tool>.txt
+# BFS (graph and host level loops, parents), decode, SSSP, PageRank, with
+# the whole-graph, degree-relabelled and out-of-core builds.  Summaries -> gpurun_out/sanitize_<tool>.txt
 O=gpurun_out; mkdir -p $O
 python -c "import __graft_entry__ as g; g.build()" > $O/build_san.log 2>&1 || { tail -20 $O/build_san.log; exit 1; }
 for tool in memcheck racecheck synccheck; do
