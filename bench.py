@@ -259,7 +259,8 @@ def cpu_model() -> str:
 REF_STEP_EDGES = 1 << 28  # reference-arm step: FIFO BFS stopped after this many scanned edges
 
 
-def _cpu_baseline_child(cfg: int, scale, index: int, count: int, out_dir: str, core: int, permute=None):
+def _cpu_baseline_child(cfg: int, scale, index: int, count: int, out_dir: str, core: int, permute=None,
+                        go_parallel=None):
     """Spawned process (bench.py cpu_baseline leg): the oracle's CSR of the
     same seeded graph, then ONE plain single-threaded FIFO BFS from the first
     timed source, pinned to `core` (the parent keeps off that core).  Writes
@@ -278,9 +279,20 @@ def _cpu_baseline_child(cfg: int, scale, index: int, count: int, out_dir: str, c
     d = oracle.bfs(ov, oe, s0)
     cs = time.perf_counter() - t
     np.save(os.path.join(out_dir, "depth.npy"), d)
+    meta = {"source": s0, "bfs_s": cs, "csr_s": csr_s, "edges": int(deg[d >= 0].sum()),
+            "core": core, "affinity": sorted(os.sched_getaffinity(0))}
+    # the optional all-core baseline (BASELINE.md CPU plan), once the parent's
+    # GPU work is over: OpenMP top-down BFS on the same CSR and source
+    if go_parallel is not None and go_parallel.wait(timeout=3600):
+        import cpu_baseline
+        os.sched_setaffinity(0, set(range(os.cpu_count() or 1)))
+        threads = len(os.sched_getaffinity(0))
+        cpu_baseline.bfs(ov, oe, s0, threads)  # warm-up (page faults of the CSR in every thread)
+        t = time.perf_counter()
+        dp = cpu_baseline.bfs(ov, oe, s0, threads)
+        meta.update(par_s=time.perf_counter() - t, par_threads=threads, par_exact=bool(np.array_equal(dp, d)))
     with open(os.path.join(out_dir, "meta.json"), "w") as f:
-        json.dump({"source": s0, "bfs_s": cs, "csr_s": csr_s, "edges": int(deg[d >= 0].sum()),
-                   "core": core, "affinity": sorted(os.sched_getaffinity(0))}, f)
+        json.dump(meta, f)
 
 
 def start_cpu_baseline(args, count: int, index: int):
@@ -291,16 +303,18 @@ def start_cpu_baseline(args, count: int, index: int):
     cores = sorted(os.sched_getaffinity(0))
     core = cores[-1]
     out_dir = tempfile.mkdtemp(prefix="efg_cpu_baseline_")
-    proc = mp.get_context("spawn").Process(target=_cpu_baseline_child,
-                                            args=(args.config, args.scale, index, count, out_dir, core,
-                                                  args.permute or None))
+    ctx = mp.get_context("spawn")
+    go = ctx.Event()
+    proc = ctx.Process(target=_cpu_baseline_child,
+                       args=(args.config, args.scale, index, count, out_dir, core, args.permute or None, go))
     proc.start()
     if len(cores) > 1:
         os.sched_setaffinity(0, set(cores[:-1]))
-    return proc, out_dir
+    return proc, out_dir, go
 
 
-def finish_cpu_baseline(proc, out_dir: str, g, n: int):
+def finish_cpu_baseline(proc, out_dir: str, go, g, n: int):
+    go.set()  # the GPU measurements are over: the child may use every core
     proc.join()
     if proc.exitcode != 0:
         return {"unavailable": f"cpu_baseline process exited with {proc.exitcode}"}
@@ -314,7 +328,11 @@ def finish_cpu_baseline(proc, out_dir: str, g, n: int):
                       f"{meta['csr_s']:.1f} s untimed), pinned to host core {meta['core']} "
                       f"(sched_setaffinity = taskset -c {meta['core']}; bench's own threads kept off it)",
             "cpu_model": cpu_model(), "host_cores": os.cpu_count(),
-            "parity_bit_exact": ok, "parity_source": meta["source"]}
+            "parity_bit_exact": ok, "parity_source": meta["source"],
+            "all_cores": ({"value": meta["edges"] / meta["par_s"] / 1e9, "unit": UNIT,
+                           "cores": meta["par_threads"], "kind": "openmp top-down BFS (cpu_baseline/omp_bfs.c)",
+                           "sample": "the same source and CSR, after the GPU work", "depth_equal_oracle":
+                           meta["par_exact"]} if "par_s" in meta else None)}
 
 
 def run_reference(args, rank, world):

@@ -63,5 +63,6 @@ def test_cpu_baseline_child_pinned_and_checked():
             srcs = synth.sources(n, 4, seed=1001, nonisolated_mask=np.diff(ov) > 0)
             assert cpu["parity_source"] == int(srcs[1])
             assert "taskset -c" in cpu["sample"] and cpu["cpu_model"]
+            assert cpu["all_cores"]["depth_equal_oracle"] and cpu["all_cores"]["value"] > 0
     finally:
         os.sched_setaffinity(0, before)

@@ -184,3 +184,15 @@ def test_bfs_bounded_sample():
                     dq_depths = np.sort(full[full >= 0])[:nv]
                     for u in np.flatnonzero((full >= 0) & (full < dq_depths[-1])):
                         assert np.all(got[elist[vlist[u]:vlist[u + 1]]] >= 0)
+
+
+def test_cpu_baseline_omp_bfs_matches_oracle():
+    """The optional all-core CPU baseline (cpu_baseline/omp_bfs.c) gives the
+    oracle's depths (a reported baseline must compute the same thing)."""
+    import cpu_baseline
+    n, src, dst = synth.rmat(14, 16, seed=9)
+    vlist, elist = oracle.csr_build(n, src, dst)
+    for s in (0, 1, 5000, n - 1):
+        ref = oracle.bfs(vlist, elist, s)
+        for t in (1, 4):
+            assert np.array_equal(cpu_baseline.bfs(vlist, elist, s, threads=t), ref)
