@@ -98,7 +98,10 @@ def partitioned_bfs(g, source: int, depth, bounds: np.ndarray, transport, make_b
 def simulated_partitioned_bfs(graphs, source: int, depths, bounds: np.ndarray, make_buffer):
     """The same protocol with all `world` rank handles in one process (one GPU):
     the all-to-all and all-gather become buffer copies.  Used by the GPU tests to
-    run the partitioned kernels without several GPUs."""
+    run the partitioned kernels without several GPUs.  The handles may run on
+    their own streams: the copies (torch's current stream) are fenced with
+    device synchronisations on both sides."""
+    import torch
     world = bounds.size - 1
     S = graphs[0].xchg_geometry(bounds)
     send = [make_buffer(world * S) for _ in range(world)]
@@ -112,13 +115,17 @@ def simulated_partitioned_bfs(graphs, source: int, depths, bounds: np.ndarray, m
         for r, g in enumerate(graphs):
             g.bfs_expand()
             g.xchg_pack(bounds, S, send[r])
+        torch.cuda.synchronize()
         for r in range(world):          # all-to-all
             for p in range(world):
                 recv[r][p * S:(p + 1) * S].copy_(send[p][r * S:(r + 1) * S])
+        torch.cuda.synchronize()
         for r, g in enumerate(graphs):
             g.xchg_reduce(world, S, recv[r], mine[r])
+        torch.cuda.synchronize()
         for r in range(world):          # all-gather
             gathered[r * S:(r + 1) * S].copy_(mine[r])
+        torch.cuda.synchronize()
         news = []
         for g in graphs:
             g.xchg_unpack(bounds, S, gathered)
