@@ -203,7 +203,8 @@ typedef struct efg_stats {
     float expand_ms;           /* device time inside the expand+decode kernel        */
     uint32_t expand_launches;  /* number of expand+decode launches                   */
     uint32_t kernel_launches;  /* all kernels launched by the call                   */
-    uint64_t expand_bytes;     /* algorithmic bytes of the expand launches (DESIGN)  */
+    uint64_t expand_bytes;     /* reserved, 0 (bench.py derives the algorithmic     *
+                                *  bytes from efg_export sizes and the levels)      */
     uint64_t *level_frontier;  /* in/out: |F_L| per level (level_cap entries)        */
     uint64_t *level_edges;     /* in/out: E_L = sum of frontier degrees per level    */
     float *level_expand_ms;    /* in/out: expand kernel time per level, or NULL      */

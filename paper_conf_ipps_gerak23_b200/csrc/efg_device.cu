@@ -196,10 +196,11 @@ FrontierArgs frontier_args(DeviceGraph &d, cudaGraphConditionalHandle cond, bool
 
 // level end + next plan: one launch (every block resident, see frontier_kernel)
 efg_status launch_level_end(DeviceGraph &d, cudaGraphConditionalHandle cond, cudaStream_t s,
-                            bool consume = false, bool cond_global = false)
+                            bool consume = false, bool cond_global = false, bool need_cvtx = true)
 {
     FrontierArgs fa = frontier_args(d, cond, consume);
     fa.cond_global = cond_global ? 1 : 0;
+    if (!need_cvtx) fa.cvtx = nullptr;  // plain BFS: the expand never reads the chunk's vertex
     CUDA_TRY(launch_frontier(fa, (unsigned)((d.nwords + d.words_per_block - 1) / d.words_per_block), s));
     return EFG_OK;
 }
@@ -273,7 +274,7 @@ efg_status build_loop_graph(DeviceGraph &d, int mode)
     cudaError_t e1 = launch_level_expand(d, emode, cs);
     efg_status st = e1 == cudaSuccess ? EFG_OK : EFG_ECUDA;
     if (st == EFG_OK && part) st = launch_peer_exchange(d, cs);
-    if (st == EFG_OK) st = launch_level_end(d, cond, cs, false, part);
+    if (st == EFG_OK) st = launch_level_end(d, cond, cs, false, part, emode != kModeVisit);
     cudaGraph_t captured;
     cudaError_t e2 = cudaStreamEndCapture(cs, &captured);
     cudaStreamDestroy(cs);
@@ -674,7 +675,7 @@ efg_status device_bfs(efg_graph *g, uint32_t source, int32_t *depth, uint32_t *p
             CUDA_TRY(launch_level_expand(d, emode, s));
             CUDA_TRY(cudaEventRecord(b, s));
             if (part) EFG_TRY(launch_peer_exchange(d, s));
-            EFG_TRY(launch_level_end(d, 0, s));
+            EFG_TRY(launch_level_end(d, 0, s, false, false, emode != kModeVisit));
             CUDA_TRY(cudaEventRecord(ec, s));
             launches += part ? 7 : 2;
             if (d.trace) {  // debug: phase end times of frontier_kernel, max over blocks (us after the first start)
@@ -839,7 +840,7 @@ efg_status device_step_finish(efg_graph *g, uint64_t *global_new)
     DeviceGraph &d = g->dev;
     CUDA_TRY(cudaSetDevice(d.device));
     cudaStream_t s = stream_of(d);
-    EFG_TRY(launch_level_end(d, 0, s));
+    EFG_TRY(launch_level_end(d, 0, s, false, false, false));  // the stepwise expand is plain BFS
     ++d.step_launches;
     CUDA_TRY(cudaMemcpyAsync(d.ctrl_host, d.ctrl, sizeof(LevelCtrl), cudaMemcpyDeviceToHost, s));
     CUDA_TRY(cudaStreamSynchronize(s));

@@ -695,7 +695,7 @@ __global__ void __launch_bounds__(kFrontierThreads, 1024 / kFrontierThreads) fro
                 if (mine && !big) {
                     if (nch == 1) {  // a4: the list's only chunk (cc = 0)
                         *reinterpret_cast<uint4 *>(a.chunks + C) = make_uint4(rv[u].x, rv[u].y, d, ub);
-                        a.cvtx[C] = (uint32_t)((w0 + jw[u]) * 32 + lane);
+                        if (a.cvtx) a.cvtx[C] = (uint32_t)((w0 + jw[u]) * 32 + lane);
                     }
                     // a3: a tile boundary t*T inside [W, W + wlen) starts at this chunk or the next
                     const uint64_t t = (W + TW - 1) / TW;
@@ -762,7 +762,7 @@ __global__ void __launch_bounds__(kFrontierThreads, 1024 / kFrontierThreads) fro
             for (uint32_t j = 0; j < nch; ++j) {
                 const uint64_t oc = off_l | ((uint64_t)j << kCcShift);
                 *reinterpret_cast<uint4 *>(a.chunks + cs + j) = make_uint4((uint32_t)oc, (uint32_t)(oc >> 32), d, ub);
-                a.cvtx[cs + j] = v;
+                if (a.cvtx) a.cvtx[cs + j] = v;
             }
             for (uint64_t t = t_lo; t < t_hi; ++t)
                 a.tiles[t] = (uint32_t)(cs + tile_chunk((uint32_t)(t * TW - W), nch));
@@ -778,7 +778,7 @@ __global__ void __launch_bounds__(kFrontierThreads, 1024 / kFrontierThreads) fro
             for (uint32_t j = lane; j < onch; j += 32) {
                 const uint64_t oc = ooff | ((uint64_t)j << kCcShift);
                 *reinterpret_cast<uint4 *>(a.chunks + ocs + j) = make_uint4((uint32_t)oc, (uint32_t)(oc >> 32), od, oub);
-                a.cvtx[ocs + j] = ov;
+                if (a.cvtx) a.cvtx[ocs + j] = ov;
             }
             const uint64_t owl = (uint64_t)onch * CW + od;
             const uint64_t ot_lo = (oW + TW - 1) / TW, ot_hi = (oW + owl + TW - 1) / TW;

@@ -94,7 +94,7 @@ struct FrontierArgs {           // level end (a7) + next level plan (a1-a4), one
     uint32_t *skipw;           // scratch (nwords): per bitmap word, the skipped lists (phase 1 -> phase 2)
     const VRec *rec;           // vertex records (pass 2)
     ChunkDesc *chunks;         // out: chunk descriptors
-    uint32_t *cvtx;            // out: source vertex of each chunk
+    uint32_t *cvtx;            // out: source vertex of each chunk, or null (plain BFS never reads it)
     uint32_t *tiles;           // out: first chunk of each tile (+ sentinel)
     LevelCtrl *ctrl;           // in: level, seq, depth ptr; out: nf, ne, nwork, nchunks, ntiles, xlevel, vmin2
     uint64_t *status;          // five per-block aggregate regions of kMaxGrid words

@@ -100,6 +100,12 @@ def _check_roundtrip(x, k):
     # size = 4*floor(n/k) + ceil(n*l/8) + ceil(((u>>l)+n)/8)  (C4, C7, C8)
     upper_bits = (u >> l) + n
     assert len(enc) == (4 * (n // k) if k else 0) + (n * l + 7) // 8 + (upper_bits + 7) // 8
+    # north_star's a-priori size n*l + n + ceil(u / 2^l) bits: the upper
+    # section's (u >> l) + n bits never exceed it, and equal it when 2^l | u
+    # (reading C4: the last stop bit is the last bit, no trailing zero bucket)
+    apriori = n * l + n + -(-u // (1 << l))
+    assert n * l + upper_bits <= apriori <= n * l + upper_bits + 1
+    assert (n * l + upper_bits == apriori) == (u % (1 << l) == 0)
     # at most n(2 + ceil(log u/n)) bits in total (u >= n case)
     if u >= n and u > 0:
         assert n * l + upper_bits <= n * (2 + math.ceil(math.log2(u / n))) + 1e-9
