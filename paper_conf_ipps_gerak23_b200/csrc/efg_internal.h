@@ -162,6 +162,10 @@ constexpr int kBitmapAlign = 1024;           // bitmap words are padded to a mul
 #endif
 constexpr uint32_t kTileWork = EFG_TILE_WORK;         // work units per tile (a3)
 constexpr uint32_t kChunkWork = 32;          // per-chunk overhead in work units
+#ifndef EFG_FRONTIER_SPARSE
+#define EFG_FRONTIER_SPARSE 1
+#endif
+constexpr bool kFrontierSparse = EFG_FRONTIER_SPARSE;  // frontier_kernel phase 2: compacted slots for sparse groups
 #ifndef EFG_TILE_BIG_MIN_WORK
 #define EFG_TILE_BIG_MIN_WORK (1ull << 27)
 #endif

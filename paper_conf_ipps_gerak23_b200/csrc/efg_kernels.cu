@@ -88,6 +88,22 @@ __device__ __forceinline__ int warp_maxle_u32(uint32_t key, uint32_t g)
     return lo;
 }
 
+// position (0..31) of the set bit of rank kk (0-based, kk < popc(w)) of w:
+// five popcount halvings (the in-word part of select1, P:96)
+__device__ __forceinline__ uint32_t select_in_word(uint32_t w, uint32_t kk)
+{
+    uint32_t pos = 0;
+#pragma unroll
+    for (uint32_t sh = 16; sh; sh >>= 1) {
+        const uint32_t c = __popc(w & ((1u << sh) - 1));
+        const bool up = kk >= c;
+        kk -= up ? c : 0u;
+        w = up ? w >> sh : w;
+        pos += up ? sh : 0u;
+    }
+    return pos;
+}
+
 __device__ __forceinline__ uint32_t ldg_u32(const uint32_t *p) { return __ldg(p); }
 
 // uint32 little-endian at an arbitrary byte offset of the 4-byte aligned data
@@ -608,7 +624,7 @@ __global__ void __launch_bounds__(kFrontierThreads, 1024 / kFrontierThreads) fro
 #ifndef EFG_KS
 #define EFG_KS 3
 #endif
-    constexpr int kS = EFG_KS;                    // non-empty words planned together
+    constexpr int kS = EFG_KS;                    // slots (words, or 32-vertex groups) planned together
     for (uint64_t w0 = 32ull * gw; w0 < a.nwords; w0 += WG) {
         const uint64_t w = w0 + lane;
         uint32_t nb = 0, skw = 0;
@@ -629,26 +645,52 @@ __global__ void __launch_bounds__(kFrontierThreads, 1024 / kFrontierThreads) fro
         const bool own = w >= a.own_lo_w && w < a.own_hi_w;
         const uint32_t nq = own ? nb & ~skw : 0u;
         uint32_t todo = __ballot_sync(FULL, nb != 0);
-        while (todo) {
-            uint32_t jw[kS], bq[kS], wl[kS], nc[kS];
+        // a slot = up to 32 new vertices, one per lane, in id order: the bits of
+        // one non-empty word (dense groups: 32 consecutive records, coalesced),
+        // or, when the group's non-empty words are sparsely filled, the next 32
+        // new vertices of the whole group (compacted: a lane finds its word by
+        // maxle over the words' popcount prefix, then its bit by select)
+        uint32_t gtot;
+        const uint32_t gex = warp_excl_u32(__popc(nb), gtot);
+        const bool sparse = kFrontierSparse && 4 * gtot <= 32u * (uint32_t)__popc(todo);
+        uint32_t cursor = 0;
+        while (sparse ? cursor < gtot : todo != 0) {
+            uint32_t vv[kS], bq[kS], wl[kS], nc[kS];
+            bool pl[kS];
             uint4 rv[kS];
 #pragma unroll
             for (int u = 0; u < kS; ++u) {
-                jw[u] = 32;
-                bq[u] = 0;
+                bool isnew = false;
+                pl[u] = false;
+                vv[u] = 0;
                 rv[u] = make_uint4(0, 0, 0, 0);
-                if (todo) {
+                if (sparse) {
+                    const uint32_t t = cursor + lane;
+                    if (cursor < gtot) {
+                        const int j = warp_maxle_u32(gex, t < gtot ? t : 0u);
+                        const uint32_t bits = __shfl_sync(FULL, nb, j), qb = __shfl_sync(FULL, nq, j);
+                        const uint32_t r = t - __shfl_sync(FULL, gex, j);
+                        if (t < gtot) {
+                            const uint32_t bit = select_in_word(bits, r);
+                            vv[u] = (uint32_t)((w0 + j) * 32 + bit);
+                            isnew = true;
+                            pl[u] = (qb >> bit) & 1;
+                        }
+                        cursor += 32;
+                    }
+                } else if (todo) {
                     const int j = __ffs(todo) - 1;
                     todo &= todo - 1;
-                    jw[u] = j;
-                    bq[u] = __shfl_sync(FULL, nq, j);
-                    const uint32_t bb = __shfl_sync(FULL, nb, j);
-                    const uint32_t v = (uint32_t)((w0 + j) * 32 + lane);
-                    if ((bq[u] >> lane) & 1) rv[u] = __ldg(reinterpret_cast<const uint4 *>(a.rec + v));
-                    if ((bb >> lane) & 1) {
-                        if (a.depth_stored) a.depth_stored[v] = (int32_t)level;  // stored-id order (coalesced)
-                        if (!a.depth_stored_only && depth) depth[v] = (int32_t)level;
-                    }
+                    const uint32_t qb = __shfl_sync(FULL, nq, j), bb = __shfl_sync(FULL, nb, j);
+                    vv[u] = (uint32_t)((w0 + j) * 32 + lane);
+                    isnew = (bb >> lane) & 1;
+                    pl[u] = (qb >> lane) & 1;
+                }
+                bq[u] = __ballot_sync(FULL, pl[u]);
+                if (pl[u]) rv[u] = __ldg(reinterpret_cast<const uint4 *>(a.rec + vv[u]));
+                if (isnew) {
+                    if (a.depth_stored) a.depth_stored[vv[u]] = (int32_t)level;  // stored-id order
+                    if (!a.depth_stored_only && depth) depth[vv[u]] = (int32_t)level;
                 }
             }
             // per-list work nch*CW + d < 2^31.1 (deg < 2^26); the 32-lane sums fit
@@ -685,7 +727,7 @@ __global__ void __launch_bounds__(kFrontierThreads, 1024 / kFrontierThreads) fro
 #pragma unroll
             for (int u = 0; u < kS; ++u) {
                 if (!bq[u]) continue;  // warp-uniform
-                const bool mine = (bq[u] >> lane) & 1;
+                const bool mine = pl[u];
                 const uint32_t d = rv[u].z, ub = rv[u].w, nch = nc[u];
                 const uint64_t off_l = ((uint64_t)rv[u].y << 32) | rv[u].x;
                 const uint64_t W = run + (narrow ? (uint64_t)wl[u] : ((uint64_t)wl[u] << 5) + wlo[u]);
@@ -695,7 +737,7 @@ __global__ void __launch_bounds__(kFrontierThreads, 1024 / kFrontierThreads) fro
                 if (mine && !big) {
                     if (nch == 1) {  // a4: the list's only chunk (cc = 0)
                         *reinterpret_cast<uint4 *>(a.chunks + C) = make_uint4(rv[u].x, rv[u].y, d, ub);
-                        if (a.cvtx) a.cvtx[C] = (uint32_t)((w0 + jw[u]) * 32 + lane);
+                        if (a.cvtx) a.cvtx[C] = vv[u];
                     }
                     // a3: a tile boundary t*T inside [W, W + wlen) starts at this chunk or the next
                     const uint64_t t = (W + TW - 1) / TW;
@@ -712,7 +754,7 @@ __global__ void __launch_bounds__(kFrontierThreads, 1024 / kFrontierThreads) fro
                         bl.off_l = off_l;
                         bl.deg = d;
                         bl.ubytes = ub;
-                        bl.v = (uint32_t)((w0 + jw[u]) * 32 + lane);
+                        bl.v = vv[u];
                         bl.nch = nch;
                         a.big[base + __popc(bm & lt)] = bl;
                     }
@@ -903,22 +945,6 @@ __device__ __forceinline__ uint32_t shf_r_wrap(uint32_t lo, uint32_t hi, uint32_
     uint32_t d;
     asm("shf.r.wrap.b32 %0, %1, %2, %3;" : "=r"(d) : "r"(lo), "r"(hi), "r"(sh));
     return d;
-}
-
-// position (0..31) of the set bit of rank kk (0-based, kk < popc(w)) of w:
-// five popcount halvings (the in-word part of select1, P:96)
-__device__ __forceinline__ uint32_t select_in_word(uint32_t w, uint32_t kk)
-{
-    uint32_t pos = 0;
-#pragma unroll
-    for (uint32_t sh = 16; sh; sh >>= 1) {
-        const uint32_t c = __popc(w & ((1u << sh) - 1));
-        const bool up = kk >= c;
-        kk -= up ? c : 0u;
-        w = up ? w >> sh : w;
-        pos += up ? sh : 0u;
-    }
-    return pos;
 }
 
 // TMA bulk copy global -> shared (16-byte aligned addresses, size a multiple of 16)
