@@ -650,9 +650,13 @@ __global__ void __launch_bounds__(kFrontierThreads, 1024 / kFrontierThreads) fro
         // or, when the group's non-empty words are sparsely filled, the next 32
         // new vertices of the whole group (compacted: a lane finds its word by
         // maxle over the words' popcount prefix, then its bit by select)
-        uint32_t gtot;
-        const uint32_t gex = warp_excl_u32(__popc(nb), gtot);
+        const uint32_t gtot = __reduce_add_sync(FULL, __popc(nb));
         const bool sparse = kFrontierSparse && 4 * gtot <= 32u * (uint32_t)__popc(todo);
+        uint32_t gex = 0;  // exclusive popcount prefix of the group's words (sparse slots only)
+        if (sparse) {
+            uint32_t t;
+            gex = warp_excl_u32(__popc(nb), t);
+        }
         uint32_t cursor = 0;
         while (sparse ? cursor < gtot : todo != 0) {
             uint32_t vv[kS], bq[kS], wl[kS], nc[kS];
@@ -999,6 +1003,7 @@ constexpr bool kFastSingle = EFG_FAST_SINGLE;  // producer fast path for batches
 #define EFG_LPC_BITSKIP 1
 #endif
 constexpr bool kLpcBitSkip = EFG_LPC_BITSKIP;  // lane-per-chunk: skip the below-vpre stop bits of the first kept word
+constexpr uint64_t kMaxSuperTile = 16;           // tiles per super-tile at most (work assignment)
 
 template <int MODE>
 __global__ void __launch_bounds__(kExpandThreads, 1) expand_kernel(ExpandArgs a)
@@ -1049,11 +1054,22 @@ __global__ void __launch_bounds__(kExpandThreads, 1) expand_kernel(ExpandArgs a)
     const uint32_t kshift = kpow2 ? (uint32_t)__ffs(a.k) - 1 : 0u;
 
     // producer cursor: chunks [cnext, cend) of the current tile
-    uint64_t tile = gw;
+    // work assignment: super-tiles of ST consecutive tiles dealt round robin to
+    // the warps; a warp's batches run across the tile boundaries inside a
+    // super-tile (fewer part-filled batches), and round robin keeps regions
+    // of the id space spread over the grid.  ST grows with the level's tile
+    // count (>= 4 super-tiles per warp) up to kMaxSuperTile.
+    uint64_t ST = 1;
+    if (a.variant & 16) {
+        ST = ntiles / (4 * nwarps);
+        ST = ST < 1 ? 1 : (ST > kMaxSuperTile ? kMaxSuperTile : ST);
+    }
+    const uint64_t nst = (ntiles + ST - 1) / ST;
+    uint64_t tile = gw;  // super-tile index
     uint64_t cnext = 0, cend = 0;
-    if (tile < ntiles) {
-        cnext = a.tiles[tile];
-        cend = a.tiles[tile + 1];
+    if (tile < nst) {
+        cnext = a.tiles[tile * ST];
+        cend = a.tiles[tile * ST + ST < ntiles ? tile * ST + ST : ntiles];
     }
     uint32_t phase = 0;  // bit b: parity of the next wait on buffer b
     uint32_t nbuf = 0;   // buffer of the next produced batch
@@ -1062,9 +1078,9 @@ __global__ void __launch_bounds__(kExpandThreads, 1) expand_kernel(ExpandArgs a)
     auto produce = [&](Batch &B) -> bool {
         while (cnext >= cend) {
             tile += nwarps;
-            if (tile >= ntiles) return false;
-            cnext = a.tiles[tile];
-            cend = a.tiles[tile + 1];
+            if (tile >= nst) return false;
+            cnext = a.tiles[tile * ST];
+            cend = a.tiles[tile * ST + ST < ntiles ? tile * ST + ST : ntiles];
         }
         const uint64_t c = cnext + lane;
         const bool valid = c < cend;
