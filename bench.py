@@ -473,15 +473,17 @@ def run_partitioned(args, rank, world, local):
     hdepth = torch.empty(n, dtype=torch.int32, pin_memory=True)
     dist.barrier()
     t1 = time.perf_counter()
+    d2h = 0
     if args.xchg == "peer":
         for s in srcs[args.warmup:]:
-            g.bfs(int(s), depth=hdepth)
+            _, _, st_e = g.bfs(int(s), depth=hdepth, stats=True)  # includes the device->host depth copy
+            d2h += st_e["d2h_bytes"]
     e2e_s = time.perf_counter() - t1
     t = torch.tensor([ms, e2e_s], dtype=torch.float64, device=cdev)
-    e = torch.tensor([edges], dtype=torch.float64, device=cdev)
+    e = torch.tensor([edges, d2h], dtype=torch.float64, device=cdev)
     dist.all_reduce(t, op=dist.ReduceOp.MAX)
     dist.all_reduce(e, op=dist.ReduceOp.SUM)
-    value = float(e.item()) / (float(t[0].item()) * 1e-3) / 1e9
+    value = float(e[0].item()) / (float(t[0].item()) * 1e-3) / 1e9
     if rank == 0:
         cfgname = synth.CONFIGS[args.config]["name"] + (f"_scale{args.scale}" if args.scale else "")
         gpus = torch.cuda.device_count()
@@ -503,11 +505,17 @@ def run_partitioned(args, rank, world, local):
                        "l2_policy": "inputs larger than L2"},
             "clocks": clocks, "gpu_launches": launches,
             "gpu_launches_note": "rank 0's kernels (every rank launches the same number per level)",
-            "e2e": ({"value": float(e.item()) / float(t[1].item()) / 1e9, "unit": UNIT, "h2d_bytes_per_step": 4,
-                     "d2h_bytes_per_step": None,
-                     "d2h_note": "every rank receives the full depth array in a pinned host buffer"}
+            "e2e": ({"value": float(e[0].item()) / float(t[1].item()) / 1e9, "unit": UNIT,
+                     "h2d_bytes_per_step": 4 * world,
+                     "d2h_bytes_per_step": int(float(e[1].item()) / max(1, args.steps)),
+                     "d2h_note": "summed over ranks: every rank receives the full depth array in a pinned "
+                                 "host buffer (4-bit codes when the BFS has < 15 levels)"}
                     if args.xchg == "peer" else None),
+            "roofline": None,
+            "roofline_note": "N > 1: the expand roofline is reported on the N = 1 line (same kernel, a "
+                             "1/N row range per rank)",
             "cpu_baseline": None,
+            "cpu_baseline_note": "rank 0 at N = 1 only (contract)",
         }
         print(json.dumps(line), flush=True)
     g.free()

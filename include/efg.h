@@ -281,7 +281,7 @@ efg_status efg_pagerank(efg_graph *g, double damping, uint32_t iters, double *ra
                                  * directed or row-range handle): push along every edge with
                                  * fp64 atomicAdd.  Same sums, other order (C21). */
 
-#define EFG_OPT_EXPAND_VARIANT 4 /* tuning / A-B switch of the expand kernel, bit mask (default 11):
+#define EFG_OPT_EXPAND_VARIANT 4 /* tuning / A-B switch of the expand kernel, bit mask (default 43):
                                   * bit 0: batches of balanced chunks are decoded lane-per-chunk
                                   * (each lane walks its own chunk) instead of by word records
                                   * split evenly over the lanes; bit 1: a batch of adjacent chunks
@@ -290,8 +290,11 @@ efg_status efg_pagerank(efg_graph *g, double damping, uint32_t iters, double *ra
                                   * a pseudo-random ("arbitrary") order instead of the bitmap's
                                   * id order; bit 3: a lane-per-chunk lane steps over the stop
                                   * bits below the visited prefix inside its first kept word
-                                  * (select0) instead of decoding them.  Results are identical
-                                  * for every value. */
+                                  * (select0) instead of decoding them; bit 4: tiles are dealt
+                                  * to the warps in super-tiles of consecutive tiles; bit 5: the
+                                  * level-end list skip uses the visited prefix of the level just
+                                  * expanded (one more grid barrier) instead of the previous one.
+                                  * Values 0..63.  Results are identical for every value. */
 
 /* Set a per-handle option.  Errors: EFG_EINVAL (unknown option / value),
  * EFG_ESTATE (host-only handle). */
@@ -359,6 +362,15 @@ efg_status efg_bfs_end(efg_graph *g, efg_stats *st);
  *                    unpack; the cross-rank barriers over flags in the regions
  *                    spin in one block each) and returns.  Every rank must call
  *                    it once per level.
+ *   efg_xchg_peer_phase  the same exchange without the device barriers, one
+ *                    phase per call (0 publish, 1 owner OR + broadcast, 2
+ *                    unpack), each synchronising the handle's stream before it
+ *                    returns: the CALLER orders the phases across ranks with a
+ *                    host barrier after every phase (no kernel waits for
+ *                    another rank — the form for ranks time-sharing one GPU,
+ *                    whose cross-rank spinning kernels nothing schedules
+ *                    together).  Errors as efg_xchg_peer, EFG_EINVAL for a bad
+ *                    phase.
  * Ranks that share one device must use distinct non-blocking streams (the
  * barrier kernels of one rank wait for the others' kernels).  A barrier that
  * waits more than 4 s gives up; the next efg_bfs_finish_level then returns
@@ -371,6 +383,7 @@ efg_status efg_peer_alloc(efg_graph *g, int world, void **region, uint8_t *ipc_h
 efg_status efg_peer_open(efg_graph *g, int world, int rank, const uint64_t *bounds, const uint8_t *ipc_handles,
                          void *const *regions);
 efg_status efg_xchg_peer(efg_graph *g);
+efg_status efg_xchg_peer_phase(efg_graph *g, int phase);
 
 /*
  * efg_partition — the 1-D row partition (efg_build_opts.row_lo / row_hi):

@@ -264,6 +264,12 @@ class Graph:
     def xchg_peer(self) -> None:
         check(lib.efg_xchg_peer(self._h), "efg_xchg_peer")
 
+    def xchg_peer_phase(self, phase: int) -> None:
+        """One phase of the peer exchange without device barriers (0 publish,
+        1 owner OR + broadcast, 2 unpack); returns after the stream is idle —
+        the caller orders the phases across ranks with a host barrier."""
+        check(lib.efg_xchg_peer_phase(self._h, phase), "efg_xchg_peer_phase")
+
     def bfs_finish_level(self) -> int:
         n = C.c_uint64()
         check(lib.efg_bfs_finish_level(self._h, C.byref(n)), "efg_bfs_finish_level")

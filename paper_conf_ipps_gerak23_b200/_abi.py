@@ -77,6 +77,7 @@ SIGNATURES = [
     ("efg_peer_alloc", C.c_int, [C.c_void_p, C.c_int, C.POINTER(C.c_void_p), C.c_void_p]),
     ("efg_peer_open", C.c_int, [C.c_void_p, C.c_int, C.c_int, C.c_void_p, C.c_void_p, C.c_void_p]),
     ("efg_xchg_peer", C.c_int, [C.c_void_p]),
+    ("efg_xchg_peer_phase", C.c_int, [C.c_void_p, C.c_int]),
     ("efg_bfs_finish_level", C.c_int, [C.c_void_p, C.POINTER(C.c_uint64)]),
     ("efg_bfs_end", C.c_int, [C.c_void_p, C.POINTER(Stats)]),
     ("efg_partition", C.c_int, [C.c_uint64, C.c_void_p, C.c_void_p, C.c_int, C.c_void_p]),

@@ -217,7 +217,7 @@ extern "C" efg_status efg_set_option(efg_graph *g, int option, int64_t value)
         }
         return EFG_OK;
     case EFG_OPT_EXPAND_VARIANT:
-        if (value < 0 || value > 31) return set_error(EFG_EINVAL, "EFG_OPT_EXPAND_VARIANT: 0..31");
+        if (value < 0 || value > 63) return set_error(EFG_EINVAL, "EFG_OPT_EXPAND_VARIANT: 0..63");
         if (g->dev.expand_variant != (int)value) {
             g->dev.expand_variant = (int)value;
             efg::device_drop_graphs(g->dev);
@@ -332,6 +332,14 @@ extern "C" efg_status efg_xchg_peer(efg_graph *g)
     clear_error();
     EFG_TRY(check_handle(g));
     return device_xchg_peer(g);
+}
+
+extern "C" efg_status efg_xchg_peer_phase(efg_graph *g, int phase)
+{
+    clear_error();
+    EFG_TRY(check_handle(g));
+    if (phase < 0 || phase > 2) return set_error(EFG_EINVAL, "efg_xchg_peer_phase: phase 0..2");
+    return device_xchg_peer_phase(g, phase);
 }
 
 extern "C" efg_status efg_bfs_finish_level(efg_graph *g, uint64_t *global_new)

@@ -171,7 +171,7 @@ FrontierArgs frontier_args(DeviceGraph &d, cudaGraphConditionalHandle cond, bool
 #ifdef EFG_NO_LSKIP
     a.lskip = 0;  // tuning experiment: record-level skip only
 #else
-    a.lskip = (d.prefix_skip && !consume) ? 1u : 0u;
+    a.lskip = (d.prefix_skip && !consume) ? ((d.expand_variant & 32) ? 2u : 1u) : 0u;
 #endif
     a.rec = d.rec;
     a.chunks = d.chunks;
@@ -196,9 +196,13 @@ FrontierArgs frontier_args(DeviceGraph &d, cudaGraphConditionalHandle cond, bool
 
 // level end + next plan: one launch (every block resident, see frontier_kernel)
 efg_status launch_level_end(DeviceGraph &d, cudaGraphConditionalHandle cond, cudaStream_t s,
-                            bool consume = false, bool cond_global = false, bool need_cvtx = true)
+                            bool consume = false, bool cond_global = false, bool need_cvtx = true,
+                            bool start = false)
 {
     FrontierArgs fa = frontier_args(d, cond, consume);
+    // a traversal's first plan has no visited prefix to skip by (decode and
+    // PageRank mark their whole vertex range visited to plan it)
+    if (start) fa.lskip = 0;
     fa.cond_global = cond_global ? 1 : 0;
     if (!need_cvtx) fa.cvtx = nullptr;  // plain BFS: the expand never reads the chunk's vertex
     CUDA_TRY(launch_frontier(fa, (unsigned)((d.nwords + d.words_per_block - 1) / d.words_per_block), s));
@@ -521,7 +525,7 @@ static efg_status start_traversal(DeviceGraph &d, uint64_t v0, uint64_t v1, int3
     ia.v0 = v0;
     ia.v1 = v1;
     CUDA_TRY(launch_init(ia, s));
-    EFG_TRY(launch_level_end(d, 0, s));
+    EFG_TRY(launch_level_end(d, 0, s, false, false, true, true));
     launches += 2;
     return EFG_OK;
 }
@@ -979,6 +983,18 @@ efg_status device_xchg_peer(efg_graph *g)
     CUDA_TRY(cudaSetDevice(d.device));
     EFG_TRY(launch_peer_exchange(d, stream_of(d)));
     d.step_launches += 5;
+    return EFG_OK;
+}
+
+efg_status device_xchg_peer_phase(efg_graph *g, int phase)
+{
+    DeviceGraph &d = g->dev;
+    if (!d.peer_ptrs) return set_error(EFG_ESTATE, "efg_xchg_peer_phase: call efg_peer_open first");
+    CUDA_TRY(cudaSetDevice(d.device));
+    cudaStream_t s = stream_of(d);
+    CUDA_TRY(launch_peer(peer_args(d, phase), d.num_sms, s));
+    CUDA_TRY(cudaStreamSynchronize(s));
+    d.step_launches += 1;
     return EFG_OK;
 }
 

@@ -226,7 +226,7 @@ struct DeviceGraph {
     int level_loop = 0;                // 0 = CUDA graph (device loop), 1 = host loop + events
     int prefix_skip = 1;               // EFG_OPT_PREFIX_SKIP
     int pr_pull = 1;                   // EFG_OPT_PAGERANK_PULL
-    int expand_variant = 11;           // EFG_OPT_EXPAND_VARIANT (bits 0, 1, 3)
+    int expand_variant = 43;           // EFG_OPT_EXPAND_VARIANT (bits 0, 1, 3, 5)
     static constexpr int kLoopGraphs = 3;                 // visit, visit+parent, partitioned visit
     cudaGraph_t loop_graph[kLoopGraphs] = {};
     cudaGraphExec_t loop_exec[kLoopGraphs] = {};
@@ -272,6 +272,7 @@ efg_status device_peer_alloc(efg_graph *g, int world, void **region, uint8_t *ip
 efg_status device_peer_open(efg_graph *g, int world, int rank, const uint64_t *bounds, const uint8_t *ipc_handles,
                             void *const *regions);
 efg_status device_xchg_peer(efg_graph *g);
+efg_status device_xchg_peer_phase(efg_graph *g, int phase);
 void device_peer_close(DeviceGraph &d);
 efg_status device_xchg(efg_graph *g, int op, int world, const uint64_t *bounds, uint64_t slice_words,
                        uint32_t *out, const uint32_t *in);

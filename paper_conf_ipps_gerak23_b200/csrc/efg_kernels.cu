@@ -339,6 +339,9 @@ __global__ void peer_kernel(PeerArgs a)
 //       whose work position is >= tT (the Fig. 4 maxle rule, once per tile).
 //
 // Persistent grid (every block resident: blocks wait on each other).  Phases:
+//   0   (list skip on the level's own prefix, lskip = 2) each warp finds the
+//       first vertex of its bitmap groups neither visited nor isolated, the
+//       minimum is reduced over the grid, grid barrier;
 //   1   a warp counts the new vertices of its bitmap word run, their work and
 //       chunks (degree loads coalesced: lanes over the bits of a word);
 //       the per-block aggregates are published, a grid barrier, then each
@@ -472,18 +475,41 @@ __global__ void __launch_bounds__(kFrontierThreads, 1024 / kFrontierThreads) fro
     // prefix the last expand used (a lower bound of the next one) cannot
     // discover anything: it is neither planned nor expanded (its degree still
     // counts in the level's edges, reading C18)
-    const uint32_t vlow = a.lskip ? ctrl->vpre_used : 0u;
+    // lskip == 2: the level's own visited prefix (phase 0: the smallest vertex
+    // neither visited nor isolated after this level's expand, reduced over the
+    // grid before the counting) — at a discovery level's end the prefix jumps,
+    // and the previous one would keep lists planned that cannot discover anything
+    uint32_t vmin = FULL;  // smallest vertex of this warp's range that is neither visited nor isolated
+    uint32_t vlow = 0;
+    if (a.lskip == 2) {
+        for (uint64_t w0 = 32ull * gw; w0 < a.nwords; w0 += WG) {  // the warp's first group with a zero
+            const uint64_t w = w0 + lane;
+            const uint32_t un = w < a.nwords ? ~(__ldcg(a.vis + w) | a.iso[w]) : 0u;
+            const uint32_t zm = __ballot_sync(FULL, un != 0);
+            if (zm) {
+                const uint32_t cand = (uint32_t)(w * 32) + (un ? (uint32_t)__ffs(un) - 1 : 0u);
+                vmin = __shfl_sync(FULL, cand, __ffs(zm) - 1);
+                break;
+            }
+        }
+        if (lane == 0 && vmin != FULL) atomicMin(&ctrl->vmin2[level & 1], vmin);
+        grid_barrier(a.barrier, &ctrl->fault);
+        vlow = __ldcg(&ctrl->vmin2[level & 1]);
+        vmin = FULL;  // already reduced
+    } else if (a.lskip) {
+        vlow = ctrl->vpre_used;
+    }
+    const bool vmin_done = a.lskip == 2;
     uint32_t cq = 0, all = 0, ch = 0;  // lane partials
     uint64_t wk = 0, sk = 0;
     uint32_t bg = 0;  // lists planned grid-wide (phase 3)
-    uint32_t vmin = FULL;  // smallest vertex of this warp's range that is neither visited nor isolated
     for (uint64_t w0 = 32ull * gw; w0 < a.nwords; w0 += WG) {
         const uint64_t w = w0 + lane;
         uint32_t nb = 0, nq = 0;
         if (w < a.nwords) {
             const uint32_t x = a.vis[w];
             nb = a.consume ? x : (x & ~a.prev[w]);
-            if (!a.consume && vmin == FULL) {
+            if (!a.consume && !vmin_done && vmin == FULL) {
                 const uint32_t un = ~(x | a.iso[w]);
                 if (un) vmin = (uint32_t)(w * 32) + (__ffs(un) - 1);
             }

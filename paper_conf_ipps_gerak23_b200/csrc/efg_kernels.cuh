@@ -90,7 +90,8 @@ struct FrontierArgs {           // level end (a7) + next level plan (a1-a4), one
     int consume;               // 1: frontier = vis itself, vis reset (SSSP relaxed set)
     const uint32_t *deg32;     // degrees (pass 1)
     const uint32_t *umax;      // largest neighbour of each list
-    uint32_t lskip;            // BFS: lists whose largest neighbour is below ctrl->vpre_used are not planned
+    uint32_t lskip;            // BFS: lists whose largest neighbour is below the visited prefix are not planned
+                               // (1: ctrl->vpre_used, the previous level's; 2: this level's, phase 0)
     uint32_t *skipw;           // scratch (nwords): per bitmap word, the skipped lists (phase 1 -> phase 2)
     const VRec *rec;           // vertex records (pass 2)
     ChunkDesc *chunks;         // out: chunk descriptors

@@ -168,6 +168,26 @@ def partitioned_bfs_peer(g, source: int, depth):
     return counts
 
 
+def partitioned_bfs_peer_hostseq(g, source: int, depth, host_barrier):
+    """The same partitioned BFS over peer memory with host-sequenced exchange
+    phases (efg_xchg_peer_phase + `host_barrier()` after each): no kernel waits
+    for another rank, so ranks may time-share one GPU."""
+    g.bfs_begin(source, depth)
+    counts = [1]
+    while True:
+        g.bfs_expand()
+        for phase in (0, 1, 2):
+            g.xchg_peer_phase(phase)
+            if phase < 2:
+                host_barrier()
+        new = g.bfs_finish_level()
+        host_barrier()  # every rank's unpack read res before the next publish / OR
+        if new == 0:
+            break
+        counts.append(new)
+    return counts
+
+
 def simulated_peer_setup(graphs, bounds: np.ndarray) -> None:
     """All `world` rank handles in one process on one device (tests): the
     regions are mapped by address instead of IPC.  Each handle must have been

@@ -1,11 +1,16 @@
 """Two processes, one per rank, running the partitioned BFS with the exchange
-over peer memory (efg_peer_alloc / efg_peer_open with CUDA IPC handles /
-efg_xchg_peer).  On a multi-GPU box each rank would own a GPU
-and the regions would be reached over NVLink; here both ranks share cuda:0
-(this run has one GPU), which exercises the same IPC mapping, the same
-system-scope flag barriers between processes and the same kernels.  The
-handles are all-gathered over gloo (torch.distributed); no data-path
-collective.  Every rank's depth must equal the oracle's.
+over peer memory (efg_peer_alloc / efg_peer_open with CUDA IPC handles;
+SURVEY §8(e)).  On a multi-GPU box each rank would own a GPU and the regions
+would be reached over NVLink; here both ranks share cuda:0 (this run has one
+GPU), which exercises the same IPC mapping and the same exchange kernels.
+Ranks time-sharing one GPU must not run kernels that wait on one another
+(nothing schedules two processes' kernels together; B200_PROFILING.md reports
+Xid 109 for exactly that), so the exchange runs host-sequenced here
+(efg_xchg_peer_phase, a gloo barrier after every phase); the device-barrier
+form (efg_xchg_peer, collective efg_bfs) is tested with simulated ranks in one
+process (tests/test_gpu_bfs.py, tests/test_gpu_boundary.py).  The handles are
+all-gathered over gloo; no data-path collective.  Every rank's depth must
+equal the oracle's.
 """
 import os
 import socket
@@ -34,7 +39,7 @@ def _worker(rank: int, port: int, q):
         import oracle
         import synth
         import paper_conf_ipps_gerak23_b200 as efg
-        from paper_conf_ipps_gerak23_b200.dist import peer_setup, partitioned_bfs_peer
+        from paper_conf_ipps_gerak23_b200.dist import peer_setup, partitioned_bfs_peer_hostseq
         dist.init_process_group("gloo", rank=rank, world_size=WORLD)
         torch.cuda.set_device(0)
         n, src, dst = synth.rmat(14, 16, seed=13)
@@ -49,22 +54,11 @@ def _worker(rank: int, port: int, q):
         for s in SOURCES:
             ref = oracle.bfs(ov, oe, s)
             depth = torch.empty(n, dtype=torch.int32, device="cuda")
-            partitioned_bfs_peer(g, s, depth)  # stepwise calls
+            depth.fill_(-7)
+            partitioned_bfs_peer_hostseq(g, s, depth, dist.barrier)
             torch.cuda.synchronize()
             if not np.array_equal(depth.cpu().numpy(), ref):
-                bad.append(("stepwise", s))
-            # collective efg_bfs: enqueue-only (device depth) and synchronous (host depth),
-            # graph loop and host loop
-            for host_loop in (False, True):
-                g.set_level_loop(host_loop)
-                depth.fill_(-7)
-                g.bfs(s, depth=depth)
-                torch.cuda.synchronize()
-                if not np.array_equal(depth.cpu().numpy(), ref):
-                    bad.append(("collective-device", host_loop, s))
-                if not np.array_equal(g.bfs(s), ref):
-                    bad.append(("collective-host", host_loop, s))
-            g.set_level_loop(False)
+                bad.append(("hostseq", s))
         dist.barrier()
         g.free()
         dist.destroy_process_group()
