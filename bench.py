@@ -279,7 +279,10 @@ def _cpu_baseline_child(cfg: int, scale, index: int, count: int, out_dir: str, c
     d = oracle.bfs(ov, oe, s0)
     cs = time.perf_counter() - t
     np.save(os.path.join(out_dir, "depth.npy"), d)
-    meta = {"source": s0, "bfs_s": cs, "csr_s": csr_s, "edges": int(deg[d >= 0].sum()),
+    # a second parity source (untimed): the next timed source
+    s1 = int(synth.sources(n, count, seed=1000 + cfg, nonisolated_mask=deg > 0)[min(index + 1, count - 1)])
+    np.save(os.path.join(out_dir, "depth1.npy"), oracle.bfs(ov, oe, s1))
+    meta = {"source": s0, "source1": s1, "bfs_s": cs, "csr_s": csr_s, "edges": int(deg[d >= 0].sum()),
             "core": core, "affinity": sorted(os.sched_getaffinity(0))}
     # the optional all-core baseline (BASELINE.md CPU plan), once the parent's
     # GPU work is over: OpenMP top-down BFS on the same CSR and source
@@ -322,13 +325,17 @@ def finish_cpu_baseline(proc, out_dir: str, go, g, n: int):
         meta = json.load(f)
     dref = np.load(os.path.join(out_dir, "depth.npy"))
     ok = bool(np.array_equal(dref, g.bfs(meta["source"])))
+    psrc = [meta["source"]]
+    if "source1" in meta:
+        ok = ok and bool(np.array_equal(np.load(os.path.join(out_dir, "depth1.npy")), g.bfs(meta["source1"])))
+        psrc.append(meta["source1"])
     return {"value": meta["edges"] / meta["bfs_s"] / 1e9, "unit": UNIT, "cores": 1, "kind": "oracle",
             "sample": f"one single-threaded FIFO BFS (source {meta['source']}, {meta['edges']} edges) over "
                       f"the oracle CSR of the same graph ({meta['bfs_s']:.1f} s; CSR build "
                       f"{meta['csr_s']:.1f} s untimed), pinned to host core {meta['core']} "
                       f"(sched_setaffinity = taskset -c {meta['core']}; bench's own threads kept off it)",
             "cpu_model": cpu_model(), "host_cores": os.cpu_count(),
-            "parity_bit_exact": ok, "parity_source": meta["source"],
+            "parity_bit_exact": ok, "parity_sources": psrc,
             "all_cores": ({"value": meta["edges"] / meta["par_s"] / 1e9, "unit": UNIT,
                            "cores": meta["par_threads"], "kind": "openmp top-down BFS (cpu_baseline/omp_bfs.c)",
                            "sample": "the same source and CSR, after the GPU work", "depth_equal_oracle":
@@ -769,7 +776,7 @@ def main():
     cpu = None
     if cpu_job is not None:
         cpu = finish_cpu_baseline(*cpu_job, g, n)
-        if "parity_source" in cpu and cpu["parity_source"] != stats[0][0]:
+        if "parity_sources" in cpu and cpu["parity_sources"][0] != stats[0][0]:
             cpu["parity_note"] = "source differs from the first timed source"
 
     if rank == 0:

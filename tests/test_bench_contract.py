@@ -61,7 +61,7 @@ def test_cpu_baseline_child_pinned_and_checked():
             assert cpu["kind"] == "oracle" and cpu["cores"] == 1 and cpu["value"] > 0
             assert cpu["parity_bit_exact"] is (not wrong)
             srcs = synth.sources(n, 4, seed=1001, nonisolated_mask=np.diff(ov) > 0)
-            assert cpu["parity_source"] == int(srcs[1])
+            assert cpu["parity_sources"] == [int(srcs[1]), int(srcs[2])]
             assert "taskset -c" in cpu["sample"] and cpu["cpu_model"]
             assert cpu["all_cores"]["depth_equal_oracle"] and cpu["all_cores"]["value"] > 0
     finally:
