@@ -79,8 +79,9 @@ def parse():
                         "read by the kernels over the host link")
     p.add_argument("--permute", action="store_true",
                    help="random relabelling of the generator's ids (P:248-258 'random ordering' arm)")
-    p.add_argument("--reorder", default="degree", choices=["none", "degree"],
-                   help="EFG_REORDER_DEGREE relabelling at build time (results stay in input ids)")
+    p.add_argument("--reorder", default=None, choices=["none", "degree"],
+                   help="EFG_REORDER_DEGREE relabelling at build time (results stay in input ids); "
+                        "default degree, none on C5 (permuted ids, sharded build without global degrees)")
     p.add_argument("--profile-levels", action="store_true", help="print per-level stats to stderr")
     p.add_argument("--no-sssp", action="store_true",
                    help="skip the SSSP (NEXT-1) timing over the same graph built with synthetic weights "
@@ -91,6 +92,8 @@ def parse():
                         "BFS and PageRank)")
     p.add_argument("--pagerank", action="store_true", help="force the PageRank timing on other configs")
     a = p.parse_args()
+    if a.reorder is None:
+        a.reorder = "none" if a.config == 5 else "degree"
     a.do_alt = (a.alt or a.config in (2, 4)) and not a.no_alt
     a.do_sssp = (a.sssp or a.config == 4) and not a.no_sssp
     a.do_pagerank = (a.pagerank or a.config == 2) and not a.no_pagerank
@@ -387,6 +390,33 @@ def run_reference(args, rank, world):
     print(json.dumps(line), flush=True)
 
 
+def stream_degree_bounds(sg, world: int, relabel: bool, chunk: int = 1 << 27):
+    """1-D partition bounds from ONE counting pass over the generator stream
+    (no EFG build): per-vertex degree estimate = endpoint count of the non-loop
+    samples (duplicates included), cost per vertex = 29 B + its estimated EF
+    list bytes deg * (2 + log2(n / deg)) / 8 (efg_partition's model, SURVEY
+    8(e)), in the relabelled order (degree descending, ties by id) when
+    `relabel`.  Cut points are 64-aligned (one owner per bitmap word).
+    Returns (bounds uint64[world + 1], degree estimate in input ids)."""
+    n, m = sg.n, sg.m
+    deg = np.zeros(n, np.int64)
+    for first in range(0, m, chunk):
+        src, dst = sg.range(first, min(chunk, m - first))
+        keep = src != dst
+        deg += np.bincount(src[keep], minlength=n)
+        deg += np.bincount(dst[keep], minlength=n)
+    order = np.lexsort((np.arange(n), -deg)) if relabel else np.arange(n)
+    d = deg[order].astype(np.float64)
+    cost = 29.0 + np.where(d > 0, d * (2.0 + np.log2(np.maximum(n / np.maximum(d, 1.0), 1.0))) / 8.0, 0.0)
+    c = np.cumsum(cost)
+    b = [0]
+    for r in range(1, world):
+        v = int(np.searchsorted(c, c[-1] * r / world))
+        b.append(min(n, max(b[-1], (v + 63) // 64 * 64)))
+    b.append(n)
+    return np.array(b, np.uint64), deg
+
+
 def run_partitioned(args, rank, world, local):
     """N ranks, one collective BFS at a time over the 1-D row partition (strong
     scaling).  Each rank builds only its rows from the generator
@@ -410,24 +440,14 @@ def run_partitioned(args, rank, world, local):
     srcs_t = torch.zeros(args.warmup + args.steps, dtype=torch.int64, device=cdev)
     nthr = max(1, (os.cpu_count() or 1) // world)
     if rank == 0:
+        # bounds from one counting pass over the generator (no whole-graph build
+        # on rank 0; every rank then builds only its rows)
         if args.reorder == "degree":
-            # byte-balanced bounds need the relabelled sizes: one host-only
-            # whole-graph build on rank 0 (efg_partition)
-            whole = efg.Graph.build_stream(n, sg.m, sg.fn, sg.user, device=-1, flags=flags,
-                                           n_threads=os.cpu_count() or 1)
-            vl, _, of, _ = whole.export()
-            b = efg.partition(vl, of, world)
-            pm = whole.perm()
-            deg = np.empty(n, np.int64)
-            deg[pm] = np.diff(vl).astype(np.int64)
-            whole.free()
+            b, deg = stream_degree_bounds(sg, world, relabel=True)
+            s = synth.sources(n, args.warmup + args.steps, seed=1000 + args.config, nonisolated_mask=deg > 0)
         else:
             # generator order (e.g. permuted RMAT, C5): equal vertex ranges, 64-aligned
             b = np.array([min(n, (n * r // world + 63) // 64 * 64) for r in range(world)] + [n], np.uint64)
-            deg = None
-        if deg is not None:
-            s = synth.sources(n, args.warmup + args.steps, seed=1000 + args.config, nonisolated_mask=deg > 0)
-        else:
             s = synth.sources(n, args.warmup + args.steps, seed=1000 + args.config)
         bounds.copy_(torch.from_numpy(b.astype(np.int64)))
         srcs_t.copy_(torch.from_numpy(s.astype(np.int64)))

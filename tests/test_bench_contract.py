@@ -66,3 +66,30 @@ def test_cpu_baseline_child_pinned_and_checked():
             assert cpu["all_cores"]["depth_equal_oracle"] and cpu["all_cores"]["value"] > 0
     finally:
         os.sched_setaffinity(0, before)
+
+
+def test_stream_degree_bounds_partition():
+    """N > 1 bench: rank 0's partition bounds come from one counting pass over
+    the generator (no whole-graph build).  Bounds are monotone, 64-aligned,
+    cover [0, n], and balance the EF bytes + 29 B per vertex of the real build
+    (efg_partition's model) within 10 % per rank; the degree estimate marks
+    exactly the non-isolated vertices."""
+    import numpy as np
+    import bench
+    import synth
+    import paper_conf_ipps_gerak23_b200 as efg
+    sg = synth.config_stream(1)
+    for world in (2, 3, 4, 8):
+        b, deg = bench.stream_degree_bounds(sg, world, relabel=True, chunk=1 << 18)
+        assert b[0] == 0 and b[-1] == sg.n and np.all(np.diff(b.astype(np.int64)) >= 0)
+        assert np.all(b[1:-1] % 64 == 0)
+        g = efg.Graph.build_stream(sg.n, sg.m, sg.fn, sg.user, device=-1,
+                                   flags=efg.EFG_DEFAULT_FLAGS | efg.EFG_REORDER_DEGREE)
+        vl, _, of, _ = g.export()
+        true_deg = np.empty(sg.n, np.int64)
+        true_deg[g.perm()] = np.diff(vl).astype(np.int64)
+        cost = np.diff(of).astype(np.float64) + 29.0
+        g.free()
+        per = np.array([cost[int(b[r]):int(b[r + 1])].sum() for r in range(world)])
+        assert per.max() / per.mean() < 1.10, (world, per)
+        assert np.array_equal(deg > 0, true_deg > 0)
