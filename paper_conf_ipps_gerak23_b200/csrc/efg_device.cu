@@ -661,10 +661,15 @@ efg_status device_bfs(efg_graph *g, uint32_t source, int32_t *depth, uint32_t *p
                 return set_error(EFG_ECUDA, "a grid or peer barrier timed out (grid not co-resident, or a rank "
                                             "missing from the collective); sticky until efg_free");
             if ((part ? c.nnew : c.nf) == 0) break;  // partitioned: the global new count
-            if (std::getenv("EFG_DEBUG_LEVELS"))  // plan statistics of the level about to be expanded
-                fprintf(stderr, "efg-level L=%u nf=%llu ne=%llu nchunks=%llu nwork=%llu ntiles=%llu vpre_used=%u\n",
+            if (std::getenv("EFG_DEBUG_LEVELS")) {  // plan statistics of the level about to be expanded
+                fprintf(stderr, "efg-level L=%u nf=%llu ne=%llu nchunks=%llu nwork=%llu ntiles=%llu vpre_used=%u"
+                        " prev-batches lpc=%llu rec=%llu chunks %llu/%llu elems %llu/%llu lpc-slots %llu words %llu\n",
                         levels, (unsigned long long)c.nf, (unsigned long long)c.ne, (unsigned long long)c.nchunks,
-                        (unsigned long long)c.nwork, (unsigned long long)c.ntiles, c.vpre_used);
+                        (unsigned long long)c.nwork, (unsigned long long)c.ntiles, c.vpre_used, c.bstat[0],
+                        c.bstat[1], c.bstat[2], c.bstat[3], c.bstat[4], c.bstat[5], c.bstat[6], c.bstat[7]);
+                CUDA_TRY(cudaMemsetAsync(reinterpret_cast<char *>(d.ctrl) + offsetof(LevelCtrl, bstat), 0,
+                                         sizeof(c.bstat), s));
+            }
             lf.push_back(c.nf);
             le.push_back(c.ne);
             cudaEvent_t a, b;

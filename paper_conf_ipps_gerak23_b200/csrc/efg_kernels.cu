@@ -1407,6 +1407,21 @@ __global__ void __launch_bounds__(kExpandThreads, 1) expand_kernel(ExpandArgs a)
     while (have) {
         // slot table of the current batch (its producer registers are about to be reused)
         const uint32_t cnt = cur.cnt, NW = cur.nw, buf = cur.buf;
+#ifdef EFG_BATCH_STATS
+        // [0/1] batches lane-per-chunk / records, [2/3] their chunks, [4/5] their
+        // elements, [6] 32 x longest chunk summed over the LPC batches, [7] words
+        if (lane == 0) {
+            const int r = cur.lpc ? 0 : 1;
+            atomicAdd(&a.ctrl->bstat[r], 1ull);
+            atomicAdd(&a.ctrl->bstat[2 + r], (unsigned long long)cnt);
+            atomicAdd(&a.ctrl->bstat[4 + r], (unsigned long long)cur.ne);
+            atomicAdd(&a.ctrl->bstat[7], (unsigned long long)NW);
+        }
+        {
+            const uint32_t mx = __reduce_max_sync(FULL, lane < cnt ? cur.nel : 0u);
+            if (lane == 0 && cur.lpc) atomicAdd(&a.ctrl->bstat[6], 32ull * mx);
+        }
+#endif
         if (lane < cnt) {
             SlotP sp;
             sp.lsmb = cur.lsmb;
