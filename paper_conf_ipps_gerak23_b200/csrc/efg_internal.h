@@ -162,6 +162,7 @@ constexpr int kBitmapAlign = 1024;           // bitmap words are padded to a mul
 #define EFG_TILE_WORK 2048
 #endif
 constexpr uint32_t kTileWork = EFG_TILE_WORK;         // work units per tile (a3)
+static_assert((kTileWork & (kTileWork - 1)) == 0, "kTileWork: a power of two (tile indices by shifts)");
 constexpr uint32_t kChunkWork = 32;          // per-chunk overhead in work units
 #ifndef EFG_FRONTIER_SPARSE
 #define EFG_FRONTIER_SPARSE 1

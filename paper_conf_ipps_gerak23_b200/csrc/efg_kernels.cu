@@ -443,6 +443,7 @@ __global__ void __launch_bounds__(kFrontierThreads, 1024 / kFrontierThreads) fro
     constexpr int NT = kFrontierThreads, NW = NT / 32;
     __shared__ uint64_t s_q[NW], s_wk[NW], s_ch[NW], s_sk[NW], s_bg[NW], s_all[NW];
     __shared__ uint64_t s_pre[5], s_tot[5];
+    __shared__ uint32_t s_skw[NW][32];  // phase 1, sparse groups: skipped lists of each word
 
     const uint32_t tid = threadIdx.x, lane = tid & 31, wid = tid >> 5, b = blockIdx.x;
 #define FTRACE(p)                                                      \
@@ -469,6 +470,9 @@ __global__ void __launch_bounds__(kFrontierThreads, 1024 / kFrontierThreads) fro
 #define EFG_KB 4
 #endif
     constexpr int kB = EFG_KB;  // pass 1: non-empty words whose degree loads are in flight together
+#ifndef EFG_P1_SPARSE
+#define EFG_P1_SPARSE 4
+#endif
 
     // ---- 1: count, work and chunks of the warp's new (owned) vertices ----
     // BFS list skip: a list whose largest neighbour is below the visited
@@ -520,6 +524,58 @@ __global__ void __launch_bounds__(kFrontierThreads, 1024 / kFrontierThreads) fro
         // a1: degrees of the new vertices, lanes over the bits of each non-empty
         // word (one coalesced 128-byte load per word)
         uint32_t todo = __ballot_sync(FULL, nq != 0);
+        const uint32_t gq = __reduce_add_sync(FULL, __popc(nq));
+        if (kFrontierSparse && gq && EFG_P1_SPARSE * gq <= 32u * (uint32_t)__popc(todo)) {
+            // sparsely filled words (<= 32 / EFG_P1_SPARSE new vertices per non-empty word): lanes
+            // over the group's new vertices instead (32 per slot, kB slots of
+            // loads in flight — a word per step would leave most lanes idle and
+            // serialise one memory round trip per few vertices)
+            uint32_t t_;
+            const uint32_t gex = warp_excl_u32(__popc(nq), t_);
+            if (vlow) s_skw[wid][lane] = 0;
+            __syncwarp();
+            for (uint32_t cursor = 0; cursor < gq; cursor += 32u * kB) {
+                uint32_t dv[kB], uv[kB];
+#pragma unroll
+                for (int u = 0; u < kB; ++u) {
+                    dv[u] = 0;
+                    uv[u] = FULL;
+                    const uint32_t t = cursor + 32u * u + lane;
+                    if (cursor + 32u * u < gq) {  // warp-uniform
+                        const int j = warp_maxle_u32(gex, t < gq ? t : 0u);
+                        const uint32_t bits = __shfl_sync(FULL, nq, j);
+                        const uint32_t r = t - __shfl_sync(FULL, gex, j);
+                        if (t < gq) {
+                            const uint32_t bit = select_in_word(bits, r);
+                            const uint64_t v = (w0 + j) * 32 + bit;
+                            dv[u] = __ldg(a.deg32 + v);
+                            if (vlow) {
+                                uv[u] = __ldg(a.umax + v);
+                                if (uv[u] < vlow) atomicOr(&s_skw[wid][j], 1u << bit);
+                            }
+                        }
+                    }
+                }
+#pragma unroll
+                for (int u = 0; u < kB; ++u) {
+                    const uint32_t d = dv[u];
+                    if (uv[u] < vlow) {  // skipped list
+                        sk += d;
+                        continue;
+                    }
+                    const uint32_t nch = d ? (uint32_t)cl.div((uint64_t)d + CH - 1) : 0u;
+                    wk += (uint64_t)nch * CW + d;
+                    ch += nch;
+                    bg += (nch > 1 || (uint64_t)nch * CW + d > kTileWork) ? 1u : 0u;
+                }
+            }
+            if (vlow) {
+                __syncwarp();
+                if (nq) a.skipw[w] = s_skw[wid][lane];
+                __syncwarp();
+            }
+            todo = 0;
+        }
         while (todo) {
             uint32_t dv[kB], uv[kB], jv[kB];
 #pragma unroll
@@ -599,11 +655,12 @@ __global__ void __launch_bounds__(kFrontierThreads, 1024 / kFrontierThreads) fro
     // (longer batches of short lists per warp), kTileWork otherwise (enough
     // tiles for every expand warp on small levels).  Lists of <= kTileWork
     // units cross at most one tile boundary either way (phase 2).
-    const uint64_t TW = s_tot[1] >= kTileBigMinWork ? 2ull * kTileWork : (uint64_t)kTileWork;
+    const uint32_t TWs = (31 - __builtin_clz(kTileWork)) + (s_tot[1] >= kTileBigMinWork ? 1 : 0);
+    const uint64_t TW = 1ull << TWs;  // a power of two: tile index = work position >> TWs
     if (b == gridDim.x - 1 && tid == 0) {  // level totals
         const uint64_t nwork = s_tot[1], nchunks = s_tot[2];
         const uint64_t ne = nwork - CW * nchunks + s_tot[3];  // every frontier list's edges
-        const uint64_t ntiles = (nwork + TW - 1) / TW;
+        const uint64_t ntiles = (nwork + TW - 1) >> TWs;
         ctrl->nf = nf;
         ctrl->nwork = nwork;
         ctrl->nchunks = nchunks;
@@ -770,7 +827,7 @@ __global__ void __launch_bounds__(kFrontierThreads, 1024 / kFrontierThreads) fro
                         if (a.cvtx) a.cvtx[C] = vv[u];
                     }
                     // a3: a tile boundary t*T inside [W, W + wlen) starts at this chunk or the next
-                    const uint64_t t = (W + TW - 1) / TW;
+                    const uint64_t t = (W + TW - 1) >> TWs;
                     if (t * TW < W + wlen) a.tiles[t] = C + (t * TW > W ? 1u : 0u);
                 }
                 const uint32_t bm = __ballot_sync(FULL, big);
@@ -828,7 +885,7 @@ __global__ void __launch_bounds__(kFrontierThreads, 1024 / kFrontierThreads) fro
             nch = __ldcg(&bp->nch);
         }
         const uint64_t wl = (uint64_t)nch * CW + d;
-        const uint64_t t_lo = (W + TW - 1) / TW, t_hi = (W + wl + TW - 1) / TW;
+        const uint64_t t_lo = (W + TW - 1) >> TWs, t_hi = (W + wl + TW - 1) >> TWs;
         const bool huge = nch > 8 || t_hi - t_lo > 8;
         if (!huge) {
             for (uint32_t j = 0; j < nch; ++j) {
@@ -853,7 +910,7 @@ __global__ void __launch_bounds__(kFrontierThreads, 1024 / kFrontierThreads) fro
                 if (a.cvtx) a.cvtx[ocs + j] = ov;
             }
             const uint64_t owl = (uint64_t)onch * CW + od;
-            const uint64_t ot_lo = (oW + TW - 1) / TW, ot_hi = (oW + owl + TW - 1) / TW;
+            const uint64_t ot_lo = (oW + TW - 1) >> TWs, ot_hi = (oW + owl + TW - 1) >> TWs;
             for (uint64_t t = ot_lo + lane; t < ot_hi; t += 32)
                 a.tiles[t] = (uint32_t)(ocs + tile_chunk((uint32_t)(t * TW - oW), onch));
         }
