@@ -70,10 +70,12 @@ def parse():
     p.add_argument("--mode", default="partition", choices=["partition", "replicas"],
                    help="N > 1: 1-D partitioned BFS with a per-level NCCL exchange (SURVEY 8(e)), "
                         "or independent replicas on disjoint sources")
-    p.add_argument("--xchg", default="peer", choices=["peer", "nccl"],
+    p.add_argument("--xchg", default="peer", choices=["peer", "hostseq", "nccl"],
                    help="N > 1 partition mode: per-level exchange by the library's kernels over "
-                        "NVLink peer memory (CUDA IPC, efg_xchg_peer) or all_to_all + all_gather "
-                        "with torch.distributed (efg_xchg_pack/reduce/unpack)")
+                        "NVLink peer memory (CUDA IPC, efg_xchg_peer; collective efg_bfs), the same "
+                        "kernels host-sequenced (efg_xchg_peer_phase + a barrier per phase: no kernel "
+                        "waits for another rank; used automatically when ranks share a GPU), or "
+                        "all_to_all + all_gather with torch.distributed (efg_xchg_pack/reduce/unpack)")
     p.add_argument("--host-resident", action="store_true",
                    help="out-of-core EFG (EFG_HOST_RESIDENT, P:34/P:222): EF data in pinned host memory, "
                         "read by the kernels over the host link")
@@ -428,7 +430,12 @@ def run_partitioned(args, rank, world, local):
     import torch.distributed as dist
     import synth
     import paper_conf_ipps_gerak23_b200 as efg
-    from paper_conf_ipps_gerak23_b200.dist import TorchTransport, partitioned_bfs, peer_setup
+    from paper_conf_ipps_gerak23_b200.dist import (TorchTransport, partitioned_bfs, partitioned_bfs_peer_hostseq,
+                                                   peer_setup)
+    if args.xchg == "peer" and world > torch.cuda.device_count():
+        # ranks time-sharing a GPU must not run kernels that wait on each other
+        # (B200_PROFILING.md: Xid 109): host-sequenced exchange instead
+        args.xchg = "hostseq"
 
     dev = torch.device("cuda", local)
     stream = torch.cuda.Stream(device=dev)
@@ -465,6 +472,9 @@ def run_partitioned(args, rank, world, local):
     if args.xchg == "peer":
         peer_setup(g, rank, b)  # IPC handles all-gathered once; no collective per level
         one_bfs = lambda s: g.bfs(s, depth=depth)  # noqa: E731  collective, enqueue-only
+    elif args.xchg == "hostseq":
+        peer_setup(g, rank, b)
+        one_bfs = lambda s: partitioned_bfs_peer_hostseq(g, s, depth, dist.barrier)  # noqa: E731
     else:
         one_bfs = lambda s: partitioned_bfs(g, s, depth, b, tr, mk)  # noqa: E731
     with torch.cuda.stream(stream):
@@ -492,7 +502,7 @@ def run_partitioned(args, rank, world, local):
         if args.xchg == "peer":
             _, _, st = g.bfs(int(s), depth=depth, stats=True)
         else:
-            partitioned_bfs(g, int(s), depth, b, tr, mk)
+            one_bfs(int(s))
             st = g.bfs_end()
         edges += st["edges_traversed"]
         launches += st["kernel_launches"]
@@ -525,6 +535,9 @@ def run_partitioned(args, rank, world, local):
                                       + ("exchange by the library's kernels over peer memory (owner OR + "
                                          "broadcast, CUDA IPC), collective efg_bfs with the level loop on "
                                          "the device" if args.xchg == "peer" else
+                                         "exchange by the library's kernels over peer memory, host-sequenced "
+                                         "(a barrier per phase; functional: ranks share a GPU)"
+                                         if args.xchg == "hostseq" else
                                          "exchange (all_to_all + OR + all_gather, torch.distributed)"),
                        "ranks_per_gpu": world / max(1, min(world, gpus)),
                        "xchg": args.xchg, "bounds": [int(x) for x in b],
@@ -552,6 +565,10 @@ def run_partitioned(args, rank, world, local):
 def main():
     args = parse()
     rank, world, local = dist_env()
+    if world > 1:
+        # torchrun sets OMP_NUM_THREADS=1; the library's host-side OpenMP work
+        # (depth widening of the e2e call) gets this rank's share of the cores
+        os.environ["OMP_NUM_THREADS"] = str(max(1, (os.cpu_count() or 1) // world))
     if args.impl == "reference":
         run_reference(args, rank, world)
         return
