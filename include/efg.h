@@ -213,6 +213,8 @@ typedef struct efg_stats {
     uint64_t d2h_bytes;        /* out: device->host bytes the call moved for host    *
                                 *       outputs (a host depth array travels as one   *
                                 *       byte per vertex when every depth < 127)      */
+    uint32_t xchg_sparse_levels; /* out (partitioned BFS over the peer exchange):    *
+                                  *  levels whose exchange took the sparse path      */
 } efg_stats;
 
 /*
@@ -347,9 +349,10 @@ efg_status efg_bfs_end(efg_graph *g, efg_stats *st);
  *   efg_bfs_expand; efg_xchg_peer; efg_bfs_finish_level
  * Setup, once per handle and partition (collective: every rank, same world):
  *   efg_peer_alloc   allocates this rank's exchange region (cudaMalloc, 4 *
- *                    (64 + 2 * ceil32(ceil(n/32))) bytes, owned by the handle,
- *                    zeroed) and returns its device address and its 64-byte
- *                    CUDA IPC handle; either may be NULL.
+ *                    (96 + 2 * W + 2 * (W / 32 + 32)) bytes with W =
+ *                    ceil32(ceil(n/32)), owned by the handle, zeroed) and
+ *                    returns its device address and its 64-byte CUDA IPC
+ *                    handle; either may be NULL.
  *   (caller)         all-gathers the handles (e.g. torch.distributed) — or, for
  *                    several handles on one device in one process, the addresses.
  *   efg_peer_open    maps the other ranks' regions: ipc_handles = world * 64
@@ -361,7 +364,12 @@ efg_status efg_bfs_end(efg_graph *g, efg_stats *st);
  *                    kernels: publish, barrier, owner OR + broadcast, barrier,
  *                    unpack; the cross-rank barriers over flags in the regions
  *                    spin in one block each) and returns.  Every rank must call
- *                    it once per level.
+ *                    it once per level.  Sparse levels: when no
+ *                    rank has more than W/32 + 32 non-zero words of new bits,
+ *                    every rank ORs the others' published (word, bits) lists
+ *                    into its bitmap instead (no owner step, traffic in
+ *                    proportion to the discoveries); all ranks take the same
+ *                    decision from the published counts.
  *   efg_xchg_peer_phase  the same exchange without the device barriers, one
  *                    phase per call (0 publish, 1 owner OR + broadcast, 2
  *                    unpack), each synchronising the handle's stream before it

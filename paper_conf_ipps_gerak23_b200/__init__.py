@@ -208,6 +208,7 @@ class Graph:
                   "vertices_reached": st.vertices_reached, "device_ms": st.device_ms,
                   "expand_ms": st.expand_ms, "expand_launches": st.expand_launches,
                   "kernel_launches": st.kernel_launches, "d2h_bytes": st.d2h_bytes,
+                  "xchg_sparse_levels": st.xchg_sparse_levels,
                   "level_frontier": arrs[0][:min(L, level_cap)].copy(),
                   "level_edges": arrs[1][:min(L, level_cap)].copy(),
                   "level_expand_ms": arrs[2][:min(L, level_cap)].copy(),
@@ -284,6 +285,7 @@ class Graph:
         L = min(st.levels + 1, level_cap)
         return {"levels": st.levels, "edges_traversed": st.edges_traversed,
                 "vertices_reached": st.vertices_reached, "kernel_launches": st.kernel_launches,
+                "xchg_sparse_levels": st.xchg_sparse_levels,
                 "level_frontier": lf[:L].copy(), "level_edges": le[:L].copy()}
 
     def sssp(self, source: int, dist=None, stats: bool = False):

@@ -49,7 +49,8 @@ class Stats(C.Structure):
                 ("expand_launches", C.c_uint32), ("kernel_launches", C.c_uint32),
                 ("expand_bytes", C.c_uint64), ("level_frontier", C.c_void_p),
                 ("level_edges", C.c_void_p), ("level_expand_ms", C.c_void_p),
-                ("level_end_ms", C.c_void_p), ("d2h_bytes", C.c_uint64)]
+                ("level_end_ms", C.c_void_p), ("d2h_bytes", C.c_uint64),
+                ("xchg_sparse_levels", C.c_uint32)]
 
 
 # (name, restype, argtypes) for every symbol include/efg.h declares

@@ -234,6 +234,7 @@ PeerArgs peer_args(DeviceGraph &d, int op)
     a.prev = d.prev;
     a.fault = &d.ctrl->fault;
     a.epoch = &d.ctrl->peer_epoch;
+    a.sparse_levels = &d.ctrl->xchg_sparse;
     a.nwords = d.nwords;
     a.world = d.peer_world;
     a.rank = d.peer_rank;
@@ -795,6 +796,7 @@ efg_status device_bfs(efg_graph *g, uint32_t source, int32_t *depth, uint32_t *p
         st->kernel_launches = launches;
         st->expand_bytes = 0;
         st->d2h_bytes = d2h;
+        st->xchg_sparse_levels = part ? d.ctrl_host->xchg_sparse : 0u;
         for (uint32_t i = 0; i < std::min<uint32_t>((uint32_t)lf.size(), st->level_cap); ++i) {
             if (st->level_frontier) st->level_frontier[i] = lf[i];
             if (st->level_edges) st->level_edges[i] = le[i];
@@ -883,6 +885,7 @@ efg_status device_step_end(efg_graph *g, efg_stats *st)
     st->vertices_reached = reached;   // this rank's rows
     st->expand_launches = d.step_levels;
     st->kernel_launches = d.step_launches;
+    st->xchg_sparse_levels = d.ctrl_host->xchg_sparse;
     for (uint32_t i = 0; i < std::min<uint32_t>((uint32_t)d.step_lf.size(), st->level_cap); ++i) {
         if (st->level_frontier) st->level_frontier[i] = d.step_lf[i];
         if (st->level_edges) st->level_edges[i] = d.step_le[i];

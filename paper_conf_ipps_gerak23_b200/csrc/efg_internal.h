@@ -105,6 +105,7 @@ struct LevelCtrl {
     uint32_t vpre_used; // visited prefix the last BFS expand used (0: none); lower bound for the next level end
     uint32_t fault;     // a frontier_kernel grid barrier timed out (sticky; reported by the host)
     uint32_t peer_epoch;  // peer exchange counter (efg_xchg_peer / partitioned efg_bfs): +2 per exchange
+    uint32_t xchg_sparse; // exchanges of the current traversal that took the sparse path
     unsigned long long bstat[8];  // debug builds (EFG_BATCH_STATS): expand batch counters of the last level
 };
 

@@ -196,6 +196,7 @@ __global__ void init_kernel(InitArgs a)
         a.ctrl->vmin2[0] = FULL;
         a.ctrl->vmin2[1] = FULL;
         a.ctrl->vpre_used = 0;
+        a.ctrl->xchg_sparse = 0;
         if (a.parent) a.parent[a.v0] = (uint32_t)a.v0;
     }
     const uint64_t w0 = a.v0 >> 5, w1 = (a.v1 + 31) >> 5;
@@ -246,10 +247,15 @@ __global__ void xchg_kernel(XchgArgs a)
 // order on each rank (the barriers are one-block kernels, the data ops never
 // spin):
 //   op 0  publish:  pub[w] = vis[w] & ~prev[w]                 (local)
+//                   + the non-zero words as a (word, bits) list while they
+//                     number <= cap (warp-aggregated appends)
 //   op 3  barrier e
-//   op 1  for owned words w: m = OR_p pub_p[w]; res_p[w] = m for all p
+//   op 1  every rank reads all ranks' list counts (same decision everywhere):
+//         sparse (every count <= cap): vis[w] |= bits for the entries of the
+//           OTHER ranks' lists (one pass, no owner step, traffic ~ discoveries)
+//         dense: for owned words w: m = OR_p pub_p[w]; res_p[w] = m for all p
 //   op 4  barrier e+1
-//   op 2  vis[w] |= res[w]                                     (local)
+//   op 2  dense: vis[w] |= res[w] (local); both: reset this rank's count
 // Barrier e: block 0 stores e into flags[rank] of every rank (release, system
 // scope), every block waits until all of its own flags reach e (acquire).
 // Reuse is safe without more barriers: a rank republishes (op 0 of the next
@@ -291,10 +297,29 @@ __device__ __forceinline__ bool peer_barrier(const PeerArgs &a, uint32_t e)
 __global__ void peer_kernel(PeerArgs a)
 {
     const uint64_t pub = kPeerFlagWords, res = kPeerFlagWords + peer_pad(a.nwords);
+    const uint64_t sp = peer_sp_off(a.nwords), lst = sp + kPeerSpWords;
+    const uint32_t cap = (uint32_t)peer_list_cap(a.nwords);
     const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
     const uint64_t t0 = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
     if (a.op == 0) {
-        for (uint64_t w = t0; w < a.nwords; w += stride) a.local[pub + w] = a.vis[w] & ~a.prev[w];
+        // whole warps iterate together (the list appends are warp-aggregated)
+        const uint64_t tw = t0 & ~31ull;
+        const uint32_t lane = threadIdx.x & 31;
+        for (uint64_t w0 = tw; w0 < a.nwords; w0 += stride) {
+            const uint64_t w = w0 + lane;
+            const uint32_t m = w < a.nwords ? a.vis[w] & ~a.prev[w] : 0u;
+            if (w < a.nwords) a.local[pub + w] = m;
+            const uint32_t bal = __ballot_sync(FULL, m != 0);
+            if (bal && __ldcg(a.local + sp) <= cap) {  // (past cap the level is dense: stop appending)
+                uint32_t base = 0;
+                if (lane == 0) base = atomicAdd(a.local + sp, (uint32_t)__popc(bal));
+                base = __shfl_sync(FULL, base, 0) + __popc(bal & ((1u << lane) - 1));
+                if (m && base < cap) {
+                    a.local[lst + 2 * (uint64_t)base] = (uint32_t)w;
+                    a.local[lst + 2 * (uint64_t)base + 1] = m;
+                }
+            }
+        }
         // barrier epochs of this exchange: E - 1 (before op 1) and E (before
         // op 2), E = the counter after this increment (a device counter, so a
         // captured level loop advances it every iteration; every rank runs the
@@ -308,6 +333,33 @@ __global__ void peer_kernel(PeerArgs a)
         return;
     }
     if (a.op == 1) {
+        // the decision: every rank sees the same published counts
+        __shared__ uint32_t s_cnt[kPeerMaxWorld];
+        __shared__ int s_sparse;
+        if (threadIdx.x == 0) s_sparse = 1;
+        __syncthreads();
+        if (threadIdx.x < (unsigned)a.world) {
+            s_cnt[threadIdx.x] = __ldcv(a.peers[threadIdx.x] + sp);
+            if (s_cnt[threadIdx.x] > cap) s_sparse = 0;
+        }
+        __syncthreads();
+        if (s_sparse) {
+            if (blockIdx.x == 0 && threadIdx.x == 0) {
+                a.local[sp + 1] = 1;
+                *a.sparse_levels += 1;
+            }
+            for (int p = 0; p < a.world; ++p) {
+                if (p == a.rank) continue;  // its own bits are in vis already
+                const uint32_t *l = a.peers[p] + lst;
+                for (uint64_t i = t0; i < s_cnt[p]; i += stride) {
+                    const uint32_t w = __ldcv(l + 2 * i), m = __ldcv(l + 2 * i + 1);
+                    atomicOr(a.vis + w, m);
+                }
+            }
+            __threadfence_system();
+            return;
+        }
+        if (blockIdx.x == 0 && threadIdx.x == 0) a.local[sp + 1] = 0;
         const uint64_t w0 = a.bounds[a.rank] / 32, w1 = (a.bounds[a.rank + 1] + 31) / 32;
         for (uint64_t w = w0 + t0; w < w1; w += stride) {
             uint32_t m = 0;
@@ -317,6 +369,11 @@ __global__ void peer_kernel(PeerArgs a)
         __threadfence_system();
         return;
     }
+    // op 2 (every peer has passed its op 1: the list and its count may be reused)
+    const bool sparse = __ldcv(a.local + sp + 1) != 0;
+    __syncthreads();
+    if (blockIdx.x == 0 && threadIdx.x == 0) a.local[sp] = 0;
+    if (sparse) return;
     for (uint64_t w = t0; w < a.nwords; w += stride) {
         const uint32_t m = __ldcv(a.local + res + w);
         if (m) a.vis[w] |= m;

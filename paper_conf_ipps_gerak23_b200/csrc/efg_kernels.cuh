@@ -61,12 +61,23 @@ struct XchgArgs {
 
 // Peer-memory exchange (efg_xchg_peer): every rank's region, mapped into every
 // rank (CUDA IPC over NVLink / NVSwitch, or plain pointers on one device), is
-//   [flags: kPeerFlagWords u32 | pub: peer_pad(nwords) u32 | res: nwords u32]
-// flags[p] = the last barrier epoch rank p signalled to this rank.
+//   [flags: kPeerFlagWords u32 | pub: peer_pad(nwords) u32 | res: peer_pad(nwords) u32 |
+//    sp: kPeerSpWords u32 | list: 2 * peer_list_cap(nwords) u32]
+// flags[p] = the last barrier epoch rank p signalled to this rank; sp[0] = the
+// number of non-zero words this rank published (its sparse list: (word, bits)
+// pairs, complete while sp[0] <= cap); sp[1] = this rank's decision for the
+// current exchange (1 sparse, 0 dense).
 constexpr int kPeerMaxWorld = 64;
 constexpr uint64_t kPeerFlagWords = 64;
+constexpr uint64_t kPeerSpWords = 32;
 __host__ __device__ inline uint64_t peer_pad(uint64_t nwords) { return (nwords + 31) & ~31ull; }
-__host__ __device__ inline uint64_t peer_region_words(uint64_t nwords) { return kPeerFlagWords + 2 * peer_pad(nwords); }
+// sparse-level exchange: at most 1/32 of the words non-zero on every rank
+__host__ __device__ inline uint64_t peer_list_cap(uint64_t nwords) { return peer_pad(nwords) / 32 + 32; }
+__host__ __device__ inline uint64_t peer_sp_off(uint64_t nwords) { return kPeerFlagWords + 2 * peer_pad(nwords); }
+__host__ __device__ inline uint64_t peer_region_words(uint64_t nwords)
+{
+    return peer_sp_off(nwords) + kPeerSpWords + 2 * peer_list_cap(nwords);
+}
 
 struct PeerArgs {
     uint32_t *const *peers;        // device array [world]: region base of every rank (own included)
@@ -78,6 +89,7 @@ struct PeerArgs {
     uint64_t nwords;
     uint32_t *epoch;               // device exchange counter (LevelCtrl.peer_epoch): op 0 adds 2,
                                    // ops 1 and 2 wait on barrier epochs counter-1 and counter
+    uint32_t *sparse_levels;       // LevelCtrl.xchg_sparse: exchanges that took the sparse path
     int world, rank;
     int op;                        // 0 publish, 1 owner OR + broadcast, 2 unpack, 3 / 4 barrier (one block)
 };

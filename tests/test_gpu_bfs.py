@@ -421,14 +421,21 @@ def test_partitioned_bfs_peer_exchange_simulated_ranks(efg, world):
         graphs = [efg.Graph.build(n, src, dst, flags=flags, stream=streams[r].cuda_stream,
                                   rows=(int(bounds[r]), int(bounds[r + 1]))) for r in range(world)]
         simulated_peer_setup(graphs, bounds)
+        sparse = dense = 0
         for s in (0, 3, 9999, n - 1):
             depths = [torch.empty(n, dtype=torch.int32, device="cuda") for _ in range(world)]
             torch.cuda.synchronize()
-            simulated_partitioned_bfs_peer(graphs, s, depths)
+            counts = simulated_partitioned_bfs_peer(graphs, s, depths)
             torch.cuda.synchronize()
             ref = oracle.bfs(ov, oe, s)
             for d in depths:
                 assert np.array_equal(d.cpu().numpy(), ref)
+            sts = [g.bfs_end() for g in graphs]
+            assert len({st["xchg_sparse_levels"] for st in sts}) == 1  # one decision on every rank
+            sparse += sts[0]["xchg_sparse_levels"]
+            dense += len(counts) - sts[0]["xchg_sparse_levels"]
+        if world > 1:  # both exchange paths ran (small levels sparse, the heavy ones dense)
+            assert sparse > 0 and dense > 0, (sparse, dense)
         for g in graphs:
             g.free()
 

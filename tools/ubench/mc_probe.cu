@@ -38,15 +38,25 @@ int main()
     if (!mcs) return 0;
     CUmulticastObjectProp mp = {};
     mp.numDevices = 1;
-    mp.handleTypes = CU_MEM_HANDLE_TYPE_NONE;
     size_t gran = 0;
     mp.size = 1 << 21;
-    CK(cuMulticastGetGranularity(&gran, &mp, CU_MULTICAST_GRANULARITY_RECOMMENDED));
-    size_t size = ((size_t)(1 << 21) + gran - 1) / gran * gran;
-    mp.size = size;
-    printf("granularity=%zu size=%zu\n", gran, size);
     CUmemGenericAllocationHandle mch;
-    CK(cuMulticastCreate(&mch, &mp));
+    bool made = false;
+    const CUmemAllocationHandleType types[] = {CU_MEM_HANDLE_TYPE_POSIX_FILE_DESCRIPTOR, CU_MEM_HANDLE_TYPE_FABRIC,
+                                               CU_MEM_HANDLE_TYPE_NONE};
+    size_t size = 0;
+    for (auto t : types) {
+        mp.handleTypes = t;
+        mp.size = 1 << 21;
+        CUresult r = cuMulticastGetGranularity(&gran, &mp, CU_MULTICAST_GRANULARITY_RECOMMENDED);
+        if (r != CUDA_SUCCESS) { printf("granularity(type %d) -> %d\n", (int)t, (int)r); continue; }
+        size = ((size_t)(1 << 21) + gran - 1) / gran * gran;
+        mp.size = size;
+        r = cuMulticastCreate(&mch, &mp);
+        printf("cuMulticastCreate(type %d, numDevices 1, size %zu, gran %zu) -> %d\n", (int)t, size, gran, (int)r);
+        if (r == CUDA_SUCCESS) { made = true; break; }
+    }
+    if (!made) return 0;
     CK(cuMulticastAddDevice(mch, dev));
     CUmemAllocationProp ap = {};
     ap.type = CU_MEM_ALLOCATION_TYPE_PINNED;
