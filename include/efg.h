@@ -42,7 +42,8 @@ typedef enum efg_status {
     EFG_ECUDA = 4,   /* a CUDA runtime error (message in efg_last_error)         */
     EFG_ENCCL = 5,   /* a NCCL error (multi-GPU)                                 */
     EFG_ENOTSUP = 6, /* the operation is not available on this handle            */
-    EFG_ESTATE = 7   /* handle in the wrong state (e.g. host-only handle)        */
+    EFG_ESTATE = 7,  /* handle in the wrong state (e.g. host-only handle)        */
+    EFG_EIO = 8      /* efg_save / efg_load: a file that cannot be written / read */
 } efg_status;
 
 /* efg_build_opts.flags (SURVEY §8(c) readings C11, C12) */
@@ -143,6 +144,28 @@ typedef void (*efg_edge_gen_fn)(void *user, uint64_t first, uint64_t count, uint
                                 float *w);
 efg_status efg_build_stream(uint64_t n, uint64_t m, efg_edge_gen_fn gen, void *user, int weighted,
                             const efg_build_opts *opts, efg_graph **out);
+
+/*
+ * efg_save / efg_load — the on-disk EFG: a built graph written once and loaded
+ * without rebuilding (the builder's minutes on C3-C5 become a file read).
+ * The file holds a fixed header (magic "EFGRAPH1", version, n, m, k, row
+ * range, section byte totals, the length of every array) followed by the
+ * P:113 arrays vlist (u64[n+1]), num_lower_bits (u8[n]), offsets (u64[n+1]),
+ * data (u8[offsets[n]]), then the builder's derived arrays: largest neighbour
+ * (u32[n]), in-edge flags (u8[n]), the EFG_REORDER_DEGREE relabelling
+ * (u32[n] twice, or absent) and the CSR-order weights (f32[m], or absent).
+ * Native byte order (little-endian on every supported host).
+ *   efg_save: g may be host-only or on a device; the host arrays are written.
+ *   efg_load: opts->device / stream / flags & EFG_HOST_RESIDENT apply as in
+ *     efg_build (NULL: defaults, device 0); the other options are the file's.
+ *     The loaded handle equals the saved one (efg_export, efg_export_perm,
+ *     every traversal).
+ * Errors: EFG_EINVAL (null argument), EFG_EIO (open / write / read failure,
+ * not an EFG file, other version, inconsistent header, truncated file), then
+ * as efg_build for the upload.
+ */
+efg_status efg_save(const efg_graph *g, const char *path);
+efg_status efg_load(const char *path, const efg_build_opts *opts, efg_graph **out);
 
 /* Release everything the handle owns (host and device).  NULL-safe. */
 void efg_free(efg_graph *g);

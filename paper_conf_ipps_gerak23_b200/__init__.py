@@ -12,6 +12,7 @@ decode lists inside the BFS frontier-expansion kernel.
 from __future__ import annotations
 
 import ctypes as C
+import os
 
 import numpy as np
 
@@ -100,6 +101,23 @@ class Graph:
         h = C.c_void_p()
         check(lib.efg_build_stream(n, m, gen_fn, gen_user, 1 if weighted else 0, C.byref(o), C.byref(h)),
               "efg_build_stream")
+        return cls(h.value, stream)
+
+    def save(self, path: str) -> None:
+        """efg_save: write the built graph to `path` (the on-disk EFG)."""
+        check(lib.efg_save(self._h, os.fsencode(path)), "efg_save")
+
+    @classmethod
+    def load(cls, path: str, *, flags: int = 0, device: int = 0, stream: int | None = None):
+        """efg_load: a graph saved with save(); `flags` may add EFG_HOST_RESIDENT,
+        `device` = -1 keeps it host-only."""
+        o = _abi.BuildOpts()
+        lib.efg_default_opts(C.byref(o))
+        o.flags = flags
+        o.device = device
+        o.stream = stream
+        h = C.c_void_p()
+        check(lib.efg_load(os.fsencode(path), C.byref(o), C.byref(h)), "efg_load")
         return cls(h.value, stream)
 
     def set_level_loop(self, host: bool) -> None:

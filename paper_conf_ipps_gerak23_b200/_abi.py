@@ -13,9 +13,9 @@ _HERE = os.path.dirname(os.path.abspath(__file__))
 # EFG_LIB: an alternative build of the same library (tuning experiments only)
 LIB_PATH = os.environ.get("EFG_LIB") or os.path.join(_HERE, "libefg.so")
 
-EFG_OK, EFG_EINVAL, EFG_ERANGE, EFG_ENOMEM, EFG_ECUDA, EFG_ENCCL, EFG_ENOTSUP, EFG_ESTATE = range(8)
+EFG_OK, EFG_EINVAL, EFG_ERANGE, EFG_ENOMEM, EFG_ECUDA, EFG_ENCCL, EFG_ENOTSUP, EFG_ESTATE, EFG_EIO = range(9)
 STATUS_NAMES = {0: "EFG_OK", 1: "EFG_EINVAL", 2: "EFG_ERANGE", 3: "EFG_ENOMEM", 4: "EFG_ECUDA",
-                5: "EFG_ENCCL", 6: "EFG_ENOTSUP", 7: "EFG_ESTATE"}
+                5: "EFG_ENCCL", 6: "EFG_ENOTSUP", 7: "EFG_ESTATE", 8: "EFG_EIO"}
 EFG_SYMMETRIZE, EFG_DEDUP, EFG_DROP_SELF_LOOPS = 0x1, 0x2, 0x4
 EFG_DEFAULT_FLAGS = 0x7
 EFG_REORDER_DEGREE = 0x8
@@ -61,6 +61,8 @@ SIGNATURES = [
     ("efg_build_stream", C.c_int, [C.c_uint64, C.c_uint64, C.c_void_p, C.c_void_p, C.c_int,
                                    C.POINTER(BuildOpts), C.POINTER(C.c_void_p)]),
     ("efg_free", None, [C.c_void_p]),
+    ("efg_save", C.c_int, [C.c_void_p, C.c_char_p]),
+    ("efg_load", C.c_int, [C.c_char_p, C.POINTER(BuildOpts), C.POINTER(C.c_void_p)]),
     ("efg_info", C.c_int, [C.c_void_p, C.POINTER(Info)]),
     ("efg_export", C.c_int, [C.c_void_p, C.c_void_p, C.c_void_p, C.c_void_p, C.c_void_p]),
     ("efg_export_perm", C.c_int, [C.c_void_p, C.c_void_p]),

@@ -12,6 +12,19 @@
 #include "efg_internal.h"
 #include "efg_kernels.cuh"
 
+#include <nvtx3/nvToolsExt.h>  // header-only NVTX v3: no-ops unless a profiler injects itself
+
+namespace {
+// NVTX range over one C-ABI call (tracing): ncu --nvtx / Nsight
+// Systems show every efg_* call of the host timeline by name
+struct NvtxRange {
+    explicit NvtxRange(const char *name) { nvtxRangePushA(name); }
+    ~NvtxRange() { nvtxRangePop(); }
+    NvtxRange(const NvtxRange &) = delete;
+    NvtxRange &operator=(const NvtxRange &) = delete;
+};
+}  // namespace
+
 using namespace efg;
 
 #define CUDA_TRY(expr)                                                                         \
@@ -91,6 +104,7 @@ efg_status build_common(uint64_t n, const efg_build_opts *opts, efg_graph **out,
 extern "C" efg_status efg_build(uint64_t n, uint64_t m, const uint32_t *src, const uint32_t *dst,
                                 const efg_build_opts *opts, efg_graph **out)
 {
+    NvtxRange nvtx_range("efg_build");
     clear_error();
     if (m && (!src || !dst)) {
         if (out) *out = nullptr;
@@ -104,6 +118,7 @@ extern "C" efg_status efg_build(uint64_t n, uint64_t m, const uint32_t *src, con
 extern "C" efg_status efg_build_stream(uint64_t n, uint64_t m, efg_edge_gen_fn gen, void *user, int weighted,
                                        const efg_build_opts *opts, efg_graph **out)
 {
+    NvtxRange nvtx_range("efg_build_stream");
     clear_error();
     if (m && !gen) {
         if (out) *out = nullptr;
@@ -114,6 +129,32 @@ extern "C" efg_status efg_build_stream(uint64_t n, uint64_t m, efg_edge_gen_fn g
         o2.weights = nullptr;
         return build_host_stream(n, m, gen, user, weighted, o2, h);
     });
+}
+
+extern "C" efg_status efg_save(const efg_graph *g, const char *path)
+{
+    NvtxRange nvtx_range("efg_save");
+    clear_error();
+    if (!g || !path) return set_error(EFG_EINVAL, "efg_save: null handle or path");
+    return save_host(g->host, path);
+}
+
+extern "C" efg_status efg_load(const char *path, const efg_build_opts *opts, efg_graph **out)
+{
+    NvtxRange nvtx_range("efg_load");
+    clear_error();
+    if (!path) {
+        if (out) *out = nullptr;
+        return set_error(EFG_EINVAL, "efg_load: path is NULL");
+    }
+    efg_build_opts o;
+    if (opts)
+        o = *opts;
+    else
+        efg_default_opts(&o);
+    o.row_lo = o.row_hi = 0;  // the file's row range applies
+    o.weights = nullptr;
+    return build_common(1, &o, out, [&](const efg_build_opts &, HostEFG &h) { return load_host(path, h); });
 }
 
 extern "C" void efg_free(efg_graph *g)
@@ -177,6 +218,7 @@ extern "C" efg_status efg_export_perm(const efg_graph *g, uint32_t *old_of_new)
 
 extern "C" efg_status efg_decode(efg_graph *g, uint32_t v0, uint32_t v1, uint32_t *out)
 {
+    NvtxRange nvtx_range("efg_decode");
     clear_error();
     EFG_TRY(check_handle(g));
     const HostEFG &h = g->host;
@@ -188,6 +230,7 @@ extern "C" efg_status efg_decode(efg_graph *g, uint32_t v0, uint32_t v1, uint32_
 
 extern "C" efg_status efg_bfs(efg_graph *g, uint32_t source, int32_t *depth, uint32_t *parent, efg_stats *st)
 {
+    NvtxRange nvtx_range("efg_bfs");
     clear_error();
     EFG_TRY(check_handle(g));
     if (source >= g->dev.n) return set_error(EFG_ERANGE, "efg_bfs: source >= n");
@@ -230,6 +273,7 @@ extern "C" efg_status efg_set_option(efg_graph *g, int option, int64_t value)
 
 extern "C" efg_status efg_sssp(efg_graph *g, uint32_t source, float *dist, efg_stats *st)
 {
+    NvtxRange nvtx_range("efg_sssp");
     clear_error();
     EFG_TRY(check_handle(g));
     if (source >= g->dev.n) return set_error(EFG_ERANGE, "efg_sssp: source >= n");
@@ -242,6 +286,7 @@ extern "C" efg_status efg_sssp(efg_graph *g, uint32_t source, float *dist, efg_s
 
 extern "C" efg_status efg_pagerank(efg_graph *g, double damping, uint32_t iters, double *rank, efg_stats *st)
 {
+    NvtxRange nvtx_range("efg_pagerank");
     clear_error();
     EFG_TRY(check_handle(g));
     if (!rank) return set_error(EFG_EINVAL, "efg_pagerank: rank is NULL");
@@ -266,6 +311,7 @@ extern "C" efg_status efg_xchg_geometry(const efg_graph *g, int world, const uin
 
 extern "C" efg_status efg_bfs_begin(efg_graph *g, uint32_t source, int32_t *depth_device)
 {
+    NvtxRange nvtx_range("efg_bfs_begin");
     clear_error();
     EFG_TRY(check_handle(g));
     if (source >= g->dev.n) return set_error(EFG_ERANGE, "efg_bfs_begin: source >= n");
@@ -276,6 +322,7 @@ extern "C" efg_status efg_bfs_begin(efg_graph *g, uint32_t source, int32_t *dept
 
 extern "C" efg_status efg_bfs_expand(efg_graph *g)
 {
+    NvtxRange nvtx_range("efg_bfs_expand");
     clear_error();
     EFG_TRY(check_handle(g));
     return device_step_expand(g);
@@ -284,6 +331,7 @@ extern "C" efg_status efg_bfs_expand(efg_graph *g)
 extern "C" efg_status efg_xchg_pack(efg_graph *g, int world, const uint64_t *bounds, uint64_t slice_words,
                                     uint32_t *send)
 {
+    NvtxRange nvtx_range("efg_xchg_pack");
     clear_error();
     EFG_TRY(check_handle(g));
     if (world < 1 || !bounds || !send) return set_error(EFG_EINVAL, "efg_xchg_pack: bad args");
@@ -293,6 +341,7 @@ extern "C" efg_status efg_xchg_pack(efg_graph *g, int world, const uint64_t *bou
 extern "C" efg_status efg_xchg_reduce(efg_graph *g, int world, uint64_t slice_words, const uint32_t *recv,
                                       uint32_t *mine)
 {
+    NvtxRange nvtx_range("efg_xchg_reduce");
     clear_error();
     EFG_TRY(check_handle(g));
     if (world < 1 || !recv || !mine) return set_error(EFG_EINVAL, "efg_xchg_reduce: bad args");
@@ -302,6 +351,7 @@ extern "C" efg_status efg_xchg_reduce(efg_graph *g, int world, uint64_t slice_wo
 extern "C" efg_status efg_xchg_unpack(efg_graph *g, int world, const uint64_t *bounds, uint64_t slice_words,
                                       const uint32_t *gathered)
 {
+    NvtxRange nvtx_range("efg_xchg_unpack");
     clear_error();
     EFG_TRY(check_handle(g));
     if (world < 1 || !bounds || !gathered) return set_error(EFG_EINVAL, "efg_xchg_unpack: bad args");
@@ -310,6 +360,7 @@ extern "C" efg_status efg_xchg_unpack(efg_graph *g, int world, const uint64_t *b
 
 extern "C" efg_status efg_peer_alloc(efg_graph *g, int world, void **region, uint8_t *ipc_handle)
 {
+    NvtxRange nvtx_range("efg_peer_alloc");
     clear_error();
     EFG_TRY(check_handle(g));
     if (world < 1 || world > kPeerMaxWorld) return set_error(EFG_EINVAL, "efg_peer_alloc: world outside [1, 64]");
@@ -319,6 +370,7 @@ extern "C" efg_status efg_peer_alloc(efg_graph *g, int world, void **region, uin
 extern "C" efg_status efg_peer_open(efg_graph *g, int world, int rank, const uint64_t *bounds,
                                     const uint8_t *ipc_handles, void *const *regions)
 {
+    NvtxRange nvtx_range("efg_peer_open");
     clear_error();
     EFG_TRY(check_handle(g));
     if (world < 1 || world > kPeerMaxWorld || rank < 0 || rank >= world || !bounds ||
@@ -329,6 +381,7 @@ extern "C" efg_status efg_peer_open(efg_graph *g, int world, int rank, const uin
 
 extern "C" efg_status efg_xchg_peer(efg_graph *g)
 {
+    NvtxRange nvtx_range("efg_xchg_peer");
     clear_error();
     EFG_TRY(check_handle(g));
     return device_xchg_peer(g);
@@ -336,6 +389,7 @@ extern "C" efg_status efg_xchg_peer(efg_graph *g)
 
 extern "C" efg_status efg_xchg_peer_phase(efg_graph *g, int phase)
 {
+    NvtxRange nvtx_range("efg_xchg_peer_phase");
     clear_error();
     EFG_TRY(check_handle(g));
     if (phase < 0 || phase > 2) return set_error(EFG_EINVAL, "efg_xchg_peer_phase: phase 0..2");
@@ -344,6 +398,7 @@ extern "C" efg_status efg_xchg_peer_phase(efg_graph *g, int phase)
 
 extern "C" efg_status efg_bfs_finish_level(efg_graph *g, uint64_t *global_new)
 {
+    NvtxRange nvtx_range("efg_bfs_finish_level");
     clear_error();
     EFG_TRY(check_handle(g));
     return device_step_finish(g, global_new);
@@ -351,6 +406,7 @@ extern "C" efg_status efg_bfs_finish_level(efg_graph *g, uint64_t *global_new)
 
 extern "C" efg_status efg_bfs_end(efg_graph *g, efg_stats *st)
 {
+    NvtxRange nvtx_range("efg_bfs_end");
     clear_error();
     EFG_TRY(check_handle(g));
     return device_step_end(g, st);
@@ -359,6 +415,7 @@ extern "C" efg_status efg_bfs_end(efg_graph *g, efg_stats *st)
 extern "C" efg_status efg_partition(uint64_t n, const uint64_t *vlist, const uint64_t *offsets, int world,
                                     uint64_t *bounds)
 {
+    NvtxRange nvtx_range("efg_partition");
     clear_error();
     if (!vlist || !offsets || !bounds || world < 1 || n == 0) return set_error(EFG_EINVAL, "efg_partition: bad args");
     // weight of a vertex: compressed bytes + 29 bytes of per-vertex state

@@ -51,6 +51,9 @@ efg_status build_host(uint64_t n, uint64_t m, const uint32_t *src, const uint32_
                       const efg_build_opts &o, HostEFG &out);
 efg_status build_host_stream(uint64_t n, uint64_t m, efg_edge_gen_fn gen, void *user, int weighted,
                              const efg_build_opts &o, HostEFG &out);
+// On-disk EFG (efg_io.cpp).
+efg_status save_host(const HostEFG &h, const char *path);
+efg_status load_host(const char *path, HostEFG &h);
 
 // ---------------------------------------------------------------------------
 // Device layout
