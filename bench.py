@@ -265,7 +265,7 @@ REF_STEP_EDGES = 1 << 28  # reference-arm step: FIFO BFS stopped after this many
 
 
 def _cpu_baseline_child(cfg: int, scale, index: int, count: int, out_dir: str, core: int, permute=None,
-                        go_parallel=None):
+                        go_parallel=None, timed_lock=None):
     """Spawned process (bench.py cpu_baseline leg): the oracle's CSR of the
     same seeded graph, then ONE plain single-threaded FIFO BFS from the first
     timed source, pinned to `core` (the parent keeps off that core).  Writes
@@ -280,9 +280,13 @@ def _cpu_baseline_child(cfg: int, scale, index: int, count: int, out_dir: str, c
     del src, dst
     deg = np.diff(ov)
     s0 = int(synth.sources(n, count, seed=1000 + cfg, nonisolated_mask=deg > 0)[index])
+    if timed_lock is not None:
+        timed_lock.acquire()  # the parent never pauses this process inside its timed BFS
     t = time.perf_counter()
     d = oracle.bfs(ov, oe, s0)
     cs = time.perf_counter() - t
+    if timed_lock is not None:
+        timed_lock.release()
     np.save(os.path.join(out_dir, "depth.npy"), d)
     # a second parity source (untimed): the next timed source
     s1 = int(synth.sources(n, count, seed=1000 + cfg, nonisolated_mask=deg > 0)[min(index + 1, count - 1)])
@@ -313,15 +317,42 @@ def start_cpu_baseline(args, count: int, index: int):
     out_dir = tempfile.mkdtemp(prefix="efg_cpu_baseline_")
     ctx = mp.get_context("spawn")
     go = ctx.Event()
+    lock = ctx.Lock()
     proc = ctx.Process(target=_cpu_baseline_child,
-                       args=(args.config, args.scale, index, count, out_dir, core, args.permute or None, go))
+                       args=(args.config, args.scale, index, count, out_dir, core, args.permute or None, go, lock))
     proc.start()
     if len(cores) > 1:
         os.sched_setaffinity(0, set(cores[:-1]))
-    return proc, out_dir, go
+    return proc, out_dir, go, lock
 
 
-def finish_cpu_baseline(proc, out_dir: str, go, g, n: int):
+def pause_cpu_baseline(job, stop: bool, was_paused: bool = True) -> bool:
+    """SIGSTOP / SIGCONT the cpu_baseline child (None-safe).  Returns whether
+    the child was stopped.  Only outside its timed BFS: the parent holds the
+    child's timing lock while the child is stopped (if the child is inside
+    its timed BFS, nothing is paused)."""
+    import signal
+    if job is None or not was_paused:
+        return False
+    proc, lock = job[0], job[3]
+    if stop:
+        if not proc.is_alive() or not lock.acquire(block=False):
+            return False
+        try:
+            os.kill(proc.pid, signal.SIGSTOP)
+        except OSError:
+            lock.release()
+            return False
+        return True
+    try:
+        os.kill(proc.pid, signal.SIGCONT)
+    except OSError:
+        pass
+    lock.release()
+    return True
+
+
+def finish_cpu_baseline(proc, out_dir: str, go, lock, g, n: int):
     go.set()  # the GPU measurements are over: the child may use every core
     proc.join()
     if proc.exitcode != 0:
@@ -694,6 +725,10 @@ def main():
     # ---- e2e: through the C ABI with a pinned host depth buffer ----
     hdepth = torch.empty(n, dtype=torch.int32, pin_memory=True)
     e2e_edges = 0
+    # the cpu_baseline child (building its CSR on another core) is paused while
+    # the host side of the e2e call is timed: the host memory bandwidth the
+    # depth widening needs is not shared with our own background job
+    paused = pause_cpu_baseline(cpu_job, True)
     torch.cuda.synchronize()
     if world > 1:
         torch.distributed.barrier()
@@ -711,6 +746,8 @@ def main():
         dist.all_reduce(e2e_t, op=dist.ReduceOp.MAX)
         dist.all_reduce(e2e_e, op=dist.ReduceOp.SUM)
     e2e_val = float(e2e_e.item()) / float(e2e_t.item()) / 1e9
+
+    pause_cpu_baseline(cpu_job, False, paused)
 
     # ---- the same measurement without the degree relabelling (transparency) ----
     alt = None

@@ -56,6 +56,14 @@ def test_cpu_baseline_child_pinned_and_checked():
     try:
         for wrong in (False, True):
             job = bench.start_cpu_baseline(Args, 4, 1)
+            if not wrong:  # the e2e pause: stopped outside its timed BFS, then resumed
+                import time
+                time.sleep(0.5)
+                if bench.pause_cpu_baseline(job, True):
+                    time.sleep(0.2)
+                    with open(f"/proc/{job[0].pid}/stat") as f:
+                        assert f.read().split(") ")[1][0] == "T"
+                    assert bench.pause_cpu_baseline(job, False, True)
             cpu = bench.finish_cpu_baseline(*job, Stub(wrong), n)
             os.sched_setaffinity(0, before)
             assert cpu["kind"] == "oracle" and cpu["cores"] == 1 and cpu["value"] > 0
