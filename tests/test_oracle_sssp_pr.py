@@ -117,9 +117,7 @@ def test_pagerank_star_ratio():
     r = oracle.pagerank(vlist, elist, 0.85, 200)
     N = s + 1
     d = 0.85
-    # c = (1-d)/N + d*s*l ; l = (1-d)/N + d*c/s
-    l = ((1 - d) / N + d * (1 - d) / N / s * s / s) / (1 - d * d)  # noqa: E501 (placeholder)
-    # solve the 2x2 linear system exactly instead
+    # centre c and leaf l: c = (1-d)/N + d*s*l ; l = (1-d)/N + d*c/s — the 2x2 linear system
     Amat = np.array([[1.0, -d * s], [-d / s, 1.0]])
     b = np.array([(1 - d) / N, (1 - d) / N])
     c_ref, l_ref = np.linalg.solve(Amat, b)
