@@ -260,7 +260,7 @@ extern "C" efg_status efg_set_option(efg_graph *g, int option, int64_t value)
         }
         return EFG_OK;
     case EFG_OPT_EXPAND_VARIANT:
-        if (value < 0 || value > 63) return set_error(EFG_EINVAL, "EFG_OPT_EXPAND_VARIANT: 0..63");
+        if (value < 0 || value > 127) return set_error(EFG_EINVAL, "EFG_OPT_EXPAND_VARIANT: 0..127");
         if (g->dev.expand_variant != (int)value) {
             g->dev.expand_variant = (int)value;
             efg::device_drop_graphs(g->dev);

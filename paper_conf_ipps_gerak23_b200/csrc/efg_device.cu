@@ -152,6 +152,7 @@ ExpandArgs expand_args(DeviceGraph &d, uint32_t *out)
     a.k = d.k;
     a.pskip = d.prefix_skip ? 1u : 0u;
     a.variant = (uint32_t)d.expand_variant;
+    a.lpc_skip_vpre = (uint32_t)(d.n / 8);
     return a;
 }
 

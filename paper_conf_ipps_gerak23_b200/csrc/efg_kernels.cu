@@ -1186,6 +1186,11 @@ __global__ void __launch_bounds__(kExpandThreads, 1) expand_kernel(ExpandArgs a)
     const uint32_t sbits = smem_u32(st32) * 8;  // shared-window bit address of the staging area
     const uint32_t vpre = kBfs ? a.ctrl->vmin2[xl & 1] : 0u;  // ids below it are visited (or never probed)
     const bool pskip = kBfs && a.pskip && vpre != 0;              // warp-uniform
+    // lane-per-chunk threshold (busy element slots >= 2/lpcf of 32 x the longest
+    // chunk): halved on skip levels (visited prefix past n/8: most elements are
+    // stepped over word by word, so a lane's chunk costs little whatever its
+    // length, while a record round is paid in full)
+    const uint32_t lpcf = (pskip && (a.variant & 64) && vpre >= a.lpc_skip_vpre) ? 4u : 2u;
     if (blockIdx.x == 0 && threadIdx.x == 0) a.ctrl->vpre_used = pskip ? vpre : 0u;
     const uint64_t gw = (uint64_t)blockIdx.x * kExpandWarps + wid;
     const uint64_t nwarps = (uint64_t)gridDim.x * kExpandWarps;
@@ -1273,7 +1278,7 @@ __global__ void __launch_bounds__(kExpandThreads, 1) expand_kernel(ExpandArgs a)
                 B.nel = nel;
                 B.cc = 0;
                 B.v = (MODE != kModeVisit && valid) ? a.cvtx[c] : 0u;
-                B.lpc = kLpc && (a.variant & 1) && 2 * B.ne >= 32 * __reduce_max_sync(FULL, nel);
+                B.lpc = kLpc && (a.variant & 1) && lpcf * B.ne >= 32 * __reduce_max_sync(FULL, nel);
                 const uint32_t sbase = buf * kStageBytes;
                 B.lsmb = sbits + 8 * (sbase + (uint32_t)(off - S)) - B.eb * l;
                 B.lflags = l | ((uint32_t)(A0 & 31) << 8) | ((uint32_t)((A1 - 1) & 31) << 16) | (1u << 24);
@@ -1394,7 +1399,7 @@ __global__ void __launch_bounds__(kExpandThreads, 1) expand_kernel(ExpandArgs a)
         // lane-per-chunk decode when the lanes' chunks are balanced enough:
         // >= 50 % of the warp's element slots busy (the degree relabelling puts
         // lists of similar length next to each other in the frontier)
-        B.lpc = kLpc && (a.variant & 1) && 2 * tot_e >= 32 * __reduce_max_sync(FULL, B.nel);
+        B.lpc = kLpc && (a.variant & 1) && lpcf * tot_e >= 32 * __reduce_max_sync(FULL, B.nel);
         // stage-area byte offset of this chunk's first staged byte
         const uint32_t base = buf * kStageBytes + (span ? (bytes ? (uint32_t)(rs - S) : 0u) : sb);
         const uint32_t lsm = sbits + (l ? base * 8 + (uint32_t)(lb - lg0 * 8) : buf * kStageBytes * 8);

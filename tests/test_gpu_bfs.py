@@ -207,7 +207,7 @@ def test_expand_variants_identical(efg, k):
         g = efg.Graph.build(n, src, dst, k=k, flags=flags, weights=w)
         u = np.repeat(np.arange(n, dtype=np.uint32), deg.astype(np.int64))
         dref = oracle.sssp(ov, oe, synth.weights(u, oe, seed=2005), int(srcs[0]))
-        for mask in (0, 1, 2, 3, 4, 8, 11, 16, 27, 32, 43, 59, 63):
+        for mask in (0, 1, 2, 3, 4, 8, 11, 16, 27, 32, 43, 59, 63, 107, 127):
             g.set_expand_variant(mask)
             _check_bfs(g, ov, oe, srcs)
             g.set_level_loop(True)
