@@ -306,7 +306,7 @@ efg_status efg_pagerank(efg_graph *g, double damping, uint32_t iters, double *ra
                                  * directed or row-range handle): push along every edge with
                                  * fp64 atomicAdd.  Same sums, other order (C21). */
 
-#define EFG_OPT_EXPAND_VARIANT 4 /* tuning / A-B switch of the expand kernel, bit mask (default 43):
+#define EFG_OPT_EXPAND_VARIANT 4 /* tuning / A-B switch of the expand kernel, bit mask (default 107):
                                   * bit 0: batches of balanced chunks are decoded lane-per-chunk
                                   * (each lane walks its own chunk) instead of by word records
                                   * split evenly over the lanes; bit 1: a batch of adjacent chunks
@@ -318,8 +318,10 @@ efg_status efg_pagerank(efg_graph *g, double damping, uint32_t iters, double *ra
                                   * (select0) instead of decoding them; bit 4: tiles are dealt
                                   * to the warps in super-tiles of consecutive tiles; bit 5: the
                                   * level-end list skip uses the visited prefix of the level just
-                                  * expanded (one more grid barrier) instead of the previous one.
-                                  * Values 0..63.  Results are identical for every value. */
+                                  * expanded (one more grid barrier) instead of the previous one;
+                                  * bit 6: on skip levels (visited prefix >= n/8) a batch goes
+                                  * lane-per-chunk from 25 % busy element slots instead of 50 %.
+                                  * Values 0..127.  Results are identical for every value. */
 
 /* Set a per-handle option.  Errors: EFG_EINVAL (unknown option / value),
  * EFG_ESTATE (host-only handle). */

@@ -232,7 +232,7 @@ struct DeviceGraph {
     int level_loop = 0;                // 0 = CUDA graph (device loop), 1 = host loop + events
     int prefix_skip = 1;               // EFG_OPT_PREFIX_SKIP
     int pr_pull = 1;                   // EFG_OPT_PAGERANK_PULL
-    int expand_variant = 43;           // EFG_OPT_EXPAND_VARIANT (bits 0, 1, 3, 5)
+    int expand_variant = 107;          // EFG_OPT_EXPAND_VARIANT (bits 0, 1, 3, 5, 6)
     static constexpr int kLoopGraphs = 3;                 // visit, visit+parent, partitioned visit
     cudaGraph_t loop_graph[kLoopGraphs] = {};
     cudaGraphExec_t loop_exec[kLoopGraphs] = {};

@@ -1,0 +1,5 @@
+python -c "import __graft_entry__ as g; g.build()" > gpurun_out/build.log 2>&1 || { tail -20 gpurun_out/build.log; exit 1; }
+timeout 600 python -m pytest tests/test_gpu_bfs.py -k "variants" -x -q 2>&1 | tail -2
+timeout 1200 python tools/ab_variant.py --config 3 --masks 43,107 --rounds 3 --levels 2>&1 | tail -1
+timeout 900 python tools/ab_variant.py --config 2 --masks 43,107 --rounds 3 --levels 2>&1 | tail -1
+timeout 1800 python tools/ab_variant.py --config 4 --masks 43,107 --rounds 2 --sources 4 --levels 2>&1 | tail -1
