@@ -319,7 +319,7 @@ efg_status efg_pagerank(efg_graph *g, double damping, uint32_t iters, double *ra
                                   * to the warps in super-tiles of consecutive tiles; bit 5: the
                                   * level-end list skip uses the visited prefix of the level just
                                   * expanded (one more grid barrier) instead of the previous one;
-                                  * bit 6: on skip levels (visited prefix >= n/8) a batch goes
+                                  * bit 6: on skip levels (visited prefix >= n/3) a batch goes
                                   * lane-per-chunk from 25 % busy element slots instead of 50 %.
                                   * Values 0..127.  Results are identical for every value. */
 

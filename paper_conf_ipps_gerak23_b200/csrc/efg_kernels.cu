@@ -1187,7 +1187,7 @@ __global__ void __launch_bounds__(kExpandThreads, 1) expand_kernel(ExpandArgs a)
     const uint32_t vpre = kBfs ? a.ctrl->vmin2[xl & 1] : 0u;  // ids below it are visited (or never probed)
     const bool pskip = kBfs && a.pskip && vpre != 0;              // warp-uniform
     // lane-per-chunk threshold (busy element slots >= 2/lpcf of 32 x the longest
-    // chunk): halved on skip levels (visited prefix past n/8: most elements are
+    // chunk): halved on skip levels (visited prefix past n/3: most elements are
     // stepped over word by word, so a lane's chunk costs little whatever its
     // length, while a record round is paid in full)
     const uint32_t lpcf = (pskip && (a.variant & 64) && vpre >= a.lpc_skip_vpre) ? 4u : 2u;

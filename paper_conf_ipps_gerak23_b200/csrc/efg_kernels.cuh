@@ -37,7 +37,7 @@ struct ExpandArgs {
     uint32_t hot_words;        // bitmap words with a shared-memory snapshot (multiple of 4)
     uint32_t k;                // forward-pointer quantum (chunk length); 0 = none
     uint32_t pskip;            // BFS: skip upper words whose ids are all below the visited prefix
-    uint32_t lpc_skip_vpre;    // visited prefix from which a level counts as a skip level (n / 8)
+    uint32_t lpc_skip_vpre;    // visited prefix from which a level counts as a skip level (n / 3)
     uint32_t variant;          // EFG_OPT_EXPAND_VARIANT: bit 0 lane-per-chunk decode, bit 1 span staging
 };
 
