@@ -34,6 +34,41 @@ for flags in (efg.EFG_DEFAULT_FLAGS, efg.EFG_DEFAULT_FLAGS | efg.EFG_REORDER_DEG
     ref = oracle.pagerank(ov, oe, 0.85, 20)
     assert np.abs(pr - ref).sum() / np.abs(ref).sum() < 1e-6
     g.free()
-# (the peer exchange is left out: the sanitizer serialises kernel launches,
-# so one rank's barrier kernel would wait for another rank that cannot start)
+# The peer exchange with device barriers is left out (the sanitizer
+# serialises kernel launches, so one rank's barrier kernel would wait for a
+# rank that cannot start); the host-sequenced form has no such wait: two
+# simulated ranks in this process, the phases issued rank by rank (dense and
+# sparse levels both occur on this graph).
+import torch  # noqa: E402
+from paper_conf_ipps_gerak23_b200.dist import simulated_peer_setup  # noqa: E402
+
+world = 2
+whole = efg.Graph.build(n, src, dst, device=-1)
+vl, _, of, _ = whole.export()
+bounds = efg.partition(vl, of, world)
+whole.free()
+streams = [torch.cuda.Stream() for _ in range(world)]
+gs = [efg.Graph.build(n, src, dst, stream=streams[r].cuda_stream, rows=(int(bounds[r]), int(bounds[r + 1])))
+      for r in range(world)]
+simulated_peer_setup(gs, bounds)
+for s in (0, 5):
+    depths = [torch.empty(n, dtype=torch.int32, device="cuda") for _ in range(world)]
+    for g, d in zip(gs, depths):
+        g.bfs_begin(s, d)
+    while True:
+        for g in gs:
+            g.bfs_expand()
+        for phase in (0, 1, 2):
+            for g in gs:
+                g.xchg_peer_phase(phase)  # synchronises its stream
+        news = [g.bfs_finish_level() for g in gs]
+        assert len(set(news)) == 1
+        if news[0] == 0:
+            break
+    torch.cuda.synchronize()
+    for d in depths:
+        assert np.array_equal(d.cpu().numpy(), oracle.bfs(ov, oe, s))
+    assert len({g.bfs_end()["xchg_sparse_levels"] for g in gs}) == 1
+for g in gs:
+    g.free()
 print("sanitize_target: all traversals match the oracle")
